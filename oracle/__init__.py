@@ -1,0 +1,9 @@
+"""CPU oracle for DyCuckoo (TEST INFRASTRUCTURE ONLY).
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+``--impl reference`` leg may import this package.  The product path
+(paper_conf_icde_lizlhs21_b200) never imports it and fails loudly without its
+CUDA library.  See oracle/dyc_oracle.c for the paper citations and for which
+outputs are pinned ("parity unpinned": placement positions, φ, eviction counts).
+"""
+from .oracle import OracleTable, build_oracle, oracle_lib  # noqa: F401
