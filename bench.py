@@ -1,0 +1,410 @@
+#!/usr/bin/env python
+"""bench.py — DyCuckoo hot path on B200 (BASELINE.json metric: insert/find/delete
+Mops/s; subtable resize ms vs full rehash).
+
+One step = one pass of the whole hot path over one batch of config C2
+("RAND static", BASELINE.json configs[1]): clear the table, insert 2^27 keys
+(fill 0.85), find 2^27 keys (50% hit), upsize one subtable (from θ = 0.85, as in
+P:L809), delete 2^26 keys, downsize that subtable back (from θ ≈ 0.34).
+`value` = (inserts + finds + deletes) / step time, whole job, in Mops/s.
+
+    python bench.py [--gpus N --steps K --warmup W] [--impl reference]
+
+For N > 1 (torchrun) every rank drives its own C2 batch through the hash-
+partitioned router (shard(k) = x_{d+1}(k) mod N, NCCL all-to-all over NVLink) and
+the per-rank work is fixed (weak scaling).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import platform
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "insert/find/delete Mops/s at 1/2/4/8 B200; subtable resize ms vs full rehash"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="dycuckoo", choices=["dycuckoo", "reference"])
+    ap.add_argument("--log2n", type=int, default=27, help="C2 batch size 2^log2n (27 = BASELINE configs[1])")
+    ap.add_argument("--bucket-slots", type=int, default=4)
+    ap.add_argument("--cpu-log2n", type=int, default=23, help="oracle sample size for cpu_baseline")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-rehash", action="store_true")
+    ap.add_argument("--profile-only", action="store_true", help="a few steps, no extras (for ncu)")
+    return ap.parse_args()
+
+
+# ---------------------------------------------------------------- clocks
+class ClockSampler:
+    """Samples SM clock and throttle reasons during the timed region (NVML)."""
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+               0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+               0x100: "display_clock_setting"}
+
+    def __init__(self, index=0, period=0.1):
+        self.index, self.period = index, period
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        self._t = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:  # noqa: BLE001
+            self.nv = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:  # noqa: BLE001
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.nv:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                "samples": len(self.samples)}
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+# ---------------------------------------------------------------- CPU oracle leg
+def run_oracle_sample(log2n: int):
+    """The oracle as it stands (single-threaded C), on C2's shape scaled to 2^log2n
+    keys (same fill 0.85, same 50% hit rate, same 1/2 delete ratio)."""
+    import oracle
+    from paper_conf_icde_lizlhs21_b200 import workload as W
+    wl = W.c2_rand_static(log2_n=log2n)
+    ins, fnd, dele = wl.batches
+    o = oracle.OracleTable(d=wl.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta)
+    t0 = time.perf_counter()
+    o.insert(ins.keys, ins.values)
+    t1 = time.perf_counter()
+    o.find(fnd.keys)
+    t2 = time.perf_counter()
+    o.delete(dele.keys)
+    t3 = time.perf_counter()
+    n_ops = ins.keys.size + fnd.keys.size + dele.keys.size
+    return {
+        "value": n_ops / (t3 - t0) / 1e6, "unit": "Mops/s", "cores": 1, "kind": "oracle",
+        "sample": f"C2 shape scaled to 2^{log2n} keys: {ins.keys.size} inserts (fill 0.85), "
+                  f"{fnd.keys.size} finds (50% hit), {dele.keys.size} deletes; oracle/dyc_oracle.c, 1 thread",
+        "seconds": t3 - t0,
+        "insert_mops": ins.keys.size / (t1 - t0) / 1e6,
+        "find_mops": fnd.keys.size / (t2 - t1) / 1e6,
+        "delete_mops": dele.keys.size / (t3 - t2) / 1e6,
+        "host_cpu": platform.processor() or platform.machine(),
+        "nproc": os.cpu_count(),
+    }
+
+
+def reference_arm(args, rank, world):
+    """--impl reference: the CPU oracle is this tier's reference arm."""
+    if rank != 0:
+        return
+    K, Wm = args.steps, args.warmup
+    log2n = min(args.cpu_log2n, 21)
+    for _ in range(min(Wm, 1)):
+        run_oracle_sample(16)
+    times, ops = [], 0
+    for _ in range(K):
+        r = run_oracle_sample(log2n)
+        times.append(r["seconds"])
+        ops = int(round(r["value"] * 1e6 * r["seconds"]))
+    ms = 1e3 * statistics.mean(times)
+    value = ops / (sum(times) / len(times)) / 1e6
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "Mops/s", "n_gpus": world,
+        "steps": K, "warmup": Wm, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": f"C2 RAND static (BASELINE configs[1]) shape, bounded sample 2^{log2n} keys",
+                   "d": 4, "alpha": 0.3, "beta": 0.85, "bucket_slots": 4},
+        "cpu_baseline": {"value": value, "unit": "Mops/s", "cores": 1, "kind": "oracle",
+                         "sample": f"C2 shape at 2^{log2n} keys per step (insert+find+delete)"},
+        "e2e": {"value": value, "unit": "Mops/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- GPU arm
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        reference_arm(args, rank, world)
+        return
+
+    import numpy as np
+    import torch
+
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    from paper_conf_icde_lizlhs21_b200 import _lib as L
+    from paper_conf_icde_lizlhs21_b200 import workload as W
+    from paper_conf_icde_lizlhs21_b200.table import Table
+
+    n = 1 << args.log2n
+    cap, k_ins, v_ins, k_find, k_del = W.c2_rand_static_torch(args.log2n, device="cuda")
+    if world > 1:
+        return multi_gpu(args, rank, world, local, dist)
+
+    stream = torch.cuda.current_stream()
+    g = Table(d=4, init_capacity=cap, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
+    st_ins = torch.empty(n, dtype=torch.uint8, device="cuda")
+    v_out = torch.empty(n, dtype=torch.int32, device="cuda")
+    f_out = torch.empty(n, dtype=torch.uint8, device="cuda")
+    dv_out = torch.empty(n // 2, dtype=torch.int32, device="cuda")
+    ds_out = torch.empty(n // 2, dtype=torch.uint8, device="cuda")
+    n_ops = n + n + n // 2
+
+    phases = ["clear", "insert", "find", "upsize", "delete", "downsize"]
+
+    def step(record=None):
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(len(phases) + 1)] if record is not None else None
+        if evs: evs[0].record(stream)
+        g.clear()
+        if evs: evs[1].record(stream)
+        g.insert(k_ins, v_ins, st_ins)
+        if evs: evs[2].record(stream)
+        g.find(k_find, v_out, f_out)
+        if evs: evs[3].record(stream)
+        g.resize(+1)
+        if evs: evs[4].record(stream)
+        g.delete(k_del, dv_out, ds_out)
+        if evs: evs[5].record(stream)
+        g.resize(-1)
+        if evs:
+            evs[6].record(stream)
+            record.append(evs)
+
+    # calibration pass (untimed): correctness spot checks + per-phase statistics
+    g.clear()
+    g.insert(k_ins, v_ins, st_ins)
+    s_ins = g.stats()
+    assert s_ins["m"] == n and s_ins["n_upsize"] == 0, s_ins
+    g.find(k_find, v_out, f_out)
+    hit_rate = float(f_out.float().mean().item())
+    phi = s_ins["n_second_table"] / max(1, s_ins["m"])
+    g.resize(+1)
+    g.delete(k_del, dv_out, ds_out)
+    assert int(ds_out.sum().item()) == n // 2
+    s_del_before = g.stats()
+    phi_after_up = s_del_before["n_second_table"] / max(1, s_del_before["m"])
+    g.resize(-1)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+
+    g.launch_count(reset=True)
+    g.profile(True)
+    records = []
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize()
+        t_start = torch.cuda.Event(enable_timing=True)
+        t_end = torch.cuda.Event(enable_timing=True)
+        t_start.record(stream)
+        for _ in range(args.steps):
+            step(records)
+        t_end.record(stream)
+        torch.cuda.synchronize()
+    total_ms = t_start.elapsed_time(t_end)
+    launches = g.launch_count()
+    prof = g.profile_read()
+    g.profile(False)
+    ms_per_step = total_ms / args.steps
+    phase_ms = {p: statistics.mean(r[i].elapsed_time(r[i + 1]) for r in records) for i, p in enumerate(phases)}
+    value = n_ops / (ms_per_step * 1e-3) / 1e6
+
+    # --------------------------------------------------------- roofline
+    peak, peak_src = measured_peaks()
+    E = s_ins["last_insert_evictions"] / max(1, s_ins["last_insert_new"])
+    pend = s_ins["last_insert_pending"]
+    sec = 32
+    bytes_alg = {
+        # find: 1 sector when the key is in its first-choice table, else 2; + key, value, flag
+        "k_find": n * ((hit_rate * (1 + phi) + (1 - hit_rate) * 2) * sec + 9),
+        # upsert on an empty table: both candidate buckets read (existence check),
+        # one sector written for each key placed here; + key, value, status
+        "k_upsert": n * (2 * sec + 9) + (n - pend) * sec,
+        # eviction kernel: per pending key 1 write + 2 sectors per hop (read + exchange)
+        "k_place": pend * sec + s_ins["last_insert_evictions"] * 2 * sec,
+        # delete (all hits): 1+φ reads, 1 write; + key, old value, status
+        "k_delete": (n // 2) * ((1 + phi_after_up) * sec + sec + 9),
+        # upsize: stream the subtable in (8 B/slot) and twice its size out
+        "k_upsize": (cap // 4 // args.bucket_slots + 1) * args.bucket_slots * 24,
+        "k_downsize": (cap // 4 // args.bucket_slots + 1) * args.bucket_slots * 24,
+    }
+    kern = {k: prof[k][0] / args.steps for k in bytes_alg if prof[k][1]}
+    dom = max(kern, key=kern.get)
+    calls = prof[dom][1] / args.steps
+    launch_ms = prof[dom][0] / max(1, prof[dom][1])
+    achieved = bytes_alg[dom] / calls / (launch_ms * 1e-3) / 1e9
+    # random 32-byte gather ceiling on a table-sized buffer (same sector count as one find launch)
+    buf = torch.empty(int(cap * 8 // (1 << 20) + 1) << 20, dtype=torch.uint8, device="cuda")
+    sink = torch.zeros(1, dtype=torch.int64, device="cuda")
+    nreads = int(n * (hit_rate * (1 + phi) + (1 - hit_rate) * 2))
+    for _ in range(2):
+        L.check(L.dyc_bench_gather(buf.data_ptr(), buf.numel(), nreads, 32, 7, sink.data_ptr(),
+                                   stream.cuda_stream), "dyc_bench_gather")
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    L.check(L.dyc_bench_gather(buf.data_ptr(), buf.numel(), nreads, 32, 9, sink.data_ptr(),
+                               stream.cuda_stream), "dyc_bench_gather")
+    e1.record(stream)
+    torch.cuda.synchronize()
+    gather_gbs = nreads * 32 / (e0.elapsed_time(e1) * 1e-3) / 1e9
+    del buf
+    roofline = {
+        "bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
+        "frac": achieved / peak, "peak_source": peak_src, "traffic": None,
+        "algorithmic_bytes_per_launch": bytes_alg[dom] / calls,
+        "launch_ms": launch_ms,
+        "random_32B_gather_gbs": gather_gbs, "frac_of_gather_ceiling": achieved / gather_gbs,
+        "kernel_ms_per_step": {k: round(v, 4) for k, v in kern.items()},
+        "model": {"phi": phi, "hit_rate": hit_rate, "evictions_per_insert": E,
+                  "pending_keys": pend, "sector_bytes": sec},
+    }
+
+    # --------------------------------------------------------- resize baselines
+    resize = {"upsize_ms": phase_ms["upsize"], "downsize_ms": phase_ms["downsize"]}
+    if not args.no_rehash and not args.profile_only:
+        def timed(fn):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            fn()
+            b.record(stream)
+            torch.cuda.synchronize()
+            return a.elapsed_time(b)
+        for name, method in (("reinsert_subtable", L.DYC_RESIZE_REINSERT_SUBTABLE),
+                             ("rehash_all", L.DYC_RESIZE_REHASH_ALL)):
+            g2 = Table(d=4, init_capacity=cap, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
+            g2.insert(k_ins, v_ins, st_ins)                                   # θ = 0.85
+            resize[f"{name}_upsize_ms"] = timed(lambda: g2.resize(+1, -1, method))
+            g2.close()
+            del g2
+        # downsize baselines from θ ≈ 0.30: upsize once, fill to 0.30 of N
+        for name, method in (("split", L.DYC_RESIZE_SPLIT),
+                             ("reinsert_subtable", L.DYC_RESIZE_REINSERT_SUBTABLE),
+                             ("rehash_all", L.DYC_RESIZE_REHASH_ALL)):
+            g2 = Table(d=4, init_capacity=cap, alpha=0.05, beta=0.85, bucket_slots=args.bucket_slots)
+            g2.resize(+1)
+            m30 = int(0.30 * g2.stats()["N"])
+            g2.insert(k_ins[:m30], v_ins[:m30], st_ins[:m30])
+            resize[f"{name}_downsize_ms_from_fill_0.30"] = timed(lambda: g2.resize(-1, -1, method))
+            g2.close()
+            del g2
+        resize["speedup_upsize_vs_rehash_all"] = resize["rehash_all_upsize_ms"] / resize["upsize_ms"]
+
+    # --------------------------------------------------------- e2e (host buffers)
+    e2e = None
+    if not args.no_e2e and not args.profile_only:
+        pin = lambda t: t.cpu().pin_memory().numpy().view(np.uint32)  # noqa: E731
+        hk, hv, hq, hd = pin(k_ins), pin(v_ins), pin(k_find), pin(k_del)
+
+        def e2e_step():
+            g.clear()
+            g.insert_host(hk, hv)
+            g.find_host(hq)
+            g.resize(+1)
+            g.delete_host(hd)
+            g.resize(-1)
+        e2e_step()
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(max(1, min(args.steps, 3))):
+            t0 = time.perf_counter()
+            e2e_step()
+            torch.cuda.synchronize()
+            ts.append(time.perf_counter() - t0)
+        e2e = {"value": n_ops / statistics.mean(ts) / 1e6, "unit": "Mops/s",
+               "h2d_bytes_per_step": 4 * n + 4 * n + 4 * n + 4 * (n // 2),
+               "d2h_bytes_per_step": n + 5 * n + 5 * (n // 2),
+               "ms_per_step": 1e3 * statistics.mean(ts),
+               "path": "dyc_{insert,find,delete}_batch_host (pinned host buffers, copies inside)"}
+
+    cpu = None
+    if not args.no_cpu_baseline and not args.profile_only:
+        cpu = run_oracle_sample(args.cpu_log2n)
+
+    line = {
+        "metric": METRIC, "value": value, "unit": "Mops/s", "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": f"C2 RAND static (BASELINE.json configs[1]): 2^{args.log2n} inserts to fill 0.85, "
+                               f"2^{args.log2n} finds (50% hit), one subtable upsize, 2^{args.log2n - 1} deletes, "
+                               "one subtable downsize",
+                   "d": 4, "alpha": 0.3, "beta": 0.85, "bucket_slots": args.bucket_slots,
+                   "table_bytes": int(s_ins["N"] * 8),
+                   "l2": "inputs and table larger than L2 (126 MB); no flush needed"},
+        "phase_ms": phase_ms,
+        "ops": {"insert_mops": n / phase_ms["insert"] / 1e3, "find_mops": n / phase_ms["find"] / 1e3,
+                "delete_mops": (n // 2) / phase_ms["delete"] / 1e3},
+        "resize": resize,
+        "roofline": roofline,
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": launches,
+        "clocks": clk.summary(),
+        "table": {"fill_after_insert": s_ins["fill"], "phi": phi,
+                  "pending_after_upsert": pend, "evictions": s_ins["last_insert_evictions"]},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def multi_gpu(args, rank, world, local, dist):
+    from paper_conf_icde_lizlhs21_b200.dist import bench_multi_gpu
+    line = bench_multi_gpu(args, rank, world, local, METRIC, ClockSampler, measured_peaks, run_oracle_sample)
+    if rank == 0 and line is not None:
+        print(json.dumps(line), flush=True)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

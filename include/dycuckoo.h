@@ -1,0 +1,259 @@
+/*
+ * dycuckoo.h — C ABI of libdyc.so, the B200-native DyCuckoo hot path.
+ *
+ * DyCuckoo: "Dynamic Hash Tables on GPUs" (Li, Zhu, Lyu, Huang, Sun, ICDE'21).
+ * P:L<n> cites line n of the paper's text with its section; Qn cites
+ * a reading of an ambiguous passage, listed in DESIGN.md §4.
+ *
+ * The table is a two-layer cuckoo hash table: d subtables (§IV-A) of
+ * buckets of B slots; a first-layer hash maps every key to an ordered pair of
+ * subtables (§V-A), a second-layer universal hash
+ * h^t(k) = ((a_t k + b_t) mod p) mod |h^t| to one bucket per subtable,
+ * so find and delete probe at most two buckets.  Inserts run bounded
+ * cuckoo eviction chains (Alg. 1).  The fill factor
+ * θ = Σm_t / Σn_t is kept inside [alpha, beta] by doubling the
+ * smallest or halving the largest subtable, one at a time (§IV-B),
+ * splitting or merging its buckets.
+ *
+ * Conventions common to every entry point
+ * ---------------------------------------
+ * - Keys and values are uint32.  Key 0xFFFFFFFF (DYC_EMPTY_KEY) is reserved to
+ *   mark free slots (reading Q25): an op on it gets status DYC_OP_NONE and has
+ *   no effect; the batch does not fail.
+ * - Every d_* pointer is DEVICE memory on the table's device, owned by the
+ *   caller, and must stay valid until the enqueued work completes.  h_* pointers
+ *   are HOST memory (pinned gives the best copy speed, pageable works).  The
+ *   table owns its subtables, scratch lists and memory pool.
+ * - Arrays are dense, element i belongs to op i.  No alignment beyond the
+ *   element type is required.
+ * - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *   Work is stream-ordered.  find never blocks the host.  insert and delete
+ *   synchronize `stream` once (twice when a resize decision needs the number of
+ *   new keys) to read the batch counters that drive the resize policy (S6).
+ * - Batches are single-type.  Keys must be distinct within a batch
+ *   (precondition, reading Q9); violating it never corrupts the table but the
+ *   final value of a duplicated key is unspecified.
+ * - n == 0 is a no-op returning DYC_OK.
+ * - Errors are returned, never thrown.  dyc_last_error() gives a thread-local
+ *   message.  A CUDA error is sticky: DYC_ERR_CUDA.  An out-of-memory during a
+ *   resize returns DYC_ERR_OOM and leaves the table consistent (no key lost).
+ * - A table belongs to one host thread at a time.
+ */
+#ifndef DYCUCKOO_H
+#define DYCUCKOO_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define DYC_MAX_D      16u            /* maximum number of subtables d          */
+#define DYC_EMPTY_KEY  0xFFFFFFFFu    /* reserved key (free slot), Q25          */
+#define DYC_NOT_FOUND  0xFFFFFFFFu    /* value written for a find/delete miss   */
+
+typedef struct dyc_table dyc_table;   /* opaque; owns subtables, scratch, pool  */
+typedef void* dyc_stream_t;           /* cudaStream_t                           */
+
+typedef enum {
+    DYC_OK = 0,
+    DYC_ERR_INVALID_ARG = 1,
+    DYC_ERR_OOM = 2,
+    DYC_ERR_CUDA = 3,
+    DYC_ERR_INSERT_FAILED = 4,        /* a key could not be placed even after upsizing */
+    DYC_ERR_NO_DEVICE = 5
+} dyc_status;
+
+/* per-op status codes written to uint8 status / found arrays */
+enum {
+    DYC_OP_NONE = 0,                  /* absent key, or reserved key            */
+    DYC_OP_INSERTED = 1,              /* insert of a key that was absent        */
+    DYC_OP_UPDATED = 2,               /* insert of a present key: value replaced (Alg. 1) */
+    DYC_OP_FOUND = 1,                 /* find hit                               */
+    DYC_OP_DELETED = 1                /* delete hit                             */
+};
+
+/* Resize methods for dyc_resize_ex (measurement baselines). */
+enum {
+    DYC_RESIZE_SPLIT = 0,             /* the paper's method: split/merge one subtable */
+    DYC_RESIZE_REINSERT_SUBTABLE = 1, /* baseline of P:L809: reinsert the subtable's entries with the insert path */
+    DYC_RESIZE_REHASH_ALL = 2         /* MegaKV-style baseline: double/halve every subtable, reinsert all */
+};
+
+typedef struct {
+    uint32_t d;              /* subtables, 2..DYC_MAX_D (paper default 4)      */
+    uint32_t bucket_slots;   /* B: 4 (32-byte bucket, default), 8, 16 or 32 (Q26)     */
+    double   alpha, beta;    /* fill bounds, 0 < alpha < beta < 1, alpha <= beta*d/(d+1) (Q14) */
+    uint64_t init_capacity;  /* slots; n0 = max(1, ceil(init_capacity/(d*B))) buckets per subtable (Q13) */
+    uint64_t seed;           /* SplitMix64 seed of the hash constants a_s, b_s (Q1)  */
+    uint32_t max_hops;       /* L_max: eviction hops per attempt before the failure list (Q6) */
+    uint32_t flags;          /* reserved, 0                                          */
+} dyc_config;
+
+typedef struct {
+    uint64_t m;                       /* live keys Σ m_t                          */
+    uint64_t N;                       /* slots Σ n_t * B                          */
+    uint32_t d, B;
+    uint64_t buckets[DYC_MAX_D];      /* |h^t|                                    */
+    uint64_t count[DYC_MAX_D];        /* m_t, counted on the device               */
+    double   fill;                    /* θ = m / N                       */
+    uint64_t n_upsize, n_downsize;    /* policy resizes                  */
+    uint64_t n_fail_upsize;           /* upsizes triggered by placement failure */
+    uint64_t n_residual;              /* downsize residuals re-placed    */
+    uint64_t n_evict;                 /* eviction hops performed                  */
+    uint64_t n_place_retry;           /* extra placement passes over failure lists */
+    uint64_t n_second_table;          /* live keys stored in their second-choice subtable (φ·m) */
+    uint64_t bytes_allocated;         /* device bytes held by subtables + scratch */
+    uint64_t last_insert_new;         /* new keys of the last insert batch               */
+    uint64_t last_insert_pending;     /* ... of which needed the eviction kernel (k_place) */
+    uint64_t last_insert_evictions;   /* eviction hops of the last insert batch          */
+} dyc_stats_t;
+
+/* Fills *cfg with the defaults: d=4, B=4, alpha=0.3, beta=0.85 (Table
+ * `tbl:parameters`), init_capacity=4096, seed=0x5EED0001, max_hops=64. */
+dyc_status dyc_config_default(dyc_config* cfg);
+
+/* Creates a table on the current CUDA device with the default config except
+ * d, init_capacity, alpha, beta.  *out receives the handle.  Errors:
+ * DYC_ERR_INVALID_ARG for d outside 2..16 or bounds violating
+ * 0 < alpha < beta < 1, alpha <= beta*d/(d+1); DYC_ERR_OOM; DYC_ERR_NO_DEVICE. */
+dyc_status dyc_create(uint32_t d, uint64_t init_capacity, double alpha, double beta, dyc_table** out);
+dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out);
+
+/* Releases all device memory of the table (synchronizes its last stream). */
+dyc_status dyc_destroy(dyc_table* t);
+
+/* Batched insert (P:L188-189 insert(k,v); Alg. 1; §V-B "Insert").
+ * d_keys[n], d_values[n]: input.  d_status[n] (nullable): DYC_OP_INSERTED,
+ * DYC_OP_UPDATED, or DYC_OP_NONE for the reserved key.  Before placing new keys
+ * the table upsizes while (m + n_new) > beta*N (Q11); a placement
+ * failure triggers further upsizes; afterwards the alpha bound is
+ * enforced.  Returns DYC_ERR_OOM / DYC_ERR_INSERT_FAILED if memory runs out
+ * (already-placed ops stay applied; the table stays consistent). */
+dyc_status dyc_insert_batch(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_values,
+                            uint8_t* d_status, uint64_t n, dyc_stream_t stream);
+
+/* Batched find (§V-B "Find"): at most two bucket probes per key.
+ * d_values_out[n]: the value, or DYC_NOT_FOUND on a miss ("NULL").
+ * d_found[n] (nullable): DYC_OP_FOUND or DYC_OP_NONE.  Never synchronizes. */
+dyc_status dyc_find_batch(dyc_table* t, const uint32_t* d_keys, uint32_t* d_values_out,
+                          uint8_t* d_found, uint64_t n, dyc_stream_t stream);
+
+/* Batched delete (§V-B "Delete"): erase on match, no locking.
+ * d_values_out[n] (nullable): the removed value or DYC_NOT_FOUND.
+ * d_status[n] (nullable): DYC_OP_DELETED or DYC_OP_NONE.  Afterwards the table
+ * halves its largest subtable while m < alpha*N (Q11-Q13). */
+dyc_status dyc_delete_batch(dyc_table* t, const uint32_t* d_keys, uint32_t* d_values_out,
+                            uint8_t* d_status, uint64_t n, dyc_stream_t stream);
+
+/* Explicit resize of one subtable (§IV-B; kernels P:L374-395).
+ * direction +1: double subtable `subtable` (-1 = the smallest, ties lowest index);
+ * direction -1: halve it (-1 = the largest, ties highest index; refused if its
+ * bucket count is odd or 1); direction 0: enforce [alpha, beta] with the policy.
+ * A choice that would leave a subtable more than twice another is
+ * DYC_ERR_INVALID_ARG.  dyc_resize_ex selects the method (DYC_RESIZE_*). */
+dyc_status dyc_resize(dyc_table* t, int direction, int subtable, dyc_stream_t stream);
+dyc_status dyc_resize_ex(dyc_table* t, int direction, int subtable, int method, dyc_stream_t stream);
+
+/* Empties the table without resizing (all slots EMPTY, m = 0). */
+dyc_status dyc_clear(dyc_table* t, dyc_stream_t stream);
+
+/* Statistics; counts m_t with a device kernel and synchronizes `stream`. */
+dyc_status dyc_stats(dyc_table* t, dyc_stats_t* out, dyc_stream_t stream);
+
+/* Copies the live contents to host arrays (tests/diagnostics, not timed).
+ * h_kv[i] = key | (uint64)value << 32; h_table[i] / h_bucket[i] (nullable) give
+ * the subtable and bucket holding it.  Order is unspecified.  At most `cap`
+ * entries are written; *n_out receives the number of live entries.
+ * Synchronizes `stream`. */
+dyc_status dyc_dump(dyc_table* t, uint64_t* h_kv, uint32_t* h_table, uint64_t* h_bucket,
+                    uint64_t cap, uint64_t* n_out, dyc_stream_t stream);
+
+/* Hash constants a_s, b_s for s = 0..d+1 (s=0 first layer, s=1..d subtables,
+ * s=d+1 shard), each array of length >= d+2.  For cross-checking the hash
+ * specification against test vectors. */
+dyc_status dyc_hash_params(const dyc_table* t, uint64_t* a, uint64_t* b);
+
+/* Evaluates the device hash for n keys (test vectors): d_x[n*(d+2)] receives
+ * x_s(k) for s = 0..d+1, d_pair[2n] the ordered pair (t1, t2). */
+dyc_status dyc_hash_probe(dyc_table* t, const uint32_t* d_keys, uint64_t n, uint32_t* d_x,
+                          uint32_t* d_pair, dyc_stream_t stream);
+
+/* Host-buffer variants (the end-to-end path): copy the inputs host->device,
+ * run the batch, copy the outputs device->host and synchronize `stream`.
+ * Staging buffers are owned by the table. */
+dyc_status dyc_insert_batch_host(dyc_table* t, const uint32_t* h_keys, const uint32_t* h_values,
+                                 uint8_t* h_status, uint64_t n, dyc_stream_t stream);
+dyc_status dyc_find_batch_host(dyc_table* t, const uint32_t* h_keys, uint32_t* h_values_out,
+                               uint8_t* h_found, uint64_t n, dyc_stream_t stream);
+dyc_status dyc_delete_batch_host(dyc_table* t, const uint32_t* h_keys, uint32_t* h_values_out,
+                                 uint8_t* h_status, uint64_t n, dyc_stream_t stream);
+
+/* Kernel launch counter (for the bench's gpu_launches claim): number of kernels
+ * this table has launched since creation or the last reset. */
+uint64_t dyc_launch_count(const dyc_table* t, int reset);
+
+/* Per-kernel timing with CUDA events recorded on the launching stream around
+ * every kernel this table launches (measurement only; off by default).
+ * dyc_profile_enable(t, 1) starts a fresh window; dyc_profile_read() waits for
+ * the recorded events and reports, for each kernel kind k < DYC_PROF_KINDS,
+ * the summed milliseconds ms[k] and launch count calls[k]. */
+#define DYC_PROF_KINDS 16
+enum {
+    DYC_PROF_FIND = 0, DYC_PROF_UPSERT = 1, DYC_PROF_PLACE = 2, DYC_PROF_DELETE = 3,
+    DYC_PROF_UPSIZE = 4, DYC_PROF_DOWNSIZE = 5, DYC_PROF_REINSERT = 6, DYC_PROF_OTHER = 7
+};
+dyc_status dyc_profile_enable(dyc_table* t, int enable);
+dyc_status dyc_profile_read(dyc_table* t, double* ms, uint64_t* calls);
+
+/* ---------------------------------------------------------------------------
+ * Hash-partitioned sharding across G GPUs (build component C1).
+ * shard(k) = x_{d+1}(k) mod G, independent of the pair and bucket hashes.
+ * The exchange itself is an NCCL all-to-all issued by the caller (one process
+ * per GPU, torch.distributed); these kernels do the data-parallel parts.
+ * ------------------------------------------------------------------------- */
+
+/* Counts ops per destination shard: d_counts[world] (uint64, device) receives
+ * the histogram.  `t` supplies the hash constants (all ranks use one seed). */
+dyc_status dyc_route_count(dyc_table* t, const uint32_t* d_keys, uint64_t n, uint32_t world,
+                           uint64_t* d_counts, dyc_stream_t stream);
+
+/* Scatters op i to position d_offsets[dest] + rank-within-dest of the send
+ * buffers (grouped by destination).  d_offsets[world] (uint64, device) holds the
+ * exclusive prefix sum of the counts and is consumed as cursors.  d_vals_in and
+ * d_vals_out may be NULL (finds/deletes).  d_pos[i] (uint32) receives op i's
+ * position in the send buffer, for dyc_route_unpermute. */
+dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_vals_in,
+                             uint64_t n, uint32_t world, uint64_t* d_offsets,
+                             uint32_t* d_keys_out, uint32_t* d_vals_out, uint32_t* d_pos,
+                             dyc_stream_t stream);
+
+/* Gathers replies back into request order: d_vals[i] = d_reply_vals[d_pos[i]],
+ * d_status[i] = d_reply_status[d_pos[i]] (either pair may be NULL). */
+dyc_status dyc_route_unpermute(const uint32_t* d_pos, uint64_t n, const uint32_t* d_reply_vals,
+                               const uint8_t* d_reply_status, uint32_t* d_vals,
+                               uint8_t* d_status, dyc_stream_t stream);
+
+/* ---------------------------------------------------------------------------
+ * Measurement helpers (bench.py; not part of the method).
+ * ------------------------------------------------------------------------- */
+
+/* Random-gather ceiling: `n_reads` reads of `bytes_per_read` (32/64/128)
+ * bytes at uniformly random aligned offsets of d_buf[buf_bytes], XOR-reduced
+ * into *d_sink.  Bounds what the one-sector-per-probe roofline can reach. */
+dyc_status dyc_bench_gather(const void* d_buf, uint64_t buf_bytes, uint64_t n_reads,
+                            uint32_t bytes_per_read, uint64_t seed, uint64_t* d_sink,
+                            dyc_stream_t stream);
+
+/* Thread-local message for the last error returned on this thread. */
+const char* dyc_last_error(void);
+
+/* Library version string. */
+const char* dyc_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* DYCUCKOO_H */

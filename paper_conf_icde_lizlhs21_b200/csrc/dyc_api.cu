@@ -1,0 +1,894 @@
+// dyc_api.cu — host control (resize policy, scratch, counters) and the C ABI of
+// libdyc.so (include/dycuckoo.h).
+//
+// Host policy (readings Q11-Q13, Q17, Q29):
+//   insert: upsize the smallest subtable while (m + n_new) > beta*N, place, settle
+//           failures (retry, then failure-triggered upsize), then the
+//           alpha loop;
+//   delete: erase, then halve the largest subtable while m < alpha*N (unless it
+//           is odd / a single bucket, or halving would exceed beta; a downsize
+//           whose residuals needed a failure upsize ends the loop, Q17b).
+// All comparisons are `(double)m <op> bound*(double)N` on the host (Q29).
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "dycuckoo.h"
+#include "dyc_device.cuh"
+#include "dyc_kernels.cuh"
+
+using namespace dyc;
+
+namespace {
+
+thread_local std::string g_err;
+
+dyc_status set_err(dyc_status s, const std::string& msg) {
+    g_err = msg;
+    return s;
+}
+
+dyc_status cuda_err(cudaError_t e, const char* what) {
+    return set_err(e == cudaErrorMemoryAllocation ? DYC_ERR_OOM : DYC_ERR_CUDA,
+                   std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+#define CU(x)                                            \
+    do {                                                 \
+        cudaError_t e_ = (x);                            \
+        if (e_ != cudaSuccess) return cuda_err(e_, #x);  \
+    } while (0)
+
+#define TRY(x)                          \
+    do {                                \
+        dyc_status s_ = (x);            \
+        if (s_ != DYC_OK) return s_;    \
+    } while (0)
+
+uint64_t splitmix64(uint64_t& s) {
+    uint64_t z = (s += 0x9E3779B97F4A7C15ull);
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+uint64_t fastmod_magic(uint64_t n) { return n <= 1 ? 0ull : (~0ull / n) + 1ull; }
+
+inline cudaStream_t S(dyc_stream_t s) { return reinterpret_cast<cudaStream_t>(s); }
+
+}  // namespace
+
+struct dyc_table {
+    dyc_config cfg{};
+    int device = 0;
+    int num_sms = 148;
+    int place_blocks = 148 * 8;            // persistent grid of k_place
+    cudaMemPool_t pool = nullptr;
+    unsigned long long* sub[DYC_MAX_D] = {};
+    uint64_t nb[DYC_MAX_D] = {};
+    uint32_t a[DYC_MAX_D + 2] = {}, b[DYC_MAX_D + 2] = {};
+    uint64_t m = 0;
+    unsigned long long* list[2] = {nullptr, nullptr};
+    uint64_t list_cap = 0;
+    unsigned long long* d_ctr = nullptr;   // C_N device counters
+    unsigned long long* h_ctr = nullptr;   // pinned mirror
+    void* stage = nullptr;                 // device staging for the host-buffer entry points
+    uint64_t stage_cap = 0;
+    uint64_t n_upsize = 0, n_downsize = 0, n_fail_upsize = 0, n_residual = 0, n_evict = 0, n_place_retry = 0;
+    uint64_t launches = 0;
+    uint64_t last_new = 0, last_pending = 0, last_evict = 0;
+    cudaStream_t last = nullptr;
+    // per-kernel event profiling (dyc_profile_*)
+    bool prof = false;
+    struct Rec { int kind; cudaEvent_t a, b; };
+    std::vector<Rec> recs;
+    std::vector<cudaEvent_t> ev_pool;
+    double prof_ms[DYC_PROF_KINDS] = {};
+    uint64_t prof_calls[DYC_PROF_KINDS] = {};
+
+    cudaEvent_t ev() {
+        if (!ev_pool.empty()) { cudaEvent_t e = ev_pool.back(); ev_pool.pop_back(); return e; }
+        cudaEvent_t e = nullptr;
+        cudaEventCreate(&e);
+        return e;
+    }
+
+    uint64_t N() const {
+        uint64_t s = 0;
+        for (uint32_t t = 0; t < cfg.d; t++) s += nb[t] * cfg.bucket_slots;
+        return s;
+    }
+    int smallest() const {      // ties -> lowest index (Q12)
+        int best = 0;
+        for (uint32_t t = 1; t < cfg.d; t++)
+            if (nb[t] < nb[best]) best = (int)t;
+        return best;
+    }
+    int largest() const {       // ties -> highest index (Q12)
+        int best = (int)cfg.d - 1;
+        for (int t = (int)cfg.d - 2; t >= 0; t--)
+            if (nb[t] > nb[best]) best = t;
+        return best;
+    }
+    TableView view() const {
+        TableView v{};
+        for (uint32_t t = 0; t < cfg.d; t++) {
+            v.sub[t].slots = sub[t];
+            v.sub[t].n = (uint32_t)nb[t];
+            v.sub[t].magic = fastmod_magic(nb[t]);
+        }
+        for (uint32_t s = 0; s < cfg.d + 2; s++) { v.a[s] = a[s]; v.b[s] = b[s]; }
+        v.d = cfg.d;
+        v.d2 = cfg.d * (cfg.d - 1);
+        v.magic_d2 = fastmod_magic(v.d2);
+        v.dm1 = cfg.d - 1;
+        v.recip_dm1 = (65536u + v.dm1 - 1) / v.dm1;
+        v.max_hops = cfg.max_hops;
+        return v;
+    }
+};
+
+namespace {
+
+// Records CUDA events around one launch when profiling is on (measurement only).
+struct ProfScope {
+    dyc_table* t;
+    int kind;
+    cudaStream_t st;
+    cudaEvent_t a = nullptr;
+    ProfScope(dyc_table* t_, int kind_, cudaStream_t st_) : t(t_), kind(kind_), st(st_) {
+        t->launches++;
+        if (t->prof) { a = t->ev(); cudaEventRecord(a, st); }
+    }
+    ~ProfScope() {
+        if (a) {
+            cudaEvent_t b = t->ev();
+            cudaEventRecord(b, st);
+            t->recs.push_back({kind, a, b});
+        }
+    }
+};
+
+unsigned grid_for(uint64_t work, uint64_t per_block) {
+    uint64_t g = (work + per_block - 1) / per_block;
+    g = std::max<uint64_t>(1, std::min<uint64_t>(g, 1u << 30));
+    return (unsigned)g;
+}
+
+dyc_status dev_alloc(dyc_table* t, void** p, uint64_t bytes, cudaStream_t st) {
+    cudaError_t e = cudaMallocFromPoolAsync(p, std::max<uint64_t>(bytes, 8), t->pool, st);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        *p = nullptr;
+        return set_err(DYC_ERR_OOM, std::string("device allocation of ") + std::to_string(bytes) + " bytes failed: " +
+                                        cudaGetErrorString(e));
+    }
+    return DYC_OK;
+}
+
+dyc_status read_ctr(dyc_table* t, cudaStream_t st) {
+    CU(cudaMemcpyAsync(t->h_ctr, t->d_ctr, C_N * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+    CU(cudaStreamSynchronize(st));
+    return DYC_OK;
+}
+
+dyc_status zero_ctr(dyc_table* t, cudaStream_t st) {
+    CU(cudaMemsetAsync(t->d_ctr, 0, C_N * sizeof(unsigned long long), st));
+    return DYC_OK;
+}
+
+dyc_status zero_one(dyc_table* t, int idx, cudaStream_t st) {
+    CU(cudaMemsetAsync(t->d_ctr + idx, 0, sizeof(unsigned long long), st));
+    return DYC_OK;
+}
+
+dyc_status ensure_lists(dyc_table* t, uint64_t n, cudaStream_t st) {
+    if (n <= t->list_cap) return DYC_OK;
+    uint64_t cap = std::max<uint64_t>(n, 2 * t->list_cap);
+    void* l0 = nullptr;
+    void* l1 = nullptr;
+    TRY(dev_alloc(t, &l0, cap * 8, st));
+    dyc_status s = dev_alloc(t, &l1, cap * 8, st);
+    if (s != DYC_OK) {
+        cudaFreeAsync(l0, st);
+        return s;
+    }
+    if (t->list[0]) cudaFreeAsync(t->list[0], st);
+    if (t->list[1]) cudaFreeAsync(t->list[1], st);
+    t->list[0] = (unsigned long long*)l0;
+    t->list[1] = (unsigned long long*)l1;
+    t->list_cap = cap;
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status upsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
+    const uint64_t n_old = t->nb[ti], n_new = 2 * n_old;
+    if (n_new > 0xFFFFFFFFull) return set_err(DYC_ERR_OOM, "subtable would exceed 2^32 buckets");
+    void* p = nullptr;
+    TRY(dev_alloc(t, &p, n_new * B * 8, st));
+    const uint64_t slots = n_old * B;
+    {
+        ProfScope ps(t, DYC_PROF_UPSIZE, st);
+        k_upsize<B><<<grid_for(slots, kThreads), kThreads, 0, st>>>(
+            t->sub[ti], (unsigned long long*)p, (uint32_t)n_old, t->a[ti + 1], t->b[ti + 1], fastmod_magic(n_new),
+            (uint32_t)n_new);
+    }
+    CU(cudaGetLastError());
+    CU(cudaFreeAsync(t->sub[ti], st));
+    t->sub[ti] = (unsigned long long*)p;
+    t->nb[ti] = n_new;
+    return DYC_OK;
+}
+
+// Place list[src][0..cnt) (count given on host or in a device counter), settling
+// failures: first a plain retry pass, then failure-triggered upsizes.
+template <int B>
+dyc_status place_and_settle(dyc_table* t, int src, const unsigned long long* d_count, uint64_t h_count,
+                            bool first_fit, cudaStream_t st) {
+    TRY(zero_one(t, C_FAIL, st));
+    TRY(zero_one(t, C_EVICT, st));
+    {
+        ProfScope ps(t, DYC_PROF_PLACE, st);
+        k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->list[src], d_count, h_count,
+                                                         t->list[1 - src], t->d_ctr, first_fit);
+    }
+    CU(cudaGetLastError());
+    TRY(read_ctr(t, st));
+    t->n_evict += t->h_ctr[C_EVICT];
+    uint64_t nfail = t->h_ctr[C_FAIL];
+    int cur = 1 - src;
+    int round = 0;
+    while (nfail > 0) {
+        if (round > 0) {
+            TRY(upsize_table<B>(t, (uint32_t)t->smallest(), st));
+            t->n_fail_upsize++;
+        }
+        round++;
+        t->n_place_retry++;
+        TRY(zero_one(t, C_FAIL, st));
+        TRY(zero_one(t, C_EVICT, st));
+        {
+            ProfScope ps(t, DYC_PROF_PLACE, st);
+            k_place<B><<<grid_for(nfail, kThreads), kThreads, 0, st>>>(t->view(), t->list[cur], nullptr, nfail,
+                                                                       t->list[1 - cur], t->d_ctr, true);
+        }
+        CU(cudaGetLastError());
+        TRY(read_ctr(t, st));
+        t->n_evict += t->h_ctr[C_EVICT];
+        nfail = t->h_ctr[C_FAIL];
+        cur = 1 - cur;
+        if (round > 64) return set_err(DYC_ERR_INSERT_FAILED, "placement kept failing after 64 upsizes");
+    }
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status downsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
+    const uint64_t n_old = t->nb[ti], h = n_old / 2;
+    if (n_old < 2 || (n_old & 1)) return set_err(DYC_ERR_INVALID_ARG, "subtable cannot be halved");
+    TRY(ensure_lists(t, h * B, st));
+    void* p = nullptr;
+    TRY(dev_alloc(t, &p, h * B * 8, st));
+    TRY(zero_one(t, C_RESIDUAL, st));
+    {
+        ProfScope ps(t, DYC_PROF_DOWNSIZE, st);
+        k_downsize<B><<<grid_for(h * B, kThreads), kThreads, 0, st>>>(t->sub[ti], (unsigned long long*)p,
+                                                                       (uint32_t)h, t->list[0], t->d_ctr);
+    }
+    CU(cudaGetLastError());
+    CU(cudaFreeAsync(t->sub[ti], st));
+    t->sub[ti] = (unsigned long long*)p;
+    t->nb[ti] = h;
+    // residuals go to the other table of their pair; run as a
+    // separate kernel, so the exclusion of t is not needed for correctness (Q16)
+    TRY(place_and_settle<B>(t, 0, t->d_ctr + C_RESIDUAL, 0, true, st));
+    t->n_residual += t->h_ctr[C_RESIDUAL];
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status enforce_lower(dyc_table* t, cudaStream_t st) {
+    bool shrank = false;
+    for (;;) {
+        const uint64_t N = t->N();
+        if (!((double)t->m < t->cfg.alpha * (double)N)) break;
+        const int ti = t->largest();
+        if (t->nb[ti] < 2 || (t->nb[ti] & 1)) break;
+        const uint64_t N_after = N - (t->nb[ti] / 2) * B;
+        if ((double)t->m > t->cfg.beta * (double)N_after) break;
+        const uint64_t fails = t->n_fail_upsize;
+        TRY(downsize_table<B>(t, (uint32_t)ti, st));
+        t->n_downsize++;
+        shrank = true;
+        if (t->n_fail_upsize != fails) break;   // Q17b
+    }
+    if (shrank) {
+        CU(cudaStreamSynchronize(st));
+        cudaMemPoolTrimTo(t->pool, 0);
+    }
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* status, uint64_t n,
+                       cudaStream_t st) {
+    TRY(ensure_lists(t, n, st));
+    TRY(zero_ctr(t, st));
+    const bool fuse = (double)(t->m + n) <= t->cfg.beta * (double)t->N();
+    const unsigned grid = grid_for(n, kThreads);
+    {
+        ProfScope ps(t, DYC_PROF_UPSERT, st);
+        if (fuse)
+            k_upsert<B, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
+        else
+            k_upsert<B, false><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
+    }
+    CU(cudaGetLastError());
+    if (!fuse) {
+        // the resize decision needs n_new before any placement (Q11)
+        TRY(read_ctr(t, st));
+        const uint64_t n_new = t->h_ctr[C_INSERTED];
+        while ((double)(t->m + n_new) > t->cfg.beta * (double)t->N()) {
+            TRY(upsize_table<B>(t, (uint32_t)t->smallest(), st));
+            t->n_upsize++;
+        }
+    }
+    const uint64_t ev0 = t->n_evict;
+    dyc_status s = place_and_settle<B>(t, 0, t->d_ctr + C_PENDING, 0, !fuse, st);
+    t->m += t->h_ctr[C_INSERTED];   // counters were read by place_and_settle
+    t->last_new = t->h_ctr[C_INSERTED];
+    t->last_pending = t->h_ctr[C_PENDING];
+    t->last_evict = t->n_evict - ev0;
+    if (s != DYC_OK) return s;
+    return enforce_lower<B>(t, st);
+}
+
+template <int B>
+dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* found, uint64_t n,
+                     cudaStream_t st) {
+    constexpr int ILP = (B <= 4) ? 4 : (B <= 8 ? 2 : 1);
+    {
+        ProfScope ps(t, DYC_PROF_FIND, st);
+        k_find<B, ILP><<<grid_for(n, (uint64_t)kThreads * ILP), kThreads, 0, st>>>(t->view(), keys, vals, found, n);
+    }
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status delete_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
+                       cudaStream_t st) {
+    TRY(zero_one(t, C_REMOVED, st));
+    {
+        ProfScope ps(t, DYC_PROF_DELETE, st);
+        k_delete<B><<<grid_for(n, kThreads), kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr);
+    }
+    CU(cudaGetLastError());
+    TRY(read_ctr(t, st));
+    t->m -= t->h_ctr[C_REMOVED];
+    return enforce_lower<B>(t, st);
+}
+
+// Baselines (measurement only): reinsert one subtable or everything.
+template <int B>
+dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaStream_t st) {
+    const uint32_t d = t->cfg.d;
+    unsigned long long* old[DYC_MAX_D] = {};
+    uint64_t old_nb[DYC_MAX_D] = {};
+    bool touched[DYC_MAX_D] = {};
+    for (uint32_t i = 0; i < d; i++) touched[i] = all || (int)i == ti;
+    uint64_t live_bound = 0;
+    for (uint32_t i = 0; i < d; i++) {
+        if (!touched[i]) continue;
+        const uint64_t nn = direction > 0 ? 2 * t->nb[i] : t->nb[i] / 2;
+        if (nn == 0 || nn > 0xFFFFFFFFull) return set_err(DYC_ERR_INVALID_ARG, "bad subtable size");
+        void* p = nullptr;
+        TRY(dev_alloc(t, &p, nn * B * 8, st));
+        CU(cudaMemsetAsync(p, 0xFF, nn * B * 8, st));
+        old[i] = t->sub[i];
+        old_nb[i] = t->nb[i];
+        t->sub[i] = (unsigned long long*)p;
+        t->nb[i] = nn;
+        live_bound += old_nb[i] * B;
+    }
+    TRY(ensure_lists(t, live_bound, st));
+    TRY(zero_ctr(t, st));
+    const TableView tv = t->view();
+    for (uint32_t i = 0; i < d; i++) {
+        if (!touched[i]) continue;
+        const uint64_t ns = old_nb[i] * B;
+        ProfScope ps(t, DYC_PROF_REINSERT, st);
+        k_reinsert<B><<<grid_for(ns, kThreads), kThreads, 0, st>>>(tv, old[i], ns, t->list[1], t->d_ctr);
+        CU(cudaGetLastError());
+    }
+    TRY(read_ctr(t, st));
+    t->n_evict += t->h_ctr[C_EVICT];
+    const uint64_t nfail = t->h_ctr[C_FAIL];
+    for (uint32_t i = 0; i < d; i++)
+        if (touched[i]) CU(cudaFreeAsync(old[i], st));
+    if (nfail) TRY(place_and_settle<B>(t, 1, nullptr, nfail, true, st));
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status resize_impl(dyc_table* t, int direction, int subtable, int method, cudaStream_t st) {
+    if (direction == 0) {
+        while ((double)t->m > t->cfg.beta * (double)t->N()) {
+            TRY(upsize_table<B>(t, (uint32_t)t->smallest(), st));
+            t->n_upsize++;
+        }
+        return enforce_lower<B>(t, st);
+    }
+    if (method == DYC_RESIZE_REHASH_ALL) {
+        TRY(reinsert_resize<B>(t, direction, -1, true, st));
+        if (direction > 0) t->n_upsize++; else t->n_downsize++;
+        return DYC_OK;
+    }
+    int ti = subtable;
+    if (direction > 0) {
+        if (ti < 0) ti = t->smallest();
+        if (ti >= (int)t->cfg.d || t->nb[ti] != t->nb[t->smallest()])
+            return set_err(DYC_ERR_INVALID_ARG, "only a smallest subtable may be doubled (P:L311-312)");
+    } else {
+        if (ti < 0) ti = t->largest();
+        if (ti >= (int)t->cfg.d || t->nb[ti] != t->nb[t->largest()])
+            return set_err(DYC_ERR_INVALID_ARG, "only a largest subtable may be halved (P:L311-312)");
+        if (t->nb[ti] < 2 || (t->nb[ti] & 1)) return set_err(DYC_ERR_INVALID_ARG, "subtable cannot be halved");
+    }
+    if (method == DYC_RESIZE_REINSERT_SUBTABLE) {
+        TRY(reinsert_resize<B>(t, direction, ti, false, st));
+    } else if (direction > 0) {
+        TRY(upsize_table<B>(t, (uint32_t)ti, st));
+    } else {
+        TRY(downsize_table<B>(t, (uint32_t)ti, st));
+    }
+    if (direction > 0) t->n_upsize++; else t->n_downsize++;
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status stats_impl(dyc_table* t, dyc_stats_t* out, cudaStream_t st) {
+    TRY(zero_ctr(t, st));
+    const TableView tv = t->view();
+    for (uint32_t i = 0; i < t->cfg.d; i++) {
+        ProfScope ps(t, DYC_PROF_OTHER, st);
+        k_count<B><<<grid_for(t->nb[i] * B, kThreads * 8), kThreads, 0, st>>>(tv, i, t->d_ctr);
+        CU(cudaGetLastError());
+    }
+    TRY(read_ctr(t, st));
+    std::memset(out, 0, sizeof(*out));
+    out->m = t->m;
+    out->N = t->N();
+    out->d = t->cfg.d;
+    out->B = B;
+    for (uint32_t i = 0; i < t->cfg.d; i++) {
+        out->buckets[i] = t->nb[i];
+        out->count[i] = t->h_ctr[C_COUNT0 + i];
+    }
+    out->fill = out->N ? (double)out->m / (double)out->N : 0.0;
+    out->n_upsize = t->n_upsize;
+    out->n_downsize = t->n_downsize;
+    out->n_fail_upsize = t->n_fail_upsize;
+    out->n_residual = t->n_residual;
+    out->n_evict = t->n_evict;
+    out->n_place_retry = t->n_place_retry;
+    out->n_second_table = t->h_ctr[C_SECOND];
+    out->bytes_allocated = out->N * 8 + 2 * t->list_cap * 8 + t->stage_cap + C_N * 8;
+    out->last_insert_new = t->last_new;
+    out->last_insert_pending = t->last_pending;
+    out->last_insert_evictions = t->last_evict;
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status dump_impl(dyc_table* t, uint64_t* h_kv, uint32_t* h_tab, uint64_t* h_bkt, uint64_t cap, uint64_t* n_out,
+                     cudaStream_t st) {
+    const uint64_t m = t->m;
+    void *kv = nullptr, *tb = nullptr, *bk = nullptr;
+    TRY(dev_alloc(t, &kv, m * 8, st));
+    TRY(dev_alloc(t, &tb, m * 4, st));
+    TRY(dev_alloc(t, &bk, m * 8, st));
+    TRY(zero_one(t, C_DUMP, st));
+    const TableView tv = t->view();
+    for (uint32_t i = 0; i < t->cfg.d; i++) {
+        ProfScope ps(t, DYC_PROF_OTHER, st);
+        k_dump<B><<<grid_for(t->nb[i] * B, kThreads), kThreads, 0, st>>>(
+            tv, i, (unsigned long long*)kv, (uint32_t*)tb, (unsigned long long*)bk, m, t->d_ctr);
+        CU(cudaGetLastError());
+    }
+    TRY(read_ctr(t, st));
+    const uint64_t cnt = t->h_ctr[C_DUMP];
+    const uint64_t ncopy = std::min(std::min(cnt, m), cap);
+    if (ncopy) {
+        if (h_kv) CU(cudaMemcpyAsync(h_kv, kv, ncopy * 8, cudaMemcpyDeviceToHost, st));
+        if (h_tab) CU(cudaMemcpyAsync(h_tab, tb, ncopy * 4, cudaMemcpyDeviceToHost, st));
+        if (h_bkt) CU(cudaMemcpyAsync(h_bkt, bk, ncopy * 8, cudaMemcpyDeviceToHost, st));
+    }
+    CU(cudaFreeAsync(kv, st));
+    CU(cudaFreeAsync(tb, st));
+    CU(cudaFreeAsync(bk, st));
+    CU(cudaStreamSynchronize(st));
+    if (n_out) *n_out = cnt;
+    if (cnt != m) return set_err(DYC_ERR_CUDA, "dump found " + std::to_string(cnt) + " live slots, expected " +
+                                                   std::to_string(m));
+    return DYC_OK;
+}
+
+#define DISPATCH_B(t, CALL)                                                        \
+    switch ((t)->cfg.bucket_slots) {                                               \
+        case 4: { constexpr int B_ = 4; return CALL; }                             \
+        case 8: { constexpr int B_ = 8; return CALL; }                             \
+        case 16: { constexpr int B_ = 16; return CALL; }                           \
+        case 32: { constexpr int B_ = 32; return CALL; }                           \
+        default: return set_err(DYC_ERR_INVALID_ARG, "unsupported bucket_slots");  \
+    }
+
+dyc_status check_table(const dyc_table* t) {
+    if (!t) return set_err(DYC_ERR_INVALID_ARG, "null table");
+    return DYC_OK;
+}
+
+dyc_status enter(dyc_table* t, dyc_stream_t s) {
+    TRY(check_table(t));
+    CU(cudaSetDevice(t->device));
+    t->last = S(s);
+    return DYC_OK;
+}
+
+dyc_status ensure_stage(dyc_table* t, uint64_t bytes, cudaStream_t st) {
+    if (bytes <= t->stage_cap) return DYC_OK;
+    if (t->stage) CU(cudaFreeAsync(t->stage, st));
+    t->stage = nullptr;
+    t->stage_cap = 0;
+    TRY(dev_alloc(t, &t->stage, bytes, st));
+    t->stage_cap = bytes;
+    return DYC_OK;
+}
+
+}  // namespace
+
+// ============================================================================ C ABI
+extern "C" {
+
+const char* dyc_last_error(void) { return g_err.c_str(); }
+const char* dyc_version(void) { return "dycuckoo-b200 0.1 (sm_100a)"; }
+
+dyc_status dyc_config_default(dyc_config* cfg) {
+    if (!cfg) return set_err(DYC_ERR_INVALID_ARG, "null cfg");
+    std::memset(cfg, 0, sizeof(*cfg));
+    cfg->d = 4;
+    cfg->bucket_slots = 4;
+    cfg->alpha = 0.3;
+    cfg->beta = 0.85;
+    cfg->init_capacity = 4096;
+    cfg->seed = 0x5EED0001ull;
+    cfg->max_hops = 64;
+    return DYC_OK;
+}
+
+dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
+    if (!cfg || !out) return set_err(DYC_ERR_INVALID_ARG, "null argument");
+    *out = nullptr;
+    const uint32_t d = cfg->d, B = cfg->bucket_slots;
+    if (d < 2 || d > DYC_MAX_D) return set_err(DYC_ERR_INVALID_ARG, "d must be in 2..16");
+    if (B != 4 && B != 8 && B != 16 && B != 32) return set_err(DYC_ERR_INVALID_ARG, "bucket_slots must be 4, 8, 16 or 32");
+    if (!(cfg->alpha > 0.0 && cfg->alpha < cfg->beta && cfg->beta < 1.0))
+        return set_err(DYC_ERR_INVALID_ARG, "need 0 < alpha < beta < 1");
+    if (cfg->alpha > cfg->beta * (double)d / (double)(d + 1))
+        return set_err(DYC_ERR_INVALID_ARG, "need alpha <= beta*d/(d+1) (P:L315-318)");
+    if (cfg->max_hops < 1) return set_err(DYC_ERR_INVALID_ARG, "max_hops must be >= 1");
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        return set_err(DYC_ERR_NO_DEVICE, "no CUDA device");
+    }
+    dyc_table* t = new dyc_table();
+    t->cfg = *cfg;
+    cudaGetDevice(&t->device);
+    cudaDeviceGetAttribute(&t->num_sms, cudaDevAttrMultiProcessorCount, t->device);
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_place<4>, kThreads, 0);
+    t->place_blocks = t->num_sms * std::max(1, occ);
+    uint64_t st = cfg->seed;
+    for (uint32_t s = 0; s < d + 2; s++) {
+        t->a[s] = (uint32_t)(1 + splitmix64(st) % (kP - 1));   // a_s in [1, p)
+        t->b[s] = (uint32_t)(splitmix64(st) % kP);             // b_s in [0, p)
+    }
+    cudaMemPoolProps props{};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = t->device;
+    cudaError_t e = cudaMemPoolCreate(&t->pool, &props);
+    if (e != cudaSuccess) {
+        delete t;
+        return cuda_err(e, "cudaMemPoolCreate");
+    }
+    uint64_t thr = ~0ull;
+    cudaMemPoolSetAttribute(t->pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    uint64_t per = (cfg->init_capacity + (uint64_t)d * B - 1) / ((uint64_t)d * B);   // Q13
+    if (per < 1) per = 1;
+    if (per > 0xFFFFFFFFull) {
+        dyc_destroy(t);
+        return set_err(DYC_ERR_INVALID_ARG, "init_capacity too large");
+    }
+    dyc_status s = DYC_OK;
+    for (uint32_t i = 0; i < d && s == DYC_OK; i++) {
+        void* p = nullptr;
+        s = dev_alloc(t, &p, per * B * 8, nullptr);
+        if (s == DYC_OK) {
+            t->sub[i] = (unsigned long long*)p;
+            t->nb[i] = per;
+            if (cudaMemsetAsync(p, 0xFF, per * B * 8, nullptr) != cudaSuccess) s = cuda_err(cudaGetLastError(), "memset");
+        }
+    }
+    if (s == DYC_OK && cudaMalloc(&t->d_ctr, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMalloc");
+    if (s == DYC_OK && cudaMallocHost(&t->h_ctr, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMallocHost");
+    if (s == DYC_OK && cudaDeviceSynchronize() != cudaSuccess) s = cuda_err(cudaGetLastError(), "create");
+    if (s != DYC_OK) {
+        dyc_destroy(t);
+        return s;
+    }
+    *out = t;
+    return DYC_OK;
+}
+
+dyc_status dyc_create(uint32_t d, uint64_t init_capacity, double alpha, double beta, dyc_table** out) {
+    dyc_config c;
+    dyc_config_default(&c);
+    c.d = d;
+    c.init_capacity = init_capacity;
+    c.alpha = alpha;
+    c.beta = beta;
+    return dyc_create_ex(&c, out);
+}
+
+dyc_status dyc_destroy(dyc_table* t) {
+    if (!t) return DYC_OK;
+    cudaSetDevice(t->device);
+    cudaDeviceSynchronize();
+    for (uint32_t i = 0; i < t->cfg.d; i++)
+        if (t->sub[i]) cudaFree(t->sub[i]);
+    for (int i = 0; i < 2; i++)
+        if (t->list[i]) cudaFree(t->list[i]);
+    if (t->stage) cudaFree(t->stage);
+    if (t->d_ctr) cudaFree(t->d_ctr);
+    if (t->h_ctr) cudaFreeHost(t->h_ctr);
+    cudaDeviceSynchronize();
+    if (t->pool) cudaMemPoolDestroy(t->pool);
+    for (auto& r : t->recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
+    for (auto e : t->ev_pool) cudaEventDestroy(e);
+    delete t;
+    return DYC_OK;
+}
+
+dyc_status dyc_insert_batch(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_values, uint8_t* d_status,
+                            uint64_t n, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (n == 0) return DYC_OK;
+    if (!d_keys || !d_values) return set_err(DYC_ERR_INVALID_ARG, "null keys/values");
+    DISPATCH_B(t, insert_impl<B_>(t, d_keys, d_values, d_status, n, S(stream)));
+}
+
+dyc_status dyc_find_batch(dyc_table* t, const uint32_t* d_keys, uint32_t* d_values_out, uint8_t* d_found, uint64_t n,
+                          dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (n == 0) return DYC_OK;
+    if (!d_keys || !d_values_out) return set_err(DYC_ERR_INVALID_ARG, "null keys/values_out");
+    DISPATCH_B(t, find_impl<B_>(t, d_keys, d_values_out, d_found, n, S(stream)));
+}
+
+dyc_status dyc_delete_batch(dyc_table* t, const uint32_t* d_keys, uint32_t* d_values_out, uint8_t* d_status,
+                            uint64_t n, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (n == 0) return DYC_OK;
+    if (!d_keys) return set_err(DYC_ERR_INVALID_ARG, "null keys");
+    DISPATCH_B(t, delete_impl<B_>(t, d_keys, d_values_out, d_status, n, S(stream)));
+}
+
+dyc_status dyc_resize_ex(dyc_table* t, int direction, int subtable, int method, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (direction < -1 || direction > 1 || method < 0 || method > 2)
+        return set_err(DYC_ERR_INVALID_ARG, "bad direction/method");
+    DISPATCH_B(t, resize_impl<B_>(t, direction, subtable, method, S(stream)));
+}
+
+dyc_status dyc_resize(dyc_table* t, int direction, int subtable, dyc_stream_t stream) {
+    return dyc_resize_ex(t, direction, subtable, DYC_RESIZE_SPLIT, stream);
+}
+
+dyc_status dyc_clear(dyc_table* t, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    for (uint32_t i = 0; i < t->cfg.d; i++)
+        CU(cudaMemsetAsync(t->sub[i], 0xFF, t->nb[i] * t->cfg.bucket_slots * 8, S(stream)));
+    t->m = 0;
+    return DYC_OK;
+}
+
+dyc_status dyc_stats(dyc_table* t, dyc_stats_t* out, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (!out) return set_err(DYC_ERR_INVALID_ARG, "null out");
+    DISPATCH_B(t, stats_impl<B_>(t, out, S(stream)));
+}
+
+dyc_status dyc_dump(dyc_table* t, uint64_t* h_kv, uint32_t* h_table, uint64_t* h_bucket, uint64_t cap,
+                    uint64_t* n_out, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    DISPATCH_B(t, dump_impl<B_>(t, h_kv, h_table, h_bucket, cap, n_out, S(stream)));
+}
+
+dyc_status dyc_hash_params(const dyc_table* t, uint64_t* a, uint64_t* b) {
+    TRY(check_table(t));
+    for (uint32_t s = 0; s < t->cfg.d + 2; s++) {
+        if (a) a[s] = t->a[s];
+        if (b) b[s] = t->b[s];
+    }
+    return DYC_OK;
+}
+
+dyc_status dyc_hash_probe(dyc_table* t, const uint32_t* d_keys, uint64_t n, uint32_t* d_x, uint32_t* d_pair,
+                          dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (n == 0) return DYC_OK;
+    {
+        ProfScope ps(t, DYC_PROF_OTHER, S(stream));
+        k_hash_probe<<<grid_for(n, 128), 128, 0, S(stream)>>>(t->view(), d_keys, n, d_x, d_pair);
+    }
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+dyc_status dyc_insert_batch_host(dyc_table* t, const uint32_t* h_keys, const uint32_t* h_values, uint8_t* h_status,
+                                 uint64_t n, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (n == 0) return DYC_OK;
+    cudaStream_t st = S(stream);
+    TRY(ensure_stage(t, n * 9 + 64, st));
+    uint32_t* k = (uint32_t*)t->stage;
+    uint32_t* v = k + n;
+    uint8_t* s = (uint8_t*)(v + n);
+    CU(cudaMemcpyAsync(k, h_keys, n * 4, cudaMemcpyHostToDevice, st));
+    CU(cudaMemcpyAsync(v, h_values, n * 4, cudaMemcpyHostToDevice, st));
+    TRY(dyc_insert_batch(t, k, v, h_status ? s : nullptr, n, stream));
+    if (h_status) CU(cudaMemcpyAsync(h_status, s, n, cudaMemcpyDeviceToHost, st));
+    CU(cudaStreamSynchronize(st));
+    return DYC_OK;
+}
+
+dyc_status dyc_find_batch_host(dyc_table* t, const uint32_t* h_keys, uint32_t* h_values_out, uint8_t* h_found,
+                               uint64_t n, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (n == 0) return DYC_OK;
+    cudaStream_t st = S(stream);
+    TRY(ensure_stage(t, n * 9 + 64, st));
+    uint32_t* k = (uint32_t*)t->stage;
+    uint32_t* v = k + n;
+    uint8_t* f = (uint8_t*)(v + n);
+    CU(cudaMemcpyAsync(k, h_keys, n * 4, cudaMemcpyHostToDevice, st));
+    TRY(dyc_find_batch(t, k, v, h_found ? f : nullptr, n, stream));
+    if (h_values_out) CU(cudaMemcpyAsync(h_values_out, v, n * 4, cudaMemcpyDeviceToHost, st));
+    if (h_found) CU(cudaMemcpyAsync(h_found, f, n, cudaMemcpyDeviceToHost, st));
+    CU(cudaStreamSynchronize(st));
+    return DYC_OK;
+}
+
+dyc_status dyc_delete_batch_host(dyc_table* t, const uint32_t* h_keys, uint32_t* h_values_out, uint8_t* h_status,
+                                 uint64_t n, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (n == 0) return DYC_OK;
+    cudaStream_t st = S(stream);
+    TRY(ensure_stage(t, n * 9 + 64, st));
+    uint32_t* k = (uint32_t*)t->stage;
+    uint32_t* v = k + n;
+    uint8_t* s = (uint8_t*)(v + n);
+    CU(cudaMemcpyAsync(k, h_keys, n * 4, cudaMemcpyHostToDevice, st));
+    TRY(dyc_delete_batch(t, k, h_values_out ? v : nullptr, h_status ? s : nullptr, n, stream));
+    if (h_values_out) CU(cudaMemcpyAsync(h_values_out, v, n * 4, cudaMemcpyDeviceToHost, st));
+    if (h_status) CU(cudaMemcpyAsync(h_status, s, n, cudaMemcpyDeviceToHost, st));
+    CU(cudaStreamSynchronize(st));
+    return DYC_OK;
+}
+
+uint64_t dyc_launch_count(const dyc_table* t, int reset) {
+    if (!t) return 0;
+    uint64_t c = t->launches;
+    if (reset) const_cast<dyc_table*>(t)->launches = 0;
+    return c;
+}
+
+dyc_status dyc_profile_enable(dyc_table* t, int enable) {
+    TRY(check_table(t));
+    for (auto& r : t->recs) { t->ev_pool.push_back(r.a); t->ev_pool.push_back(r.b); }
+    t->recs.clear();
+    for (int k = 0; k < DYC_PROF_KINDS; k++) { t->prof_ms[k] = 0; t->prof_calls[k] = 0; }
+    t->prof = enable != 0;
+    return DYC_OK;
+}
+
+dyc_status dyc_profile_read(dyc_table* t, double* ms, uint64_t* calls) {
+    TRY(check_table(t));
+    for (auto& r : t->recs) {
+        CU(cudaEventSynchronize(r.b));
+        float x = 0.f;
+        CU(cudaEventElapsedTime(&x, r.a, r.b));
+        t->prof_ms[r.kind] += x;
+        t->prof_calls[r.kind]++;
+        t->ev_pool.push_back(r.a);
+        t->ev_pool.push_back(r.b);
+    }
+    t->recs.clear();
+    for (int k = 0; k < DYC_PROF_KINDS; k++) {
+        if (ms) ms[k] = t->prof_ms[k];
+        if (calls) calls[k] = t->prof_calls[k];
+    }
+    return DYC_OK;
+}
+
+dyc_status dyc_route_count(dyc_table* t, const uint32_t* d_keys, uint64_t n, uint32_t world, uint64_t* d_counts,
+                           dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (world < 1 || world > 4096) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..4096");
+    CU(cudaMemsetAsync(d_counts, 0, world * 8, S(stream)));
+    if (n == 0) return DYC_OK;
+    const uint32_t sh = t->cfg.d + 1;
+    {
+        ProfScope ps(t, DYC_PROF_OTHER, S(stream));
+        k_route_count<<<std::min<unsigned>(grid_for(n, kThreads), t->num_sms * 8), kThreads, world * 8, S(stream)>>>(
+            t->a[sh], t->b[sh], fastmod_magic(world), world, d_keys, n, (unsigned long long*)d_counts);
+    }
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_vals_in, uint64_t n,
+                             uint32_t world, uint64_t* d_offsets, uint32_t* d_keys_out, uint32_t* d_vals_out,
+                             uint32_t* d_pos, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (world < 1 || world > 4096) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..4096");
+    if (n == 0) return DYC_OK;
+    if (n > 0xFFFFFFFFull) return set_err(DYC_ERR_INVALID_ARG, "route batch must be < 2^32 ops");
+    const uint32_t sh = t->cfg.d + 1;
+    {
+        ProfScope ps(t, DYC_PROF_OTHER, S(stream));
+        k_route_scatter<<<grid_for(n, kThreads), kThreads, 0, S(stream)>>>(
+            t->a[sh], t->b[sh], fastmod_magic(world), world, d_keys, d_vals_in, n, (unsigned long long*)d_offsets,
+            d_keys_out, d_vals_out, d_pos);
+    }
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+dyc_status dyc_route_unpermute(const uint32_t* d_pos, uint64_t n, const uint32_t* d_reply_vals,
+                               const uint8_t* d_reply_status, uint32_t* d_vals, uint8_t* d_status,
+                               dyc_stream_t stream) {
+    if (n == 0) return DYC_OK;
+    k_route_unpermute<<<grid_for(n, kThreads), kThreads, 0, S(stream)>>>(d_pos, n, d_reply_vals, d_reply_status,
+                                                                        d_vals, d_status);
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+dyc_status dyc_bench_gather(const void* d_buf, uint64_t buf_bytes, uint64_t n_reads, uint32_t bytes_per_read,
+                            uint64_t seed, uint64_t* d_sink, dyc_stream_t stream) {
+    if (bytes_per_read != 32 && bytes_per_read != 64 && bytes_per_read != 128)
+        return set_err(DYC_ERR_INVALID_ARG, "bytes_per_read must be 32, 64 or 128");
+    const uint64_t units = buf_bytes / bytes_per_read;
+    if (units == 0) return set_err(DYC_ERR_INVALID_ARG, "buffer too small");
+    const unsigned grid = grid_for(n_reads, kThreads);
+    const unsigned long long* buf = (const unsigned long long*)d_buf;
+    unsigned long long* sink = (unsigned long long*)d_sink;
+    switch (bytes_per_read) {
+        case 32: k_gather<1><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
+        case 64: k_gather<2><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
+        default: k_gather<4><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
+    }
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,495 @@
+// dyc_kernels.cuh — the sm_100a kernels of the DyCuckoo hot path.
+//
+// Rows of SURVEY.md §8(a) and the kernel implementing each:
+//   S2+S3 find ............. k_find      (<= 2 probes)
+//   S2+S5 insert phase 1 ... k_upsert    (Alg. 1 L536-539 upsert; FUSE: first-fit CAS)
+//   S7    insert phase 2 ... k_place     (eviction chains; failure list P:L737)
+//   S4    delete ........... k_delete    (no lock)
+//   S8    upsize ........... k_upsize    (bucket b -> b or b+|h|)
+//   S9    downsize ......... k_downsize  (merge b, b+|h|/2; residuals)
+//   S10   stats / dump ..... k_count, k_dump
+//   S11   routing .......... k_route_count, k_route_scatter, k_route_unpermute
+// The paper's voter/lock mechanism (Alg. 1) was designed around
+// Pascal's slow contended atomics; here a key-value pair is one 64-bit word, so
+// lock-free atomicCAS (into an EMPTY slot) and atomicExch (eviction) on the slot
+// itself replace the bucket lock.
+#pragma once
+#include "dyc_device.cuh"
+
+namespace dyc {
+
+constexpr int kThreads = 256;
+
+enum CounterIdx : int {
+    C_PENDING = 0,    // new keys handed to k_place
+    C_INSERTED = 1,   // ops with status INSERTED
+    C_UPDATED = 2,    // ops with status UPDATED
+    C_FAIL = 3,       // homeless pairs appended by k_place
+    C_EVICT = 4,      // eviction hops
+    C_REMOVED = 5,    // delete hits
+    C_RESIDUAL = 6,   // downsize residuals
+    C_DUMP = 7,       // dump cursor
+    C_SECOND = 8,     // keys in their second-choice subtable (stats)
+    C_COUNT0 = 16,    // per-subtable live counts [16, 32)
+    C_N = 32
+};
+
+// ----------------------------------------------------------------- find (S3)
+// ILP queries per thread; all first probes are issued back to back, then the
+// second probes (predicated, only for first-probe misses: <= 2 lookups).
+template <int B, int ILP>
+__global__ void __launch_bounds__(kThreads) k_find(TableView tv, const uint32_t* __restrict__ keys,
+                                                   uint32_t* __restrict__ vals, uint8_t* __restrict__ found,
+                                                   uint64_t n) {
+    __shared__ SmemView sv;
+    load_view(tv, sv);
+    const uint64_t tile = (uint64_t)kThreads * ILP;
+    for (uint64_t base = (uint64_t)blockIdx.x * tile; base < n; base += (uint64_t)gridDim.x * tile) {
+        uint32_t k[ILP], v[ILP];
+        bool f[ILP];
+        const unsigned long long* p2[ILP];
+        unsigned long long s[ILP][B];
+#pragma unroll
+        for (int j = 0; j < ILP; j++) {
+            const uint64_t i = base + (uint64_t)j * kThreads + threadIdx.x;
+            k[j] = i < n ? __ldg(keys + i) : kEmptyKey;
+        }
+#pragma unroll
+        for (int j = 0; j < ILP; j++) {
+            const Pair p = pair_of(tv, k[j]);
+            p2[j] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[j]), B);
+            load_bucket_nc<B>(bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[j]), B), s[j]);
+        }
+#pragma unroll
+        for (int j = 0; j < ILP; j++) {
+            v[j] = kEmptyKey;
+            f[j] = lookup_slot<B>(s[j], k[j], v[j]) && k[j] != kEmptyKey;
+        }
+#pragma unroll
+        for (int j = 0; j < ILP; j++) load_bucket_nc_pred<B>(p2[j], s[j], !f[j] && k[j] != kEmptyKey);
+#pragma unroll
+        for (int j = 0; j < ILP; j++) {
+            if (!f[j] && k[j] != kEmptyKey) f[j] = lookup_slot<B>(s[j], k[j], v[j]);
+            const uint64_t i = base + (uint64_t)j * kThreads + threadIdx.x;
+            if (i < n) {
+                vals[i] = f[j] ? v[j] : kEmptyKey;
+                if (found) found[i] = f[j] ? 1 : 0;
+            }
+        }
+    }
+}
+
+// --------------------------------------------------------- placement helpers
+template <int B>
+__device__ __forceinline__ bool try_insert_empty(unsigned long long* bp, unsigned long long kv) {
+    unsigned long long s[B];
+    load_bucket_cg<B>(bp, s);
+#pragma unroll
+    for (int j = 0; j < B; j++) {
+        if (s[j] == kEmptySlot) {
+            if (cas_slot(bp + j, kEmptySlot, kv) == kEmptySlot) return true;
+        }
+    }
+    return false;
+}
+
+__device__ __forceinline__ uint32_t mix32(uint32_t x) {
+    x ^= x >> 16; x *= 0x7FEB352Du; x ^= x >> 15; x *= 0x846CA68Bu; x ^= x >> 16;
+    return x;
+}
+
+// Cuckoo placement of a pair known to be absent (S7).  First-fit over the
+// ordered pair (reading Q3); then an eviction chain: swap with a pseudo-random
+// victim slot (Q5) and carry the victim to the OTHER table of ITS pair
+// (P:L444).  Every pair is held by exactly one thread or one slot at any
+// time (atomicExch), so nothing is lost or duplicated.  After max_hops hops
+// (Q6) the carried pair is returned as homeless.
+template <int B>
+__device__ __forceinline__ bool place_kv(const TableView& tv, const SmemView& sv, unsigned long long kv,
+                                         unsigned long long& homeless, uint32_t& evictions, bool first_fit) {
+    uint32_t k = key_of(kv);
+    const Pair p = pair_of(tv, k);
+    if (first_fit) {
+        if (try_insert_empty<B>(bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B), kv)) return true;
+        if (try_insert_empty<B>(bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B), kv)) return true;
+    }
+    uint32_t t = (mix32(k) & 1u) ? p.t2 : p.t1;
+    for (uint32_t hop = 0; hop < tv.max_hops; hop++) {
+        unsigned long long* bp = bucket_ptr(sv, t, bucket_of(sv, t, k), B);
+        if (hop > 0 && try_insert_empty<B>(bp, kv)) return true;
+        const uint32_t victim = (mix32(k ^ (hop * 0x9E3779B9u)) >> 8) & (B - 1);
+        const unsigned long long old = exch_slot(bp + victim, kv);
+        evictions++;
+        if (old == kEmptySlot) return true;
+        kv = old;
+        k = key_of(kv);
+        const Pair q = pair_of(tv, k);
+        t = (t == q.t1) ? q.t2 : q.t1;
+    }
+    homeless = kv;
+    return false;
+}
+
+// ------------------------------------------------------ insert phase 1 (S5)
+// Upsert: probe t1's bucket, then t2's; an existing key gets its value replaced
+// (Alg. 1, status UPDATED).  A new key (status INSERTED) is, with FUSE,
+// CAS-ed into a free slot of its first-fit bucket right away; otherwise (or if
+// both candidate buckets are full) it is appended to `pending` for k_place.
+// Keys never move during this kernel (no evictions), so the existence check is
+// exact; FUSE is only used when no upsize can be needed ((m+n) <= beta*N).
+template <int B, bool FUSE>
+__global__ void __launch_bounds__(kThreads) k_upsert(TableView tv, const uint32_t* __restrict__ keys,
+                                                     const uint32_t* __restrict__ vals,
+                                                     uint8_t* __restrict__ status, uint64_t n,
+                                                     unsigned long long* __restrict__ pending,
+                                                     unsigned long long* __restrict__ ctr) {
+    __shared__ SmemView sv;
+    load_view(tv, sv);
+    unsigned long long n_ins = 0, n_upd = 0;
+    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < n; base += (uint64_t)gridDim.x * kThreads) {
+        const uint64_t i = base + threadIdx.x;
+        const bool valid = i < n;
+        const uint32_t k = valid ? __ldg(keys + i) : kEmptyKey;
+        const uint32_t v = valid ? __ldg(vals + i) : 0u;
+        const unsigned long long kv = make_kv(k, v);
+        uint8_t st = 0;
+        bool pend = false;
+        if (k != kEmptyKey) {
+            const Pair p = pair_of(tv, k);
+            unsigned long long* b1 = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B);
+            unsigned long long s1[B];
+            load_bucket_cg<B>(b1, s1);
+            int h = match_slot<B>(s1, k);
+            if (h >= 0) {
+                st_u64_cg(b1 + h, kv);
+                st = 2;
+            } else {
+                unsigned long long* b2 = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B);
+                unsigned long long s2[B];
+                load_bucket_cg<B>(b2, s2);
+                h = match_slot<B>(s2, k);
+                if (h >= 0) {
+                    st_u64_cg(b2 + h, kv);
+                    st = 2;
+                } else {
+                    st = 1;
+                    bool placed = false;
+                    if (FUSE) {
+#pragma unroll
+                        for (int j = 0; j < B; j++)
+                            if (!placed && s1[j] == kEmptySlot)
+                                placed = cas_slot(b1 + j, kEmptySlot, kv) == kEmptySlot;
+#pragma unroll
+                        for (int j = 0; j < B; j++)
+                            if (!placed && s2[j] == kEmptySlot)
+                                placed = cas_slot(b2 + j, kEmptySlot, kv) == kEmptySlot;
+                    }
+                    pend = !placed;
+                }
+            }
+        }
+        if (valid && status) status[i] = st;
+        warp_append(pend, kv, pending, ctr + C_PENDING);
+        n_ins += (st == 1);
+        n_upd += (st == 2);
+    }
+    block_add<kThreads>(ctr + C_INSERTED, n_ins);
+    block_add<kThreads>(ctr + C_UPDATED, n_upd);
+}
+
+// ------------------------------------------------------ insert phase 2 (S7)
+// Persistent grid-stride over list[0 .. *count) (count read on the device, so
+// no host round trip is needed between phase 1 and phase 2).  first_fit=false
+// skips the free-slot probe when the caller already found both buckets full
+// (pending keys of a FUSE upsert: nothing is deleted in between).
+template <int B>
+__global__ void __launch_bounds__(kThreads) k_place(TableView tv, const unsigned long long* __restrict__ list,
+                                                    const unsigned long long* count_ptr, uint64_t count_host,
+                                                    unsigned long long* __restrict__ fail_list,
+                                                    unsigned long long* __restrict__ ctr, bool first_fit) {
+    __shared__ SmemView sv;
+    load_view(tv, sv);
+    const uint64_t cnt = count_ptr ? *(volatile const unsigned long long*)count_ptr : count_host;
+    uint32_t ev = 0;
+    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < cnt; base += (uint64_t)gridDim.x * kThreads) {
+        const uint64_t i = base + threadIdx.x;
+        bool fail = false;
+        unsigned long long hl = kEmptySlot;
+        if (i < cnt) fail = !place_kv<B>(tv, sv, list[i], hl, ev, first_fit);
+        warp_append(fail, hl, fail_list, ctr + C_FAIL);
+    }
+    block_add<kThreads>(ctr + C_EVICT, ev);
+}
+
+// Reinsert every live slot of a detached buffer through the insert path (the
+// resize baselines of P:L736 and P:L809).
+template <int B>
+__global__ void __launch_bounds__(kThreads) k_reinsert(TableView tv, const unsigned long long* __restrict__ slots,
+                                                       uint64_t nslots, unsigned long long* __restrict__ fail_list,
+                                                       unsigned long long* __restrict__ ctr) {
+    __shared__ SmemView sv;
+    load_view(tv, sv);
+    uint32_t ev = 0;
+    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < nslots; base += (uint64_t)gridDim.x * kThreads) {
+        const uint64_t i = base + threadIdx.x;
+        bool fail = false;
+        unsigned long long hl = kEmptySlot;
+        if (i < nslots) {
+            const unsigned long long e = slots[i];
+            if (e != kEmptySlot) fail = !place_kv<B>(tv, sv, e, hl, ev, true);
+        }
+        warp_append(fail, hl, fail_list, ctr + C_FAIL);
+    }
+    block_add<kThreads>(ctr + C_EVICT, ev);
+}
+
+// ------------------------------------------------------------- delete (S4)
+template <int B>
+__global__ void __launch_bounds__(kThreads) k_delete(TableView tv, const uint32_t* __restrict__ keys,
+                                                     uint32_t* __restrict__ old_vals,
+                                                     uint8_t* __restrict__ status, uint64_t n,
+                                                     unsigned long long* __restrict__ ctr) {
+    __shared__ SmemView sv;
+    load_view(tv, sv);
+    unsigned long long removed = 0;
+    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < n; base += (uint64_t)gridDim.x * kThreads) {
+        const uint64_t i = base + threadIdx.x;
+        const bool valid = i < n;
+        const uint32_t k = valid ? __ldg(keys + i) : kEmptyKey;
+        uint32_t ov = kEmptyKey;
+        uint8_t st = 0;
+        if (k != kEmptyKey) {
+            const Pair p = pair_of(tv, k);
+            unsigned long long* b1 = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B);
+            unsigned long long s[B];
+            load_bucket_cg<B>(b1, s);
+            int h = match_slot<B>(s, k);
+            unsigned long long* bp = b1;
+            if (h < 0) {
+                bp = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B);
+                load_bucket_cg<B>(bp, s);
+                h = match_slot<B>(s, k);
+            }
+            if (h >= 0) {
+                unsigned long long e = kEmptySlot;
+#pragma unroll
+                for (int q = 0; q < B; q++)
+                    if (h == q) e = s[q];
+                ov = val_of(e);
+                st_u64_cg(bp + h, kEmptySlot);
+                st = 1;
+            }
+        }
+        if (valid) {
+            if (old_vals) old_vals[i] = ov;
+            if (status) status[i] = st;
+        }
+        removed += st;
+    }
+    block_add<kThreads>(ctr + C_REMOVED, removed);
+}
+
+// ------------------------------------------------------------- upsize (S8)
+// One lane per old slot; the B lanes of a bucket rank their entries with a
+// ballot (the warp-cooperative bucket pass of P:L379-380).  New bucket b gets the
+// entries that stay, b+n_old the ones that move; unused slots are written EMPTY,
+// so the new buffer needs no memset.  Streams: read 8 B, write 16 B per old slot.
+template <int B>
+__global__ void __launch_bounds__(kThreads) k_upsize(const unsigned long long* __restrict__ old_s,
+                                                     unsigned long long* __restrict__ new_s, uint32_t n_old,
+                                                     uint32_t a, uint32_t b, uint64_t magic2, uint32_t n2) {
+    static_assert(B <= 32 && (32 % B) == 0, "bucket must divide a warp");
+    const uint64_t total = (uint64_t)n_old * B;
+    const unsigned lane = threadIdx.x & 31;
+    const unsigned gmask = (B == 32) ? kFull : (((1u << B) - 1u) << (lane & ~(unsigned)(B - 1)));
+    const unsigned lt = lanemask_lt() & gmask;
+    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < total; base += (uint64_t)gridDim.x * kThreads) {
+        const uint64_t g = base + threadIdx.x;
+        const bool valid = g < total;
+        const unsigned long long e = valid ? __ldcs(old_s + g) : kEmptySlot;
+        const uint32_t bucket = (uint32_t)(g / B);
+        const uint32_t s = (uint32_t)(g % B);
+        const bool occ = key_of(e) != kEmptyKey;
+        bool hi = false;
+        if (occ) hi = fastmod(hx(a, b, key_of(e)), magic2, n2) != bucket;
+        const unsigned hb = __ballot_sync(kFull, occ && hi) & gmask;
+        const unsigned lb = __ballot_sync(kFull, occ && !hi) & gmask;
+        if (valid) {
+            const uint64_t lo_base = (uint64_t)bucket * B;
+            const uint64_t hi_base = ((uint64_t)bucket + n_old) * B;
+            if (occ) new_s[(hi ? hi_base : lo_base) + __popc((hi ? hb : lb) & lt)] = e;
+            if (s >= (uint32_t)__popc(lb)) new_s[lo_base + s] = kEmptySlot;
+            if (s >= (uint32_t)__popc(hb)) new_s[hi_base + s] = kEmptySlot;
+        }
+    }
+}
+
+// ----------------------------------------------------------- downsize (S9)
+// One lane per slot of the halved table: new bucket b' takes old b' then old
+// b'+h in slot order, keeps the first B (reading Q18) and appends the rest to
+// the residual list, which k_place then inserts into the pairs' other tables
+// (P:L392-393).  Streams: read 16 B, write 8 B per new slot.
+template <int B>
+__global__ void __launch_bounds__(kThreads) k_downsize(const unsigned long long* __restrict__ old_s,
+                                                       unsigned long long* __restrict__ new_s, uint32_t h,
+                                                       unsigned long long* __restrict__ residual,
+                                                       unsigned long long* __restrict__ ctr) {
+    static_assert(B <= 32 && (32 % B) == 0, "bucket must divide a warp");
+    const uint64_t total = (uint64_t)h * B;
+    const unsigned lane = threadIdx.x & 31;
+    const unsigned gmask = (B == 32) ? kFull : (((1u << B) - 1u) << (lane & ~(unsigned)(B - 1)));
+    const unsigned lt = lanemask_lt() & gmask;
+    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < total; base += (uint64_t)gridDim.x * kThreads) {
+        const uint64_t g = base + threadIdx.x;
+        const bool valid = g < total;
+        const unsigned long long e1 = valid ? __ldcs(old_s + g) : kEmptySlot;
+        const unsigned long long e2 = valid ? __ldcs(old_s + g + total) : kEmptySlot;
+        const bool o1 = key_of(e1) != kEmptyKey, o2 = key_of(e2) != kEmptyKey;
+        const unsigned m1 = __ballot_sync(kFull, o1) & gmask;
+        const unsigned m2 = __ballot_sync(kFull, o2) & gmask;
+        const uint32_t c1 = __popc(m1), ctot = c1 + __popc(m2);
+        const uint32_t r1 = __popc(m1 & lt), r2 = c1 + __popc(m2 & lt);
+        const uint64_t bb = (g / B) * B;
+        const uint32_t s = (uint32_t)(g % B);
+        bool res = false;
+        if (valid) {
+            if (o1) new_s[bb + r1] = e1;                 // r1 < c1 <= B always fits
+            if (o2) {
+                if (r2 < (uint32_t)B) new_s[bb + r2] = e2;
+                else res = true;
+            }
+            if (s >= ctot) new_s[bb + s] = kEmptySlot;
+        }
+        warp_append(res, e2, residual, ctr + C_RESIDUAL);
+    }
+}
+
+// ---------------------------------------------------------- stats / dump (S10)
+template <int B>
+__global__ void __launch_bounds__(kThreads) k_count(TableView tv, uint32_t t, unsigned long long* __restrict__ ctr) {
+    const unsigned long long* slots = tv.sub[t].slots;
+    const uint64_t total = (uint64_t)tv.sub[t].n * B;
+    unsigned long long cnt = 0, second = 0;
+    for (uint64_t g = (uint64_t)blockIdx.x * kThreads + threadIdx.x; g < total; g += (uint64_t)gridDim.x * kThreads) {
+        const unsigned long long e = slots[g];
+        if (key_of(e) != kEmptyKey) {
+            cnt++;
+            if (pair_of(tv, key_of(e)).t2 == t) second++;
+        }
+    }
+    block_add<kThreads>(ctr + C_COUNT0 + t, cnt);
+    block_add<kThreads>(ctr + C_SECOND, second);
+}
+
+template <int B>
+__global__ void __launch_bounds__(kThreads) k_dump(TableView tv, uint32_t t, unsigned long long* __restrict__ kv,
+                                                   uint32_t* __restrict__ tab, unsigned long long* __restrict__ bkt,
+                                                   uint64_t cap, unsigned long long* __restrict__ ctr) {
+    const unsigned long long* slots = tv.sub[t].slots;
+    const uint64_t total = (uint64_t)tv.sub[t].n * B;
+    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < total; base += (uint64_t)gridDim.x * kThreads) {
+        const uint64_t g = base + threadIdx.x;
+        const unsigned long long e = g < total ? slots[g] : kEmptySlot;
+        const bool occ = key_of(e) != kEmptyKey;
+        const unsigned m = __ballot_sync(kFull, occ);
+        if (!m) continue;
+        const int leader = __ffs(m) - 1;
+        unsigned long long pos = 0;
+        if ((int)(threadIdx.x & 31) == leader) pos = atomicAdd(ctr + C_DUMP, (unsigned long long)__popc(m));
+        pos = __shfl_sync(kFull, pos, leader) + __popc(m & lanemask_lt());
+        if (occ && pos < cap) {
+            kv[pos] = e;
+            tab[pos] = t;
+            bkt[pos] = g / B;
+        }
+    }
+}
+
+__global__ void k_hash_probe(TableView tv, const uint32_t* __restrict__ keys, uint64_t n, uint32_t* __restrict__ x,
+                             uint32_t* __restrict__ pr) {
+    const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const uint32_t k = keys[i];
+    for (uint32_t s = 0; s < tv.d + 2; s++) x[i * (tv.d + 2) + s] = hx(tv.a[s], tv.b[s], k);
+    const Pair p = pair_of(tv, k);
+    pr[2 * i] = p.t1;
+    pr[2 * i + 1] = p.t2;
+}
+
+// --------------------------------------------------------------- routing (S11)
+__global__ void __launch_bounds__(kThreads) k_route_count(uint32_t a, uint32_t b, uint64_t magic, uint32_t world,
+                                                          const uint32_t* __restrict__ keys, uint64_t n,
+                                                          unsigned long long* __restrict__ counts) {
+    extern __shared__ unsigned long long hist[];
+    for (uint32_t w = threadIdx.x; w < world; w += blockDim.x) hist[w] = 0;
+    __syncthreads();
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        atomicAdd(&hist[fastmod(hx(a, b, keys[i]), magic, world)], 1ull);
+    __syncthreads();
+    for (uint32_t w = threadIdx.x; w < world; w += blockDim.x)
+        if (hist[w]) atomicAdd(&counts[w], hist[w]);
+}
+
+// Lanes bound for the same shard are grouped with __match_any_sync; one atomic
+// per group claims their positions.
+__global__ void __launch_bounds__(kThreads) k_route_scatter(uint32_t a, uint32_t b, uint64_t magic, uint32_t world,
+                                                            const uint32_t* __restrict__ keys,
+                                                            const uint32_t* __restrict__ vals_in, uint64_t n,
+                                                            unsigned long long* __restrict__ cursor,
+                                                            uint32_t* __restrict__ keys_out,
+                                                            uint32_t* __restrict__ vals_out,
+                                                            uint32_t* __restrict__ pos_out) {
+    for (uint64_t base = (uint64_t)blockIdx.x * blockDim.x; base < n; base += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t i = base + threadIdx.x;
+        const bool valid = i < n;
+        const uint32_t k = valid ? keys[i] : 0u;
+        const uint32_t dest = valid ? fastmod(hx(a, b, k), magic, world) : 0xFFFFFFFFu;
+        const unsigned peers = __match_any_sync(kFull, dest);
+        const int leader = __ffs(peers) - 1;
+        unsigned long long p0 = 0;
+        if (valid && (int)(threadIdx.x & 31) == leader) p0 = atomicAdd(&cursor[dest], (unsigned long long)__popc(peers));
+        p0 = __shfl_sync(kFull, p0, leader);
+        if (valid) {
+            const uint64_t pos = p0 + __popc(peers & lanemask_lt());
+            keys_out[pos] = k;
+            if (vals_in && vals_out) vals_out[pos] = vals_in[i];
+            pos_out[i] = (uint32_t)pos;
+        }
+    }
+}
+
+__global__ void __launch_bounds__(kThreads) k_route_unpermute(const uint32_t* __restrict__ pos, uint64_t n,
+                                                              const uint32_t* __restrict__ rv,
+                                                              const uint8_t* __restrict__ rs,
+                                                              uint32_t* __restrict__ vals, uint8_t* __restrict__ st) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t p = pos[i];
+        if (rv && vals) vals[i] = rv[p];
+        if (rs && st) st[i] = rs[p];
+    }
+}
+
+// ------------------------------------------------------ random-gather ceiling
+template <int NSEC>
+__global__ void __launch_bounds__(kThreads) k_gather(const unsigned long long* __restrict__ buf, uint64_t n_units,
+                                                     uint64_t n_reads, uint64_t seed,
+                                                     unsigned long long* __restrict__ sink) {
+    unsigned long long acc = 0;
+    for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n_reads; i += (uint64_t)gridDim.x * kThreads) {
+        uint64_t h = (i + seed) * 0x9E3779B97F4A7C15ull;
+        h ^= h >> 29;
+        h *= 0xBF58476D1CE4E5B9ull;
+        h ^= h >> 32;
+        const uint64_t u = __umul64hi(h, n_units);
+        const unsigned long long* p = buf + u * (NSEC * 4);
+#pragma unroll
+        for (int q = 0; q < NSEC; q++) {
+            unsigned long long s[4];
+            ld4_nc(p + 4 * q, s);
+            acc ^= s[0] ^ s[1] ^ s[2] ^ s[3];
+        }
+    }
+    if (acc == 0x0123456789ABCDEFull) *sink = acc;   // keeps the loads alive
+}
+
+}  // namespace dyc

@@ -1,0 +1,207 @@
+"""Python view of a libdyc.so table.  PyTorch supplies device memory and streams
+only; every step of the hot path runs in the CUDA kernels behind the C ABI.
+
+Keys/values are passed as CUDA tensors of dtype torch.int32 or torch.uint32
+(reinterpreted as uint32; element i is op i).  Status/found arrays are uint8.
+"""
+from __future__ import annotations
+
+import ctypes as C
+from typing import Dict, Optional, Tuple
+
+import numpy as np
+
+from . import _lib as L
+
+_U32_DTYPES = None
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def _check_u32(t, name):
+    torch = _torch()
+    if not t.is_cuda:
+        raise ValueError(f"{name} must be a CUDA tensor")
+    if t.dtype not in (torch.int32, torch.uint32):
+        raise TypeError(f"{name} must be int32/uint32, got {t.dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+
+
+def _stream_ptr(stream) -> int:
+    torch = _torch()
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return int(s.cuda_stream)
+
+
+class Table:
+    """A DyCuckoo table (two-layer cuckoo hash, d subtables; see include/dycuckoo.h)."""
+
+    def __init__(self, d: int = 4, init_capacity: int = 4096, alpha: float = 0.3, beta: float = 0.85,
+                 bucket_slots: int = 4, seed: int = 0x5EED0001, max_hops: int = 64, device=None):
+        torch = _torch()
+        self._lib = L.load_library()
+        if not torch.cuda.is_available():
+            raise RuntimeError("dycuckoo needs a CUDA device (no CPU fallback)")
+        self.device = torch.device("cuda", torch.cuda.current_device() if device is None else
+                                   torch.device(device).index or 0)
+        cfg = L.dyc_config()
+        L.check(self._lib.dyc_config_default(C.byref(cfg)), "dyc_config_default")
+        cfg.d, cfg.bucket_slots, cfg.alpha, cfg.beta = d, bucket_slots, alpha, beta
+        cfg.init_capacity, cfg.seed, cfg.max_hops = init_capacity, seed, max_hops
+        self.cfg = cfg
+        h = C.c_void_p()
+        with torch.cuda.device(self.device):
+            L.check(self._lib.dyc_create_ex(C.byref(cfg), C.byref(h)), "dyc_create_ex")
+        self._h = h
+        self.d, self.B = d, bucket_slots
+
+    @property
+    def handle(self) -> int:
+        return self._h.value
+
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            self._lib.dyc_destroy(self._h)
+            self._h = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # noqa: BLE001
+            pass
+
+    # ------------------------------------------------------------ batches
+    def insert(self, keys, values, status=None, stream=None):
+        torch = _torch()
+        _check_u32(keys, "keys")
+        _check_u32(values, "values")
+        n = keys.numel()
+        if values.numel() != n:
+            raise ValueError("keys/values length mismatch")
+        if status is None:
+            status = torch.empty(n, dtype=torch.uint8, device=keys.device)
+        L.check(self._lib.dyc_insert_batch(self._h, keys.data_ptr(), values.data_ptr(),
+                                           status.data_ptr() if n else None, n, _stream_ptr(stream)),
+                "dyc_insert_batch")
+        return status
+
+    def find(self, keys, values_out=None, found=None, stream=None):
+        torch = _torch()
+        _check_u32(keys, "keys")
+        n = keys.numel()
+        if values_out is None:
+            values_out = torch.empty(n, dtype=torch.int32, device=keys.device)
+        if found is None:
+            found = torch.empty(n, dtype=torch.uint8, device=keys.device)
+        L.check(self._lib.dyc_find_batch(self._h, keys.data_ptr(), values_out.data_ptr(),
+                                         found.data_ptr() if n else None, n, _stream_ptr(stream)),
+                "dyc_find_batch")
+        return values_out, found
+
+    def delete(self, keys, values_out=None, status=None, stream=None, want_values=True):
+        torch = _torch()
+        _check_u32(keys, "keys")
+        n = keys.numel()
+        if values_out is None and want_values:
+            values_out = torch.empty(n, dtype=torch.int32, device=keys.device)
+        if status is None:
+            status = torch.empty(n, dtype=torch.uint8, device=keys.device)
+        L.check(self._lib.dyc_delete_batch(self._h, keys.data_ptr(),
+                                           values_out.data_ptr() if (values_out is not None and n) else None,
+                                           status.data_ptr() if n else None, n, _stream_ptr(stream)),
+                "dyc_delete_batch")
+        return values_out, status
+
+    # host-buffer entry points (end-to-end path: copies inside the call)
+    def insert_host(self, keys: np.ndarray, values: np.ndarray, stream=None) -> np.ndarray:
+        keys = np.ascontiguousarray(keys, dtype=np.uint32)
+        values = np.ascontiguousarray(values, dtype=np.uint32)
+        st = np.empty(keys.size, dtype=np.uint8)
+        L.check(self._lib.dyc_insert_batch_host(self._h, keys.ctypes.data, values.ctypes.data, st.ctypes.data,
+                                                keys.size, _stream_ptr(stream)), "dyc_insert_batch_host")
+        return st
+
+    def find_host(self, keys: np.ndarray, stream=None) -> Tuple[np.ndarray, np.ndarray]:
+        keys = np.ascontiguousarray(keys, dtype=np.uint32)
+        v = np.empty(keys.size, dtype=np.uint32)
+        f = np.empty(keys.size, dtype=np.uint8)
+        L.check(self._lib.dyc_find_batch_host(self._h, keys.ctypes.data, v.ctypes.data, f.ctypes.data,
+                                              keys.size, _stream_ptr(stream)), "dyc_find_batch_host")
+        return v, f
+
+    def delete_host(self, keys: np.ndarray, stream=None) -> Tuple[np.ndarray, np.ndarray]:
+        keys = np.ascontiguousarray(keys, dtype=np.uint32)
+        v = np.empty(keys.size, dtype=np.uint32)
+        s = np.empty(keys.size, dtype=np.uint8)
+        L.check(self._lib.dyc_delete_batch_host(self._h, keys.ctypes.data, v.ctypes.data, s.ctypes.data,
+                                                keys.size, _stream_ptr(stream)), "dyc_delete_batch_host")
+        return v, s
+
+    # ------------------------------------------------------------ control
+    def resize(self, direction: int, subtable: int = -1, method: int = L.DYC_RESIZE_SPLIT, stream=None):
+        L.check(self._lib.dyc_resize_ex(self._h, direction, subtable, method, _stream_ptr(stream)),
+                "dyc_resize_ex")
+
+    def clear(self, stream=None):
+        L.check(self._lib.dyc_clear(self._h, _stream_ptr(stream)), "dyc_clear")
+
+    def stats(self, stream=None) -> Dict:
+        s = L.dyc_stats_t()
+        L.check(self._lib.dyc_stats(self._h, C.byref(s), _stream_ptr(stream)), "dyc_stats")
+        d = s.d
+        return dict(m=s.m, N=s.N, d=d, B=s.B, buckets=list(s.buckets[:d]), count=list(s.count[:d]),
+                    fill=s.fill, n_upsize=s.n_upsize, n_downsize=s.n_downsize,
+                    n_fail_upsize=s.n_fail_upsize, n_residual=s.n_residual, n_evict=s.n_evict,
+                    n_place_retry=s.n_place_retry, n_second_table=s.n_second_table,
+                    bytes_allocated=s.bytes_allocated, last_insert_new=s.last_insert_new,
+                    last_insert_pending=s.last_insert_pending,
+                    last_insert_evictions=s.last_insert_evictions)
+
+    def dump(self, stream=None):
+        """(kv uint64, table uint32, bucket uint64) host arrays, unspecified order."""
+        n = C.c_uint64()
+        st = self.stats(stream)
+        m = st["m"]
+        kv = np.empty(m, dtype=np.uint64)
+        tb = np.empty(m, dtype=np.uint32)
+        bk = np.empty(m, dtype=np.uint64)
+        L.check(self._lib.dyc_dump(self._h, kv.ctypes.data, tb.ctypes.data, bk.ctypes.data, m, C.byref(n),
+                                   _stream_ptr(stream)), "dyc_dump")
+        return kv, tb, bk
+
+    def sorted_kv(self, stream=None) -> np.ndarray:
+        kv, _, _ = self.dump(stream)
+        keys = (kv & np.uint64(0xFFFFFFFF)).astype(np.uint32)
+        return kv[np.argsort(keys, kind="stable")]
+
+    def hash_params(self) -> Tuple[np.ndarray, np.ndarray]:
+        a = np.zeros(self.d + 2, dtype=np.uint64)
+        b = np.zeros(self.d + 2, dtype=np.uint64)
+        L.check(self._lib.dyc_hash_params(self._h, a.ctypes.data, b.ctypes.data), "dyc_hash_params")
+        return a, b
+
+    def hash_probe(self, keys, stream=None):
+        torch = _torch()
+        _check_u32(keys, "keys")
+        n = keys.numel()
+        x = torch.empty(n * (self.d + 2), dtype=torch.int32, device=keys.device)
+        pr = torch.empty(2 * n, dtype=torch.int32, device=keys.device)
+        L.check(self._lib.dyc_hash_probe(self._h, keys.data_ptr(), n, x.data_ptr(), pr.data_ptr(),
+                                         _stream_ptr(stream)), "dyc_hash_probe")
+        return x.view(n, self.d + 2), pr.view(n, 2)
+
+    def profile(self, enable: bool = True) -> None:
+        L.check(self._lib.dyc_profile_enable(self._h, 1 if enable else 0), "dyc_profile_enable")
+
+    def profile_read(self) -> Dict[str, Tuple[float, int]]:
+        ms = np.zeros(L.DYC_PROF_KINDS, dtype=np.float64)
+        calls = np.zeros(L.DYC_PROF_KINDS, dtype=np.uint64)
+        L.check(self._lib.dyc_profile_read(self._h, ms.ctypes.data, calls.ctypes.data), "dyc_profile_read")
+        return {name: (float(ms[i]), int(calls[i])) for i, name in enumerate(L.PROF_NAMES)}
+
+    def launch_count(self, reset: bool = False) -> int:
+        return int(self._lib.dyc_launch_count(self._h, 1 if reset else 0))

@@ -116,26 +116,46 @@ def c1_rand_small(seed_cfg: Optional[int] = None, n_keys: int = 65536,
     return w
 
 
+def perm_pow2(x: np.ndarray, log2n: int, seed: int) -> np.ndarray:
+    """A seeded bijection on [0, 2^log2n): xor-shift and odd-multiply rounds
+    (each invertible mod 2^log2n).  Used instead of shuffles so that 2^27-op
+    batches are generated in O(n) vectorised passes."""
+    mask = np.uint64((1 << log2n) - 1)
+    sh = np.uint64(max(1, (log2n + 1) // 2))
+    x = (np.asarray(x, dtype=np.uint64) ^ np.uint64(seed & ((1 << log2n) - 1))) & mask
+    with np.errstate(over="ignore"):
+        for c in (0x2C1B3C6D, 0x297A2D39, 0x9E3779B1):
+            x ^= x >> sh
+            x = (x * np.uint64(c)) & mask
+        x ^= x >> sh
+    return x
+
+
 def c2_rand_static(log2_n: int = 27, seed_cfg: Optional[int] = None,
                    beta: float = 0.85) -> Workload:
     """Config C2 (BASELINE.json configs[1]): 2^27 inserts into a table sized for
-    fill beta, then 2^27 finds (50% hit, shuffled) and 2^26 deletes of live keys.
+    fill beta, then 2^27 finds (50% hit: 2^26 distinct live keys and 2^26 misses,
+    interleaved pseudo-randomly) and 2^26 deletes of distinct live keys.
     `log2_n` scales it down for parity tests."""
     s = config_seed(2) if seed_cfg is None else seed_cfg
     n = 1 << log2_n
-    rng = np.random.Generator(np.random.PCG64(s))
     keys = key_range(0, n, s)
     vals = val_of(keys, 0)
     cap = int(math.ceil(n / beta))
     w = Workload(f"C2-rand-static-2^{log2_n}", 4, 0.3, beta, cap)
     w.batches.append(Batch("insert", keys, vals))
-    perm = rng.permutation(n)
-    hits = keys[perm[: n // 2]]
-    miss = key_range(MISS_BASE, n // 2, s)
-    q = np.concatenate([hits, miss])
-    rng.shuffle(q)
+    i = np.arange(n, dtype=np.uint64)
+    j = perm_pow2(i, log2_n, s ^ 0x1234567)            # position -> draw index
+    half = np.uint64(n // 2)
+    hit = j < half
+    hit_idx = perm_pow2(j, log2_n, s ^ 0x7654321)      # distinct indices of live keys
+    q = np.where(hit, keys[hit_idx.astype(np.int64) & (n - 1)],
+                 key_of(np.uint64(MISS_BASE) + (j - half), s)).astype(np.uint32)
+    # the miss range may contain the single EMPTY preimage: replace it by a live key's twin miss
+    q[q == np.uint32(EMPTY_KEY)] = key_of(np.array([MISS_BASE + n], dtype=np.uint64), s)[0]
     w.batches.append(Batch("find", q))
-    w.batches.append(Batch("delete", keys[perm[n // 2: n // 2 + n // 2]].copy()))
+    del_idx = perm_pow2(np.arange(n // 2, dtype=np.uint64), log2_n, s ^ 0x5A5A5A5)
+    w.batches.append(Batch("delete", np.ascontiguousarray(keys[del_idx.astype(np.int64)])))
     return w
 
 
@@ -160,3 +180,60 @@ def random_op_stream(seed: int, n_batches: int, batch: int, universe: int,
         for j in range(0, universe, max(1, batch)):
             w.batches.append(Batch("delete", univ[order[j:j + batch]].copy()))
     return w
+
+
+# ---------------------------------------------------------------------------
+# The same C2 recipe evaluated with torch int64 tensor ops (on the GPU or on
+# many CPU threads), for the full 2^27-op benchmark batches.  Bit-identical to
+# c2_rand_static (tests/test_workload.py); still no arithmetic of the method.
+def _lowbias32_t(x):
+    m = 0xFFFFFFFF
+    x = x ^ (x >> 16)
+    x = (x * 0x7FEB352D) & m
+    x = x ^ (x >> 15)
+    x = (x * 0x846CA68B) & m
+    x = x ^ (x >> 16)
+    return x
+
+
+def _key_of_t(idx, seed):
+    return _lowbias32_t((idx & 0xFFFFFFFF) ^ (seed & 0xFFFFFFFF))
+
+
+def _perm_pow2_t(x, log2n, seed):
+    mask = (1 << log2n) - 1
+    sh = max(1, (log2n + 1) // 2)
+    x = (x ^ (seed & mask)) & mask
+    for c in (0x2C1B3C6D, 0x297A2D39, 0x9E3779B1):
+        x = x ^ (x >> sh)
+        x = (x * c) & mask
+    return x ^ (x >> sh)
+
+
+def _as_i32(x):
+    import torch
+    return torch.where(x >= (1 << 31), x - (1 << 32), x).to(torch.int32)
+
+
+def c2_rand_static_torch(log2_n: int = 27, device="cuda", seed_cfg: Optional[int] = None, beta: float = 0.85):
+    """Returns (init_capacity, ins_keys, ins_vals, find_keys, del_keys) as int32
+    tensors holding the uint32 bit patterns of c2_rand_static(log2_n)."""
+    import torch
+    s = config_seed(2) if seed_cfg is None else seed_cfg
+    n = 1 << log2_n
+    idx = torch.arange(n + 1, dtype=torch.int64, device=device)
+    k = _key_of_t(idx, s)
+    k = k[k != EMPTY_KEY][:n]                                    # key_range(0, n, s)
+    mix = (0x9E3779B9 * 1) & 0xFFFFFFFF
+    v = _lowbias32_t(k ^ mix)                                    # val_of(keys, 0)
+    i = torch.arange(n, dtype=torch.int64, device=device)
+    j = _perm_pow2_t(i, log2_n, s ^ 0x1234567)
+    hit = j < n // 2
+    hit_idx = _perm_pow2_t(j, log2_n, s ^ 0x7654321) & (n - 1)
+    miss = _key_of_t(MISS_BASE + (j - n // 2), s)
+    q = torch.where(hit, k[hit_idx], miss)
+    q = torch.where(q == EMPTY_KEY, _key_of_t(torch.tensor(MISS_BASE + n, device=device), s), q)
+    del_idx = _perm_pow2_t(torch.arange(n // 2, dtype=torch.int64, device=device), log2_n, s ^ 0x5A5A5A5)
+    dk = k[del_idx]
+    cap = int(math.ceil(n / beta))
+    return cap, _as_i32(k), _as_i32(v), _as_i32(q), _as_i32(dk)

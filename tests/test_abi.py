@@ -1,0 +1,90 @@
+"""The C-ABI library builds, loads and exports every symbol include/*.h declares;
+host-only entry points behave without a GPU.  No compute calls here."""
+import ctypes as C
+import glob
+import os
+import re
+
+import pytest
+
+from paper_conf_icde_lizlhs21_b200 import _lib as L
+from paper_conf_icde_lizlhs21_b200.build import build_library, INCLUDE
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def declared_functions():
+    names = set()
+    for h in glob.glob(os.path.join(INCLUDE, "*.h")):
+        text = open(h).read()
+        text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
+        for m in re.finditer(r"^\s*[A-Za-z_][\w\s\*]*?\b(dyc_\w+)\s*\(", text, flags=re.M):
+            names.add(m.group(1))
+    return names
+
+
+@pytest.fixture(scope="module")
+def lib():
+    build_library()
+    return L.load_library()
+
+
+def test_header_declares_the_boundary():
+    names = declared_functions()
+    for required in ("dyc_create", "dyc_insert_batch", "dyc_find_batch", "dyc_delete_batch",
+                     "dyc_resize", "dyc_stats", "dyc_destroy", "dyc_dump"):
+        assert required in names
+
+
+def test_library_exports_every_declared_symbol(lib):
+    names = declared_functions()
+    missing = [n for n in sorted(names) if not hasattr(lib, n)]
+    assert not missing, missing
+    # the binding wraps exactly the declared functions
+    assert set(L.SIGNATURES) == names
+
+
+def test_binding_has_no_torch_in_abi():
+    text = open(os.path.join(INCLUDE, "dycuckoo.h")).read()
+    assert "torch" not in text.lower().replace("torch.distributed", "")
+    assert 'extern "C"' in text
+
+
+def test_host_only_calls_without_gpu(lib):
+    cfg = L.dyc_config()
+    assert lib.dyc_config_default(C.byref(cfg)) == L.DYC_OK
+    assert (cfg.d, cfg.bucket_slots, cfg.max_hops) == (4, 4, 64)
+    assert abs(cfg.alpha - 0.3) < 1e-12 and abs(cfg.beta - 0.85) < 1e-12
+    assert lib.dyc_version().decode().startswith("dycuckoo-b200")
+    h = C.c_void_p()
+    # infeasible bounds are rejected before touching a device (Q14)
+    cfg.alpha = 0.7
+    assert lib.dyc_create_ex(C.byref(cfg), C.byref(h)) == L.DYC_ERR_INVALID_ARG
+    assert "alpha" in L.last_error()
+    cfg.alpha, cfg.bucket_slots = 0.3, 6
+    assert lib.dyc_create_ex(C.byref(cfg), C.byref(h)) == L.DYC_ERR_INVALID_ARG
+    assert lib.dyc_destroy(None) == L.DYC_OK
+    assert lib.dyc_launch_count(None, 0) == 0
+
+
+def test_library_is_sm100a(lib):
+    """The fatbin carries sm_100a SASS (cuobjdump), with 256-bit probe loads."""
+    import shutil
+    import subprocess
+    cuobjdump = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+    if not os.path.exists(cuobjdump):
+        pytest.skip("cuobjdump not available")
+    out = subprocess.run([cuobjdump, "-lelf", L.LIB], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+    sass = subprocess.run([cuobjdump, "-sass", L.LIB], capture_output=True, text=True).stdout
+    assert "LDG.E.NA.ENL2.256" in sass      # one 256-bit load per 32-byte bucket probe
+    assert "ATOMG.E.CAS.64" in sass and "ATOMG.E.EXCH.64" in sass
+
+
+def test_product_does_not_import_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_icde_lizlhs21_b200")
+    for path in glob.glob(os.path.join(pkg, "**", "*.*"), recursive=True):
+        if path.endswith((".py", ".cu", ".cuh", ".h")):
+            text = open(path).read()
+            assert "import oracle" not in text and "from oracle" not in text, path
+            assert "dyc_oracle" not in text, path
