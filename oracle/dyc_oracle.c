@@ -426,6 +426,7 @@ static int cmp_u32(const void *x, const void *y)
  * ops in batch order (upsert or place); settle failures; then the α check. */
 void dyo_insert_batch(dyo_table *T, const uint32_t *keys, const uint32_t *vals, uint8_t *status, uint64_t n)
 {
+    if (n == 0) return;   /* reading Q32: an empty batch is a no-op (no resize check) */
     uint32_t *sorted = (uint32_t *)malloc((n + 1) * sizeof(uint32_t));
     memcpy(sorted, keys, n * sizeof(uint32_t));
     qsort(sorted, n, sizeof(uint32_t), cmp_u32);
@@ -473,6 +474,7 @@ void dyo_find_batch(dyo_table *T, const uint32_t *keys, uint32_t *vals_out, uint
 /* delete_batch: erase on match; then the α check. */
 void dyo_delete_batch(dyo_table *T, const uint32_t *keys, uint32_t *old_vals, uint8_t *status, uint64_t n)
 {
+    if (n == 0) return;   /* reading Q32 */
     for (uint64_t i = 0; i < n; i++) {
         uint32_t pr = 0;
         dyo_slot *sl = (keys[i] == DYO_EMPTY) ? NULL : lookup(T, keys[i], &pr);

@@ -63,6 +63,9 @@ def replay_sizes(d, B, init_capacity, alpha, beta, m_after_batches):
     n = [per] * d
     out = []
     for kind, target, m in m_after_batches:
+        if kind == "empty":          # reading Q32: an empty batch is a no-op
+            out.append(list(n))
+            continue
         if kind == "insert":
             while target > beta * (B * sum(n)):
                 t = min(range(d), key=lambda i: (n[i], i))
