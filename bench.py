@@ -40,12 +40,13 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="dycuckoo", choices=["dycuckoo", "reference"])
     ap.add_argument("--log2n", type=int, default=27, help="C2 batch size 2^log2n (27 = BASELINE configs[1])")
-    ap.add_argument("--bucket-slots", type=int, default=4)
+    ap.add_argument("--bucket-slots", type=int, default=8)
     ap.add_argument("--cpu-log2n", type=int, default=23, help="oracle sample size for cpu_baseline")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-rehash", action="store_true")
     ap.add_argument("--profile-only", action="store_true", help="a few steps, no extras (for ncu)")
+    ap.add_argument("--l2-fetch", type=int, default=None, help="set cudaLimitMaxL2FetchGranularity (bytes)")
     return ap.parse_args()
 
 
@@ -158,7 +159,7 @@ def reference_arm(args, rank, world):
         "steps": K, "warmup": Wm, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
         "config": {"workload": f"C2 RAND static (BASELINE configs[1]) shape, bounded sample 2^{log2n} keys",
-                   "d": 4, "alpha": 0.3, "beta": 0.85, "bucket_slots": 4},
+                   "d": 4, "alpha": 0.3, "beta": 0.85, "bucket_slots": 8},
         "cpu_baseline": {"value": value, "unit": "Mops/s", "cores": 1, "kind": "oracle",
                          "sample": f"C2 shape at 2^{log2n} keys per step (insert+find+delete)"},
         "e2e": {"value": value, "unit": "Mops/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -188,6 +189,8 @@ def main():
     from paper_conf_icde_lizlhs21_b200 import workload as W
     from paper_conf_icde_lizlhs21_b200.table import Table
 
+    if args.l2_fetch is not None:
+        L.check(L.dyc_set_l2_fetch_granularity(args.l2_fetch), "dyc_set_l2_fetch_granularity")
     n = 1 << args.log2n
     cap, k_ins, v_ins, k_find, k_del = W.c2_rand_static_torch(args.log2n, device="cuda")
     if world > 1:

@@ -83,7 +83,7 @@ enum {
 
 typedef struct {
     uint32_t d;              /* subtables, 2..DYC_MAX_D (paper default 4)      */
-    uint32_t bucket_slots;   /* B: 4 (32-byte bucket, default), 8, 16 or 32 (Q26)     */
+    uint32_t bucket_slots;   /* B: 4, 8 (64-byte bucket, default), 16 or 32 (Q26)     */
     double   alpha, beta;    /* fill bounds, 0 < alpha < beta < 1, alpha <= beta*d/(d+1) (Q14) */
     uint64_t init_capacity;  /* slots; n0 = max(1, ceil(init_capacity/(d*B))) buckets per subtable (Q13) */
     uint64_t seed;           /* SplitMix64 seed of the hash constants a_s, b_s (Q1)  */
@@ -110,7 +110,7 @@ typedef struct {
     uint64_t last_insert_evictions;   /* eviction hops of the last insert batch          */
 } dyc_stats_t;
 
-/* Fills *cfg with the defaults: d=4, B=4, alpha=0.3, beta=0.85 (Table
+/* Fills *cfg with the defaults: d=4, B=8, alpha=0.3, beta=0.85 (Table
  * `tbl:parameters`), init_capacity=4096, seed=0x5EED0001, max_hops=64. */
 dyc_status dyc_config_default(dyc_config* cfg);
 
@@ -245,6 +245,12 @@ dyc_status dyc_route_unpermute(const uint32_t* d_pos, uint64_t n, const uint32_t
 dyc_status dyc_bench_gather(const void* d_buf, uint64_t buf_bytes, uint64_t n_reads,
                             uint32_t bytes_per_read, uint64_t seed, uint64_t* d_sink,
                             dyc_stream_t stream);
+
+/* Device-wide L2 fetch granularity (cudaLimitMaxL2FetchGranularity, bytes in
+ * 0..128, a hint) for the current device: how much the L2 pulls from HBM on a
+ * sector miss.  Random 32-byte bucket probes want 32. */
+dyc_status dyc_set_l2_fetch_granularity(uint32_t bytes);
+dyc_status dyc_get_l2_fetch_granularity(uint32_t* bytes);
 
 /* Thread-local message for the last error returned on this thread. */
 const char* dyc_last_error(void);

@@ -76,6 +76,8 @@ SIGNATURES = {
     "dyc_route_scatter": (_I, [_TP, _P, _P, _U64, _U32, _P, _P, _P, _P, _P]),
     "dyc_route_unpermute": (_I, [_P, _U64, _P, _P, _P, _P, _P]),
     "dyc_bench_gather": (_I, [_P, _U64, _U64, _U32, _U64, _P, _P]),
+    "dyc_set_l2_fetch_granularity": (_I, [_U32]),
+    "dyc_get_l2_fetch_granularity": (_I, [C.POINTER(_U32)]),
     "dyc_last_error": (C.c_char_p, []),
     "dyc_version": (C.c_char_p, []),
 }
@@ -83,11 +85,13 @@ SIGNATURES = {
 _lib = None
 
 
-def load_library(path: str = LIB):
-    """Loads libdyc.so (building it first if nvcc is present and it is stale)."""
+def load_library(path: str = None):
+    """Loads libdyc.so (building it first if nvcc is present and it is stale).
+    DYC_LIB overrides the path (tuning experiments only)."""
     global _lib
     if _lib is not None:
         return _lib
+    path = path or os.environ.get("DYC_LIB") or LIB
     if not os.path.exists(path):
         try:
             from .build import build_library

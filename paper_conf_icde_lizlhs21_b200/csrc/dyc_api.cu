@@ -255,7 +255,7 @@ dyc_status place_and_settle(dyc_table* t, int src, const unsigned long long* d_c
         TRY(zero_one(t, C_EVICT, st));
         {
             ProfScope ps(t, DYC_PROF_PLACE, st);
-            k_place<B><<<grid_for(nfail, kThreads), kThreads, 0, st>>>(t->view(), t->list[cur], nullptr, nfail,
+            k_place<B><<<grid_for(nfail, kThreads / (B / 4)), kThreads, 0, st>>>(t->view(), t->list[cur], nullptr, nfail,
                                                                        t->list[1 - cur], t->d_ctr, true);
         }
         CU(cudaGetLastError());
@@ -321,7 +321,7 @@ dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals,
     TRY(ensure_lists(t, n, st));
     TRY(zero_ctr(t, st));
     const bool fuse = (double)(t->m + n) <= t->cfg.beta * (double)t->N();
-    const unsigned grid = grid_for(n, kThreads);
+    const unsigned grid = grid_for(n, kThreads / (B / 4));
     {
         ProfScope ps(t, DYC_PROF_UPSERT, st);
         if (fuse)
@@ -352,10 +352,11 @@ dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals,
 template <int B>
 dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* found, uint64_t n,
                      cudaStream_t st) {
-    constexpr int ILP = (B <= 4) ? 4 : (B <= 8 ? 2 : 1);
+    constexpr int ILP = (B <= 16) ? 4 : 2;
+    constexpr uint64_t per_block = (uint64_t)(kThreads / (B / 4)) * ILP;   // queries per block per pass
     {
         ProfScope ps(t, DYC_PROF_FIND, st);
-        k_find<B, ILP><<<grid_for(n, (uint64_t)kThreads * ILP), kThreads, 0, st>>>(t->view(), keys, vals, found, n);
+        k_find<B, ILP><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n);
     }
     CU(cudaGetLastError());
     return DYC_OK;
@@ -367,7 +368,8 @@ dyc_status delete_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8
     TRY(zero_one(t, C_REMOVED, st));
     {
         ProfScope ps(t, DYC_PROF_DELETE, st);
-        k_delete<B><<<grid_for(n, kThreads), kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr);
+        k_delete<B><<<grid_for(n, kThreads / (B / 4)), kThreads, 0, st>>>(t->view(), keys, vals, status, n,
+                                                                         t->d_ctr);
     }
     CU(cudaGetLastError());
     TRY(read_ctr(t, st));
@@ -404,7 +406,7 @@ dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaSt
         if (!touched[i]) continue;
         const uint64_t ns = old_nb[i] * B;
         ProfScope ps(t, DYC_PROF_REINSERT, st);
-        k_reinsert<B><<<grid_for(ns, kThreads), kThreads, 0, st>>>(tv, old[i], ns, t->list[1], t->d_ctr);
+        k_reinsert<B><<<grid_for(ns, kThreads / (B / 4)), kThreads, 0, st>>>(tv, old[i], ns, t->list[1], t->d_ctr);
         CU(cudaGetLastError());
     }
     TRY(read_ctr(t, st));
@@ -563,7 +565,7 @@ dyc_status dyc_config_default(dyc_config* cfg) {
     if (!cfg) return set_err(DYC_ERR_INVALID_ARG, "null cfg");
     std::memset(cfg, 0, sizeof(*cfg));
     cfg->d = 4;
-    cfg->bucket_slots = 4;
+    cfg->bucket_slots = 8;   // 64-byte buckets read by 2-lane groups
     cfg->alpha = 0.3;
     cfg->beta = 0.85;
     cfg->init_capacity = 4096;
@@ -870,6 +872,19 @@ dyc_status dyc_route_unpermute(const uint32_t* d_pos, uint64_t n, const uint32_t
     k_route_unpermute<<<grid_for(n, kThreads), kThreads, 0, S(stream)>>>(d_pos, n, d_reply_vals, d_reply_status,
                                                                         d_vals, d_status);
     CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+dyc_status dyc_set_l2_fetch_granularity(uint32_t bytes) {
+    if (bytes > 128) return set_err(DYC_ERR_INVALID_ARG, "granularity must be 0..128");
+    CU(cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, bytes));
+    return DYC_OK;
+}
+
+dyc_status dyc_get_l2_fetch_granularity(uint32_t* bytes) {
+    size_t v = 0;
+    CU(cudaDeviceGetLimit(&v, cudaLimitMaxL2FetchGranularity));
+    if (bytes) *bytes = (uint32_t)v;
     return DYC_OK;
 }
 

@@ -19,6 +19,19 @@
 namespace dyc {
 
 constexpr int kThreads = 256;
+// minimum resident blocks per SM requested from ptxas (register budget) per kernel family
+#ifndef DYC_FIND_MINB
+#define DYC_FIND_MINB 1
+#endif
+#ifndef DYC_UPSERT_MINB
+#define DYC_UPSERT_MINB 1
+#endif
+#ifndef DYC_DELETE_MINB
+#define DYC_DELETE_MINB 1
+#endif
+#ifndef DYC_PLACE_MINB
+#define DYC_PLACE_MINB 1
+#endif
 
 enum CounterIdx : int {
     C_PENDING = 0,    // new keys handed to k_place
@@ -34,63 +47,40 @@ enum CounterIdx : int {
     C_N = 32
 };
 
-// ----------------------------------------------------------------- find (S3)
-// ILP queries per thread; all first probes are issued back to back, then the
-// second probes (predicated, only for first-probe misses: <= 2 lookups).
-template <int B, int ILP>
-__global__ void __launch_bounds__(kThreads) k_find(TableView tv, const uint32_t* __restrict__ keys,
-                                                   uint32_t* __restrict__ vals, uint8_t* __restrict__ found,
-                                                   uint64_t n) {
-    __shared__ SmemView sv;
-    load_view(tv, sv);
-    const uint64_t tile = (uint64_t)kThreads * ILP;
-    for (uint64_t base = (uint64_t)blockIdx.x * tile; base < n; base += (uint64_t)gridDim.x * tile) {
-        uint32_t k[ILP], v[ILP];
-        bool f[ILP];
-        const unsigned long long* p2[ILP];
-        unsigned long long s[ILP][B];
-#pragma unroll
-        for (int j = 0; j < ILP; j++) {
-            const uint64_t i = base + (uint64_t)j * kThreads + threadIdx.x;
-            k[j] = i < n ? __ldg(keys + i) : kEmptyKey;
-        }
-#pragma unroll
-        for (int j = 0; j < ILP; j++) {
-            const Pair p = pair_of(tv, k[j]);
-            p2[j] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[j]), B);
-            load_bucket_nc<B>(bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[j]), B), s[j]);
-        }
-#pragma unroll
-        for (int j = 0; j < ILP; j++) {
-            v[j] = kEmptyKey;
-            f[j] = lookup_slot<B>(s[j], k[j], v[j]) && k[j] != kEmptyKey;
-        }
-#pragma unroll
-        for (int j = 0; j < ILP; j++) load_bucket_nc_pred<B>(p2[j], s[j], !f[j] && k[j] != kEmptyKey);
-#pragma unroll
-        for (int j = 0; j < ILP; j++) {
-            if (!f[j] && k[j] != kEmptyKey) f[j] = lookup_slot<B>(s[j], k[j], v[j]);
-            const uint64_t i = base + (uint64_t)j * kThreads + threadIdx.x;
-            if (i < n) {
-                vals[i] = f[j] ? v[j] : kEmptyKey;
-                if (found) found[i] = f[j] ? 1 : 0;
-            }
-        }
+// ------------------------------------------------------------- lane groups
+// G = B/4 lanes cooperate on one bucket: lane `sub` of the group holds slots
+// [4*sub, 4*sub+4) of it (one 256-bit load), so one warp-wide load instruction
+// probes 32/G buckets and a 128-byte bucket (B = 16) costs ONE line request.
+// Measured on B200: ~53 G random line requests/s whether a
+// request carries 32 or 128 bytes, so wide buckets read cooperatively are free
+// bytes that cut second-table probes (φ) and evictions.  This is the warp-
+// cooperative bucket scan of the paper with
+// __ballot_sync deciding the hit lane.
+template <int G>
+struct Grp {
+    unsigned lane, sub, base, gmask;
+    __device__ __forceinline__ Grp() {
+        lane = threadIdx.x & 31;
+        sub = lane & (G - 1);
+        base = lane - sub;
+        gmask = (G == 32) ? kFull : (((1u << G) - 1u) << base);
     }
-}
+    // group-local ballot: bit s <=> lane `s` of this group voted true
+    __device__ __forceinline__ unsigned ballot(bool p) const { return (__ballot_sync(kFull, p) & gmask) >> base; }
+    __device__ __forceinline__ unsigned long long bcast(unsigned long long v, unsigned src) const {
+        return __shfl_sync(kFull, v, base + src);
+    }
+    __device__ __forceinline__ uint32_t bcast32(uint32_t v, unsigned src) const {
+        return __shfl_sync(kFull, v, base + src);
+    }
+};
 
-// --------------------------------------------------------- placement helpers
-template <int B>
-__device__ __forceinline__ bool try_insert_empty(unsigned long long* bp, unsigned long long kv) {
-    unsigned long long s[B];
-    load_bucket_cg<B>(bp, s);
-#pragma unroll
-    for (int j = 0; j < B; j++) {
-        if (s[j] == kEmptySlot) {
-            if (cas_slot(bp + j, kEmptySlot, kv) == kEmptySlot) return true;
-        }
-    }
-    return false;
+__device__ __forceinline__ unsigned first_lane(unsigned bits) { return bits ? (unsigned)(__ffs(bits) - 1) : 0u; }
+
+__device__ __forceinline__ void ld4_cg_pred(const unsigned long long* p, unsigned long long* s, bool pred) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %5, 0;\n\t"
+                 "@q ld.global.cg.v4.u64 {%0,%1,%2,%3}, [%4];\n\t}"
+                 : "+l"(s[0]), "+l"(s[1]), "+l"(s[2]), "+l"(s[3]) : "l"(p), "r"((unsigned)pred) : "memory");
 }
 
 __device__ __forceinline__ uint32_t mix32(uint32_t x) {
@@ -98,36 +88,139 @@ __device__ __forceinline__ uint32_t mix32(uint32_t x) {
     return x;
 }
 
-// Cuckoo placement of a pair known to be absent (S7).  First-fit over the
-// ordered pair (reading Q3); then an eviction chain: swap with a pseudo-random
-// victim slot (Q5) and carry the victim to the OTHER table of ITS pair
-// (P:L444).  Every pair is held by exactly one thread or one slot at any
-// time (atomicExch), so nothing is lost or duplicated.  After max_hops hops
-// (Q6) the carried pair is returned as homeless.
+// First-fit CAS of kv into an EMPTY slot of the bucket whose group snapshot is s
+// (slot order).  Called by every lane of the warp (ballots); `want` is uniform
+// within a group.  A failed CAS means another key took that slot: try the next.
+template <int G>
+__device__ __forceinline__ bool coop_cas_empty(const Grp<G>& g, unsigned long long* bp,
+                                               const unsigned long long (&s)[4], bool want,
+                                               unsigned long long kv) {
+    unsigned emask = 0;
+#pragma unroll
+    for (int j = 0; j < 4; j++)
+        if (s[j] == kEmptySlot) emask |= 1u << j;
+    bool placed = false;
+    for (;;) {
+        const unsigned cand = g.ballot(want && !placed && emask != 0);
+        if (!__any_sync(kFull, cand != 0)) break;
+        const unsigned owner = first_lane(cand);
+        bool ok = false;
+        if (cand && g.sub == owner) {
+            const unsigned j = __ffs(emask) - 1;
+            ok = cas_slot(bp + 4 * g.sub + j, kEmptySlot, kv) == kEmptySlot;
+            emask &= ~(1u << j);
+        }
+        ok = __shfl_sync(kFull, ok, g.base + owner);
+        if (cand && ok) placed = true;
+    }
+    return placed;
+}
+
+// ----------------------------------------------------------------- find (S3)
+// ILP queries per group; all first probes are issued back to back, then the
+// second probes (predicated, only after a first-probe miss: <= 2 lookups).
+template <int B, int ILP>
+__global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, const uint32_t* __restrict__ keys,
+                                                   uint32_t* __restrict__ vals, uint8_t* __restrict__ found,
+                                                   uint64_t n) {
+    constexpr int G = B / 4, QPW = 32 / G;
+    __shared__ SmemView sv;
+    load_view(tv, sv);
+    const Grp<G> g;
+    const unsigned grp = g.lane / G;
+    const uint64_t wtile = (uint64_t)QPW * ILP;
+    const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
+    const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
+    for (uint64_t base = w * wtile; base < n; base += nwarps * wtile) {
+        uint32_t k[ILP], v[ILP];
+        bool f[ILP];
+        const unsigned long long* p2[ILP];
+        unsigned long long s[ILP][4];
+#pragma unroll
+        for (int j = 0; j < ILP; j++) {
+            const uint64_t i = base + (uint64_t)j * QPW + grp;
+            k[j] = i < n ? __ldg(keys + i) : kEmptyKey;
+        }
+#pragma unroll
+        for (int j = 0; j < ILP; j++) {
+            const Pair p = pair_of(tv, k[j]);
+            p2[j] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[j]), B) + 4 * g.sub;
+            ld4_nc(bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[j]), B) + 4 * g.sub, s[j]);
+        }
+#pragma unroll
+        for (int j = 0; j < ILP; j++) {
+            uint32_t lv = 0;
+            const bool lh = lookup_slot<4>(s[j], k[j], lv) && k[j] != kEmptyKey;
+            const unsigned hb = g.ballot(lh);
+            f[j] = hb != 0;
+            v[j] = g.bcast32(lv, first_lane(hb));
+        }
+#pragma unroll
+        for (int j = 0; j < ILP; j++) ld4_nc_pred(p2[j], s[j], !f[j] && k[j] != kEmptyKey);
+#pragma unroll
+        for (int j = 0; j < ILP; j++) {
+            uint32_t lv = 0;
+            const bool lh = !f[j] && k[j] != kEmptyKey && lookup_slot<4>(s[j], k[j], lv);
+            const unsigned hb = g.ballot(lh);
+            const uint32_t v2 = g.bcast32(lv, first_lane(hb));
+            if (hb) { f[j] = true; v[j] = v2; }
+            const uint64_t i = base + (uint64_t)j * QPW + grp;
+            if (g.sub == 0 && i < n) {
+                vals[i] = f[j] ? v[j] : kEmptyKey;
+                if (found) found[i] = f[j] ? 1 : 0;
+            }
+        }
+    }
+}
+
+// ------------------------------------------------------- placement (S7 core)
+// Cuckoo placement of a pair known to be absent, by one lane group.  First-fit
+// over the ordered pair (reading Q3); then an eviction chain: exchange with a
+// pseudo-random victim slot (Q5) and carry the victim to the OTHER table of ITS
+// pair.  Every pair is held by exactly one group or one slot at
+// any time (atomicExch), so nothing is lost or duplicated.  After max_hops hops
+// (Q6) the carried pair is returned as homeless.  Returns true when placed;
+// groups that enter with done == true only take part in the ballots.
 template <int B>
-__device__ __forceinline__ bool place_kv(const TableView& tv, const SmemView& sv, unsigned long long kv,
-                                         unsigned long long& homeless, uint32_t& evictions, bool first_fit) {
+__device__ __forceinline__ bool coop_place(const Grp<B / 4>& g, const TableView& tv, const SmemView& sv,
+                                           unsigned long long& kv, bool done, bool first_fit, uint32_t& ev) {
     uint32_t k = key_of(kv);
     const Pair p = pair_of(tv, k);
+    unsigned long long s[4] = {kEmptySlot, kEmptySlot, kEmptySlot, kEmptySlot};
     if (first_fit) {
-        if (try_insert_empty<B>(bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B), kv)) return true;
-        if (try_insert_empty<B>(bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B), kv)) return true;
+        unsigned long long* b1 = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B);
+        ld4_cg_pred(b1 + 4 * g.sub, s, !done);
+        done |= coop_cas_empty(g, b1, s, !done, kv);
+        unsigned long long* b2 = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B);
+        ld4_cg_pred(b2 + 4 * g.sub, s, !done);
+        done |= coop_cas_empty(g, b2, s, !done, kv);
     }
     uint32_t t = (mix32(k) & 1u) ? p.t2 : p.t1;
     for (uint32_t hop = 0; hop < tv.max_hops; hop++) {
+        if (!__any_sync(kFull, !done)) break;
         unsigned long long* bp = bucket_ptr(sv, t, bucket_of(sv, t, k), B);
-        if (hop > 0 && try_insert_empty<B>(bp, kv)) return true;
+        if (hop > 0) {
+            ld4_cg_pred(bp + 4 * g.sub, s, !done);
+            done |= coop_cas_empty(g, bp, s, !done, kv);
+        }
         const uint32_t victim = (mix32(k ^ (hop * 0x9E3779B9u)) >> 8) & (B - 1);
-        const unsigned long long old = exch_slot(bp + victim, kv);
-        evictions++;
-        if (old == kEmptySlot) return true;
-        kv = old;
-        k = key_of(kv);
-        const Pair q = pair_of(tv, k);
-        t = (t == q.t1) ? q.t2 : q.t1;
+        const unsigned owner = victim >> 2;
+        unsigned long long old = kEmptySlot;
+        if (!done && g.sub == owner) old = exch_slot(bp + victim, kv);
+        old = g.bcast(old, owner);
+        if (!done) {
+            ev += (g.sub == 0);
+            if (old == kEmptySlot) {
+                done = true;
+            } else {
+                kv = old;
+                k = key_of(kv);
+                const Pair q = pair_of(tv, k);
+                t = (t == q.t1) ? q.t2 : q.t1;
+            }
+        }
     }
-    homeless = kv;
-    return false;
+    return done;
 }
 
 // ------------------------------------------------------ insert phase 1 (S5)
@@ -138,60 +231,51 @@ __device__ __forceinline__ bool place_kv(const TableView& tv, const SmemView& sv
 // Keys never move during this kernel (no evictions), so the existence check is
 // exact; FUSE is only used when no upsize can be needed ((m+n) <= beta*N).
 template <int B, bool FUSE>
-__global__ void __launch_bounds__(kThreads) k_upsert(TableView tv, const uint32_t* __restrict__ keys,
+__global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView tv, const uint32_t* __restrict__ keys,
                                                      const uint32_t* __restrict__ vals,
                                                      uint8_t* __restrict__ status, uint64_t n,
                                                      unsigned long long* __restrict__ pending,
                                                      unsigned long long* __restrict__ ctr) {
+    constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
+    const Grp<G> g;
+    const unsigned grp = g.lane / G;
+    const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
+    const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     unsigned long long n_ins = 0, n_upd = 0;
-    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < n; base += (uint64_t)gridDim.x * kThreads) {
-        const uint64_t i = base + threadIdx.x;
+    for (uint64_t base = w * QPW; base < n; base += nwarps * QPW) {
+        const uint64_t i = base + grp;
         const bool valid = i < n;
         const uint32_t k = valid ? __ldg(keys + i) : kEmptyKey;
         const uint32_t v = valid ? __ldg(vals + i) : 0u;
         const unsigned long long kv = make_kv(k, v);
-        uint8_t st = 0;
-        bool pend = false;
-        if (k != kEmptyKey) {
-            const Pair p = pair_of(tv, k);
-            unsigned long long* b1 = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B);
-            unsigned long long s1[B];
-            load_bucket_cg<B>(b1, s1);
-            int h = match_slot<B>(s1, k);
-            if (h >= 0) {
-                st_u64_cg(b1 + h, kv);
-                st = 2;
-            } else {
-                unsigned long long* b2 = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B);
-                unsigned long long s2[B];
-                load_bucket_cg<B>(b2, s2);
-                h = match_slot<B>(s2, k);
-                if (h >= 0) {
-                    st_u64_cg(b2 + h, kv);
-                    st = 2;
-                } else {
-                    st = 1;
-                    bool placed = false;
-                    if (FUSE) {
-#pragma unroll
-                        for (int j = 0; j < B; j++)
-                            if (!placed && s1[j] == kEmptySlot)
-                                placed = cas_slot(b1 + j, kEmptySlot, kv) == kEmptySlot;
-#pragma unroll
-                        for (int j = 0; j < B; j++)
-                            if (!placed && s2[j] == kEmptySlot)
-                                placed = cas_slot(b2 + j, kEmptySlot, kv) == kEmptySlot;
-                    }
-                    pend = !placed;
-                }
-            }
+        const bool active = k != kEmptyKey;
+        const Pair p = pair_of(tv, k);
+        unsigned long long* b1 = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B);
+        unsigned long long* b2 = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B);
+        unsigned long long s1[4], s2[4] = {kEmptySlot, kEmptySlot, kEmptySlot, kEmptySlot};
+        ld4_cg(b1 + 4 * g.sub, s1);
+        const int j1 = match_slot<4>(s1, k);
+        const unsigned h1 = g.ballot(active && j1 >= 0);
+        const bool need2 = active && h1 == 0;
+        ld4_cg_pred(b2 + 4 * g.sub, s2, need2);
+        const int j2 = match_slot<4>(s2, k);
+        const unsigned h2 = g.ballot(need2 && j2 >= 0);
+        if (h1 && g.sub == first_lane(h1)) st_u64_cg(b1 + 4 * g.sub + j1, kv);
+        if (h2 && g.sub == first_lane(h2)) st_u64_cg(b2 + 4 * g.sub + j2, kv);
+        const bool isnew = need2 && h2 == 0;
+        bool placed = false;
+        if (FUSE) {
+            placed = coop_cas_empty(g, b1, s1, isnew, kv);
+            placed |= coop_cas_empty(g, b2, s2, isnew && !placed, kv);
         }
-        if (valid && status) status[i] = st;
-        warp_append(pend, kv, pending, ctr + C_PENDING);
-        n_ins += (st == 1);
-        n_upd += (st == 2);
+        const uint8_t st = !active ? 0 : ((h1 | h2) ? 2 : 1);
+        const bool lead = g.sub == 0;
+        if (lead && valid && status) status[i] = st;
+        warp_append(lead && isnew && !placed, kv, pending, ctr + C_PENDING);
+        n_ins += lead && st == 1;
+        n_upd += lead && st == 2;
     }
     block_add<kThreads>(ctr + C_INSERTED, n_ins);
     block_add<kThreads>(ctr + C_UPDATED, n_upd);
@@ -203,20 +287,24 @@ __global__ void __launch_bounds__(kThreads) k_upsert(TableView tv, const uint32_
 // skips the free-slot probe when the caller already found both buckets full
 // (pending keys of a FUSE upsert: nothing is deleted in between).
 template <int B>
-__global__ void __launch_bounds__(kThreads) k_place(TableView tv, const unsigned long long* __restrict__ list,
+__global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv, const unsigned long long* __restrict__ list,
                                                     const unsigned long long* count_ptr, uint64_t count_host,
                                                     unsigned long long* __restrict__ fail_list,
                                                     unsigned long long* __restrict__ ctr, bool first_fit) {
+    constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
+    const Grp<G> g;
+    const unsigned grp = g.lane / G;
     const uint64_t cnt = count_ptr ? *(volatile const unsigned long long*)count_ptr : count_host;
+    const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
+    const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     uint32_t ev = 0;
-    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < cnt; base += (uint64_t)gridDim.x * kThreads) {
-        const uint64_t i = base + threadIdx.x;
-        bool fail = false;
-        unsigned long long hl = kEmptySlot;
-        if (i < cnt) fail = !place_kv<B>(tv, sv, list[i], hl, ev, first_fit);
-        warp_append(fail, hl, fail_list, ctr + C_FAIL);
+    for (uint64_t base = w * QPW; base < cnt; base += nwarps * QPW) {
+        const uint64_t i = base + grp;
+        unsigned long long kv = i < cnt ? list[i] : kEmptySlot;
+        const bool done = coop_place<B>(g, tv, sv, kv, i >= cnt, first_fit, ev);
+        warp_append(g.sub == 0 && !done, kv, fail_list, ctr + C_FAIL);
     }
     block_add<kThreads>(ctr + C_EVICT, ev);
 }
@@ -227,64 +315,66 @@ template <int B>
 __global__ void __launch_bounds__(kThreads) k_reinsert(TableView tv, const unsigned long long* __restrict__ slots,
                                                        uint64_t nslots, unsigned long long* __restrict__ fail_list,
                                                        unsigned long long* __restrict__ ctr) {
+    constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
+    const Grp<G> g;
+    const unsigned grp = g.lane / G;
+    const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
+    const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     uint32_t ev = 0;
-    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < nslots; base += (uint64_t)gridDim.x * kThreads) {
-        const uint64_t i = base + threadIdx.x;
-        bool fail = false;
-        unsigned long long hl = kEmptySlot;
-        if (i < nslots) {
-            const unsigned long long e = slots[i];
-            if (e != kEmptySlot) fail = !place_kv<B>(tv, sv, e, hl, ev, true);
-        }
-        warp_append(fail, hl, fail_list, ctr + C_FAIL);
+    for (uint64_t base = w * QPW; base < nslots; base += nwarps * QPW) {
+        const uint64_t i = base + grp;
+        unsigned long long kv = i < nslots ? slots[i] : kEmptySlot;
+        const bool done = coop_place<B>(g, tv, sv, kv, kv == kEmptySlot, true, ev);
+        warp_append(g.sub == 0 && !done, kv, fail_list, ctr + C_FAIL);
     }
     block_add<kThreads>(ctr + C_EVICT, ev);
 }
 
 // ------------------------------------------------------------- delete (S4)
 template <int B>
-__global__ void __launch_bounds__(kThreads) k_delete(TableView tv, const uint32_t* __restrict__ keys,
+__global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView tv, const uint32_t* __restrict__ keys,
                                                      uint32_t* __restrict__ old_vals,
                                                      uint8_t* __restrict__ status, uint64_t n,
                                                      unsigned long long* __restrict__ ctr) {
+    constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
+    const Grp<G> g;
+    const unsigned grp = g.lane / G;
+    const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
+    const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     unsigned long long removed = 0;
-    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < n; base += (uint64_t)gridDim.x * kThreads) {
-        const uint64_t i = base + threadIdx.x;
+    for (uint64_t base = w * QPW; base < n; base += nwarps * QPW) {
+        const uint64_t i = base + grp;
         const bool valid = i < n;
         const uint32_t k = valid ? __ldg(keys + i) : kEmptyKey;
-        uint32_t ov = kEmptyKey;
-        uint8_t st = 0;
-        if (k != kEmptyKey) {
-            const Pair p = pair_of(tv, k);
-            unsigned long long* b1 = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B);
-            unsigned long long s[B];
-            load_bucket_cg<B>(b1, s);
-            int h = match_slot<B>(s, k);
-            unsigned long long* bp = b1;
-            if (h < 0) {
-                bp = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B);
-                load_bucket_cg<B>(bp, s);
-                h = match_slot<B>(s, k);
-            }
-            if (h >= 0) {
-                unsigned long long e = kEmptySlot;
-#pragma unroll
-                for (int q = 0; q < B; q++)
-                    if (h == q) e = s[q];
-                ov = val_of(e);
-                st_u64_cg(bp + h, kEmptySlot);
-                st = 1;
-            }
+        const bool active = k != kEmptyKey;
+        const Pair p = pair_of(tv, k);
+        unsigned long long* b1 = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B);
+        unsigned long long* b2 = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B);
+        unsigned long long s1[4], s2[4] = {kEmptySlot, kEmptySlot, kEmptySlot, kEmptySlot};
+        ld4_cg(b1 + 4 * g.sub, s1);
+        uint32_t lv1 = 0, lv2 = 0;
+        const int j1 = active ? match_slot<4>(s1, k) : -1;
+        lookup_slot<4>(s1, k, lv1);
+        const unsigned h1 = g.ballot(j1 >= 0);
+        const bool need2 = active && h1 == 0;
+        ld4_cg_pred(b2 + 4 * g.sub, s2, need2);
+        const int j2 = need2 ? match_slot<4>(s2, k) : -1;
+        lookup_slot<4>(s2, k, lv2);
+        const unsigned h2 = g.ballot(j2 >= 0);
+        if (h1 && g.sub == first_lane(h1)) st_u64_cg(b1 + 4 * g.sub + j1, kEmptySlot);
+        if (h2 && g.sub == first_lane(h2)) st_u64_cg(b2 + 4 * g.sub + j2, kEmptySlot);
+        const uint32_t o1 = g.bcast32(lv1, first_lane(h1));
+        const uint32_t o2 = g.bcast32(lv2, first_lane(h2));
+        const bool hit = (h1 | h2) != 0;
+        if (g.sub == 0 && valid) {
+            if (old_vals) old_vals[i] = h1 ? o1 : (h2 ? o2 : kEmptyKey);
+            if (status) status[i] = hit ? 1 : 0;
         }
-        if (valid) {
-            if (old_vals) old_vals[i] = ov;
-            if (status) status[i] = st;
-        }
-        removed += st;
+        removed += (g.sub == 0 && hit);
     }
     block_add<kThreads>(ctr + C_REMOVED, removed);
 }

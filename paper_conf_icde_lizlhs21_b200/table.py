@@ -41,7 +41,7 @@ class Table:
     """A DyCuckoo table (two-layer cuckoo hash, d subtables; see include/dycuckoo.h)."""
 
     def __init__(self, d: int = 4, init_capacity: int = 4096, alpha: float = 0.3, beta: float = 0.85,
-                 bucket_slots: int = 4, seed: int = 0x5EED0001, max_hops: int = 64, device=None):
+                 bucket_slots: int = 8, seed: int = 0x5EED0001, max_hops: int = 64, device=None):
         torch = _torch()
         self._lib = L.load_library()
         if not torch.cuda.is_available():

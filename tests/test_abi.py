@@ -53,7 +53,7 @@ def test_binding_has_no_torch_in_abi():
 def test_host_only_calls_without_gpu(lib):
     cfg = L.dyc_config()
     assert lib.dyc_config_default(C.byref(cfg)) == L.DYC_OK
-    assert (cfg.d, cfg.bucket_slots, cfg.max_hops) == (4, 4, 64)
+    assert (cfg.d, cfg.bucket_slots, cfg.max_hops) == (4, 8, 64)
     assert abs(cfg.alpha - 0.3) < 1e-12 and abs(cfg.beta - 0.85) < 1e-12
     assert lib.dyc_version().decode().startswith("dycuckoo-b200")
     h = C.c_void_p()

@@ -157,8 +157,6 @@ def test_edge_cases(oracle_mod):
 def test_example2_scenario_semantics(oracle_mod):
     """Example 2 as one GPU batch: k1 into a free bucket, k33 updated
     in place, k65 evicting from a full bucket; every key ends present once."""
-    wl = W.Workload("ex2", 4, 0.01, 0.99, 4 * 2 * 8)
-    o = oracle_mod.OracleTable(d=4, init_capacity=64, bucket_slots=2, alpha=0.01, beta=0.99)
     keys = W.key_range(0, 40, 77)
     # fill a tiny table so inserts must evict, then insert/update a mix
     g = Table(d=4, init_capacity=64, bucket_slots=4, alpha=0.01, beta=0.99)
@@ -250,8 +248,9 @@ def test_resize_refusals():
 # ------------------------------------------------------------------ host-buffer path
 def test_host_entry_points_match_device(oracle_mod):
     wl = W.c2_rand_static(log2_n=15)
-    g = Table(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta)
-    o = oracle_mod.OracleTable(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta)
+    g = Table(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=8)
+    o = oracle_mod.OracleTable(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta,
+                               bucket_slots=8)
     ins, fnd, dele = wl.batches
     np.testing.assert_array_equal(g.insert_host(ins.keys, ins.values), o.insert(ins.keys, ins.values))
     v, f = g.find_host(fnd.keys)
@@ -275,7 +274,7 @@ def test_c2_full_size_sampled():
     (checked on a sample of 2^20 keys one by one)."""
     wl = W.c2_rand_static(log2_n=27)
     ins, fnd, dele = wl.batches
-    g = Table(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta)
+    g = Table(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=8)
     st = g.insert(dev(ins.keys), dev(ins.values))
     assert int((st == 1).sum()) == ins.keys.size
     s = g.stats()
