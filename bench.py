@@ -58,7 +58,7 @@ class ClockSampler:
                0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
                0x100: "display_clock_setting"}
 
-    def __init__(self, index=0, period=0.1):
+    def __init__(self, index=0, period=0.02):
         self.index, self.period = index, period
         self.samples, self.reasons, self.max_mhz = [], set(), None
         self._stop = threading.Event()
@@ -265,97 +265,133 @@ def main():
     value = n_ops / (ms_per_step * 1e-3) / 1e6
 
     # --------------------------------------------------------- roofline
+    # Algorithmic bytes: every probe reads one whole bucket (8*B bytes, the unit
+    # the method compares), every slot write costs one 32-byte sector, plus the
+    # streamed keys/values/status (DESIGN.md §5 "algorithmic bytes per op").
     peak, peak_src = measured_peaks()
     E = s_ins["last_insert_evictions"] / max(1, s_ins["last_insert_new"])
     pend = s_ins["last_insert_pending"]
+    bkt = 8 * args.bucket_slots
     sec = 32
+    probes_find = hit_rate * (1 + phi) + (1 - hit_rate) * 2
+    slots_sub = (cap // 4 // args.bucket_slots + 1) * args.bucket_slots     # slots of one subtable
     bytes_alg = {
-        # find: 1 sector when the key is in its first-choice table, else 2; + key, value, flag
-        "k_find": n * ((hit_rate * (1 + phi) + (1 - hit_rate) * 2) * sec + 9),
+        # find: first-choice bucket, then the second one unless hit; + key, value, flag
+        "k_find": n * (probes_find * bkt + 9),
         # upsert on an empty table: both candidate buckets read (existence check),
         # one sector written for each key placed here; + key, value, status
-        "k_upsert": n * (2 * sec + 9) + (n - pend) * sec,
-        # eviction kernel: per pending key 1 write + 2 sectors per hop (read + exchange)
-        "k_place": pend * sec + s_ins["last_insert_evictions"] * 2 * sec,
-        # delete (all hits): 1+φ reads, 1 write; + key, old value, status
-        "k_delete": (n // 2) * ((1 + phi_after_up) * sec + sec + 9),
-        # upsize: stream the subtable in (8 B/slot) and twice its size out
-        "k_upsize": (cap // 4 // args.bucket_slots + 1) * args.bucket_slots * 24,
-        "k_downsize": (cap // 4 // args.bucket_slots + 1) * args.bucket_slots * 24,
+        "k_upsert": n * (2 * bkt + 9) + (n - pend) * sec,
+        # eviction kernel: per pending key one write; per hop one bucket read + one exchange
+        "k_place": pend * sec + s_ins["last_insert_evictions"] * (bkt + sec),
+        # delete (all hits): 1+φ bucket reads, one sector written; + key, old value, status
+        "k_delete": (n // 2) * ((1 + phi_after_up) * bkt + sec + 9),
+        # upsize: stream the subtable in (8 B/slot) and twice its size out (16 B/slot)
+        "k_upsize": slots_sub * 24,
+        # downsize: stream twice the new size in, the new size out
+        "k_downsize": slots_sub * 12,
     }
     kern = {k: prof[k][0] / args.steps for k in bytes_alg if prof[k][1]}
     dom = max(kern, key=kern.get)
     calls = prof[dom][1] / args.steps
     launch_ms = prof[dom][0] / max(1, prof[dom][1])
     achieved = bytes_alg[dom] / calls / (launch_ms * 1e-3) / 1e9
-    # random 32-byte gather ceiling on a table-sized buffer (same sector count as one find launch)
+    achieved_all = {k: bytes_alg[k] / (kern[k] * 1e-3) / 1e9 for k in kern}
+    # random-bucket ceiling: the probe access pattern alone, on a table-sized buffer
     buf = torch.empty(int(cap * 8 // (1 << 20) + 1) << 20, dtype=torch.uint8, device="cuda")
     sink = torch.zeros(1, dtype=torch.int64, device="cuda")
-    nreads = int(n * (hit_rate * (1 + phi) + (1 - hit_rate) * 2))
+    nreads = int(n * probes_find)
     for _ in range(2):
-        L.check(L.dyc_bench_gather(buf.data_ptr(), buf.numel(), nreads, 32, 7, sink.data_ptr(),
+        L.check(L.dyc_bench_gather(buf.data_ptr(), buf.numel(), nreads, bkt, 7, sink.data_ptr(),
                                    stream.cuda_stream), "dyc_bench_gather")
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)
-    L.check(L.dyc_bench_gather(buf.data_ptr(), buf.numel(), nreads, 32, 9, sink.data_ptr(),
+    L.check(L.dyc_bench_gather(buf.data_ptr(), buf.numel(), nreads, bkt, 9, sink.data_ptr(),
                                stream.cuda_stream), "dyc_bench_gather")
     e1.record(stream)
     torch.cuda.synchronize()
-    gather_gbs = nreads * 32 / (e0.elapsed_time(e1) * 1e-3) / 1e9
+    gather_ms = e0.elapsed_time(e1)
+    gather_gbs = nreads * bkt / (gather_ms * 1e-3) / 1e9
     del buf
     roofline = {
         "bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
         "frac": achieved / peak, "peak_source": peak_src, "traffic": None,
         "algorithmic_bytes_per_launch": bytes_alg[dom] / calls,
         "launch_ms": launch_ms,
-        "random_32B_gather_gbs": gather_gbs, "frac_of_gather_ceiling": achieved / gather_gbs,
+        "achieved_gbs_per_kernel": {k: round(v, 1) for k, v in achieved_all.items()},
+        "random_bucket_ceiling": {"bytes_per_probe": bkt, "gbs": gather_gbs,
+                                  "gprobes_per_s": nreads / (gather_ms * 1e-3) / 1e9,
+                                  "what": "dyc_bench_gather: random bucket reads, probe access pattern only"},
+        "frac_of_random_ceiling": achieved / gather_gbs,
         "kernel_ms_per_step": {k: round(v, 4) for k, v in kern.items()},
-        "model": {"phi": phi, "hit_rate": hit_rate, "evictions_per_insert": E,
-                  "pending_keys": pend, "sector_bytes": sec},
+        "model": {"phi": phi, "hit_rate": hit_rate, "evictions_per_insert": E, "probes_per_find": probes_find,
+                  "pending_keys": pend, "bucket_bytes": bkt, "sector_bytes": sec},
     }
 
     # --------------------------------------------------------- resize baselines
-    resize = {"upsize_ms": phase_ms["upsize"], "downsize_ms": phase_ms["downsize"]}
+    resize = {"upsize_ms": phase_ms["upsize"], "downsize_ms": phase_ms["downsize"],
+              "note": "split = the paper's method (P:L374-395); reinsert_subtable = P:L809 baseline; "
+                      "rehash_all = MegaKV-style double/halve everything (P:L736). *_cold = first run on a "
+                      "fresh table (allocation included), others = second run with the memory pool warm."}
     if not args.no_rehash and not args.profile_only:
         def timed(fn):
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
             a.record(stream)
             fn()
             b.record(stream)
             torch.cuda.synchronize()
             return a.elapsed_time(b)
-        for name, method in (("reinsert_subtable", L.DYC_RESIZE_REINSERT_SUBTABLE),
-                             ("rehash_all", L.DYC_RESIZE_REHASH_ALL)):
-            g2 = Table(d=4, init_capacity=cap, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
-            g2.insert(k_ins, v_ins, st_ins)                                   # θ = 0.85
-            resize[f"{name}_upsize_ms"] = timed(lambda: g2.resize(+1, -1, method))
-            g2.close()
-            del g2
-        # downsize baselines from θ ≈ 0.30: upsize once, fill to 0.30 of N
+
+        def undo(t2, direction, method):
+            t2.clear()
+            t2.resize(-direction, -1, L.DYC_RESIZE_REHASH_ALL if method == L.DYC_RESIZE_REHASH_ALL
+                      else L.DYC_RESIZE_SPLIT)
+
         for name, method in (("split", L.DYC_RESIZE_SPLIT),
                              ("reinsert_subtable", L.DYC_RESIZE_REINSERT_SUBTABLE),
                              ("rehash_all", L.DYC_RESIZE_REHASH_ALL)):
-            g2 = Table(d=4, init_capacity=cap, alpha=0.05, beta=0.85, bucket_slots=args.bucket_slots)
-            g2.resize(+1)
-            m30 = int(0.30 * g2.stats()["N"])
-            g2.insert(k_ins[:m30], v_ins[:m30], st_ins[:m30])
-            resize[f"{name}_downsize_ms_from_fill_0.30"] = timed(lambda: g2.resize(-1, -1, method))
-            g2.close()
-            del g2
-        resize["speedup_upsize_vs_rehash_all"] = resize["rehash_all_upsize_ms"] / resize["upsize_ms"]
+            # upsize one subtable from θ = 0.85: cold (fresh pool), then warm
+            t2 = Table(d=4, init_capacity=cap, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
+            t2.insert(k_ins, v_ins, st_ins)
+            resize[f"{name}_upsize_ms_cold"] = timed(lambda: t2.resize(+1, -1, method))
+            undo(t2, +1, method)
+            t2.insert(k_ins, v_ins, st_ins)
+            resize[f"{name}_upsize_ms"] = timed(lambda: t2.resize(+1, -1, method))
+            t2.close()
+            # downsize from θ = 0.30
+            t2 = Table(d=4, init_capacity=cap, alpha=0.05, beta=0.85, bucket_slots=args.bucket_slots)
+            t2.resize(+1)
+            m30 = int(0.30 * t2.stats()["N"])
+            t2.insert(k_ins[:m30], v_ins[:m30], st_ins[:m30])
+            resize[f"{name}_downsize_ms_cold"] = timed(lambda: t2.resize(-1, -1, method))
+            undo(t2, -1, method)
+            t2.insert(k_ins[:m30], v_ins[:m30], st_ins[:m30])
+            resize[f"{name}_downsize_ms"] = timed(lambda: t2.resize(-1, -1, method))
+            t2.close()
+            del t2
+        resize["speedup_upsize_vs_rehash_all"] = resize["rehash_all_upsize_ms"] / resize["split_upsize_ms"]
+        resize["speedup_upsize_vs_reinsert_subtable"] = (resize["reinsert_subtable_upsize_ms"]
+                                                         / resize["split_upsize_ms"])
+        resize["speedup_downsize_vs_rehash_all"] = resize["rehash_all_downsize_ms"] / resize["split_downsize_ms"]
+        resize["speedup_downsize_vs_reinsert_subtable"] = (resize["reinsert_subtable_downsize_ms"]
+                                                           / resize["split_downsize_ms"])
 
     # --------------------------------------------------------- e2e (host buffers)
     e2e = None
     if not args.no_e2e and not args.profile_only:
         pin = lambda t: t.cpu().pin_memory().numpy().view(np.uint32)  # noqa: E731
         hk, hv, hq, hd = pin(k_ins), pin(v_ins), pin(k_find), pin(k_del)
+        pinned = lambda m, dt: torch.empty(m, dtype=dt, pin_memory=True).numpy()  # noqa: E731
+        o_st = pinned(n, torch.uint8)
+        o_v, o_f = pinned(n, torch.int32).view(np.uint32), pinned(n, torch.uint8)
+        o_dv, o_ds = pinned(n // 2, torch.int32).view(np.uint32), pinned(n // 2, torch.uint8)
 
         def e2e_step():
             g.clear()
-            g.insert_host(hk, hv)
-            g.find_host(hq)
+            g.insert_host(hk, hv, o_st)
+            g.find_host(hq, o_v, o_f)
             g.resize(+1)
-            g.delete_host(hd)
+            g.delete_host(hd, o_dv, o_ds)
             g.resize(-1)
         e2e_step()
         torch.cuda.synchronize()

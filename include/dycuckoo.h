@@ -239,9 +239,11 @@ dyc_status dyc_route_unpermute(const uint32_t* d_pos, uint64_t n, const uint32_t
  * Measurement helpers (bench.py; not part of the method).
  * ------------------------------------------------------------------------- */
 
-/* Random-gather ceiling: `n_reads` reads of `bytes_per_read` (32/64/128)
- * bytes at uniformly random aligned offsets of d_buf[buf_bytes], XOR-reduced
- * into *d_sink.  Bounds what the one-sector-per-probe roofline can reach. */
+/* Random-access ceiling: `n_reads` reads of one bucket of `bytes_per_read`
+ * (32/64/128/256) bytes at uniformly random aligned offsets of d_buf[buf_bytes],
+ * with the probe kernels' access pattern (bytes_per_read/32 lanes, one 256-bit
+ * load each, same L2 prefetch size), XOR-reduced into *d_sink.  Bounds what
+ * the probe kernels can reach. */
 dyc_status dyc_bench_gather(const void* d_buf, uint64_t buf_bytes, uint64_t n_reads,
                             uint32_t bytes_per_read, uint64_t seed, uint64_t* d_sink,
                             dyc_stream_t stream);

@@ -79,6 +79,7 @@ struct dyc_table {
     unsigned long long* h_ctr = nullptr;   // pinned mirror
     void* stage = nullptr;                 // device staging for the host-buffer entry points
     uint64_t stage_cap = 0;
+    cudaStream_t cp_in = nullptr, cp_out = nullptr;   // copy streams of the host-buffer path
     uint64_t n_upsize = 0, n_downsize = 0, n_fail_upsize = 0, n_residual = 0, n_evict = 0, n_place_retry = 0;
     uint64_t launches = 0;
     uint64_t last_new = 0, last_pending = 0, last_evict = 0;
@@ -315,21 +316,37 @@ dyc_status enforce_lower(dyc_table* t, cudaStream_t st) {
     return DYC_OK;
 }
 
+// insert = begin (scratch, counters, FUSE decision) + one k_upsert per chunk of
+// the batch + end (resize decision, placement, failures, alpha loop).  Splitting
+// the upsert into chunks is invisible to the semantics: every chunk only probes,
+// updates and CASes into free slots (or queues to the pending list), and all
+// placement with evictions happens once, in insert_end.
 template <int B>
-dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* status, uint64_t n,
-                       cudaStream_t st) {
+dyc_status insert_begin(dyc_table* t, uint64_t n, cudaStream_t st, bool& fuse) {
     TRY(ensure_lists(t, n, st));
     TRY(zero_ctr(t, st));
-    const bool fuse = (double)(t->m + n) <= t->cfg.beta * (double)t->N();
-    const unsigned grid = grid_for(n, kThreads / (B / 4));
+    fuse = (double)(t->m + n) <= t->cfg.beta * (double)t->N();
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status insert_chunk(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* status, uint64_t n,
+                        bool fuse, cudaStream_t st) {
+    constexpr int U = DYC_UPSERT_U;
+    const unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
     {
         ProfScope ps(t, DYC_PROF_UPSERT, st);
         if (fuse)
-            k_upsert<B, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
+            k_upsert<B, true, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
         else
-            k_upsert<B, false><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
+            k_upsert<B, false, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
     }
     CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
     if (!fuse) {
         // the resize decision needs n_new before any placement (Q11)
         TRY(read_ctr(t, st));
@@ -350,6 +367,15 @@ dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals,
 }
 
 template <int B>
+dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* status, uint64_t n,
+                       cudaStream_t st) {
+    bool fuse = false;
+    TRY(insert_begin<B>(t, n, st, fuse));
+    TRY(insert_chunk<B>(t, keys, vals, status, n, fuse, st));
+    return insert_end<B>(t, fuse, st);
+}
+
+template <int B>
 dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* found, uint64_t n,
                      cudaStream_t st) {
     constexpr int ILP = (B <= 16) ? 4 : 2;
@@ -363,18 +389,161 @@ dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t
 }
 
 template <int B>
-dyc_status delete_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
-                       cudaStream_t st) {
-    TRY(zero_one(t, C_REMOVED, st));
+dyc_status delete_chunk(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
+                        cudaStream_t st) {
     {
         ProfScope ps(t, DYC_PROF_DELETE, st);
-        k_delete<B><<<grid_for(n, kThreads / (B / 4)), kThreads, 0, st>>>(t->view(), keys, vals, status, n,
-                                                                         t->d_ctr);
+        constexpr int U = DYC_DELETE_U;
+        k_delete<B, U><<<grid_for(n, (uint64_t)(kThreads / (B / 4)) * U), kThreads, 0, st>>>(t->view(), keys, vals,
+                                                                                            status, n, t->d_ctr);
     }
     CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status delete_end(dyc_table* t, cudaStream_t st) {
     TRY(read_ctr(t, st));
     t->m -= t->h_ctr[C_REMOVED];
     return enforce_lower<B>(t, st);
+}
+
+template <int B>
+dyc_status delete_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
+                       cudaStream_t st) {
+    TRY(zero_one(t, C_REMOVED, st));
+    TRY(delete_chunk<B>(t, keys, vals, status, n, st));
+    return delete_end<B>(t, st);
+}
+
+// ------------------------------------------------------------------ host-buffer path
+// The batch is staged on the device chunk by chunk: H2D of chunk c+1 (copy-in
+// stream) overlaps the kernel of chunk c (the caller's stream) and the D2H of
+// chunk c-1 (copy-out stream), so PCIe and HBM work concurrently.
+constexpr uint64_t kChunk = 1ull << 22;
+
+struct HostPipe {
+    dyc_table* t;
+    cudaStream_t st;
+    std::vector<cudaEvent_t> evs;
+    cudaEvent_t ev() { evs.push_back(t->ev()); return evs.back(); }
+    ~HostPipe() { for (auto e : evs) t->ev_pool.push_back(e); }
+};
+
+dyc_status ensure_stage(dyc_table* t, uint64_t bytes, cudaStream_t st);
+
+dyc_status ensure_copy_streams(dyc_table* t) {
+    if (!t->cp_in) CU(cudaStreamCreateWithFlags(&t->cp_in, cudaStreamNonBlocking));
+    if (!t->cp_out) CU(cudaStreamCreateWithFlags(&t->cp_out, cudaStreamNonBlocking));
+    return DYC_OK;
+}
+
+// copy `bytes_per_op` x len of each input from host to the staging slices, make st wait
+dyc_status pipe_in(HostPipe& P, void* const* dst, const void* const* src, const uint64_t* esz, int nin,
+                   uint64_t off, uint64_t len) {
+    dyc_table* t = P.t;
+    for (int q = 0; q < nin; q++)
+        CU(cudaMemcpyAsync((char*)dst[q] + off * esz[q], (const char*)src[q] + off * esz[q], len * esz[q],
+                           cudaMemcpyHostToDevice, t->cp_in));
+    cudaEvent_t e = P.ev();
+    CU(cudaEventRecord(e, t->cp_in));
+    CU(cudaStreamWaitEvent(P.st, e, 0));
+    return DYC_OK;
+}
+
+dyc_status pipe_out(HostPipe& P, void* const* dst, const void* const* src, const uint64_t* esz, int nout,
+                    uint64_t off, uint64_t len) {
+    dyc_table* t = P.t;
+    cudaEvent_t e = P.ev();
+    CU(cudaEventRecord(e, P.st));
+    CU(cudaStreamWaitEvent(t->cp_out, e, 0));
+    for (int q = 0; q < nout; q++)
+        if (dst[q])
+            CU(cudaMemcpyAsync((char*)dst[q] + off * esz[q], (const char*)src[q] + off * esz[q], len * esz[q],
+                               cudaMemcpyDeviceToHost, t->cp_out));
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status insert_host_impl(dyc_table* t, const uint32_t* hk, const uint32_t* hv, uint8_t* hs, uint64_t n,
+                            cudaStream_t st) {
+    TRY(ensure_copy_streams(t));
+    TRY(ensure_stage(t, n * 9 + 64, st));
+    uint32_t* k = (uint32_t*)t->stage;
+    uint32_t* v = k + n;
+    uint8_t* s = (uint8_t*)(v + n);
+    HostPipe P{t, st, {}};
+    bool fuse = false;
+    TRY(insert_begin<B>(t, n, st, fuse));
+    for (uint64_t off = 0; off < n; off += kChunk) {
+        const uint64_t len = std::min(kChunk, n - off);
+        void* d_in[2] = {k, v};
+        const void* h_in[2] = {hk, hv};
+        const uint64_t es[2] = {4, 4};
+        TRY(pipe_in(P, d_in, h_in, es, 2, off, len));
+        TRY(insert_chunk<B>(t, k + off, v + off, hs ? s + off : nullptr, len, fuse, st));
+        void* h_out[1] = {hs};
+        const void* d_out[1] = {s};
+        const uint64_t eo[1] = {1};
+        if (hs) TRY(pipe_out(P, h_out, d_out, eo, 1, off, len));
+    }
+    TRY(insert_end<B>(t, fuse, st));
+    CU(cudaStreamSynchronize(t->cp_out));
+    CU(cudaStreamSynchronize(st));
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status find_host_impl(dyc_table* t, const uint32_t* hk, uint32_t* hv, uint8_t* hf, uint64_t n, cudaStream_t st) {
+    TRY(ensure_copy_streams(t));
+    TRY(ensure_stage(t, n * 9 + 64, st));
+    uint32_t* k = (uint32_t*)t->stage;
+    uint32_t* v = k + n;
+    uint8_t* f = (uint8_t*)(v + n);
+    HostPipe P{t, st, {}};
+    for (uint64_t off = 0; off < n; off += kChunk) {
+        const uint64_t len = std::min(kChunk, n - off);
+        void* d_in[1] = {k};
+        const void* h_in[1] = {hk};
+        const uint64_t es[1] = {4};
+        TRY(pipe_in(P, d_in, h_in, es, 1, off, len));
+        TRY(find_impl<B>(t, k + off, v + off, hf ? f + off : nullptr, len, st));
+        void* h_out[2] = {hv, hf};
+        const void* d_out[2] = {v, f};
+        const uint64_t eo[2] = {4, 1};
+        TRY(pipe_out(P, h_out, d_out, eo, 2, off, len));
+    }
+    CU(cudaStreamSynchronize(t->cp_out));
+    CU(cudaStreamSynchronize(st));
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status delete_host_impl(dyc_table* t, const uint32_t* hk, uint32_t* hv, uint8_t* hs, uint64_t n,
+                            cudaStream_t st) {
+    TRY(ensure_copy_streams(t));
+    TRY(ensure_stage(t, n * 9 + 64, st));
+    uint32_t* k = (uint32_t*)t->stage;
+    uint32_t* v = k + n;
+    uint8_t* s = (uint8_t*)(v + n);
+    HostPipe P{t, st, {}};
+    TRY(zero_one(t, C_REMOVED, st));
+    for (uint64_t off = 0; off < n; off += kChunk) {
+        const uint64_t len = std::min(kChunk, n - off);
+        void* d_in[1] = {k};
+        const void* h_in[1] = {hk};
+        const uint64_t es[1] = {4};
+        TRY(pipe_in(P, d_in, h_in, es, 1, off, len));
+        TRY(delete_chunk<B>(t, k + off, hv ? v + off : nullptr, hs ? s + off : nullptr, len, st));
+        void* h_out[2] = {hv, hs};
+        const void* d_out[2] = {v, s};
+        const uint64_t eo[2] = {4, 1};
+        TRY(pipe_out(P, h_out, d_out, eo, 2, off, len));
+    }
+    TRY(delete_end<B>(t, st));
+    CU(cudaStreamSynchronize(t->cp_out));
+    CU(cudaStreamSynchronize(st));
+    return DYC_OK;
 }
 
 // Baselines (measurement only): reinsert one subtable or everything.
@@ -659,6 +828,8 @@ dyc_status dyc_destroy(dyc_table* t) {
     for (int i = 0; i < 2; i++)
         if (t->list[i]) cudaFree(t->list[i]);
     if (t->stage) cudaFree(t->stage);
+    if (t->cp_in) cudaStreamDestroy(t->cp_in);
+    if (t->cp_out) cudaStreamDestroy(t->cp_out);
     if (t->d_ctr) cudaFree(t->d_ctr);
     if (t->h_ctr) cudaFreeHost(t->h_ctr);
     cudaDeviceSynchronize();
@@ -749,51 +920,24 @@ dyc_status dyc_insert_batch_host(dyc_table* t, const uint32_t* h_keys, const uin
                                  uint64_t n, dyc_stream_t stream) {
     TRY(enter(t, stream));
     if (n == 0) return DYC_OK;
-    cudaStream_t st = S(stream);
-    TRY(ensure_stage(t, n * 9 + 64, st));
-    uint32_t* k = (uint32_t*)t->stage;
-    uint32_t* v = k + n;
-    uint8_t* s = (uint8_t*)(v + n);
-    CU(cudaMemcpyAsync(k, h_keys, n * 4, cudaMemcpyHostToDevice, st));
-    CU(cudaMemcpyAsync(v, h_values, n * 4, cudaMemcpyHostToDevice, st));
-    TRY(dyc_insert_batch(t, k, v, h_status ? s : nullptr, n, stream));
-    if (h_status) CU(cudaMemcpyAsync(h_status, s, n, cudaMemcpyDeviceToHost, st));
-    CU(cudaStreamSynchronize(st));
-    return DYC_OK;
+    if (!h_keys || !h_values) return set_err(DYC_ERR_INVALID_ARG, "null keys/values");
+    DISPATCH_B(t, insert_host_impl<B_>(t, h_keys, h_values, h_status, n, S(stream)));
 }
 
 dyc_status dyc_find_batch_host(dyc_table* t, const uint32_t* h_keys, uint32_t* h_values_out, uint8_t* h_found,
                                uint64_t n, dyc_stream_t stream) {
     TRY(enter(t, stream));
     if (n == 0) return DYC_OK;
-    cudaStream_t st = S(stream);
-    TRY(ensure_stage(t, n * 9 + 64, st));
-    uint32_t* k = (uint32_t*)t->stage;
-    uint32_t* v = k + n;
-    uint8_t* f = (uint8_t*)(v + n);
-    CU(cudaMemcpyAsync(k, h_keys, n * 4, cudaMemcpyHostToDevice, st));
-    TRY(dyc_find_batch(t, k, v, h_found ? f : nullptr, n, stream));
-    if (h_values_out) CU(cudaMemcpyAsync(h_values_out, v, n * 4, cudaMemcpyDeviceToHost, st));
-    if (h_found) CU(cudaMemcpyAsync(h_found, f, n, cudaMemcpyDeviceToHost, st));
-    CU(cudaStreamSynchronize(st));
-    return DYC_OK;
+    if (!h_keys || !h_values_out) return set_err(DYC_ERR_INVALID_ARG, "null keys/values_out");
+    DISPATCH_B(t, find_host_impl<B_>(t, h_keys, h_values_out, h_found, n, S(stream)));
 }
 
 dyc_status dyc_delete_batch_host(dyc_table* t, const uint32_t* h_keys, uint32_t* h_values_out, uint8_t* h_status,
                                  uint64_t n, dyc_stream_t stream) {
     TRY(enter(t, stream));
     if (n == 0) return DYC_OK;
-    cudaStream_t st = S(stream);
-    TRY(ensure_stage(t, n * 9 + 64, st));
-    uint32_t* k = (uint32_t*)t->stage;
-    uint32_t* v = k + n;
-    uint8_t* s = (uint8_t*)(v + n);
-    CU(cudaMemcpyAsync(k, h_keys, n * 4, cudaMemcpyHostToDevice, st));
-    TRY(dyc_delete_batch(t, k, h_values_out ? v : nullptr, h_status ? s : nullptr, n, stream));
-    if (h_values_out) CU(cudaMemcpyAsync(h_values_out, v, n * 4, cudaMemcpyDeviceToHost, st));
-    if (h_status) CU(cudaMemcpyAsync(h_status, s, n, cudaMemcpyDeviceToHost, st));
-    CU(cudaStreamSynchronize(st));
-    return DYC_OK;
+    if (!h_keys) return set_err(DYC_ERR_INVALID_ARG, "null keys");
+    DISPATCH_B(t, delete_host_impl<B_>(t, h_keys, h_values_out, h_status, n, S(stream)));
 }
 
 uint64_t dyc_launch_count(const dyc_table* t, int reset) {
@@ -890,17 +1034,21 @@ dyc_status dyc_get_l2_fetch_granularity(uint32_t* bytes) {
 
 dyc_status dyc_bench_gather(const void* d_buf, uint64_t buf_bytes, uint64_t n_reads, uint32_t bytes_per_read,
                             uint64_t seed, uint64_t* d_sink, dyc_stream_t stream) {
-    if (bytes_per_read != 32 && bytes_per_read != 64 && bytes_per_read != 128)
-        return set_err(DYC_ERR_INVALID_ARG, "bytes_per_read must be 32, 64 or 128");
+    if (bytes_per_read != 32 && bytes_per_read != 64 && bytes_per_read != 128 && bytes_per_read != 256)
+        return set_err(DYC_ERR_INVALID_ARG, "bytes_per_read must be 32, 64, 128 or 256");
     const uint64_t units = buf_bytes / bytes_per_read;
     if (units == 0) return set_err(DYC_ERR_INVALID_ARG, "buffer too small");
-    const unsigned grid = grid_for(n_reads, kThreads);
+    const uint64_t lanes_per_read = bytes_per_read / 32;
+    const unsigned grid = grid_for(n_reads * lanes_per_read, (uint64_t)kThreads * 4);
     const unsigned long long* buf = (const unsigned long long*)d_buf;
     unsigned long long* sink = (unsigned long long*)d_sink;
-    switch (bytes_per_read) {
-        case 32: k_gather<1><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
-        case 64: k_gather<2><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
-        default: k_gather<4><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
+    for (uint64_t s_ = 0; s_ < 1; s_++) {
+        switch (bytes_per_read) {
+            case 32: k_gather<4><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
+            case 64: k_gather<8><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
+            case 128: k_gather<16><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
+            default: k_gather<32><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
+        }
     }
     CU(cudaGetLastError());
     return DYC_OK;

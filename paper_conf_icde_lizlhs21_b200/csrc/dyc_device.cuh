@@ -106,32 +106,64 @@ __device__ __forceinline__ unsigned long long make_kv(uint32_t k, uint32_t v) {
 }
 
 // ---------------------------------------------------------------- loads/stores
-// Read-only probe (find): 256-bit non-coherent load, no L1 allocation (no reuse).
+// Each lane reads 4 slots (32 bytes) of its group's bucket with ONE 256-bit load
+// (LDG.E.ENL2.256).  The L2 prefetch-size qualifier is matched to the bucket:
+// without it a miss pulls a whole 128-byte line from HBM (measured: 3.7-3.9
+// DRAM sectors per 32- or 64-byte random request), so 64-byte buckets ask for
+// .L2::64B and halve the HBM bytes per probe.
+template <int B> struct Pf;                      // L2 prefetch size per bucket width
+template <> struct Pf<4>  { static constexpr const char* q = ".L2::64B"; };
+template <> struct Pf<8>  { static constexpr const char* q = ".L2::64B"; };
+template <> struct Pf<16> { static constexpr const char* q = ".L2::128B"; };
+template <> struct Pf<32> { static constexpr const char* q = ".L2::256B"; };
+
+#define DYC_LD4(NAME, COP, PF)                                                                   \
+    __device__ __forceinline__ void NAME(const unsigned long long* p, unsigned long long* s) {    \
+        asm volatile("ld.global" COP PF ".v4.u64 {%0,%1,%2,%3}, [%4];"                            \
+                     : "=l"(s[0]), "=l"(s[1]), "=l"(s[2]), "=l"(s[3]) : "l"(p) : "memory");       \
+    }                                                                                            \
+    __device__ __forceinline__ void NAME##_pred(const unsigned long long* p, unsigned long long* s, \
+                                                bool pred) {                                     \
+        asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %5, 0;\n\t"                          \
+                     "@q ld.global" COP PF ".v4.u64 {%0,%1,%2,%3}, [%4];\n\t}"                  \
+                     : "+l"(s[0]), "+l"(s[1]), "+l"(s[2]), "+l"(s[3])                             \
+                     : "l"(p), "r"((unsigned)pred) : "memory");                                  \
+    }
+
+// read-only probes (find): non-coherent path, no L1 allocation (no reuse)
+DYC_LD4(ld4_nc_64, ".nc.L1::no_allocate", ".L2::64B")
+DYC_LD4(ld4_nc_128, ".nc.L1::no_allocate", ".L2::128B")
+DYC_LD4(ld4_nc_256, ".nc.L1::no_allocate", ".L2::256B")
+// probes in kernels that mutate the table: served by L2 (coherent)
+DYC_LD4(ld4_cg_64, ".cg", ".L2::64B")
+DYC_LD4(ld4_cg_128, ".cg", ".L2::128B")
+DYC_LD4(ld4_cg_256, ".cg", ".L2::256B")
+#undef DYC_LD4
+
+template <int B>
+__device__ __forceinline__ void probe_nc(const unsigned long long* p, unsigned long long* s) {
+    if (B <= 8) ld4_nc_64(p, s); else if (B == 16) ld4_nc_128(p, s); else ld4_nc_256(p, s);
+}
+template <int B>
+__device__ __forceinline__ void probe_nc_pred(const unsigned long long* p, unsigned long long* s, bool q) {
+    if (B <= 8) ld4_nc_64_pred(p, s, q); else if (B == 16) ld4_nc_128_pred(p, s, q); else ld4_nc_256_pred(p, s, q);
+}
+template <int B>
+__device__ __forceinline__ void probe_cg(const unsigned long long* p, unsigned long long* s) {
+    if (B <= 8) ld4_cg_64(p, s); else if (B == 16) ld4_cg_128(p, s); else ld4_cg_256(p, s);
+}
+template <int B>
+__device__ __forceinline__ void probe_cg_pred(const unsigned long long* p, unsigned long long* s, bool q) {
+    if (B <= 8) ld4_cg_64_pred(p, s, q); else if (B == 16) ld4_cg_128_pred(p, s, q); else ld4_cg_256_pred(p, s, q);
+}
+
+// plain 256-bit streaming read (measurement kernels)
 __device__ __forceinline__ void ld4_nc(const unsigned long long* p, unsigned long long* s) {
     asm volatile("ld.global.nc.L1::no_allocate.v4.u64 {%0,%1,%2,%3}, [%4];"
                  : "=l"(s[0]), "=l"(s[1]), "=l"(s[2]), "=l"(s[3]) : "l"(p));
 }
-// Probe in a kernel that mutates the table: 256-bit load served by L2 (coherent).
-__device__ __forceinline__ void ld4_cg(const unsigned long long* p, unsigned long long* s) {
-    asm volatile("ld.global.cg.v4.u64 {%0,%1,%2,%3}, [%4];"
-                 : "=l"(s[0]), "=l"(s[1]), "=l"(s[2]), "=l"(s[3]) : "l"(p) : "memory");
-}
 
-// Predicated variant: when !pred the registers keep their previous contents and
-// no memory request is issued (no branch, so independent probes stay in flight).
-__device__ __forceinline__ void ld4_nc_pred(const unsigned long long* p, unsigned long long* s, bool pred) {
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %5, 0;\n\t"
-                 "@q ld.global.nc.L1::no_allocate.v4.u64 {%0,%1,%2,%3}, [%4];\n\t}"
-                 : "+l"(s[0]), "+l"(s[1]), "+l"(s[2]), "+l"(s[3]) : "l"(p), "r"((unsigned)pred));
-}
-
-template <int B>
-__device__ __forceinline__ void load_bucket_nc_pred(const unsigned long long* p, unsigned long long (&s)[B], bool pred) {
-#pragma unroll
-    for (int j = 0; j < B; j += 4) ld4_nc_pred(p + j, s + j, pred);
-}
-
-// Value of key k in the bucket snapshot (branch-free select chain).
+// Value of key k in a 4-slot snapshot (branch-free select chain).
 template <int B>
 __device__ __forceinline__ bool lookup_slot(const unsigned long long (&s)[B], uint32_t k, uint32_t& v) {
     bool f = false;
@@ -142,17 +174,6 @@ __device__ __forceinline__ bool lookup_slot(const unsigned long long (&s)[B], ui
         f |= h;
     }
     return f;
-}
-
-template <int B>
-__device__ __forceinline__ void load_bucket_nc(const unsigned long long* p, unsigned long long (&s)[B]) {
-#pragma unroll
-    for (int j = 0; j < B; j += 4) ld4_nc(p + j, s + j);
-}
-template <int B>
-__device__ __forceinline__ void load_bucket_cg(const unsigned long long* p, unsigned long long (&s)[B]) {
-#pragma unroll
-    for (int j = 0; j < B; j += 4) ld4_cg(p + j, s + j);
 }
 
 template <int B>

@@ -32,6 +32,12 @@ constexpr int kThreads = 256;
 #ifndef DYC_PLACE_MINB
 #define DYC_PLACE_MINB 1
 #endif
+#ifndef DYC_UPSERT_U
+#define DYC_UPSERT_U 2
+#endif
+#ifndef DYC_DELETE_U
+#define DYC_DELETE_U 2
+#endif
 
 enum CounterIdx : int {
     C_PENDING = 0,    // new keys handed to k_place
@@ -76,12 +82,6 @@ struct Grp {
 };
 
 __device__ __forceinline__ unsigned first_lane(unsigned bits) { return bits ? (unsigned)(__ffs(bits) - 1) : 0u; }
-
-__device__ __forceinline__ void ld4_cg_pred(const unsigned long long* p, unsigned long long* s, bool pred) {
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %5, 0;\n\t"
-                 "@q ld.global.cg.v4.u64 {%0,%1,%2,%3}, [%4];\n\t}"
-                 : "+l"(s[0]), "+l"(s[1]), "+l"(s[2]), "+l"(s[3]) : "l"(p), "r"((unsigned)pred) : "memory");
-}
 
 __device__ __forceinline__ uint32_t mix32(uint32_t x) {
     x ^= x >> 16; x *= 0x7FEB352Du; x ^= x >> 15; x *= 0x846CA68Bu; x ^= x >> 16;
@@ -145,7 +145,7 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
         for (int j = 0; j < ILP; j++) {
             const Pair p = pair_of(tv, k[j]);
             p2[j] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[j]), B) + 4 * g.sub;
-            ld4_nc(bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[j]), B) + 4 * g.sub, s[j]);
+            probe_nc<B>(bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[j]), B) + 4 * g.sub, s[j]);
         }
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
@@ -156,7 +156,7 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
             v[j] = g.bcast32(lv, first_lane(hb));
         }
 #pragma unroll
-        for (int j = 0; j < ILP; j++) ld4_nc_pred(p2[j], s[j], !f[j] && k[j] != kEmptyKey);
+        for (int j = 0; j < ILP; j++) probe_nc_pred<B>(p2[j], s[j], !f[j] && k[j] != kEmptyKey);
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
             uint32_t lv = 0;
@@ -189,10 +189,10 @@ __device__ __forceinline__ bool coop_place(const Grp<B / 4>& g, const TableView&
     unsigned long long s[4] = {kEmptySlot, kEmptySlot, kEmptySlot, kEmptySlot};
     if (first_fit) {
         unsigned long long* b1 = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B);
-        ld4_cg_pred(b1 + 4 * g.sub, s, !done);
+        probe_cg_pred<B>(b1 + 4 * g.sub, s, !done);
         done |= coop_cas_empty(g, b1, s, !done, kv);
         unsigned long long* b2 = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B);
-        ld4_cg_pred(b2 + 4 * g.sub, s, !done);
+        probe_cg_pred<B>(b2 + 4 * g.sub, s, !done);
         done |= coop_cas_empty(g, b2, s, !done, kv);
     }
     uint32_t t = (mix32(k) & 1u) ? p.t2 : p.t1;
@@ -200,7 +200,7 @@ __device__ __forceinline__ bool coop_place(const Grp<B / 4>& g, const TableView&
         if (!__any_sync(kFull, !done)) break;
         unsigned long long* bp = bucket_ptr(sv, t, bucket_of(sv, t, k), B);
         if (hop > 0) {
-            ld4_cg_pred(bp + 4 * g.sub, s, !done);
+            probe_cg_pred<B>(bp + 4 * g.sub, s, !done);
             done |= coop_cas_empty(g, bp, s, !done, kv);
         }
         const uint32_t victim = (mix32(k ^ (hop * 0x9E3779B9u)) >> 8) & (B - 1);
@@ -223,6 +223,48 @@ __device__ __forceinline__ bool coop_place(const Grp<B / 4>& g, const TableView&
     return done;
 }
 
+// First-fit CAS for U independent ops of a group at once: each round, every op
+// that still has a candidate EMPTY slot issues one CAS (all U in flight
+// together), so the atomic round trips of different ops overlap.
+template <int G, int U>
+__device__ __forceinline__ void coop_cas_multi(const Grp<G>& g, unsigned long long* const (&bp)[U],
+                                               const unsigned long long (&s)[U][4], const bool (&want)[U],
+                                               const unsigned long long (&kv)[U], bool (&placed)[U]) {
+    unsigned em[U];
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+        em[u] = 0;
+#pragma unroll
+        for (int j = 0; j < 4; j++)
+            if (s[u][j] == kEmptySlot) em[u] |= 1u << j;
+    }
+    for (;;) {
+        unsigned cand[U];
+        bool any = false;
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            cand[u] = g.ballot(want[u] && !placed[u] && em[u] != 0);
+            any |= cand[u] != 0;
+        }
+        if (!__any_sync(kFull, any)) break;
+        unsigned long long old[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            old[u] = 0;
+            if (cand[u] && g.sub == first_lane(cand[u])) {
+                const unsigned j = __ffs(em[u]) - 1;
+                old[u] = cas_slot(bp[u] + 4 * g.sub + j, kEmptySlot, kv[u]);
+                em[u] &= ~(1u << j);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const unsigned long long o = g.bcast(old[u], first_lane(cand[u]));
+            if (cand[u] && o == kEmptySlot) placed[u] = true;
+        }
+    }
+}
+
 // ------------------------------------------------------ insert phase 1 (S5)
 // Upsert: probe t1's bucket, then t2's; an existing key gets its value replaced
 // (Alg. 1, status UPDATED).  A new key (status INSERTED) is, with FUSE,
@@ -230,7 +272,9 @@ __device__ __forceinline__ bool coop_place(const Grp<B / 4>& g, const TableView&
 // both candidate buckets are full) it is appended to `pending` for k_place.
 // Keys never move during this kernel (no evictions), so the existence check is
 // exact; FUSE is only used when no upsize can be needed ((m+n) <= beta*N).
-template <int B, bool FUSE>
+// Each group carries U ops whose probes are issued together (memory-level
+// parallelism: the kernel is bound by random line requests).
+template <int B, bool FUSE, int U>
 __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView tv, const uint32_t* __restrict__ keys,
                                                      const uint32_t* __restrict__ vals,
                                                      uint8_t* __restrict__ status, uint64_t n,
@@ -244,38 +288,58 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     unsigned long long n_ins = 0, n_upd = 0;
-    for (uint64_t base = w * QPW; base < n; base += nwarps * QPW) {
-        const uint64_t i = base + grp;
-        const bool valid = i < n;
-        const uint32_t k = valid ? __ldg(keys + i) : kEmptyKey;
-        const uint32_t v = valid ? __ldg(vals + i) : 0u;
-        const unsigned long long kv = make_kv(k, v);
-        const bool active = k != kEmptyKey;
-        const Pair p = pair_of(tv, k);
-        unsigned long long* b1 = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B);
-        unsigned long long* b2 = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B);
-        unsigned long long s1[4], s2[4] = {kEmptySlot, kEmptySlot, kEmptySlot, kEmptySlot};
-        ld4_cg(b1 + 4 * g.sub, s1);
-        const int j1 = match_slot<4>(s1, k);
-        const unsigned h1 = g.ballot(active && j1 >= 0);
-        const bool need2 = active && h1 == 0;
-        ld4_cg_pred(b2 + 4 * g.sub, s2, need2);
-        const int j2 = match_slot<4>(s2, k);
-        const unsigned h2 = g.ballot(need2 && j2 >= 0);
-        if (h1 && g.sub == first_lane(h1)) st_u64_cg(b1 + 4 * g.sub + j1, kv);
-        if (h2 && g.sub == first_lane(h2)) st_u64_cg(b2 + 4 * g.sub + j2, kv);
-        const bool isnew = need2 && h2 == 0;
-        bool placed = false;
-        if (FUSE) {
-            placed = coop_cas_empty(g, b1, s1, isnew, kv);
-            placed |= coop_cas_empty(g, b2, s2, isnew && !placed, kv);
+    for (uint64_t base = w * (QPW * U); base < n; base += nwarps * (QPW * U)) {
+        uint64_t i[U];
+        uint32_t k[U];
+        unsigned long long kv[U], s1[U][4], s2[U][4];
+        unsigned long long* b1[U];
+        unsigned long long* b2[U];
+        unsigned h1[U], h2[U];
+        bool need2[U], isnew[U], placed[U];
+        int j1[U], j2[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            i[u] = base + (uint64_t)u * QPW + grp;
+            const bool valid = i[u] < n;
+            k[u] = valid ? __ldg(keys + i[u]) : kEmptyKey;
+            kv[u] = make_kv(k[u], valid ? __ldg(vals + i[u]) : 0u);
+            const Pair p = pair_of(tv, k[u]);
+            b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
+            b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
+            probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
         }
-        const uint8_t st = !active ? 0 : ((h1 | h2) ? 2 : 1);
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const bool active = k[u] != kEmptyKey;
+            j1[u] = match_slot<4>(s1[u], k[u]);
+            h1[u] = g.ballot(active && j1[u] >= 0);
+            need2[u] = active && h1[u] == 0;
+#pragma unroll
+            for (int q = 0; q < 4; q++) s2[u][q] = kEmptySlot;
+            probe_cg_pred<B>(b2[u] + 4 * g.sub, s2[u], need2[u]);
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            j2[u] = match_slot<4>(s2[u], k[u]);
+            h2[u] = g.ballot(need2[u] && j2[u] >= 0);
+            if (h1[u] && g.sub == first_lane(h1[u])) st_u64_cg(b1[u] + 4 * g.sub + j1[u], kv[u]);
+            if (h2[u] && g.sub == first_lane(h2[u])) st_u64_cg(b2[u] + 4 * g.sub + j2[u], kv[u]);
+            isnew[u] = need2[u] && h2[u] == 0;
+            placed[u] = false;
+        }
+        if (FUSE) {
+            coop_cas_multi<G, U>(g, b1, s1, isnew, kv, placed);
+            coop_cas_multi<G, U>(g, b2, s2, isnew, kv, placed);
+        }
         const bool lead = g.sub == 0;
-        if (lead && valid && status) status[i] = st;
-        warp_append(lead && isnew && !placed, kv, pending, ctr + C_PENDING);
-        n_ins += lead && st == 1;
-        n_upd += lead && st == 2;
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const uint8_t st = k[u] == kEmptyKey ? 0 : ((h1[u] | h2[u]) ? 2 : 1);
+            if (lead && i[u] < n && status) status[i[u]] = st;
+            warp_append(lead && isnew[u] && !placed[u], kv[u], pending, ctr + C_PENDING);
+            n_ins += lead && st == 1;
+            n_upd += lead && st == 2;
+        }
     }
     block_add<kThreads>(ctr + C_INSERTED, n_ins);
     block_add<kThreads>(ctr + C_UPDATED, n_upd);
@@ -333,7 +397,9 @@ __global__ void __launch_bounds__(kThreads) k_reinsert(TableView tv, const unsig
 }
 
 // ------------------------------------------------------------- delete (S4)
-template <int B>
+// Probe t1 then t2; the lane holding the key overwrites its slot with EMPTY (no
+// lock: keys in a batch are distinct).  U ops per group in flight.
+template <int B, int U>
 __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView tv, const uint32_t* __restrict__ keys,
                                                      uint32_t* __restrict__ old_vals,
                                                      uint8_t* __restrict__ status, uint64_t n,
@@ -346,35 +412,52 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     unsigned long long removed = 0;
-    for (uint64_t base = w * QPW; base < n; base += nwarps * QPW) {
-        const uint64_t i = base + grp;
-        const bool valid = i < n;
-        const uint32_t k = valid ? __ldg(keys + i) : kEmptyKey;
-        const bool active = k != kEmptyKey;
-        const Pair p = pair_of(tv, k);
-        unsigned long long* b1 = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B);
-        unsigned long long* b2 = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B);
-        unsigned long long s1[4], s2[4] = {kEmptySlot, kEmptySlot, kEmptySlot, kEmptySlot};
-        ld4_cg(b1 + 4 * g.sub, s1);
-        uint32_t lv1 = 0, lv2 = 0;
-        const int j1 = active ? match_slot<4>(s1, k) : -1;
-        lookup_slot<4>(s1, k, lv1);
-        const unsigned h1 = g.ballot(j1 >= 0);
-        const bool need2 = active && h1 == 0;
-        ld4_cg_pred(b2 + 4 * g.sub, s2, need2);
-        const int j2 = need2 ? match_slot<4>(s2, k) : -1;
-        lookup_slot<4>(s2, k, lv2);
-        const unsigned h2 = g.ballot(j2 >= 0);
-        if (h1 && g.sub == first_lane(h1)) st_u64_cg(b1 + 4 * g.sub + j1, kEmptySlot);
-        if (h2 && g.sub == first_lane(h2)) st_u64_cg(b2 + 4 * g.sub + j2, kEmptySlot);
-        const uint32_t o1 = g.bcast32(lv1, first_lane(h1));
-        const uint32_t o2 = g.bcast32(lv2, first_lane(h2));
-        const bool hit = (h1 | h2) != 0;
-        if (g.sub == 0 && valid) {
-            if (old_vals) old_vals[i] = h1 ? o1 : (h2 ? o2 : kEmptyKey);
-            if (status) status[i] = hit ? 1 : 0;
+    for (uint64_t base = w * (QPW * U); base < n; base += nwarps * (QPW * U)) {
+        uint64_t i[U];
+        uint32_t k[U];
+        unsigned long long s1[U][4], s2[U][4];
+        unsigned long long* b1[U];
+        unsigned long long* b2[U];
+        unsigned h1[U];
+        bool need2[U];
+        int j1[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            i[u] = base + (uint64_t)u * QPW + grp;
+            k[u] = i[u] < n ? __ldg(keys + i[u]) : kEmptyKey;
+            const Pair p = pair_of(tv, k[u]);
+            b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
+            b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
+            probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
         }
-        removed += (g.sub == 0 && hit);
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const bool active = k[u] != kEmptyKey;
+            j1[u] = active ? match_slot<4>(s1[u], k[u]) : -1;
+            h1[u] = g.ballot(j1[u] >= 0);
+            need2[u] = active && h1[u] == 0;
+#pragma unroll
+            for (int q = 0; q < 4; q++) s2[u][q] = kEmptySlot;
+            probe_cg_pred<B>(b2[u] + 4 * g.sub, s2[u], need2[u]);
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            uint32_t lv1 = 0, lv2 = 0;
+            lookup_slot<4>(s1[u], k[u], lv1);
+            lookup_slot<4>(s2[u], k[u], lv2);
+            const int j2 = need2[u] ? match_slot<4>(s2[u], k[u]) : -1;
+            const unsigned h2 = g.ballot(j2 >= 0);
+            if (h1[u] && g.sub == first_lane(h1[u])) st_u64_cg(b1[u] + 4 * g.sub + j1[u], kEmptySlot);
+            if (h2 && g.sub == first_lane(h2)) st_u64_cg(b2[u] + 4 * g.sub + j2, kEmptySlot);
+            const uint32_t o1 = g.bcast32(lv1, first_lane(h1[u]));
+            const uint32_t o2 = g.bcast32(lv2, first_lane(h2));
+            const bool hit = (h1[u] | h2) != 0;
+            if (g.sub == 0 && i[u] < n) {
+                if (old_vals) old_vals[i[u]] = h1[u] ? o1 : (h2 ? o2 : kEmptyKey);
+                if (status) status[i[u]] = hit ? 1 : 0;
+            }
+            removed += (g.sub == 0 && hit);
+        }
     }
     block_add<kThreads>(ctr + C_REMOVED, removed);
 }
@@ -560,24 +643,34 @@ __global__ void __launch_bounds__(kThreads) k_route_unpermute(const uint32_t* __
 }
 
 // ------------------------------------------------------ random-gather ceiling
-template <int NSEC>
+// The probe access pattern with no table logic: reads of one B-slot bucket at
+// uniformly random bucket-aligned offsets, by a G = B/4 lane group with the same
+// 256-bit loads and L2 prefetch size as k_find.  Its rate is the random-access
+// ceiling the probe kernels are compared with.
+template <int B>
 __global__ void __launch_bounds__(kThreads) k_gather(const unsigned long long* __restrict__ buf, uint64_t n_units,
                                                      uint64_t n_reads, uint64_t seed,
                                                      unsigned long long* __restrict__ sink) {
+    constexpr int G = B / 4, QPW = 32 / G, ILP = 4;
+    const Grp<G> g;
+    const unsigned grp = g.lane / G;
+    const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
+    const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     unsigned long long acc = 0;
-    for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n_reads; i += (uint64_t)gridDim.x * kThreads) {
-        uint64_t h = (i + seed) * 0x9E3779B97F4A7C15ull;
-        h ^= h >> 29;
-        h *= 0xBF58476D1CE4E5B9ull;
-        h ^= h >> 32;
-        const uint64_t u = __umul64hi(h, n_units);
-        const unsigned long long* p = buf + u * (NSEC * 4);
+    for (uint64_t base = w * QPW * ILP; base < n_reads; base += nwarps * QPW * ILP) {
+        unsigned long long s[ILP][4];
 #pragma unroll
-        for (int q = 0; q < NSEC; q++) {
-            unsigned long long s[4];
-            ld4_nc(p + 4 * q, s);
-            acc ^= s[0] ^ s[1] ^ s[2] ^ s[3];
+        for (int j = 0; j < ILP; j++) {
+            const uint64_t i = base + (uint64_t)j * QPW + grp;
+            uint64_t h = (i + seed) * 0x9E3779B97F4A7C15ull;
+            h ^= h >> 29;
+            h *= 0xBF58476D1CE4E5B9ull;
+            h ^= h >> 32;
+            const unsigned long long* p = buf + __umul64hi(h, n_units) * B + 4 * g.sub;
+            probe_nc_pred<B>(p, s[j], i < n_reads);
         }
+#pragma unroll
+        for (int j = 0; j < ILP; j++) acc ^= s[j][0] ^ s[j][1] ^ s[j][2] ^ s[j][3];
     }
     if (acc == 0x0123456789ABCDEFull) *sink = acc;   // keeps the loads alive
 }

@@ -116,27 +116,32 @@ class Table:
                 "dyc_delete_batch")
         return values_out, status
 
-    # host-buffer entry points (end-to-end path: copies inside the call)
-    def insert_host(self, keys: np.ndarray, values: np.ndarray, stream=None) -> np.ndarray:
+    # host-buffer entry points (end-to-end path: copies inside the call, chunked
+    # so PCIe transfers overlap the kernels).  Output arrays may be supplied
+    # (e.g. pinned numpy views) to avoid pageable-memory copies.
+    def insert_host(self, keys: np.ndarray, values: np.ndarray, status: Optional[np.ndarray] = None,
+                    stream=None) -> np.ndarray:
         keys = np.ascontiguousarray(keys, dtype=np.uint32)
         values = np.ascontiguousarray(values, dtype=np.uint32)
-        st = np.empty(keys.size, dtype=np.uint8)
+        st = np.empty(keys.size, dtype=np.uint8) if status is None else status
         L.check(self._lib.dyc_insert_batch_host(self._h, keys.ctypes.data, values.ctypes.data, st.ctypes.data,
                                                 keys.size, _stream_ptr(stream)), "dyc_insert_batch_host")
         return st
 
-    def find_host(self, keys: np.ndarray, stream=None) -> Tuple[np.ndarray, np.ndarray]:
+    def find_host(self, keys: np.ndarray, values_out: Optional[np.ndarray] = None,
+                  found: Optional[np.ndarray] = None, stream=None) -> Tuple[np.ndarray, np.ndarray]:
         keys = np.ascontiguousarray(keys, dtype=np.uint32)
-        v = np.empty(keys.size, dtype=np.uint32)
-        f = np.empty(keys.size, dtype=np.uint8)
+        v = np.empty(keys.size, dtype=np.uint32) if values_out is None else values_out
+        f = np.empty(keys.size, dtype=np.uint8) if found is None else found
         L.check(self._lib.dyc_find_batch_host(self._h, keys.ctypes.data, v.ctypes.data, f.ctypes.data,
                                               keys.size, _stream_ptr(stream)), "dyc_find_batch_host")
         return v, f
 
-    def delete_host(self, keys: np.ndarray, stream=None) -> Tuple[np.ndarray, np.ndarray]:
+    def delete_host(self, keys: np.ndarray, values_out: Optional[np.ndarray] = None,
+                    status: Optional[np.ndarray] = None, stream=None) -> Tuple[np.ndarray, np.ndarray]:
         keys = np.ascontiguousarray(keys, dtype=np.uint32)
-        v = np.empty(keys.size, dtype=np.uint32)
-        s = np.empty(keys.size, dtype=np.uint8)
+        v = np.empty(keys.size, dtype=np.uint32) if values_out is None else values_out
+        s = np.empty(keys.size, dtype=np.uint8) if status is None else status
         L.check(self._lib.dyc_delete_batch_host(self._h, keys.ctypes.data, v.ctypes.data, s.ctypes.data,
                                                 keys.size, _stream_ptr(stream)), "dyc_delete_batch_host")
         return v, s

@@ -264,6 +264,31 @@ def test_host_entry_points_match_device(oracle_mod):
     np.testing.assert_array_equal(g.sorted_kv(), o.sorted_kv())
 
 
+def test_host_entry_points_chunked(oracle_mod):
+    """The host-buffer path pipelines 2^22-op chunks: a batch spanning several
+    chunks with a ragged tail gives the oracle's results."""
+    n = (1 << 22) * 2 + 12345
+    keys = W.key_range(0, n, 321)
+    vals = W.val_of(keys, 0)
+    g = Table(d=4, init_capacity=int(n / 0.8), alpha=0.3, beta=0.85, bucket_slots=8)
+    o = oracle_mod.OracleTable(d=4, init_capacity=int(n / 0.8), alpha=0.3, beta=0.85, bucket_slots=8)
+    np.testing.assert_array_equal(g.insert_host(keys, vals), o.insert(keys, vals))
+    upd = keys[::3].copy()
+    np.testing.assert_array_equal(g.insert_host(upd, W.val_of(upd, 1)), o.insert(upd, W.val_of(upd, 1)))
+    q = np.concatenate([keys[::2], W.key_range(1 << 31, n // 2, 321)])
+    v, f = g.find_host(q)
+    ov, of = o.find(q)
+    np.testing.assert_array_equal(f, of)
+    np.testing.assert_array_equal(v, ov)
+    dk = keys[1::2].copy()
+    v, s = g.delete_host(dk)
+    ov, os_ = o.delete(dk)
+    np.testing.assert_array_equal(s, os_)
+    np.testing.assert_array_equal(v, ov)
+    np.testing.assert_array_equal(g.sorted_kv(), o.sorted_kv())
+    assert g.stats()["buckets"] == o.stats()["buckets"]
+
+
 # ------------------------------------------------------------------ full size (C2)
 @pytest.mark.slow
 def test_c2_full_size_sampled():
