@@ -77,7 +77,7 @@ def test_library_is_sm100a(lib):
     out = subprocess.run([cuobjdump, "-lelf", L.LIB], capture_output=True, text=True).stdout
     assert "sm_100a" in out
     sass = subprocess.run([cuobjdump, "-sass", L.LIB], capture_output=True, text=True).stdout
-    assert "LDG.E.NA.ENL2.256" in sass      # one 256-bit load per 32-byte bucket probe
+    assert re.search(r"LDG\.E\.NA\.ENL2\.LTC64B\.256", sass)   # 256-bit probe loads, 64-byte L2 prefetch
     assert "ATOMG.E.CAS.64" in sass and "ATOMG.E.EXCH.64" in sass
 
 
