@@ -312,9 +312,16 @@ def main():
     gather_ms = e0.elapsed_time(e1)
     gather_gbs = nreads * bkt / (gather_ms * 1e-3) / 1e9
     del buf
+    traffic, traffic_src = None, None
+    tr_files = sorted(f for f in os.listdir(os.path.join(ROOT, "profiles")) if f.endswith("_traffic.json")) \
+        if os.path.isdir(os.path.join(ROOT, "profiles")) else []
+    if tr_files and args.log2n == 27 and args.bucket_slots == 8:
+        tr = json.load(open(os.path.join(ROOT, "profiles", tr_files[-1])))
+        if dom in tr:
+            traffic, traffic_src = tr[dom], f"profiles/{tr_files[-1]} (ncu --set full, dram read+write per launch)"
     roofline = {
         "bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
-        "frac": achieved / peak, "peak_source": peak_src, "traffic": None,
+        "frac": achieved / peak, "peak_source": peak_src, "traffic": traffic, "traffic_source": traffic_src,
         "algorithmic_bytes_per_launch": bytes_alg[dom] / calls,
         "launch_ms": launch_ms,
         "achieved_gbs_per_kernel": {k: round(v, 1) for k, v in achieved_all.items()},

@@ -147,6 +147,20 @@ dyc_status dyc_find_batch(dyc_table* t, const uint32_t* d_keys, uint32_t* d_valu
 dyc_status dyc_delete_batch(dyc_table* t, const uint32_t* d_keys, uint32_t* d_values_out,
                             uint8_t* d_status, uint64_t n, dyc_stream_t stream);
 
+/* Mixed batch (configs C4/C5): op i is d_ops[i] in {DYC_MIX_FIND, DYC_MIX_INSERT,
+ * DYC_MIX_DELETE}.  The paper batches one op type at a time and calls
+ * mixed batches ambiguous (commented); reading Q10: keys are distinct
+ * across the whole batch and the phases run find -> insert -> delete, so finds
+ * observe the table before the batch.  The ops are grouped by type on the
+ * device, run as three single-type batches, and the results returned in request
+ * order: d_values_out[i] (nullable) = found / removed value, DYC_NOT_FOUND on a
+ * miss and for inserts; d_status[i] (nullable) = the op's status code.
+ * Synchronizes `stream` (the phase sizes are needed on the host). */
+enum { DYC_MIX_FIND = 0, DYC_MIX_INSERT = 1, DYC_MIX_DELETE = 2 };
+dyc_status dyc_mixed_batch(dyc_table* t, const uint8_t* d_ops, const uint32_t* d_keys,
+                           const uint32_t* d_values, uint32_t* d_values_out, uint8_t* d_status,
+                           uint64_t n, dyc_stream_t stream);
+
 /* Explicit resize of one subtable (§IV-B; kernels P:L374-395).
  * direction +1: double subtable `subtable` (-1 = the smallest, ties lowest index);
  * direction -1: halve it (-1 = the largest, ties highest index; refused if its
@@ -219,13 +233,16 @@ dyc_status dyc_profile_read(dyc_table* t, double* ms, uint64_t* calls);
 dyc_status dyc_route_count(dyc_table* t, const uint32_t* d_keys, uint64_t n, uint32_t world,
                            uint64_t* d_counts, dyc_stream_t stream);
 
-/* Scatters op i to position d_offsets[dest] + rank-within-dest of the send
- * buffers (grouped by destination).  d_offsets[world] (uint64, device) holds the
- * exclusive prefix sum of the counts and is consumed as cursors.  d_vals_in and
- * d_vals_out may be NULL (finds/deletes).  d_pos[i] (uint32) receives op i's
- * position in the send buffer, for dyc_route_unpermute. */
+/* Groups the ops by destination shard: op i goes to position
+ * offset[dest] + (rank of i among ops bound to dest) of d_keys_out / d_vals_out,
+ * where offset is the exclusive prefix sum of d_counts[world] (the histogram
+ * from dyc_route_count, computed on the device here).  d_cursor[world]
+ * (uint64, device) is scratch.  d_vals_in and d_vals_out may be NULL
+ * (finds/deletes).  d_pos[i] (uint32) receives op i's position in the send
+ * buffer, for dyc_route_unpermute.  Positions within one destination are in
+ * unspecified order. */
 dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_vals_in,
-                             uint64_t n, uint32_t world, uint64_t* d_offsets,
+                             uint64_t n, uint32_t world, const uint64_t* d_counts, uint64_t* d_cursor,
                              uint32_t* d_keys_out, uint32_t* d_vals_out, uint32_t* d_pos,
                              dyc_stream_t stream);
 

@@ -59,6 +59,7 @@ SIGNATURES = {
     "dyc_insert_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
     "dyc_find_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
     "dyc_delete_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
+    "dyc_mixed_batch": (_I, [_TP, _P, _P, _P, _P, _P, _U64, _P]),
     "dyc_resize": (_I, [_TP, _I, _I, _P]),
     "dyc_resize_ex": (_I, [_TP, _I, _I, _I, _P]),
     "dyc_clear": (_I, [_TP, _P]),
@@ -73,7 +74,7 @@ SIGNATURES = {
     "dyc_profile_enable": (_I, [_TP, _I]),
     "dyc_profile_read": (_I, [_TP, _P, _P]),
     "dyc_route_count": (_I, [_TP, _P, _U64, _U32, _P, _P]),
-    "dyc_route_scatter": (_I, [_TP, _P, _P, _U64, _U32, _P, _P, _P, _P, _P]),
+    "dyc_route_scatter": (_I, [_TP, _P, _P, _U64, _U32, _P, _P, _P, _P, _P, _P]),
     "dyc_route_unpermute": (_I, [_P, _U64, _P, _P, _P, _P, _P]),
     "dyc_bench_gather": (_I, [_P, _U64, _U64, _U32, _U64, _P, _P]),
     "dyc_set_l2_fetch_granularity": (_I, [_U32]),

@@ -80,6 +80,8 @@ struct dyc_table {
     void* stage = nullptr;                 // device staging for the host-buffer entry points
     uint64_t stage_cap = 0;
     cudaStream_t cp_in = nullptr, cp_out = nullptr;   // copy streams of the host-buffer path
+    void* mix = nullptr;                   // scratch of dyc_mixed_batch
+    uint64_t mix_cap = 0;
     uint64_t n_upsize = 0, n_downsize = 0, n_fail_upsize = 0, n_residual = 0, n_evict = 0, n_place_retry = 0;
     uint64_t launches = 0;
     uint64_t last_new = 0, last_pending = 0, last_evict = 0;
@@ -828,6 +830,7 @@ dyc_status dyc_destroy(dyc_table* t) {
     for (int i = 0; i < 2; i++)
         if (t->list[i]) cudaFree(t->list[i]);
     if (t->stage) cudaFree(t->stage);
+    if (t->mix) cudaFree(t->mix);
     if (t->cp_in) cudaStreamDestroy(t->cp_in);
     if (t->cp_out) cudaStreamDestroy(t->cp_out);
     if (t->d_ctr) cudaFree(t->d_ctr);
@@ -862,6 +865,53 @@ dyc_status dyc_delete_batch(dyc_table* t, const uint32_t* d_keys, uint32_t* d_va
     if (n == 0) return DYC_OK;
     if (!d_keys) return set_err(DYC_ERR_INVALID_ARG, "null keys");
     DISPATCH_B(t, delete_impl<B_>(t, d_keys, d_values_out, d_status, n, S(stream)));
+}
+
+dyc_status dyc_mixed_batch(dyc_table* t, const uint8_t* d_ops, const uint32_t* d_keys, const uint32_t* d_values,
+                           uint32_t* d_values_out, uint8_t* d_status, uint64_t n, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (n == 0) return DYC_OK;
+    if (!d_ops || !d_keys) return set_err(DYC_ERR_INVALID_ARG, "null ops/keys");
+    if (n > 0xFFFFFFFFull) return set_err(DYC_ERR_INVALID_ARG, "mixed batch must be < 2^32 ops");
+    cudaStream_t st = S(stream);
+    // scratch: keys, values, out values (u32 x n each), pos (u32 x n), status (u8 x n), 8 counters
+    const uint64_t need = n * 17 + 128;
+    if (need > t->mix_cap) {
+        if (t->mix) CU(cudaFreeAsync(t->mix, st));
+        t->mix = nullptr;
+        t->mix_cap = 0;
+        TRY(dev_alloc(t, &t->mix, need, st));
+        t->mix_cap = need;
+    }
+    unsigned long long* cnt = (unsigned long long*)t->mix;      // [0..4) counts, [4..8) cursors
+    uint32_t* k = (uint32_t*)(cnt + 8);
+    uint32_t* v = k + n;
+    uint32_t* ov = v + n;
+    uint32_t* pos = ov + n;
+    uint8_t* sts = (uint8_t*)(pos + n);
+    CU(cudaMemsetAsync(cnt, 0, 8 * 8, st));
+    {
+        ProfScope ps(t, DYC_PROF_OTHER, st);
+        k_op_count<<<std::min<unsigned>(grid_for(n, kThreads), t->num_sms * 8), kThreads, 0, st>>>(d_ops, n, cnt);
+        k_route_offsets<<<1, 32, 0, st>>>(cnt, 4, cnt + 4);
+        k_op_scatter<<<grid_for(n, kThreads), kThreads, 0, st>>>(d_ops, d_keys, d_values, n, cnt + 4, k, v, pos);
+    }
+    CU(cudaGetLastError());
+    unsigned long long h[4];
+    CU(cudaMemcpyAsync(h, cnt, sizeof(h), cudaMemcpyDeviceToHost, st));
+    CU(cudaStreamSynchronize(st));
+    if (h[3]) return set_err(DYC_ERR_INVALID_ARG, "op codes must be 0 (find), 1 (insert) or 2 (delete)");
+    const uint64_t nf = h[0], ni = h[1], nd = h[2];
+    // phases: find -> insert -> delete (Q10)
+    if (nf) TRY(dyc_find_batch(t, k, ov, sts, nf, stream));
+    if (ni) {
+        TRY(dyc_insert_batch(t, k + nf, v + nf, sts + nf, ni, stream));
+        CU(cudaMemsetAsync(ov + nf, 0xFF, ni * 4, st));
+    }
+    if (nd) TRY(dyc_delete_batch(t, k + nf + ni, ov + nf + ni, sts + nf + ni, nd, stream));
+    TRY(dyc_route_unpermute(pos, n, d_values_out ? ov : nullptr, d_status ? sts : nullptr, d_values_out, d_status,
+                            stream));
+    return DYC_OK;
 }
 
 dyc_status dyc_resize_ex(dyc_table* t, int direction, int subtable, int method, dyc_stream_t stream) {
@@ -992,8 +1042,8 @@ dyc_status dyc_route_count(dyc_table* t, const uint32_t* d_keys, uint64_t n, uin
 }
 
 dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_vals_in, uint64_t n,
-                             uint32_t world, uint64_t* d_offsets, uint32_t* d_keys_out, uint32_t* d_vals_out,
-                             uint32_t* d_pos, dyc_stream_t stream) {
+                             uint32_t world, const uint64_t* d_counts, uint64_t* d_cursor, uint32_t* d_keys_out,
+                             uint32_t* d_vals_out, uint32_t* d_pos, dyc_stream_t stream) {
     TRY(enter(t, stream));
     if (world < 1 || world > 4096) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..4096");
     if (n == 0) return DYC_OK;
@@ -1001,8 +1051,13 @@ dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_
     const uint32_t sh = t->cfg.d + 1;
     {
         ProfScope ps(t, DYC_PROF_OTHER, S(stream));
+        k_route_offsets<<<1, 32, 0, S(stream)>>>((const unsigned long long*)d_counts, world,
+                                                 (unsigned long long*)d_cursor);
+    }
+    {
+        ProfScope ps(t, DYC_PROF_OTHER, S(stream));
         k_route_scatter<<<grid_for(n, kThreads), kThreads, 0, S(stream)>>>(
-            t->a[sh], t->b[sh], fastmod_magic(world), world, d_keys, d_vals_in, n, (unsigned long long*)d_offsets,
+            t->a[sh], t->b[sh], fastmod_magic(world), world, d_keys, d_vals_in, n, (unsigned long long*)d_cursor,
             d_keys_out, d_vals_out, d_pos);
     }
     CU(cudaGetLastError());

@@ -603,6 +603,55 @@ __global__ void __launch_bounds__(kThreads) k_route_count(uint32_t a, uint32_t b
         if (hist[w]) atomicAdd(&counts[w], hist[w]);
 }
 
+// Mixed batches: histogram and grouping by op code (3 "destinations").
+__global__ void __launch_bounds__(kThreads) k_op_count(const uint8_t* __restrict__ ops, uint64_t n,
+                                                       unsigned long long* __restrict__ counts) {
+    __shared__ unsigned long long hist[4];
+    if (threadIdx.x < 4) hist[threadIdx.x] = 0;
+    __syncthreads();
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        atomicAdd(&hist[ops[i] & 3], 1ull);
+    __syncthreads();
+    if (threadIdx.x < 4 && hist[threadIdx.x]) atomicAdd(&counts[threadIdx.x], hist[threadIdx.x]);
+}
+
+__global__ void __launch_bounds__(kThreads) k_op_scatter(const uint8_t* __restrict__ ops,
+                                                         const uint32_t* __restrict__ keys,
+                                                         const uint32_t* __restrict__ vals_in, uint64_t n,
+                                                         unsigned long long* __restrict__ cursor,
+                                                         uint32_t* __restrict__ keys_out,
+                                                         uint32_t* __restrict__ vals_out,
+                                                         uint32_t* __restrict__ pos_out) {
+    for (uint64_t base = (uint64_t)blockIdx.x * blockDim.x; base < n; base += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t i = base + threadIdx.x;
+        const bool valid = i < n;
+        const uint32_t dest = valid ? (ops[i] & 3u) : 0xFFFFFFFFu;
+        const unsigned peers = __match_any_sync(kFull, dest);
+        const int leader = __ffs(peers) - 1;
+        unsigned long long p0 = 0;
+        if (valid && (int)(threadIdx.x & 31) == leader) p0 = atomicAdd(&cursor[dest], (unsigned long long)__popc(peers));
+        p0 = __shfl_sync(kFull, p0, leader);
+        if (valid) {
+            const uint64_t pos = p0 + __popc(peers & lanemask_lt());
+            keys_out[pos] = keys[i];
+            vals_out[pos] = vals_in ? vals_in[i] : 0u;
+            pos_out[i] = (uint32_t)pos;
+        }
+    }
+}
+
+// Exclusive prefix sum of the per-shard counts into the scatter cursors (one block).
+__global__ void k_route_offsets(const unsigned long long* __restrict__ counts, uint32_t world,
+                                unsigned long long* __restrict__ cursor) {
+    if (threadIdx.x == 0) {
+        unsigned long long acc = 0;
+        for (uint32_t w = 0; w < world; w++) {
+            cursor[w] = acc;
+            acc += counts[w];
+        }
+    }
+}
+
 // Lanes bound for the same shard are grouped with __match_any_sync; one atomic
 // per group claims their positions.
 __global__ void __launch_bounds__(kThreads) k_route_scatter(uint32_t a, uint32_t b, uint64_t magic, uint32_t world,

@@ -116,6 +116,21 @@ class Table:
                 "dyc_delete_batch")
         return values_out, status
 
+    def mixed(self, ops, keys, values, values_out=None, status=None, stream=None):
+        """Mixed batch (find=0, insert=1, delete=2; phases find -> insert -> delete, Q10)."""
+        torch = _torch()
+        _check_u32(keys, "keys")
+        _check_u32(values, "values")
+        n = keys.numel()
+        if values_out is None:
+            values_out = torch.empty(n, dtype=torch.int32, device=keys.device)
+        if status is None:
+            status = torch.empty(n, dtype=torch.uint8, device=keys.device)
+        L.check(self._lib.dyc_mixed_batch(self._h, ops.data_ptr(), keys.data_ptr(), values.data_ptr(),
+                                          values_out.data_ptr(), status.data_ptr(), n, _stream_ptr(stream)),
+                "dyc_mixed_batch")
+        return values_out, status
+
     # host-buffer entry points (end-to-end path: copies inside the call, chunked
     # so PCIe transfers overlap the kernels).  Output arrays may be supplied
     # (e.g. pinned numpy views) to avoid pageable-memory copies.
@@ -207,6 +222,46 @@ class Table:
         calls = np.zeros(L.DYC_PROF_KINDS, dtype=np.uint64)
         L.check(self._lib.dyc_profile_read(self._h, ms.ctypes.data, calls.ctypes.data), "dyc_profile_read")
         return {name: (float(ms[i]), int(calls[i])) for i, name in enumerate(L.PROF_NAMES)}
+
+    # ------------------------------------------------------------ routing (S11)
+    def route_count(self, keys, world: int, counts=None, stream=None):
+        """Per-shard histogram (uint64 -> int64 tensor of length world)."""
+        torch = _torch()
+        _check_u32(keys, "keys")
+        if counts is None:
+            counts = torch.empty(world, dtype=torch.int64, device=keys.device)
+        L.check(self._lib.dyc_route_count(self._h, keys.data_ptr(), keys.numel(), world, counts.data_ptr(),
+                                          _stream_ptr(stream)), "dyc_route_count")
+        return counts
+
+    def route_scatter(self, keys, values, world: int, counts, stream=None):
+        """Groups ops by destination shard; returns (keys_out, values_out|None, pos)."""
+        torch = _torch()
+        _check_u32(keys, "keys")
+        n = keys.numel()
+        kout = torch.empty(n, dtype=torch.int32, device=keys.device)
+        vout = torch.empty(n, dtype=torch.int32, device=keys.device) if values is not None else None
+        pos = torch.empty(n, dtype=torch.int32, device=keys.device)
+        cursor = torch.empty(world, dtype=torch.int64, device=keys.device)
+        L.check(self._lib.dyc_route_scatter(self._h, keys.data_ptr(), values.data_ptr() if values is not None else None,
+                                            n, world, counts.data_ptr(), cursor.data_ptr(), kout.data_ptr(),
+                                            vout.data_ptr() if vout is not None else None, pos.data_ptr(),
+                                            _stream_ptr(stream)), "dyc_route_scatter")
+        return kout, vout, pos
+
+    def route_unpermute(self, pos, reply_vals=None, reply_status=None, stream=None):
+        """vals[i] = reply_vals[pos[i]], status[i] = reply_status[pos[i]]."""
+        torch = _torch()
+        n = pos.numel()
+        v = torch.empty(n, dtype=torch.int32, device=pos.device) if reply_vals is not None else None
+        s = torch.empty(n, dtype=torch.uint8, device=pos.device) if reply_status is not None else None
+        L.check(self._lib.dyc_route_unpermute(pos.data_ptr(), n,
+                                              reply_vals.data_ptr() if reply_vals is not None else None,
+                                              reply_status.data_ptr() if reply_status is not None else None,
+                                              v.data_ptr() if v is not None else None,
+                                              s.data_ptr() if s is not None else None, _stream_ptr(stream)),
+                "dyc_route_unpermute")
+        return v, s
 
     def launch_count(self, reset: bool = False) -> int:
         return int(self._lib.dyc_launch_count(self._h, 1 if reset else 0))

@@ -215,13 +215,16 @@ def _as_i32(x):
     return torch.where(x >= (1 << 31), x - (1 << 32), x).to(torch.int32)
 
 
-def c2_rand_static_torch(log2_n: int = 27, device="cuda", seed_cfg: Optional[int] = None, beta: float = 0.85):
+def c2_rand_static_torch(log2_n: int = 27, device="cuda", seed_cfg: Optional[int] = None, beta: float = 0.85,
+                         key_base: int = 0, miss_base: int = 0):
     """Returns (init_capacity, ins_keys, ins_vals, find_keys, del_keys) as int32
-    tensors holding the uint32 bit patterns of c2_rand_static(log2_n)."""
+    tensors holding the uint32 bit patterns of c2_rand_static(log2_n).
+    key_base / miss_base shift the key index ranges (disjoint per-rank batches
+    for the sharded bench: key(key_base + i), misses key(2^31 + miss_base + j))."""
     import torch
     s = config_seed(2) if seed_cfg is None else seed_cfg
     n = 1 << log2_n
-    idx = torch.arange(n + 1, dtype=torch.int64, device=device)
+    idx = key_base + torch.arange(n + 1, dtype=torch.int64, device=device)
     k = _key_of_t(idx, s)
     k = k[k != EMPTY_KEY][:n]                                    # key_range(0, n, s)
     mix = (0x9E3779B9 * 1) & 0xFFFFFFFF
@@ -230,9 +233,9 @@ def c2_rand_static_torch(log2_n: int = 27, device="cuda", seed_cfg: Optional[int
     j = _perm_pow2_t(i, log2_n, s ^ 0x1234567)
     hit = j < n // 2
     hit_idx = _perm_pow2_t(j, log2_n, s ^ 0x7654321) & (n - 1)
-    miss = _key_of_t(MISS_BASE + (j - n // 2), s)
+    miss = _key_of_t(MISS_BASE + miss_base + (j - n // 2), s)
     q = torch.where(hit, k[hit_idx], miss)
-    q = torch.where(q == EMPTY_KEY, _key_of_t(torch.tensor(MISS_BASE + n, device=device), s), q)
+    q = torch.where(q == EMPTY_KEY, _key_of_t(torch.tensor(MISS_BASE + miss_base + n, device=device), s), q)
     del_idx = _perm_pow2_t(torch.arange(n // 2, dtype=torch.int64, device=device), log2_n, s ^ 0x5A5A5A5)
     dk = k[del_idx]
     cap = int(math.ceil(n / beta))
