@@ -494,6 +494,36 @@ void dyo_delete_batch(dyo_table *T, const uint32_t *keys, uint32_t *old_vals, ui
     enforce_lower(T);
 }
 
+/* Mixed batch (configs C4/C5).  The paper batches one op type at a time
+ * and calls mixed batches ambiguous (commented).  Reading Q10: keys are
+ * distinct across the batch; the finds run first (they see the table before the
+ * batch), then the inserts, then the deletes, each as a single-type batch in
+ * request order.  ops[i]: 0 find, 1 insert, 2 delete.  vals_out[i]: the found /
+ * removed value, 0xFFFFFFFF on a miss and for inserts; status[i]: the op's code. */
+void dyo_mixed_batch(dyo_table *T, const uint8_t *ops, const uint32_t *keys, const uint32_t *vals,
+                     uint32_t *vals_out, uint8_t *status, uint64_t n)
+{
+    uint64_t *idx = (uint64_t *)malloc((n + 1) * sizeof(uint64_t));
+    uint32_t *k = (uint32_t *)malloc((n + 1) * sizeof(uint32_t));
+    uint32_t *v = (uint32_t *)malloc((n + 1) * sizeof(uint32_t));
+    uint32_t *ov = (uint32_t *)malloc((n + 1) * sizeof(uint32_t));
+    uint8_t *st = (uint8_t *)malloc(n + 1);
+    for (uint8_t op = 0; op < 3; op++) {
+        uint64_t c = 0;
+        for (uint64_t i = 0; i < n; i++)
+            if (ops[i] == op) { idx[c] = i; k[c] = keys[i]; v[c] = vals ? vals[i] : 0; c++; }
+        if (c == 0) continue;
+        if (op == 0) dyo_find_batch(T, k, ov, st, c);
+        else if (op == 1) { dyo_insert_batch(T, k, v, st, c); for (uint64_t j = 0; j < c; j++) ov[j] = DYO_EMPTY; }
+        else dyo_delete_batch(T, k, ov, st, c);
+        for (uint64_t j = 0; j < c; j++) {
+            if (vals_out) vals_out[idx[j]] = ov[j];
+            if (status) status[idx[j]] = st[j];
+        }
+    }
+    free(idx); free(k); free(v); free(ov); free(st);
+}
+
 /* Explicit resize (dyc_resize analogue): direction +1 upsizes (the smallest, or
  * `t` if given), -1 downsizes (the largest, or `t`).  A choice that would break
  * "no subtable more than double any other" (I6) is refused (-1). */

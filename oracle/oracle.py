@@ -54,6 +54,7 @@ def oracle_lib():
         lib.dyo_destroy.argtypes = [P]
         for name in ("dyo_insert_batch", "dyo_find_batch", "dyo_delete_batch"):
             getattr(lib, name).argtypes = [P, P, P, P, U64]
+        lib.dyo_mixed_batch.argtypes = [P, P, P, P, P, P, U64]
         lib.dyo_resize.argtypes = [P, I32, I32]
         lib.dyo_resize.restype = I32
         lib.dyo_stats.argtypes = [P, C.POINTER(_Stats)]
@@ -123,6 +124,15 @@ class OracleTable:
         v = np.zeros(keys.size, dtype=np.uint32)
         st = np.zeros(keys.size, dtype=np.uint8)
         self._lib.dyo_delete_batch(self._t, _ptr(keys), _ptr(v), _ptr(st), keys.size)
+        return v, st
+
+    def mixed(self, ops: np.ndarray, keys: np.ndarray, values: np.ndarray):
+        ops = np.ascontiguousarray(ops, dtype=np.uint8)
+        keys = np.ascontiguousarray(keys, dtype=np.uint32)
+        values = np.ascontiguousarray(values, dtype=np.uint32)
+        v = np.zeros(keys.size, dtype=np.uint32)
+        st = np.zeros(keys.size, dtype=np.uint8)
+        self._lib.dyo_mixed_batch(self._t, _ptr(ops), _ptr(keys), _ptr(values), _ptr(v), _ptr(st), keys.size)
         return v, st
 
     def resize(self, direction: int, subtable: int = -1) -> int:

@@ -240,3 +240,168 @@ def c2_rand_static_torch(log2_n: int = 27, device="cuda", seed_cfg: Optional[int
     dk = k[del_idx]
     cap = int(math.ceil(n / beta))
     return cap, _as_i32(k), _as_i32(v), _as_i32(q), _as_i32(dk)
+
+
+# ---------------------------------------------------------------------------
+# Config C3: TW/RE-shaped dynamic stream (§VI-A "Dynamic Hashing
+# Comparison"; datasets Table `table:exp_data_sets` P:L671-672).
+def c3_dynamic(scale: float = 1.0, shape: str = "TW", batch: int = 1_000_000, r: float = 0.2,
+               cycles: int = 2, seed_cfg: Optional[int] = None, init_capacity: int = 1 << 20) -> Workload:
+    """Insert stream shaped like TW (50,876,784 ops over 44,523,684 unique keys,
+    multiplicity <= 4) or RE (48,104,875 / 41,466,682, <= 2), scaled by `scale`.
+    Each step: one insert batch (distinct keys), one find batch of `batch` ops
+    (50% live / 50% never inserted), one delete batch of r*batch OLDEST live keys
+    (sliding window; r = #delete/#insert, reading Q22).  After the
+    stream is exhausted the batches are replayed with insert and delete key sets
+    swapped (reading Q27); `cycles` repeats the whole thing."""
+    s = config_seed(3) if seed_cfg is None else seed_cfg
+    rng = np.random.Generator(np.random.PCG64(s))
+    total, uniq, mult = {"TW": (50_876_784, 44_523_684, 4), "RE": (48_104_875, 41_466_682, 2)}[shape]
+    T, U = max(1, int(total * scale)), max(1, int(uniq * scale))
+    batch = max(1, int(batch))
+    keys = key_range(0, U, s)
+    # repeats: T-U extra occurrences of random keys, each key at most mult-1 times,
+    # each repeat in a strictly later batch than the key's previous occurrence
+    n_rep = T - U
+    rep_keys = rng.choice(U, size=min(n_rep, U * (mult - 1)), replace=True)
+    cnt = np.bincount(rep_keys, minlength=U)
+    cnt = np.minimum(cnt, mult - 1)
+    first_batch = np.arange(U) // batch
+    n_batches = (U + batch - 1) // batch
+    rep_slots = [[] for _ in range(n_batches + 4 * mult)]
+    ids = np.nonzero(cnt)[0]
+    for kid in ids:
+        b = int(first_batch[kid])
+        for j in range(int(cnt[kid])):
+            b += 1 + int(rng.integers(0, 3))
+            if b < len(rep_slots):
+                rep_slots[b].append(int(kid))
+    w = Workload(f"C3-{shape}-x{scale:g}", 4, 0.3, 0.85, init_capacity)
+    ins_batches = []
+    for b in range(len(rep_slots)):
+        fresh = np.arange(b * batch, min((b + 1) * batch, U)) if b < n_batches else np.zeros(0, np.int64)
+        ids_b = np.concatenate([fresh, np.array(rep_slots[b], dtype=np.int64)])
+        if ids_b.size:
+            ins_batches.append(np.unique(ids_b))          # distinct within the batch
+    live = {}                                              # key id -> insertion order (FIFO)
+    order = 0
+    miss_ctr = 0
+    del_batches = []
+    for b, ids_b in enumerate(ins_batches):
+        ver = b + 1
+        w.batches.append(Batch("insert", keys[ids_b], val_of(keys[ids_b], ver)))
+        for kid in ids_b.tolist():
+            if kid not in live:
+                live[kid] = order
+                order += 1
+        nf = batch
+        lv = np.fromiter(live.keys(), dtype=np.int64, count=len(live))
+        hits = keys[rng.choice(lv, size=min(nf // 2, lv.size), replace=False)] if lv.size else np.zeros(0, np.uint32)
+        miss = key_range(MISS_BASE + miss_ctr, nf - hits.size, s)
+        miss_ctr += nf - hits.size
+        q = np.concatenate([hits, miss])
+        rng.shuffle(q)
+        w.batches.append(Batch("find", q))
+        nd = int(r * batch)
+        oldest = sorted(live, key=live.get)[:nd]
+        for kid in oldest:
+            del live[kid]
+        del_ids = np.array(oldest, dtype=np.int64)
+        del_batches.append(del_ids)
+        w.batches.append(Batch("delete", keys[del_ids]))
+    base = list(w.batches)
+    for c in range(cycles):
+        if c == 0:
+            # swap pass of the first cycle
+            for b, ids_b in enumerate(ins_batches):
+                d_ids = del_batches[b]
+                w.batches.append(Batch("insert", keys[d_ids], val_of(keys[d_ids], 1000 + b)))
+                w.batches.append(Batch("delete", keys[ids_b]))
+        else:
+            # later cycles replay the forward stream, then the swap pass again
+            for bt in base:
+                w.batches.append(Batch(bt.op, bt.keys.copy(), None if bt.values is None else bt.values.copy()))
+            for b, ids_b in enumerate(ins_batches):
+                d_ids = del_batches[b]
+                w.batches.append(Batch("insert", keys[d_ids], val_of(keys[d_ids], 2000 + b)))
+                w.batches.append(Batch("delete", keys[ids_b]))
+    return w
+
+
+# ---------------------------------------------------------------------------
+# Config C4: LINE/COM-shaped Zipf(0.99) mixed batches (P:L673-674; SURVEY §8(d)).
+@dataclass
+class MixedBatch:
+    ops: np.ndarray      # uint8: 0 find, 1 insert, 2 delete
+    keys: np.ndarray     # uint32, distinct within the batch
+    values: np.ndarray   # uint32
+
+
+def zipf_distinct(rng, cdf: np.ndarray, count: int, exclude=None) -> np.ndarray:
+    """Draw Zipf ranks (inverse CDF) until `count` distinct ranks are collected."""
+    got = []
+    seen = set() if exclude is None else set(exclude)
+    while len(got) < count:
+        draw = np.searchsorted(cdf, rng.random(max(1024, 2 * (count - len(got)))), side="right")
+        for x in draw.tolist():
+            if x not in seen:
+                seen.add(x)
+                got.append(x)
+                if len(got) == count:
+                    break
+    return np.array(got, dtype=np.int64)
+
+
+def c4_zipf_mixed(U: int = 45_159_880, distinct: int = 4_000_000, grow_batches: int = 16, cycles: int = 2,
+                  exponent: float = 0.99, seed_cfg: Optional[int] = None, init_capacity: int = 1 << 20,
+                  drain_floor: float = 0.10):
+    """Mixed 50/30/20 find/insert/delete batches over Zipf(0.99) ranks of a
+    universe of U keys (LINE-shaped: U = 45,159,880; COM-shaped: U = 4,583,941
+    with 1M-distinct batches).  Grow phase: `grow_batches` batches; drain phase:
+    50% find / 5% insert / 45% delete (deletes drawn from the live set) until
+    the live count is below drain_floor of its peak.  Returns (Workload meta, list of
+    MixedBatch)."""
+    s = config_seed(4) if seed_cfg is None else seed_cfg
+    rng = np.random.Generator(np.random.PCG64(s))
+    ranks = np.arange(1, U + 1, dtype=np.float64)
+    pmf = ranks ** (-exponent)
+    cdf = np.cumsum(pmf)
+    cdf /= cdf[-1]
+    keys_of = lambda r: key_of(np.asarray(r, dtype=np.uint64), s)  # noqa: E731  (rank -> key, a bijection)
+    meta = Workload(f"C4-zipf-U{U}", 4, 0.3, 0.85, init_capacity)
+    out = []
+    live = set()
+    ver = 0
+    for c in range(cycles):
+        for b in range(grow_batches):
+            ver += 1
+            r = zipf_distinct(rng, cdf, distinct)
+            u = rng.random(r.size)
+            ops = np.where(u < 0.5, 0, np.where(u < 0.8, 1, 2)).astype(np.uint8)
+            k = keys_of(r)
+            out.append(MixedBatch(ops, k, val_of(k, ver)))
+            for rr, op in zip(r.tolist(), ops.tolist()):
+                if op == 1:
+                    live.add(rr)
+                elif op == 2:
+                    live.discard(rr)
+        peak = len(live)
+        while len(live) > drain_floor * peak and live:
+            ver += 1
+            nd = min(len(live), int(0.45 * distinct))
+            dl = rng.choice(np.fromiter(live, dtype=np.int64, count=len(live)), size=nd, replace=False)
+            rest = zipf_distinct(rng, cdf, distinct - nd, exclude=dl.tolist())
+            u = rng.random(rest.size)
+            ops_rest = np.where(u < 0.5 / 0.55, 0, 1).astype(np.uint8)      # 50 find : 5 insert
+            r = np.concatenate([dl, rest])
+            ops = np.concatenate([np.full(nd, 2, np.uint8), ops_rest])
+            perm = rng.permutation(r.size)
+            r, ops = r[perm], ops[perm]
+            k = keys_of(r)
+            out.append(MixedBatch(ops, k, val_of(k, ver)))
+            for rr, op in zip(r.tolist(), ops.tolist()):
+                if op == 1:
+                    live.add(rr)
+                elif op == 2:
+                    live.discard(rr)
+    return meta, out

@@ -46,6 +46,20 @@ class BruteMap:
                 st[i] = 1
         return v, st
 
+    def mixed(self, ops, keys, vals):
+        """Reading Q10: finds see the pre-batch map, then inserts, then deletes."""
+        v = np.full(len(keys), EMPTY, dtype=np.uint32)
+        st = np.zeros(len(keys), dtype=np.uint8)
+        for op in (0, 1, 2):
+            sel = np.nonzero(ops == op)[0]
+            if op == 0:
+                v[sel], st[sel] = self.find(keys[sel])
+            elif op == 1:
+                st[sel] = self.insert(keys[sel], vals[sel])
+            else:
+                v[sel], st[sel] = self.delete(keys[sel])
+        return v, st
+
     def sorted_kv(self):
         ks = np.array(sorted(self.m), dtype=np.uint64)
         vs = np.array([self.m[int(k)] for k in ks], dtype=np.uint64)

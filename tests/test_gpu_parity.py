@@ -323,3 +323,34 @@ def test_c2_full_size_sampled():
     deleted = np.isin(sample, dele.keys)
     np.testing.assert_array_equal(f.cpu().numpy().astype(bool), ~deleted)
     np.testing.assert_array_equal(host_u32(v)[~deleted], W.val_of(sample[~deleted], 0))
+
+
+# ------------------------------------------------------------------ dynamic configs
+@pytest.mark.parametrize("shape", ["TW", "RE"])
+def test_c3_dynamic_parity(oracle_mod, shape):
+    """Config C3's shape (sliding window, swap pass, two cycles) at small scale:
+    up- and downsizes repeat; contents and the resize schedule match every batch."""
+    wl = W.c3_dynamic(scale=0.001, shape=shape, batch=5000, cycles=2, init_capacity=1024)
+    g, o = run_parity(oracle_mod, wl, B=8, layout_every=False)
+    check_layout(g, o)
+    s = g.stats()
+    assert s["n_upsize"] > 0 and s["n_downsize"] > 0
+
+
+def test_c4_zipf_mixed_parity(oracle_mod):
+    """Config C4's shape: Zipf(0.99) mixed 50/30/20 batches through dyc_mixed_batch
+    (reading Q10: find -> insert -> delete), grow then drain, two cycles."""
+    meta, batches = W.c4_zipf_mixed(U=60000, distinct=6000, grow_batches=6, cycles=2, init_capacity=1024)
+    g = Table(d=4, init_capacity=meta.init_capacity, alpha=meta.alpha, beta=meta.beta, bucket_slots=8)
+    o = oracle_mod.OracleTable(d=4, init_capacity=meta.init_capacity, alpha=meta.alpha, beta=meta.beta,
+                               bucket_slots=8)
+    for i, b in enumerate(batches):
+        ops = torch.from_numpy(b.ops).cuda()
+        v, st = g.mixed(ops, dev(b.keys), dev(b.values))
+        ov, os_ = o.mixed(b.ops, b.keys, b.values)
+        np.testing.assert_array_equal(st.cpu().numpy(), os_, err_msg=f"batch {i} status")
+        np.testing.assert_array_equal(host_u32(v), ov, err_msg=f"batch {i} values")
+        np.testing.assert_array_equal(g.sorted_kv(), o.sorted_kv(), err_msg=f"contents after {i}")
+        assert g.stats()["buckets"] == o.stats()["buckets"]
+    check_layout(g, o)
+    assert g.stats()["n_downsize"] > 0
