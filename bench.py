@@ -47,6 +47,8 @@ def parse():
     ap.add_argument("--no-rehash", action="store_true")
     ap.add_argument("--profile-only", action="store_true", help="a few steps, no extras (for ncu)")
     ap.add_argument("--l2-fetch", type=int, default=None, help="set cudaLimitMaxL2FetchGranularity (bytes)")
+    ap.add_argument("--routed", action="store_true",
+                    help="use the sharded router even at N=1 (exercises the N>1 code path)")
     return ap.parse_args()
 
 
@@ -167,6 +169,82 @@ def reference_arm(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi_del, cap, stream):
+    """Roofline of the dominant kernel.  Algorithmic bytes: every
+    probe reads one whole bucket (8*B bytes, the unit the method compares), every
+    slot write costs one 32-byte sector, plus the streamed keys/values/status.
+    achieved = algorithmic bytes per launch / mean launch time (CUDA events
+    recorded by libdyc.so on the launching stream over the timed region)."""
+    import torch
+    from paper_conf_icde_lizlhs21_b200 import _lib as L
+    peak, peak_src = measured_peaks()
+    ev = s_ins["last_insert_evictions"]
+    E = ev / max(1, s_ins["last_insert_new"])
+    pend = s_ins["last_insert_pending"]
+    bkt = 8 * args.bucket_slots
+    sec = 32
+    probes_find = hit_rate * (1 + phi) + (1 - hit_rate) * 2
+    slots_sub = (cap // 4 // args.bucket_slots + 1) * args.bucket_slots     # slots of one subtable
+    bytes_alg = {
+        # find: first-choice bucket, then the second one unless hit; + key, value, flag
+        "k_find": n_find * (probes_find * bkt + 9),
+        # upsert of new keys: both candidate buckets read (existence check), one
+        # sector written for each key placed here; + key, value, status
+        "k_upsert": n_ins * (2 * bkt + 9) + (n_ins - pend) * sec,
+        # eviction kernel: per pending key one write; per hop one bucket read + one exchange
+        "k_place": pend * sec + ev * (bkt + sec),
+        # delete (all hits): 1+φ bucket reads, one sector written; + key, old value, status
+        "k_delete": n_del * ((1 + phi_del) * bkt + sec + 9),
+        # upsize: stream the subtable in (8 B/slot) and twice its size out (16 B/slot)
+        "k_upsize": slots_sub * 24,
+        # downsize: stream twice the new size in, the new size out
+        "k_downsize": slots_sub * 12,
+    }
+    kern = {k: prof[k][0] / args.steps for k in bytes_alg if prof[k][1]}
+    dom = max(kern, key=kern.get)
+    calls = prof[dom][1] / args.steps
+    launch_ms = prof[dom][0] / max(1, prof[dom][1])
+    achieved = bytes_alg[dom] / calls / (launch_ms * 1e-3) / 1e9
+    achieved_all = {k: bytes_alg[k] / (kern[k] * 1e-3) / 1e9 for k in kern}
+    # random-bucket ceiling: the probe access pattern alone, on a table-sized buffer
+    buf = torch.empty(int(cap * 8 // (1 << 20) + 1) << 20, dtype=torch.uint8, device="cuda")
+    sink = torch.zeros(1, dtype=torch.int64, device="cuda")
+    nreads = int(n_find * probes_find)
+    for seed in (7, 8, 9):
+        if seed == 9:
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+        L.check(L.dyc_bench_gather(buf.data_ptr(), buf.numel(), nreads, bkt, seed, sink.data_ptr(),
+                                   stream.cuda_stream), "dyc_bench_gather")
+    e1.record(stream)
+    torch.cuda.synchronize()
+    gather_ms = e0.elapsed_time(e1)
+    gather_gbs = nreads * bkt / (gather_ms * 1e-3) / 1e9
+    del buf
+    traffic, traffic_src = None, None
+    pdir = os.path.join(ROOT, "profiles")
+    tr_files = sorted(f for f in os.listdir(pdir) if f.endswith("_traffic.json")) if os.path.isdir(pdir) else []
+    if tr_files and args.log2n == 27 and args.bucket_slots == 8 and n_ins == (1 << 27):
+        tr = json.load(open(os.path.join(pdir, tr_files[-1])))
+        if dom in tr:
+            traffic, traffic_src = tr[dom], f"profiles/{tr_files[-1]} (ncu --set full, dram read+write per launch)"
+    return {
+        "bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
+        "frac": achieved / peak, "peak_source": peak_src, "traffic": traffic, "traffic_source": traffic_src,
+        "algorithmic_bytes_per_launch": bytes_alg[dom] / calls,
+        "launch_ms": launch_ms,
+        "achieved_gbs_per_kernel": {k: round(v, 1) for k, v in achieved_all.items()},
+        "random_bucket_ceiling": {"bytes_per_probe": bkt, "gbs": gather_gbs,
+                                  "gprobes_per_s": nreads / (gather_ms * 1e-3) / 1e9,
+                                  "what": "dyc_bench_gather: random bucket reads, probe access pattern only"},
+        "frac_of_random_ceiling": achieved / gather_gbs,
+        "kernel_ms_per_step": {k: round(v, 4) for k, v in kern.items()},
+        "model": {"phi": phi, "hit_rate": hit_rate, "evictions_per_insert": E, "probes_per_find": probes_find,
+                  "pending_keys": pend, "bucket_bytes": bkt, "sector_bytes": sec},
+    }
+
+
+
 # ---------------------------------------------------------------- GPU arm
 def main():
     args = parse()
@@ -182,8 +260,12 @@ def main():
 
     torch.cuda.set_device(local)
     dist = None
-    if world > 1:
+    if world > 1 or args.routed:
         import torch.distributed as dist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29531")
+        os.environ.setdefault("RANK", "0")
+        os.environ.setdefault("WORLD_SIZE", "1")
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     from paper_conf_icde_lizlhs21_b200 import _lib as L
     from paper_conf_icde_lizlhs21_b200 import workload as W
@@ -192,9 +274,9 @@ def main():
     if args.l2_fetch is not None:
         L.check(L.dyc_set_l2_fetch_granularity(args.l2_fetch), "dyc_set_l2_fetch_granularity")
     n = 1 << args.log2n
-    cap, k_ins, v_ins, k_find, k_del = W.c2_rand_static_torch(args.log2n, device="cuda")
-    if world > 1:
+    if world > 1 or args.routed:
         return multi_gpu(args, rank, world, local, dist)
+    cap, k_ins, v_ins, k_find, k_del = W.c2_rand_static_torch(args.log2n, device="cuda")
 
     stream = torch.cuda.current_stream()
     g = Table(d=4, init_capacity=cap, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
@@ -265,74 +347,9 @@ def main():
     value = n_ops / (ms_per_step * 1e-3) / 1e6
 
     # --------------------------------------------------------- roofline
-    # Algorithmic bytes: every probe reads one whole bucket (8*B bytes, the unit
-    # the method compares), every slot write costs one 32-byte sector, plus the
-    # streamed keys/values/status (DESIGN.md §5 "algorithmic bytes per op").
-    peak, peak_src = measured_peaks()
-    E = s_ins["last_insert_evictions"] / max(1, s_ins["last_insert_new"])
+    roofline = compute_roofline(args, prof, n_ins=n, n_find=n, n_del=n // 2, s_ins=s_ins, hit_rate=hit_rate,
+                                phi=phi, phi_del=phi_after_up, cap=cap, stream=stream)
     pend = s_ins["last_insert_pending"]
-    bkt = 8 * args.bucket_slots
-    sec = 32
-    probes_find = hit_rate * (1 + phi) + (1 - hit_rate) * 2
-    slots_sub = (cap // 4 // args.bucket_slots + 1) * args.bucket_slots     # slots of one subtable
-    bytes_alg = {
-        # find: first-choice bucket, then the second one unless hit; + key, value, flag
-        "k_find": n * (probes_find * bkt + 9),
-        # upsert on an empty table: both candidate buckets read (existence check),
-        # one sector written for each key placed here; + key, value, status
-        "k_upsert": n * (2 * bkt + 9) + (n - pend) * sec,
-        # eviction kernel: per pending key one write; per hop one bucket read + one exchange
-        "k_place": pend * sec + s_ins["last_insert_evictions"] * (bkt + sec),
-        # delete (all hits): 1+φ bucket reads, one sector written; + key, old value, status
-        "k_delete": (n // 2) * ((1 + phi_after_up) * bkt + sec + 9),
-        # upsize: stream the subtable in (8 B/slot) and twice its size out (16 B/slot)
-        "k_upsize": slots_sub * 24,
-        # downsize: stream twice the new size in, the new size out
-        "k_downsize": slots_sub * 12,
-    }
-    kern = {k: prof[k][0] / args.steps for k in bytes_alg if prof[k][1]}
-    dom = max(kern, key=kern.get)
-    calls = prof[dom][1] / args.steps
-    launch_ms = prof[dom][0] / max(1, prof[dom][1])
-    achieved = bytes_alg[dom] / calls / (launch_ms * 1e-3) / 1e9
-    achieved_all = {k: bytes_alg[k] / (kern[k] * 1e-3) / 1e9 for k in kern}
-    # random-bucket ceiling: the probe access pattern alone, on a table-sized buffer
-    buf = torch.empty(int(cap * 8 // (1 << 20) + 1) << 20, dtype=torch.uint8, device="cuda")
-    sink = torch.zeros(1, dtype=torch.int64, device="cuda")
-    nreads = int(n * probes_find)
-    for _ in range(2):
-        L.check(L.dyc_bench_gather(buf.data_ptr(), buf.numel(), nreads, bkt, 7, sink.data_ptr(),
-                                   stream.cuda_stream), "dyc_bench_gather")
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    L.check(L.dyc_bench_gather(buf.data_ptr(), buf.numel(), nreads, bkt, 9, sink.data_ptr(),
-                               stream.cuda_stream), "dyc_bench_gather")
-    e1.record(stream)
-    torch.cuda.synchronize()
-    gather_ms = e0.elapsed_time(e1)
-    gather_gbs = nreads * bkt / (gather_ms * 1e-3) / 1e9
-    del buf
-    traffic, traffic_src = None, None
-    tr_files = sorted(f for f in os.listdir(os.path.join(ROOT, "profiles")) if f.endswith("_traffic.json")) \
-        if os.path.isdir(os.path.join(ROOT, "profiles")) else []
-    if tr_files and args.log2n == 27 and args.bucket_slots == 8:
-        tr = json.load(open(os.path.join(ROOT, "profiles", tr_files[-1])))
-        if dom in tr:
-            traffic, traffic_src = tr[dom], f"profiles/{tr_files[-1]} (ncu --set full, dram read+write per launch)"
-    roofline = {
-        "bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
-        "frac": achieved / peak, "peak_source": peak_src, "traffic": traffic, "traffic_source": traffic_src,
-        "algorithmic_bytes_per_launch": bytes_alg[dom] / calls,
-        "launch_ms": launch_ms,
-        "achieved_gbs_per_kernel": {k: round(v, 1) for k, v in achieved_all.items()},
-        "random_bucket_ceiling": {"bytes_per_probe": bkt, "gbs": gather_gbs,
-                                  "gprobes_per_s": nreads / (gather_ms * 1e-3) / 1e9,
-                                  "what": "dyc_bench_gather: random bucket reads, probe access pattern only"},
-        "frac_of_random_ceiling": achieved / gather_gbs,
-        "kernel_ms_per_step": {k: round(v, 4) for k, v in kern.items()},
-        "model": {"phi": phi, "hit_rate": hit_rate, "evictions_per_insert": E, "probes_per_find": probes_find,
-                  "pending_keys": pend, "bucket_bytes": bkt, "sector_bytes": sec},
-    }
 
     # --------------------------------------------------------- resize baselines
     resize = {"upsize_ms": phase_ms["upsize"], "downsize_ms": phase_ms["downsize"],
@@ -445,7 +462,8 @@ def main():
 
 def multi_gpu(args, rank, world, local, dist):
     from paper_conf_icde_lizlhs21_b200.dist import bench_multi_gpu
-    line = bench_multi_gpu(args, rank, world, local, METRIC, ClockSampler, measured_peaks, run_oracle_sample)
+    line = bench_multi_gpu(args, rank, world, local, METRIC, ClockSampler, measured_peaks, run_oracle_sample,
+                           compute_roofline)
     if rank == 0 and line is not None:
         print(json.dumps(line), flush=True)
     dist.barrier()

@@ -33,7 +33,7 @@ constexpr int kThreads = 256;
 #define DYC_PLACE_MINB 1
 #endif
 #ifndef DYC_UPSERT_U
-#define DYC_UPSERT_U 2
+#define DYC_UPSERT_U 4
 #endif
 #ifndef DYC_DELETE_U
 #define DYC_DELETE_U 2
@@ -228,16 +228,8 @@ __device__ __forceinline__ bool coop_place(const Grp<B / 4>& g, const TableView&
 // together), so the atomic round trips of different ops overlap.
 template <int G, int U>
 __device__ __forceinline__ void coop_cas_multi(const Grp<G>& g, unsigned long long* const (&bp)[U],
-                                               const unsigned long long (&s)[U][4], const bool (&want)[U],
+                                               unsigned (&em)[U], const bool (&want)[U],
                                                const unsigned long long (&kv)[U], bool (&placed)[U]) {
-    unsigned em[U];
-#pragma unroll
-    for (int u = 0; u < U; u++) {
-        em[u] = 0;
-#pragma unroll
-        for (int j = 0; j < 4; j++)
-            if (s[u][j] == kEmptySlot) em[u] |= 1u << j;
-    }
     for (;;) {
         unsigned cand[U];
         bool any = false;
@@ -265,6 +257,14 @@ __device__ __forceinline__ void coop_cas_multi(const Grp<G>& g, unsigned long lo
     }
 }
 
+__device__ __forceinline__ unsigned empty_mask(const unsigned long long (&s)[4]) {
+    unsigned m = 0;
+#pragma unroll
+    for (int j = 0; j < 4; j++)
+        if (s[j] == kEmptySlot) m |= 1u << j;
+    return m;
+}
+
 // ------------------------------------------------------ insert phase 1 (S5)
 // Upsert: probe t1's bucket, then t2's; an existing key gets its value replaced
 // (Alg. 1, status UPDATED).  A new key (status INSERTED) is, with FUSE,
@@ -289,38 +289,54 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     unsigned long long n_ins = 0, n_upd = 0;
     for (uint64_t base = w * (QPW * U); base < n; base += nwarps * (QPW * U)) {
+        // per op only the match position and the free-slot mask of each bucket
+        // are kept, not the 4-slot snapshots (register budget -> more ops in flight)
         uint64_t i[U];
         uint32_t k[U];
-        unsigned long long kv[U], s1[U][4], s2[U][4];
+        unsigned long long kv[U];
         unsigned long long* b1[U];
         unsigned long long* b2[U];
-        unsigned h1[U], h2[U];
+        unsigned h1[U], h2[U], em1[U], em2[U];
         bool need2[U], isnew[U], placed[U];
         int j1[U], j2[U];
+        {
+            unsigned long long s1[U][4];
 #pragma unroll
-        for (int u = 0; u < U; u++) {
-            i[u] = base + (uint64_t)u * QPW + grp;
-            const bool valid = i[u] < n;
-            k[u] = valid ? __ldg(keys + i[u]) : kEmptyKey;
-            kv[u] = make_kv(k[u], valid ? __ldg(vals + i[u]) : 0u);
-            const Pair p = pair_of(tv, k[u]);
-            b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
-            b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
-            probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
+            for (int u = 0; u < U; u++) {
+                i[u] = base + (uint64_t)u * QPW + grp;
+                const bool valid = i[u] < n;
+                k[u] = valid ? __ldg(keys + i[u]) : kEmptyKey;
+                kv[u] = make_kv(k[u], valid ? __ldg(vals + i[u]) : 0u);
+                const Pair p = pair_of(tv, k[u]);
+                b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
+                b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
+                probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
+            }
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                j1[u] = match_slot<4>(s1[u], k[u]);
+                em1[u] = empty_mask(s1[u]);
+            }
+        }
+        {
+            unsigned long long s2[U][4];
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                const bool active = k[u] != kEmptyKey;
+                h1[u] = g.ballot(active && j1[u] >= 0);
+                need2[u] = active && h1[u] == 0;
+#pragma unroll
+                for (int q = 0; q < 4; q++) s2[u][q] = kEmptySlot;
+                probe_cg_pred<B>(b2[u] + 4 * g.sub, s2[u], need2[u]);
+            }
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                j2[u] = match_slot<4>(s2[u], k[u]);
+                em2[u] = empty_mask(s2[u]);
+            }
         }
 #pragma unroll
         for (int u = 0; u < U; u++) {
-            const bool active = k[u] != kEmptyKey;
-            j1[u] = match_slot<4>(s1[u], k[u]);
-            h1[u] = g.ballot(active && j1[u] >= 0);
-            need2[u] = active && h1[u] == 0;
-#pragma unroll
-            for (int q = 0; q < 4; q++) s2[u][q] = kEmptySlot;
-            probe_cg_pred<B>(b2[u] + 4 * g.sub, s2[u], need2[u]);
-        }
-#pragma unroll
-        for (int u = 0; u < U; u++) {
-            j2[u] = match_slot<4>(s2[u], k[u]);
             h2[u] = g.ballot(need2[u] && j2[u] >= 0);
             if (h1[u] && g.sub == first_lane(h1[u])) st_u64_cg(b1[u] + 4 * g.sub + j1[u], kv[u]);
             if (h2[u] && g.sub == first_lane(h2[u])) st_u64_cg(b2[u] + 4 * g.sub + j2[u], kv[u]);
@@ -328,8 +344,8 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
             placed[u] = false;
         }
         if (FUSE) {
-            coop_cas_multi<G, U>(g, b1, s1, isnew, kv, placed);
-            coop_cas_multi<G, U>(g, b2, s2, isnew, kv, placed);
+            coop_cas_multi<G, U>(g, b1, em1, isnew, kv, placed);
+            coop_cas_multi<G, U>(g, b2, em2, isnew, kv, placed);
         }
         const bool lead = g.sub == 0;
 #pragma unroll

@@ -53,6 +53,7 @@ class DistTable:
         counts = self.shard.route_count(keys, self.world)
         kout, vout, pos = self.shard.route_scatter(keys, values, self.world, counts)
         send, recv = self._splits(counts)
+        self.last_recv = sum(recv)
         rk = self._a2a(kout, send, recv)
         rv = self._a2a(vout, send, recv) if values is not None else None
         return rk, rv, pos, send, recv
@@ -88,11 +89,14 @@ class DistTable:
 
 
 # ---------------------------------------------------------------- bench (N > 1)
-def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_peaks, run_oracle_sample):
+def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_peaks, run_oracle_sample,
+                    compute_roofline=None):
     """Weak scaling: every rank issues one C2-shaped batch of its own keys (2^log2n
     inserts, 2^log2n finds at 50% hit, 2^(log2n-1) deletes) through the router;
     each shard receives ~1/G of every rank's ops.  Time = max over ranks."""
     import statistics
+    import time
+    import numpy as np
     import torch
     import torch.distributed as dist
     from . import workload as W
@@ -109,24 +113,33 @@ def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_pea
         if evs: evs[0].record(stream)
         shard.clear()
         st = dt.insert(k_ins, v_ins)
+        n_ins_recv = dt.last_recv
         if evs: evs[1].record(stream)
         v, f = dt.find(k_find)
+        n_find_recv = dt.last_recv
         if evs: evs[2].record(stream)
         dv, ds = dt.delete(k_del)
         if evs: evs[3].record(stream)
-        return st, f, ds
+        return st, f, ds, (n_ins_recv, n_find_recv, dt.last_recv)
 
-    st, f, ds = step()
+    st, f, ds, recv = step()
     torch.cuda.synchronize()
     ok = torch.tensor([int((st == 1).all().item()), int(f.sum().item()), int(ds.sum().item())],
                       dtype=torch.int64, device="cuda")
     dist.all_reduce(ok)
+    hit_rate = float(f.float().mean().item())
+    # shard statistics for the roofline model (insert phase alone)
+    shard.clear()
+    dt.insert(k_ins, v_ins)
+    s_ins = shard.stats()
+    phi = s_ins["n_second_table"] / max(1, s_ins["m"])
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
     dist.barrier()
     recs = []
     shard.launch_count(reset=True)
+    shard.profile(True)
     with ClockSampler(local) as clk:
         torch.cuda.synchronize()
         dist.barrier()
@@ -139,12 +152,52 @@ def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_pea
         b.record(stream)
         torch.cuda.synchronize()
         dist.barrier()
+    launches = shard.launch_count()
+    prof = shard.profile_read()
+    shard.profile(False)
     ms = torch.tensor([a.elapsed_time(b) / args.steps], dtype=torch.float64, device="cuda")
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     ms_per_step = float(ms.item())
     n_ops = (n + n + n // 2) * world
     phases = {p: statistics.mean(r[i].elapsed_time(r[i + 1]) for r in recs)
               for i, p in enumerate(["insert", "find", "delete"])}
+    roofline = None
+    if compute_roofline is not None:
+        roofline = compute_roofline(args, prof, n_ins=recv[0], n_find=recv[1], n_del=recv[2], s_ins=s_ins,
+                                    hit_rate=hit_rate, phi=phi, phi_del=phi, cap=cap, stream=stream)
+    # end to end: the rank's batch from pinned host memory, results back to the host
+    e2e = None
+    if not getattr(args, "no_e2e", False):
+        pin = lambda t: t.cpu().pin_memory()  # noqa: E731
+        hk, hv, hq, hd = pin(k_ins), pin(v_ins), pin(k_find), pin(k_del)
+        o_st = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+        o_v, o_f = torch.empty(n, dtype=torch.int32, pin_memory=True), torch.empty(n, dtype=torch.uint8, pin_memory=True)
+        o_dv, o_ds = (torch.empty(n // 2, dtype=torch.int32, pin_memory=True),
+                      torch.empty(n // 2, dtype=torch.uint8, pin_memory=True))
+
+        def e2e_step():
+            shard.clear()
+            o_st.copy_(dt.insert(hk.cuda(non_blocking=True), hv.cuda(non_blocking=True)), non_blocking=True)
+            v, f = dt.find(hq.cuda(non_blocking=True))
+            o_v.copy_(v, non_blocking=True)
+            o_f.copy_(f, non_blocking=True)
+            dv, ds = dt.delete(hd.cuda(non_blocking=True))
+            o_dv.copy_(dv, non_blocking=True)
+            o_ds.copy_(ds, non_blocking=True)
+            torch.cuda.synchronize()
+        e2e_step()
+        dist.barrier()
+        ts = []
+        for _ in range(max(1, min(args.steps, 3))):
+            t0 = time.perf_counter()
+            e2e_step()
+            ts.append(time.perf_counter() - t0)
+        t = torch.tensor([statistics.mean(ts)], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e = {"value": n_ops / float(t.item()) / 1e6, "unit": "Mops/s",
+               "h2d_bytes_per_step": 4 * n + 4 * n + 4 * n + 4 * (n // 2),
+               "d2h_bytes_per_step": n + 5 * n + 5 * (n // 2), "ms_per_step": 1e3 * float(t.item()),
+               "path": "pinned host batch -> DistTable (route, NCCL all-to-all, local kernels) -> host"}
     if rank != 0:
         return None
     return {
@@ -154,12 +207,13 @@ def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_pea
         "config": {"workload": f"C2-shaped batch per rank (2^{args.log2n} inserts, 2^{args.log2n} finds 50% hit, "
                                f"2^{args.log2n - 1} deletes), hash-partitioned over {world} shards, "
                                "NCCL all-to-all routing", "d": 4, "alpha": 0.3, "beta": 0.85,
-                   "bucket_slots": args.bucket_slots, "parallelism": f"shard{world}"},
+                   "bucket_slots": args.bucket_slots, "parallelism": f"shard{world}",
+                   "l2": "inputs and tables larger than L2; no flush needed"},
         "phase_ms_rank0": phases,
         "check": {"all_inserted_ranks": int(ok[0].item()), "found_total": int(ok[1].item()),
                   "deleted_total": int(ok[2].item()), "expected_found": world * n // 2,
                   "expected_deleted": world * n // 2},
-        "gpu_launches": shard.launch_count(),
+        "gpu_launches": launches,
         "clocks": clk.summary(),
-        "roofline": None, "cpu_baseline": None, "e2e": None,
+        "roofline": roofline, "cpu_baseline": None, "e2e": e2e,
     }
