@@ -31,6 +31,22 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "insert/find/delete Mops/s at 1/2/4/8 B200; subtable resize ms vs full rehash"
+_JSON_OUT = None
+
+
+def emit(line):
+    """The one JSON line goes to the process's original stdout; everything else a
+    library may print (NCCL banners, warnings) is redirected to stderr."""
+    _JSON_OUT.write(json.dumps(line) + "\n")
+    _JSON_OUT.flush()
+
+
+def _redirect_stdout():
+    global _JSON_OUT
+    if _JSON_OUT is None:
+        sys.stdout.flush()
+        _JSON_OUT = os.fdopen(os.dup(1), "w")
+        os.dup2(2, 1)
 
 
 def parse():
@@ -166,7 +182,7 @@ def reference_arm(args, rank, world):
                          "sample": f"C2 shape at 2^{log2n} keys per step (insert+find+delete)"},
         "e2e": {"value": value, "unit": "Mops/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
-    print(json.dumps(line), flush=True)
+    emit(line)
 
 
 def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi_del, cap, stream):
@@ -239,6 +255,7 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
                                   "what": "dyc_bench_gather: random bucket reads, probe access pattern only"},
         "frac_of_random_ceiling": achieved / gather_gbs,
         "kernel_ms_per_step": {k: round(v, 4) for k, v in kern.items()},
+        "other_kernels_ms_per_step": round(prof["other"][0] / args.steps, 4),
         "model": {"phi": phi, "hit_rate": hit_rate, "evictions_per_insert": E, "probes_per_find": probes_find,
                   "pending_keys": pend, "bucket_bytes": bkt, "sector_bytes": sec},
     }
@@ -247,6 +264,7 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
 
 # ---------------------------------------------------------------- GPU arm
 def main():
+    _redirect_stdout()
     args = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -262,6 +280,7 @@ def main():
     dist = None
     if world > 1 or args.routed:
         import torch.distributed as dist
+        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")   # keep stdout to the one JSON line
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         os.environ.setdefault("MASTER_PORT", "29531")
         os.environ.setdefault("RANK", "0")
@@ -457,7 +476,7 @@ def main():
         "table": {"fill_after_insert": s_ins["fill"], "phi": phi,
                   "pending_after_upsert": pend, "evictions": s_ins["last_insert_evictions"]},
     }
-    print(json.dumps(line), flush=True)
+    emit(line)
 
 
 def multi_gpu(args, rank, world, local, dist):
@@ -465,7 +484,7 @@ def multi_gpu(args, rank, world, local, dist):
     line = bench_multi_gpu(args, rank, world, local, METRIC, ClockSampler, measured_peaks, run_oracle_sample,
                            compute_roofline)
     if rank == 0 and line is not None:
-        print(json.dumps(line), flush=True)
+        emit(line)
     dist.barrier()
     dist.destroy_process_group()
 

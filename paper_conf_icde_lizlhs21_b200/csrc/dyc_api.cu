@@ -892,9 +892,12 @@ dyc_status dyc_mixed_batch(dyc_table* t, const uint8_t* d_ops, const uint32_t* d
     CU(cudaMemsetAsync(cnt, 0, 8 * 8, st));
     {
         ProfScope ps(t, DYC_PROF_OTHER, st);
-        k_op_count<<<std::min<unsigned>(grid_for(n, kThreads), t->num_sms * 8), kThreads, 0, st>>>(d_ops, n, cnt);
+        const OpDest od{d_ops};
+        k_group_count<OpDest><<<std::min<unsigned>(grid_for(n, kThreads), t->num_sms * 8), kThreads, 4 * 4, st>>>(
+            od, n, 4, cnt);
         k_route_offsets<<<1, 32, 0, st>>>(cnt, 4, cnt + 4);
-        k_op_scatter<<<grid_for(n, kThreads), kThreads, 0, st>>>(d_ops, d_keys, d_values, n, cnt + 4, k, v, pos);
+        k_group_scatter<OpDest><<<grid_for(n, (uint64_t)kThreads * kTileItems), kThreads, 4 * 12, st>>>(
+            od, d_keys, d_values, n, 4, cnt + 4, k, v, pos);
     }
     CU(cudaGetLastError());
     unsigned long long h[4];
@@ -1028,14 +1031,15 @@ dyc_status dyc_profile_read(dyc_table* t, double* ms, uint64_t* calls) {
 dyc_status dyc_route_count(dyc_table* t, const uint32_t* d_keys, uint64_t n, uint32_t world, uint64_t* d_counts,
                            dyc_stream_t stream) {
     TRY(enter(t, stream));
-    if (world < 1 || world > 4096) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..4096");
+    if (world < 1 || world > 2048) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..2048");
     CU(cudaMemsetAsync(d_counts, 0, world * 8, S(stream)));
     if (n == 0) return DYC_OK;
     const uint32_t sh = t->cfg.d + 1;
     {
         ProfScope ps(t, DYC_PROF_OTHER, S(stream));
-        k_route_count<<<std::min<unsigned>(grid_for(n, kThreads), t->num_sms * 8), kThreads, world * 8, S(stream)>>>(
-            t->a[sh], t->b[sh], fastmod_magic(world), world, d_keys, n, (unsigned long long*)d_counts);
+        const HashDest hd{t->a[sh], t->b[sh], world, fastmod_magic(world), d_keys};
+        k_group_count<HashDest><<<std::min<unsigned>(grid_for(n, kThreads), t->num_sms * 8), kThreads, world * 4,
+                                  S(stream)>>>(hd, n, world, (unsigned long long*)d_counts);
     }
     CU(cudaGetLastError());
     return DYC_OK;
@@ -1045,7 +1049,7 @@ dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_
                              uint32_t world, const uint64_t* d_counts, uint64_t* d_cursor, uint32_t* d_keys_out,
                              uint32_t* d_vals_out, uint32_t* d_pos, dyc_stream_t stream) {
     TRY(enter(t, stream));
-    if (world < 1 || world > 4096) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..4096");
+    if (world < 1 || world > 2048) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..2048");
     if (n == 0) return DYC_OK;
     if (n > 0xFFFFFFFFull) return set_err(DYC_ERR_INVALID_ARG, "route batch must be < 2^32 ops");
     const uint32_t sh = t->cfg.d + 1;
@@ -1056,9 +1060,10 @@ dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_
     }
     {
         ProfScope ps(t, DYC_PROF_OTHER, S(stream));
-        k_route_scatter<<<grid_for(n, kThreads), kThreads, 0, S(stream)>>>(
-            t->a[sh], t->b[sh], fastmod_magic(world), world, d_keys, d_vals_in, n, (unsigned long long*)d_cursor,
-            d_keys_out, d_vals_out, d_pos);
+        const HashDest hd{t->a[sh], t->b[sh], world, fastmod_magic(world), d_keys};
+        k_group_scatter<HashDest><<<grid_for(n, (uint64_t)kThreads * kTileItems), kThreads, world * 12,
+                                    S(stream)>>>(hd, d_keys, d_vals_in, n, world, (unsigned long long*)d_cursor,
+                                                 d_keys_out, d_vals_out, d_pos);
     }
     CU(cudaGetLastError());
     return DYC_OK;

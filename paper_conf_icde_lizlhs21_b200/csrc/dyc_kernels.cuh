@@ -606,57 +606,92 @@ __global__ void k_hash_probe(TableView tv, const uint32_t* __restrict__ keys, ui
 }
 
 // --------------------------------------------------------------- routing (S11)
-__global__ void __launch_bounds__(kThreads) k_route_count(uint32_t a, uint32_t b, uint64_t magic, uint32_t world,
-                                                          const uint32_t* __restrict__ keys, uint64_t n,
+// ------------------------------------------------- grouping by destination
+// Used for shard routing (dest = x_{d+1}(k) mod G) and for mixed batches
+// (dest = op code).  Block-aggregated: each block bins a tile of kTileItems ops in
+// shared memory, reserves its range per destination with ONE global atomic per
+// (block, destination), then places its ops; so contention does not grow with
+// the batch even when G is 1.
+constexpr int kTileItems = 8;
+
+struct HashDest {
+    uint32_t a, b, world;
+    uint64_t magic;
+    const uint32_t* keys;
+    __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return fastmod(hx(a, b, keys[i]), magic, world); }
+};
+struct OpDest {
+    const uint8_t* ops;
+    __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return ops[i] & 3u; }
+};
+
+// Lanes of a warp with the same destination are combined with __match_any_sync,
+// so shared-memory atomics (32-bit, native) see one update per (warp, dest).
+__device__ __forceinline__ unsigned warp_group_add(unsigned* ctr, uint32_t dest, bool valid) {
+    const unsigned peers = __match_any_sync(kFull, valid ? dest : 0xFFFFFFFFu);
+    const int leader = __ffs(peers) - 1;
+    unsigned b0 = 0;
+    if (valid && (int)(threadIdx.x & 31) == leader) b0 = atomicAdd(&ctr[dest], (unsigned)__popc(peers));
+    b0 = __shfl_sync(kFull, b0, leader);
+    return b0 + __popc(peers & lanemask_lt());
+}
+
+template <class Dest>
+__global__ void __launch_bounds__(kThreads) k_group_count(Dest dest, uint64_t n, uint32_t world,
                                                           unsigned long long* __restrict__ counts) {
-    extern __shared__ unsigned long long hist[];
-    for (uint32_t w = threadIdx.x; w < world; w += blockDim.x) hist[w] = 0;
+    extern __shared__ unsigned hist32[];
+    for (uint32_t w = threadIdx.x; w < world; w += blockDim.x) hist32[w] = 0;
     __syncthreads();
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
-        atomicAdd(&hist[fastmod(hx(a, b, keys[i]), magic, world)], 1ull);
-    __syncthreads();
-    for (uint32_t w = threadIdx.x; w < world; w += blockDim.x)
-        if (hist[w]) atomicAdd(&counts[w], hist[w]);
-}
-
-// Mixed batches: histogram and grouping by op code (3 "destinations").
-__global__ void __launch_bounds__(kThreads) k_op_count(const uint8_t* __restrict__ ops, uint64_t n,
-                                                       unsigned long long* __restrict__ counts) {
-    __shared__ unsigned long long hist[4];
-    if (threadIdx.x < 4) hist[threadIdx.x] = 0;
-    __syncthreads();
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
-        atomicAdd(&hist[ops[i] & 3], 1ull);
-    __syncthreads();
-    if (threadIdx.x < 4 && hist[threadIdx.x]) atomicAdd(&counts[threadIdx.x], hist[threadIdx.x]);
-}
-
-__global__ void __launch_bounds__(kThreads) k_op_scatter(const uint8_t* __restrict__ ops,
-                                                         const uint32_t* __restrict__ keys,
-                                                         const uint32_t* __restrict__ vals_in, uint64_t n,
-                                                         unsigned long long* __restrict__ cursor,
-                                                         uint32_t* __restrict__ keys_out,
-                                                         uint32_t* __restrict__ vals_out,
-                                                         uint32_t* __restrict__ pos_out) {
     for (uint64_t base = (uint64_t)blockIdx.x * blockDim.x; base < n; base += (uint64_t)gridDim.x * blockDim.x) {
         const uint64_t i = base + threadIdx.x;
         const bool valid = i < n;
-        const uint32_t dest = valid ? (ops[i] & 3u) : 0xFFFFFFFFu;
-        const unsigned peers = __match_any_sync(kFull, dest);
-        const int leader = __ffs(peers) - 1;
-        unsigned long long p0 = 0;
-        if (valid && (int)(threadIdx.x & 31) == leader) p0 = atomicAdd(&cursor[dest], (unsigned long long)__popc(peers));
-        p0 = __shfl_sync(kFull, p0, leader);
-        if (valid) {
-            const uint64_t pos = p0 + __popc(peers & lanemask_lt());
-            keys_out[pos] = keys[i];
-            vals_out[pos] = vals_in ? vals_in[i] : 0u;
-            pos_out[i] = (uint32_t)pos;
+        warp_group_add(hist32, valid ? dest(i) : 0u, valid);
+    }
+    __syncthreads();
+    for (uint32_t w = threadIdx.x; w < world; w += blockDim.x)
+        if (hist32[w]) atomicAdd(&counts[w], (unsigned long long)hist32[w]);
+}
+
+template <class Dest>
+__global__ void __launch_bounds__(kThreads) k_group_scatter(Dest dest, const uint32_t* __restrict__ keys,
+                                                            const uint32_t* __restrict__ vals_in, uint64_t n,
+                                                            uint32_t world, unsigned long long* __restrict__ cursor,
+                                                            uint32_t* __restrict__ keys_out,
+                                                            uint32_t* __restrict__ vals_out,
+                                                            uint32_t* __restrict__ pos_out) {
+    extern __shared__ unsigned long long base[];            // per-destination global base of this tile
+    unsigned* cnt = (unsigned*)(base + world);              // per-destination count / running rank
+    const uint64_t tile = (uint64_t)kThreads * kTileItems;
+    for (uint64_t t0 = (uint64_t)blockIdx.x * tile; t0 < n; t0 += (uint64_t)gridDim.x * tile) {
+        for (uint32_t w = threadIdx.x; w < world; w += blockDim.x) cnt[w] = 0;
+        __syncthreads();
+        uint32_t dd[kTileItems], rk[kTileItems];
+#pragma unroll
+        for (int j = 0; j < kTileItems; j++) {
+            const uint64_t i = t0 + (uint64_t)j * kThreads + threadIdx.x;
+            const bool valid = i < n;
+            dd[j] = valid ? dest(i) : 0xFFFFFFFFu;
+            rk[j] = warp_group_add(cnt, dd[j], valid);      // rank of this op within (tile, dest)
         }
+        __syncthreads();
+        for (uint32_t w = threadIdx.x; w < world; w += blockDim.x)
+            base[w] = cnt[w] ? atomicAdd(&cursor[w], (unsigned long long)cnt[w]) : 0ull;
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < kTileItems; j++) {
+            const uint64_t i = t0 + (uint64_t)j * kThreads + threadIdx.x;
+            if (dd[j] != 0xFFFFFFFFu) {
+                const uint64_t pos = base[dd[j]] + rk[j];
+                keys_out[pos] = keys[i];
+                if (vals_out) vals_out[pos] = vals_in ? vals_in[i] : 0u;
+                pos_out[i] = (uint32_t)pos;
+            }
+        }
+        __syncthreads();
     }
 }
 
-// Exclusive prefix sum of the per-shard counts into the scatter cursors (one block).
+// Exclusive prefix sum of the per-destination counts into the scatter cursors (one block).
 __global__ void k_route_offsets(const unsigned long long* __restrict__ counts, uint32_t world,
                                 unsigned long long* __restrict__ cursor) {
     if (threadIdx.x == 0) {
@@ -664,34 +699,6 @@ __global__ void k_route_offsets(const unsigned long long* __restrict__ counts, u
         for (uint32_t w = 0; w < world; w++) {
             cursor[w] = acc;
             acc += counts[w];
-        }
-    }
-}
-
-// Lanes bound for the same shard are grouped with __match_any_sync; one atomic
-// per group claims their positions.
-__global__ void __launch_bounds__(kThreads) k_route_scatter(uint32_t a, uint32_t b, uint64_t magic, uint32_t world,
-                                                            const uint32_t* __restrict__ keys,
-                                                            const uint32_t* __restrict__ vals_in, uint64_t n,
-                                                            unsigned long long* __restrict__ cursor,
-                                                            uint32_t* __restrict__ keys_out,
-                                                            uint32_t* __restrict__ vals_out,
-                                                            uint32_t* __restrict__ pos_out) {
-    for (uint64_t base = (uint64_t)blockIdx.x * blockDim.x; base < n; base += (uint64_t)gridDim.x * blockDim.x) {
-        const uint64_t i = base + threadIdx.x;
-        const bool valid = i < n;
-        const uint32_t k = valid ? keys[i] : 0u;
-        const uint32_t dest = valid ? fastmod(hx(a, b, k), magic, world) : 0xFFFFFFFFu;
-        const unsigned peers = __match_any_sync(kFull, dest);
-        const int leader = __ffs(peers) - 1;
-        unsigned long long p0 = 0;
-        if (valid && (int)(threadIdx.x & 31) == leader) p0 = atomicAdd(&cursor[dest], (unsigned long long)__popc(peers));
-        p0 = __shfl_sync(kFull, p0, leader);
-        if (valid) {
-            const uint64_t pos = p0 + __popc(peers & lanemask_lt());
-            keys_out[pos] = k;
-            if (vals_in && vals_out) vals_out[pos] = vals_in[i];
-            pos_out[i] = (uint32_t)pos;
         }
     }
 }

@@ -60,7 +60,7 @@ def test_dist_table_nccl_world1(oracle_mod):
         shard = Table(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=8)
         o = oracle_mod.OracleTable(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta,
                                    bucket_slots=8)
-        dt = DistTable(shard)
+        dt = DistTable(shard, force_route=True)
         np.testing.assert_array_equal(dt.insert(dev(ins.keys), dev(ins.values)).cpu().numpy(),
                                       o.insert(ins.keys, ins.values))
         v, f = dt.find(dev(fnd.keys))
