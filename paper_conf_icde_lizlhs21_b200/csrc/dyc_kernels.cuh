@@ -362,29 +362,88 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
 }
 
 // ------------------------------------------------------ insert phase 2 (S7)
-// Persistent grid-stride over list[0 .. *count) (count read on the device, so
-// no host round trip is needed between phase 1 and phase 2).  first_fit=false
-// skips the free-slot probe when the caller already found both buckets full
-// (pending keys of a FUSE upsert: nothing is deleted in between).
+// Persistent kernel over list[0 .. *count) (count read on the device, so no host
+// round trip is needed between phase 1 and phase 2).  Each warp owns a
+// contiguous range of the list; its lane groups pull the next key from that
+// range as soon as their current chain ends, so a long eviction chain does not
+// hold the other groups of the warp idle.  Per group a small state machine:
+//   phase 0/1 : first-fit probe of t1 / t2 (reading Q3; skipped when
+//               first_fit = false, i.e. the upsert already found both full),
+//   phase 2   : eviction hops: probe for a free slot (after the first hop), else
+//               exchange a pseudo-random victim (Q5) and carry it to the other
+//               table of ITS pair; after max_hops (Q6) the
+//               carried pair goes to the failure list.
 template <int B>
 __global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv, const unsigned long long* __restrict__ list,
                                                     const unsigned long long* count_ptr, uint64_t count_host,
                                                     unsigned long long* __restrict__ fail_list,
                                                     unsigned long long* __restrict__ ctr, bool first_fit) {
-    constexpr int G = B / 4, QPW = 32 / G;
+    constexpr int G = B / 4;
     __shared__ SmemView sv;
     load_view(tv, sv);
     const Grp<G> g;
-    const unsigned grp = g.lane / G;
     const uint64_t cnt = count_ptr ? *(volatile const unsigned long long*)count_ptr : count_host;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
-    uint32_t ev = 0;
-    for (uint64_t base = w * QPW; base < cnt; base += nwarps * QPW) {
-        const uint64_t i = base + grp;
-        unsigned long long kv = i < cnt ? list[i] : kEmptySlot;
-        const bool done = coop_place<B>(g, tv, sv, kv, i >= cnt, first_fit, ev);
-        warp_append(g.sub == 0 && !done, kv, fail_list, ctr + C_FAIL);
+    const uint64_t per = (cnt + nwarps - 1) / nwarps;
+    uint64_t next = w * per;
+    const uint64_t end = min(cnt, next + per);
+    unsigned long long kv = kEmptySlot;
+    uint32_t k = 0, t = 0, hop = 0, ev = 0;
+    int phase = -1;                       // -1 idle, 0/1 first-fit t1/t2, 2 evicting
+    for (;;) {
+        // refill idle groups from the warp's range (one ballot, no atomics)
+        const bool idle = phase < 0;
+        const unsigned want = __ballot_sync(kFull, idle && g.sub == 0);   // one bit per idle group leader
+        const uint64_t mine = next + __popc(want & ((1u << g.base) - 1u)); // idle leaders before this group
+        next += __popc(want);
+        if (idle && mine < end) {
+            kv = list[mine];
+            k = key_of(kv);
+            const Pair p = pair_of(tv, k);
+            phase = first_fit ? 0 : 2;
+            t = first_fit ? p.t1 : ((mix32(k) & 1u) ? p.t2 : p.t1);
+            hop = 0;
+        }
+        if (!__any_sync(kFull, phase >= 0)) break;
+        const bool act = phase >= 0;
+        unsigned long long* bp = bucket_ptr(sv, t, bucket_of(sv, t, k), B);
+        const bool try_free = act && (phase < 2 || hop > 0);
+        unsigned long long s[4] = {kEmptySlot, kEmptySlot, kEmptySlot, kEmptySlot};
+        probe_cg_pred<B>(bp + 4 * g.sub, s, try_free);
+        unsigned em[1] = {try_free ? empty_mask(s) : 0u};
+        unsigned long long* const bpa[1] = {bp};
+        const bool want1[1] = {try_free};
+        const unsigned long long kva[1] = {kv};
+        bool placed[1] = {false};
+        coop_cas_multi<G, 1>(g, bpa, em, want1, kva, placed);
+        const bool evict = act && !placed[0] && phase == 2;
+        const uint32_t victim = (mix32(k ^ (hop * 0x9E3779B9u)) >> 8) & (B - 1);
+        const unsigned owner = victim >> 2;
+        unsigned long long old = kEmptySlot;
+        if (evict && g.sub == owner) old = exch_slot(bp + victim, kv);
+        old = g.bcast(old, owner);
+        bool fail = false;
+        if (act && placed[0]) {
+            phase = -1;
+        } else if (act && phase < 2) {
+            const Pair p = pair_of(tv, k);
+            if (phase == 0) { phase = 1; t = p.t2; }
+            else { phase = 2; hop = 0; t = (mix32(k) & 1u) ? p.t2 : p.t1; }
+        } else if (evict) {
+            ev += (g.sub == 0);
+            hop++;
+            if (old == kEmptySlot) {
+                phase = -1;
+            } else {
+                kv = old;
+                k = key_of(kv);
+                const Pair q = pair_of(tv, k);
+                t = (t == q.t1) ? q.t2 : q.t1;
+                if (hop >= tv.max_hops) { fail = true; phase = -1; }
+            }
+        }
+        warp_append(g.sub == 0 && fail, kv, fail_list, ctr + C_FAIL);
     }
     block_add<kThreads>(ctr + C_EVICT, ev);
 }
