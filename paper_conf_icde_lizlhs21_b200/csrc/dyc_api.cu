@@ -70,7 +70,6 @@ struct dyc_table {
     int place_blocks = 148 * 8;            // persistent grid of k_place
     cudaMemPool_t pool = nullptr;
     unsigned long long* sub[DYC_MAX_D] = {};
-    unsigned* hint[DYC_MAX_D] = {};        // overflow-hint bitmaps, one bit per bucket
     uint64_t nb[DYC_MAX_D] = {};
     uint32_t a[DYC_MAX_D + 2] = {}, b[DYC_MAX_D + 2] = {};
     uint64_t m = 0;
@@ -123,7 +122,6 @@ struct dyc_table {
         TableView v{};
         for (uint32_t t = 0; t < cfg.d; t++) {
             v.sub[t].slots = sub[t];
-            v.sub[t].hint = hint[t];
             v.sub[t].n = (uint32_t)nb[t];
             v.sub[t].magic = fastmod_magic(nb[t]);
         }
@@ -211,28 +209,6 @@ dyc_status ensure_lists(dyc_table* t, uint64_t n, cudaStream_t st) {
     return DYC_OK;
 }
 
-inline uint64_t hint_bytes(uint64_t nb) { return ((nb + 31) / 32) * 4; }
-
-// The hint bitmap of subtable ti follows a size change n -> n_new (split when
-// doubling, OR-merge when halving).
-dyc_status resize_hints(dyc_table* t, uint32_t ti, uint64_t n_new, cudaStream_t st) {
-    const uint64_t n_old = t->nb[ti];
-    void* p = nullptr;
-    TRY(dev_alloc(t, &p, hint_bytes(n_new), st));
-    if (n_new == 2 * n_old) {
-        k_hint_split<<<grid_for((n_new + 31) / 32, 256), 256, 0, st>>>(t->hint[ti], (unsigned*)p, (uint32_t)n_old);
-    } else if (2 * n_new == n_old) {
-        k_hint_merge<<<grid_for((n_new + 31) / 32, 256), 256, 0, st>>>(t->hint[ti], (unsigned*)p, (uint32_t)n_new);
-    } else {
-        CU(cudaMemsetAsync(p, 0xFF, hint_bytes(n_new), st));   // unknown mapping: all bits set is always safe
-    }
-    t->launches++;
-    CU(cudaGetLastError());
-    CU(cudaFreeAsync(t->hint[ti], st));
-    t->hint[ti] = (unsigned*)p;
-    return DYC_OK;
-}
-
 template <int B>
 dyc_status upsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
     const uint64_t n_old = t->nb[ti], n_new = 2 * n_old;
@@ -247,7 +223,6 @@ dyc_status upsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
             (uint32_t)n_new);
     }
     CU(cudaGetLastError());
-    TRY(resize_hints(t, ti, n_new, st));
     CU(cudaFreeAsync(t->sub[ti], st));
     t->sub[ti] = (unsigned long long*)p;
     t->nb[ti] = n_new;
@@ -310,7 +285,6 @@ dyc_status downsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
                                                                        (uint32_t)h, t->list[0], t->d_ctr);
     }
     CU(cudaGetLastError());
-    TRY(resize_hints(t, ti, h, st));
     CU(cudaFreeAsync(t->sub[ti], st));
     t->sub[ti] = (unsigned long long*)p;
     t->nb[ti] = h;
@@ -590,7 +564,6 @@ dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaSt
         void* p = nullptr;
         TRY(dev_alloc(t, &p, nn * B * 8, st));
         CU(cudaMemsetAsync(p, 0xFF, nn * B * 8, st));
-        TRY(resize_hints(t, i, nn, st));
         old[i] = t->sub[i];
         old_nb[i] = t->nb[i];
         t->sub[i] = (unsigned long long*)p;
@@ -679,9 +652,7 @@ dyc_status stats_impl(dyc_table* t, dyc_stats_t* out, cudaStream_t st) {
     out->n_evict = t->n_evict;
     out->n_place_retry = t->n_place_retry;
     out->n_second_table = t->h_ctr[C_SECOND];
-    uint64_t hb = 0;
-    for (uint32_t i = 0; i < t->cfg.d; i++) hb += hint_bytes(t->nb[i]);
-    out->bytes_allocated = out->N * 8 + hb + 2 * t->list_cap * 8 + t->stage_cap + C_N * 8;
+    out->bytes_allocated = out->N * 8 + 2 * t->list_cap * 8 + t->stage_cap + C_N * 8;
     out->last_insert_new = t->last_new;
     out->last_insert_pending = t->last_pending;
     out->last_insert_evictions = t->last_evict;
@@ -828,12 +799,6 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
             t->nb[i] = per;
             if (cudaMemsetAsync(p, 0xFF, per * B * 8, nullptr) != cudaSuccess) s = cuda_err(cudaGetLastError(), "memset");
         }
-        void* hp = nullptr;
-        if (s == DYC_OK) s = dev_alloc(t, &hp, hint_bytes(per), nullptr);
-        if (s == DYC_OK) {
-            t->hint[i] = (unsigned*)hp;
-            if (cudaMemsetAsync(hp, 0, hint_bytes(per), nullptr) != cudaSuccess) s = cuda_err(cudaGetLastError(), "memset");
-        }
     }
     if (s == DYC_OK && cudaMalloc(&t->d_ctr, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMalloc");
     if (s == DYC_OK && cudaMallocHost(&t->h_ctr, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMallocHost");
@@ -862,8 +827,6 @@ dyc_status dyc_destroy(dyc_table* t) {
     cudaDeviceSynchronize();
     for (uint32_t i = 0; i < t->cfg.d; i++)
         if (t->sub[i]) cudaFree(t->sub[i]);
-    for (uint32_t i = 0; i < t->cfg.d; i++)
-        if (t->hint[i]) cudaFree(t->hint[i]);
     for (int i = 0; i < 2; i++)
         if (t->list[i]) cudaFree(t->list[i]);
     if (t->stage) cudaFree(t->stage);
@@ -967,10 +930,8 @@ dyc_status dyc_resize(dyc_table* t, int direction, int subtable, dyc_stream_t st
 
 dyc_status dyc_clear(dyc_table* t, dyc_stream_t stream) {
     TRY(enter(t, stream));
-    for (uint32_t i = 0; i < t->cfg.d; i++) {
+    for (uint32_t i = 0; i < t->cfg.d; i++)
         CU(cudaMemsetAsync(t->sub[i], 0xFF, t->nb[i] * t->cfg.bucket_slots * 8, S(stream)));
-        CU(cudaMemsetAsync(t->hint[i], 0, hint_bytes(t->nb[i]), S(stream)));
-    }
     t->m = 0;
     return DYC_OK;
 }

@@ -29,7 +29,6 @@ constexpr unsigned kFull = 0xFFFFFFFFu;
 // Per-launch view of the table (passed by value as a kernel parameter).
 struct SubView {
     unsigned long long* slots;   // n * B slots
-    unsigned* hint;              // n bits: "a key whose first choice is this bucket lives in its second table"
     uint64_t magic;              // fastmod magic for n
     uint32_t n;                  // buckets
     uint32_t pad;
@@ -99,28 +98,6 @@ __device__ __forceinline__ uint32_t bucket_of(const SmemView& s, uint32_t t, uin
 __device__ __forceinline__ unsigned long long* bucket_ptr(const SmemView& s, uint32_t t, uint32_t b, int B) {
     return s.sub[t].slots + (uint64_t)b * B;
 }
-
-// ---------------------------------------------------------------- overflow hints
-// One bit per bucket: set on bucket_t1(k) whenever a key k is
-// stored in the second table of its pair.  Invariant: every key living in its
-// t2 has its t1 bucket's bit set (bits are conservative: never cleared except by
-// clear(); split/OR-merged on resize).  A first-probe miss on a bucket whose bit
-// is clear proves the key is absent from t2, so the second lookup is skipped.
-// The bitmap (n_buckets/8 bytes, 2.5 MB at C2) stays resident in the 126 MB L2.
-__device__ __forceinline__ void hint_set(const SmemView& s, uint32_t t, uint32_t b) {
-    atomicOr(s.sub[t].hint + (b >> 5), 1u << (b & 31));
-}
-__device__ __forceinline__ unsigned hint_word_nc(const SmemView& s, uint32_t t, uint32_t b) {
-    unsigned w;
-    asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(w) : "l"(s.sub[t].hint + (b >> 5)));
-    return w;
-}
-__device__ __forceinline__ unsigned hint_word_cg(const SmemView& s, uint32_t t, uint32_t b) {
-    unsigned w;
-    asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(w) : "l"(s.sub[t].hint + (b >> 5)) : "memory");
-    return w;
-}
-__device__ __forceinline__ bool hint_bit(unsigned word, uint32_t b) { return (word >> (b & 31)) & 1u; }
 
 __device__ __forceinline__ uint32_t key_of(unsigned long long e) { return (uint32_t)e; }
 __device__ __forceinline__ uint32_t val_of(unsigned long long e) { return (uint32_t)(e >> 32); }

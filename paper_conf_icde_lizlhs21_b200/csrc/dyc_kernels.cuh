@@ -88,11 +88,37 @@ __device__ __forceinline__ uint32_t mix32(uint32_t x) {
     return x;
 }
 
+// First-fit CAS of kv into an EMPTY slot of the bucket whose group snapshot is s
+// (slot order).  Called by every lane of the warp (ballots); `want` is uniform
+// within a group.  A failed CAS means another key took that slot: try the next.
+template <int G>
+__device__ __forceinline__ bool coop_cas_empty(const Grp<G>& g, unsigned long long* bp,
+                                               const unsigned long long (&s)[4], bool want,
+                                               unsigned long long kv) {
+    unsigned emask = 0;
+#pragma unroll
+    for (int j = 0; j < 4; j++)
+        if (s[j] == kEmptySlot) emask |= 1u << j;
+    bool placed = false;
+    for (;;) {
+        const unsigned cand = g.ballot(want && !placed && emask != 0);
+        if (!__any_sync(kFull, cand != 0)) break;
+        const unsigned owner = first_lane(cand);
+        bool ok = false;
+        if (cand && g.sub == owner) {
+            const unsigned j = __ffs(emask) - 1;
+            ok = cas_slot(bp + 4 * g.sub + j, kEmptySlot, kv) == kEmptySlot;
+            emask &= ~(1u << j);
+        }
+        ok = __shfl_sync(kFull, ok, g.base + owner);
+        if (cand && ok) placed = true;
+    }
+    return placed;
+}
+
 // ----------------------------------------------------------------- find (S3)
-// ILP queries per group; all first probes (and their overflow-hint words, L2
-// resident) are issued back to back, then the second probes, predicated: only
-// after a first-probe miss on a bucket whose hint bit is set (<= 2 lookups,
-// P:L145; the hint only removes second lookups that cannot hit).
+// ILP queries per group; all first probes are issued back to back, then the
+// second probes (predicated, only after a first-probe miss: <= 2 lookups).
 template <int B, int ILP>
 __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, const uint32_t* __restrict__ keys,
                                                    uint32_t* __restrict__ vals, uint8_t* __restrict__ found,
@@ -106,7 +132,7 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     for (uint64_t base = w * wtile; base < n; base += nwarps * wtile) {
-        uint32_t k[ILP], v[ILP], b1[ILP], hw[ILP];
+        uint32_t k[ILP], v[ILP];
         bool f[ILP];
         const unsigned long long* p2[ILP];
         unsigned long long s[ILP][4];
@@ -118,10 +144,8 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
             const Pair p = pair_of(tv, k[j]);
-            b1[j] = bucket_of(sv, p.t1, k[j]);
             p2[j] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[j]), B) + 4 * g.sub;
-            probe_nc<B>(bucket_ptr(sv, p.t1, b1[j], B) + 4 * g.sub, s[j]);
-            hw[j] = hint_word_nc(sv, p.t1, b1[j]);
+            probe_nc<B>(bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[j]), B) + 4 * g.sub, s[j]);
         }
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
@@ -132,12 +156,11 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
             v[j] = g.bcast32(lv, first_lane(hb));
         }
 #pragma unroll
-        for (int j = 0; j < ILP; j++)
-            probe_nc_pred<B>(p2[j], s[j], !f[j] && k[j] != kEmptyKey && hint_bit(hw[j], b1[j]));
+        for (int j = 0; j < ILP; j++) probe_nc_pred<B>(p2[j], s[j], !f[j] && k[j] != kEmptyKey);
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
             uint32_t lv = 0;
-            const bool lh = !f[j] && k[j] != kEmptyKey && hint_bit(hw[j], b1[j]) && lookup_slot<4>(s[j], k[j], lv);
+            const bool lh = !f[j] && k[j] != kEmptyKey && lookup_slot<4>(s[j], k[j], lv);
             const unsigned hb = g.ballot(lh);
             const uint32_t v2 = g.bcast32(lv, first_lane(hb));
             if (hb) { f[j] = true; v[j] = v2; }
@@ -150,19 +173,59 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
     }
 }
 
-__device__ __forceinline__ unsigned empty_mask(const unsigned long long (&s)[4]) {
-    unsigned m = 0;
-#pragma unroll
-    for (int j = 0; j < 4; j++)
-        if (s[j] == kEmptySlot) m |= 1u << j;
-    return m;
+// ------------------------------------------------------- placement (S7 core)
+// Cuckoo placement of a pair known to be absent, by one lane group.  First-fit
+// over the ordered pair (reading Q3); then an eviction chain: exchange with a
+// pseudo-random victim slot (Q5) and carry the victim to the OTHER table of ITS
+// pair.  Every pair is held by exactly one group or one slot at
+// any time (atomicExch), so nothing is lost or duplicated.  After max_hops hops
+// (Q6) the carried pair is returned as homeless.  Returns true when placed;
+// groups that enter with done == true only take part in the ballots.
+template <int B>
+__device__ __forceinline__ bool coop_place(const Grp<B / 4>& g, const TableView& tv, const SmemView& sv,
+                                           unsigned long long& kv, bool done, bool first_fit, uint32_t& ev) {
+    uint32_t k = key_of(kv);
+    const Pair p = pair_of(tv, k);
+    unsigned long long s[4] = {kEmptySlot, kEmptySlot, kEmptySlot, kEmptySlot};
+    if (first_fit) {
+        unsigned long long* b1 = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k), B);
+        probe_cg_pred<B>(b1 + 4 * g.sub, s, !done);
+        done |= coop_cas_empty(g, b1, s, !done, kv);
+        unsigned long long* b2 = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k), B);
+        probe_cg_pred<B>(b2 + 4 * g.sub, s, !done);
+        done |= coop_cas_empty(g, b2, s, !done, kv);
+    }
+    uint32_t t = (mix32(k) & 1u) ? p.t2 : p.t1;
+    for (uint32_t hop = 0; hop < tv.max_hops; hop++) {
+        if (!__any_sync(kFull, !done)) break;
+        unsigned long long* bp = bucket_ptr(sv, t, bucket_of(sv, t, k), B);
+        if (hop > 0) {
+            probe_cg_pred<B>(bp + 4 * g.sub, s, !done);
+            done |= coop_cas_empty(g, bp, s, !done, kv);
+        }
+        const uint32_t victim = (mix32(k ^ (hop * 0x9E3779B9u)) >> 8) & (B - 1);
+        const unsigned owner = victim >> 2;
+        unsigned long long old = kEmptySlot;
+        if (!done && g.sub == owner) old = exch_slot(bp + victim, kv);
+        old = g.bcast(old, owner);
+        if (!done) {
+            ev += (g.sub == 0);
+            if (old == kEmptySlot) {
+                done = true;
+            } else {
+                kv = old;
+                k = key_of(kv);
+                const Pair q = pair_of(tv, k);
+                t = (t == q.t1) ? q.t2 : q.t1;
+            }
+        }
+    }
+    return done;
 }
 
-// First-fit CAS for U independent ops of a group at once (slot order within the
-// bucket; a failed CAS means another key took that slot: try the next).  Each
-// round every op that still has a candidate EMPTY slot issues one CAS, all U in
-// flight together.  Called by every lane of the warp (ballots); want[u] is
-// uniform within a group.
+// First-fit CAS for U independent ops of a group at once: each round, every op
+// that still has a candidate EMPTY slot issues one CAS (all U in flight
+// together), so the atomic round trips of different ops overlap.
 template <int G, int U>
 __device__ __forceinline__ void coop_cas_multi(const Grp<G>& g, unsigned long long* const (&bp)[U],
                                                unsigned (&em)[U], const bool (&want)[U],
@@ -194,17 +257,23 @@ __device__ __forceinline__ void coop_cas_multi(const Grp<G>& g, unsigned long lo
     }
 }
 
+__device__ __forceinline__ unsigned empty_mask(const unsigned long long (&s)[4]) {
+    unsigned m = 0;
+#pragma unroll
+    for (int j = 0; j < 4; j++)
+        if (s[j] == kEmptySlot) m |= 1u << j;
+    return m;
+}
+
 // ------------------------------------------------------ insert phase 1 (S5)
-// Upsert: probe t1's bucket, then (only if the key is not there and the bucket's
-// overflow hint says a key may have spilled to its second table, or FUSE needs
-// t2's free slots) t2's; an existing key gets its value replaced (Alg. 1
-// L536-539, status UPDATED).  A new key (status INSERTED) is, with FUSE,
-// CAS-ed into a free slot of its first-fit bucket right away (storing into t2
-// sets t1's hint bit); otherwise (or if both candidate buckets are full) it is
-// appended to `pending` for k_place.  Keys never move during this kernel (no
-// evictions), so the existence check is exact; FUSE is only used when no upsize
-// can be needed ((m+n) <= beta*N).  Each group carries U ops whose probes are
-// issued together (the kernel is bound by random line requests).
+// Upsert: probe t1's bucket, then t2's; an existing key gets its value replaced
+// (Alg. 1, status UPDATED).  A new key (status INSERTED) is, with FUSE,
+// CAS-ed into a free slot of its first-fit bucket right away; otherwise (or if
+// both candidate buckets are full) it is appended to `pending` for k_place.
+// Keys never move during this kernel (no evictions), so the existence check is
+// exact; FUSE is only used when no upsize can be needed ((m+n) <= beta*N).
+// Each group carries U ops whose probes are issued together (memory-level
+// parallelism: the kernel is bound by random line requests).
 template <int B, bool FUSE, int U>
 __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView tv, const uint32_t* __restrict__ keys,
                                                      const uint32_t* __restrict__ vals,
@@ -220,14 +289,14 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     unsigned long long n_ins = 0, n_upd = 0;
     for (uint64_t base = w * (QPW * U); base < n; base += nwarps * (QPW * U)) {
-        // per op only the match position, the free-slot mask of each bucket and
-        // the hint bit are kept, not the 4-slot snapshots (registers -> more ops in flight)
+        // per op only the match position and the free-slot mask of each bucket
+        // are kept, not the 4-slot snapshots (register budget -> more ops in flight)
         uint64_t i[U];
-        uint32_t k[U], t1[U], b1i[U];
+        uint32_t k[U];
         unsigned long long kv[U];
         unsigned long long* b1[U];
         unsigned long long* b2[U];
-        unsigned h1[U], h2[U], em1[U], em2[U], hw[U];
+        unsigned h1[U], h2[U], em1[U], em2[U];
         bool need2[U], isnew[U], placed[U];
         int j1[U], j2[U];
         {
@@ -239,12 +308,9 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                 k[u] = valid ? __ldg(keys + i[u]) : kEmptyKey;
                 kv[u] = make_kv(k[u], valid ? __ldg(vals + i[u]) : 0u);
                 const Pair p = pair_of(tv, k[u]);
-                t1[u] = p.t1;
-                b1i[u] = bucket_of(sv, p.t1, k[u]);
-                b1[u] = bucket_ptr(sv, p.t1, b1i[u], B);
+                b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
                 b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
                 probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
-                hw[u] = hint_word_cg(sv, p.t1, b1i[u]);
             }
 #pragma unroll
             for (int u = 0; u < U; u++) {
@@ -258,35 +324,28 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
             for (int u = 0; u < U; u++) {
                 const bool active = k[u] != kEmptyKey;
                 h1[u] = g.ballot(active && j1[u] >= 0);
-                const bool t1_full = g.ballot(em1[u] != 0) == 0;
-                need2[u] = active && h1[u] == 0 && (hint_bit(hw[u], b1i[u]) || (FUSE && t1_full));
+                need2[u] = active && h1[u] == 0;
 #pragma unroll
                 for (int q = 0; q < 4; q++) s2[u][q] = kEmptySlot;
                 probe_cg_pred<B>(b2[u] + 4 * g.sub, s2[u], need2[u]);
             }
 #pragma unroll
             for (int u = 0; u < U; u++) {
-                j2[u] = need2[u] ? match_slot<4>(s2[u], k[u]) : -1;
-                em2[u] = need2[u] ? empty_mask(s2[u]) : 0u;
+                j2[u] = match_slot<4>(s2[u], k[u]);
+                em2[u] = empty_mask(s2[u]);
             }
         }
 #pragma unroll
         for (int u = 0; u < U; u++) {
-            h2[u] = g.ballot(j2[u] >= 0);
+            h2[u] = g.ballot(need2[u] && j2[u] >= 0);
             if (h1[u] && g.sub == first_lane(h1[u])) st_u64_cg(b1[u] + 4 * g.sub + j1[u], kv[u]);
             if (h2[u] && g.sub == first_lane(h2[u])) st_u64_cg(b2[u] + 4 * g.sub + j2[u], kv[u]);
-            isnew[u] = k[u] != kEmptyKey && h1[u] == 0 && h2[u] == 0;
+            isnew[u] = need2[u] && h2[u] == 0;
             placed[u] = false;
         }
         if (FUSE) {
             coop_cas_multi<G, U>(g, b1, em1, isnew, kv, placed);
-            bool p1[U];
-#pragma unroll
-            for (int u = 0; u < U; u++) p1[u] = placed[u];
             coop_cas_multi<G, U>(g, b2, em2, isnew, kv, placed);
-#pragma unroll
-            for (int u = 0; u < U; u++)
-                if (placed[u] && !p1[u] && g.sub == 0) hint_set(sv, t1[u], b1i[u]);   // stored in its t2
         }
         const bool lead = g.sub == 0;
 #pragma unroll
@@ -303,29 +362,27 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
 }
 
 // ------------------------------------------------------ insert phase 2 (S7)
-// Persistent kernel over a list (count read on the device, so no host round
-// trip is needed between phase 1 and phase 2).  Each warp owns a contiguous
-// range of the list; its lane groups pull the next key from that range as soon
-// as their current chain ends, so a long eviction chain does not hold the other
-// groups of the warp idle.  Per group a small state machine:
+// Persistent kernel over list[0 .. *count) (count read on the device, so no host
+// round trip is needed between phase 1 and phase 2).  Each warp owns a
+// contiguous range of the list; its lane groups pull the next key from that
+// range as soon as their current chain ends, so a long eviction chain does not
+// hold the other groups of the warp idle.  Per group a small state machine:
 //   phase 0/1 : first-fit probe of t1 / t2 (reading Q3; skipped when
 //               first_fit = false, i.e. the upsert already found both full),
 //   phase 2   : eviction hops: probe for a free slot (after the first hop), else
 //               exchange a pseudo-random victim (Q5) and carry it to the other
 //               table of ITS pair; after max_hops (Q6) the
 //               carried pair goes to the failure list.
-// Every pair is held by exactly one group or one slot at any time (atomicExch),
-// so nothing is lost or duplicated.  A pair stored in the second table of its
-// pair sets its first-choice bucket's hint bit.  SLOTS = true reads a detached
-// subtable buffer and skips its EMPTY slots (the resize baselines of P:L736 and
-// P:L809 re-insert through this kernel).
-template <int B, bool SLOTS>
-__device__ __forceinline__ void place_list(const TableView& tv, const SmemView& sv,
-                                           const unsigned long long* __restrict__ list, uint64_t cnt,
-                                           unsigned long long* __restrict__ fail_list,
-                                           unsigned long long* __restrict__ ctr, bool first_fit) {
+template <int B>
+__global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv, const unsigned long long* __restrict__ list,
+                                                    const unsigned long long* count_ptr, uint64_t count_host,
+                                                    unsigned long long* __restrict__ fail_list,
+                                                    unsigned long long* __restrict__ ctr, bool first_fit) {
     constexpr int G = B / 4;
+    __shared__ SmemView sv;
+    load_view(tv, sv);
     const Grp<G> g;
+    const uint64_t cnt = count_ptr ? *(volatile const unsigned long long*)count_ptr : count_host;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     const uint64_t per = (cnt + nwarps - 1) / nwarps;
@@ -342,22 +399,15 @@ __device__ __forceinline__ void place_list(const TableView& tv, const SmemView& 
         next += __popc(want);
         if (idle && mine < end) {
             kv = list[mine];
-            if (!SLOTS || kv != kEmptySlot) {
-                k = key_of(kv);
-                const Pair p = pair_of(tv, k);
-                phase = first_fit ? 0 : 2;
-                t = first_fit ? p.t1 : ((mix32(k) & 1u) ? p.t2 : p.t1);
-                hop = 0;
-            }
+            k = key_of(kv);
+            const Pair p = pair_of(tv, k);
+            phase = first_fit ? 0 : 2;
+            t = first_fit ? p.t1 : ((mix32(k) & 1u) ? p.t2 : p.t1);
+            hop = 0;
         }
-        if (!__any_sync(kFull, phase >= 0)) {
-            if (!__any_sync(kFull, next < end)) break;   // SLOTS: all remaining entries may be EMPTY
-            continue;
-        }
+        if (!__any_sync(kFull, phase >= 0)) break;
         const bool act = phase >= 0;
-        const Pair pk = pair_of(tv, k);
-        const uint32_t bk = bucket_of(sv, t, k);
-        unsigned long long* bp = bucket_ptr(sv, t, bk, B);
+        unsigned long long* bp = bucket_ptr(sv, t, bucket_of(sv, t, k), B);
         const bool try_free = act && (phase < 2 || hop > 0);
         unsigned long long s[4] = {kEmptySlot, kEmptySlot, kEmptySlot, kEmptySlot};
         probe_cg_pred<B>(bp + 4 * g.sub, s, try_free);
@@ -373,14 +423,13 @@ __device__ __forceinline__ void place_list(const TableView& tv, const SmemView& 
         unsigned long long old = kEmptySlot;
         if (evict && g.sub == owner) old = exch_slot(bp + victim, kv);
         old = g.bcast(old, owner);
-        // kv now lives in table t (CAS or exchange): second choice -> hint on its t1 bucket
-        if ((placed[0] || evict) && t == pk.t2 && g.sub == 0) hint_set(sv, pk.t1, bucket_of(sv, pk.t1, k));
         bool fail = false;
         if (act && placed[0]) {
             phase = -1;
         } else if (act && phase < 2) {
-            if (phase == 0) { phase = 1; t = pk.t2; }
-            else { phase = 2; hop = 0; t = (mix32(k) & 1u) ? pk.t2 : pk.t1; }
+            const Pair p = pair_of(tv, k);
+            if (phase == 0) { phase = 1; t = p.t2; }
+            else { phase = 2; hop = 0; t = (mix32(k) & 1u) ? p.t2 : p.t1; }
         } else if (evict) {
             ev += (g.sub == 0);
             hop++;
@@ -399,30 +448,32 @@ __device__ __forceinline__ void place_list(const TableView& tv, const SmemView& 
     block_add<kThreads>(ctr + C_EVICT, ev);
 }
 
+// Reinsert every live slot of a detached buffer through the insert path (the
+// resize baselines of P:L736 and P:L809).
 template <int B>
-__global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv, const unsigned long long* __restrict__ list,
-                                                    const unsigned long long* count_ptr, uint64_t count_host,
-                                                    unsigned long long* __restrict__ fail_list,
-                                                    unsigned long long* __restrict__ ctr, bool first_fit) {
-    __shared__ SmemView sv;
-    load_view(tv, sv);
-    const uint64_t cnt = count_ptr ? *(volatile const unsigned long long*)count_ptr : count_host;
-    place_list<B, false>(tv, sv, list, cnt, fail_list, ctr, first_fit);
-}
-
-template <int B>
-__global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_reinsert(TableView tv, const unsigned long long* __restrict__ slots,
+__global__ void __launch_bounds__(kThreads) k_reinsert(TableView tv, const unsigned long long* __restrict__ slots,
                                                        uint64_t nslots, unsigned long long* __restrict__ fail_list,
                                                        unsigned long long* __restrict__ ctr) {
+    constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
-    place_list<B, true>(tv, sv, slots, nslots, fail_list, ctr, true);
+    const Grp<G> g;
+    const unsigned grp = g.lane / G;
+    const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
+    const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
+    uint32_t ev = 0;
+    for (uint64_t base = w * QPW; base < nslots; base += nwarps * QPW) {
+        const uint64_t i = base + grp;
+        unsigned long long kv = i < nslots ? slots[i] : kEmptySlot;
+        const bool done = coop_place<B>(g, tv, sv, kv, kv == kEmptySlot, true, ev);
+        warp_append(g.sub == 0 && !done, kv, fail_list, ctr + C_FAIL);
+    }
+    block_add<kThreads>(ctr + C_EVICT, ev);
 }
 
 // ------------------------------------------------------------- delete (S4)
-// Probe t1, then t2 if the hint allows; the lane holding the key overwrites its
-// slot with EMPTY (no lock: keys in a batch are distinct).  Hint bits
-// are left set (conservative).  U ops per group in flight.
+// Probe t1 then t2; the lane holding the key overwrites its slot with EMPTY (no
+// lock: keys in a batch are distinct).  U ops per group in flight.
 template <int B, int U>
 __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView tv, const uint32_t* __restrict__ keys,
                                                      uint32_t* __restrict__ old_vals,
@@ -438,7 +489,7 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
     unsigned long long removed = 0;
     for (uint64_t base = w * (QPW * U); base < n; base += nwarps * (QPW * U)) {
         uint64_t i[U];
-        uint32_t k[U], b1i[U], hw[U];
+        uint32_t k[U];
         unsigned long long s1[U][4], s2[U][4];
         unsigned long long* b1[U];
         unsigned long long* b2[U];
@@ -450,18 +501,16 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
             i[u] = base + (uint64_t)u * QPW + grp;
             k[u] = i[u] < n ? __ldg(keys + i[u]) : kEmptyKey;
             const Pair p = pair_of(tv, k[u]);
-            b1i[u] = bucket_of(sv, p.t1, k[u]);
-            b1[u] = bucket_ptr(sv, p.t1, b1i[u], B);
+            b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
             b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
             probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
-            hw[u] = hint_word_cg(sv, p.t1, b1i[u]);
         }
 #pragma unroll
         for (int u = 0; u < U; u++) {
             const bool active = k[u] != kEmptyKey;
             j1[u] = active ? match_slot<4>(s1[u], k[u]) : -1;
             h1[u] = g.ballot(j1[u] >= 0);
-            need2[u] = active && h1[u] == 0 && hint_bit(hw[u], b1i[u]);
+            need2[u] = active && h1[u] == 0;
 #pragma unroll
             for (int q = 0; q < 4; q++) s2[u][q] = kEmptySlot;
             probe_cg_pred<B>(b2[u] + 4 * g.sub, s2[u], need2[u]);
@@ -486,38 +535,6 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
         }
     }
     block_add<kThreads>(ctr + C_REMOVED, removed);
-}
-
-// Hint bitmaps follow their subtable through a resize (bits are conservative):
-// doubling copies bit b to b and b+n, halving ORs b' and b'+h.
-__global__ void k_hint_split(const unsigned* __restrict__ oldh, unsigned* __restrict__ newh, uint32_t n_old) {
-    const uint64_t n_new = 2ull * n_old;
-    for (uint64_t wd = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; wd < (n_new + 31) / 32;
-         wd += (uint64_t)gridDim.x * blockDim.x) {
-        unsigned out = 0;
-        for (uint32_t j = 0; j < 32; j++) {
-            const uint64_t b = wd * 32 + j;
-            if (b >= n_new) break;
-            const uint64_t ob = b % n_old;
-            out |= ((oldh[ob >> 5] >> (ob & 31)) & 1u) << j;
-        }
-        newh[wd] = out;
-    }
-}
-
-__global__ void k_hint_merge(const unsigned* __restrict__ oldh, unsigned* __restrict__ newh, uint32_t h) {
-    for (uint64_t wd = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; wd < ((uint64_t)h + 31) / 32;
-         wd += (uint64_t)gridDim.x * blockDim.x) {
-        unsigned out = 0;
-        for (uint32_t j = 0; j < 32; j++) {
-            const uint64_t b = wd * 32 + j;
-            if (b >= h) break;
-            const uint64_t c = b + h;
-            const unsigned bit = ((oldh[b >> 5] >> (b & 31)) | (oldh[c >> 5] >> (c & 31))) & 1u;
-            out |= bit << j;
-        }
-        newh[wd] = out;
-    }
 }
 
 // ------------------------------------------------------------- upsize (S8)
