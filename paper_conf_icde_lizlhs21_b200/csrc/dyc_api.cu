@@ -380,7 +380,7 @@ dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals,
 template <int B>
 dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* found, uint64_t n,
                      cudaStream_t st) {
-    constexpr int ILP = (B <= 16) ? 4 : 2;
+    constexpr int ILP = (B <= 16) ? DYC_FIND_ILP : 2;
     constexpr uint64_t per_block = (uint64_t)(kThreads / (B / 4)) * ILP;   // queries per block per pass
     {
         ProfScope ps(t, DYC_PROF_FIND, st);

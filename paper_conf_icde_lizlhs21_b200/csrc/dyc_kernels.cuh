@@ -38,6 +38,9 @@ constexpr int kThreads = 256;
 #ifndef DYC_DELETE_U
 #define DYC_DELETE_U 2
 #endif
+#ifndef DYC_FIND_ILP
+#define DYC_FIND_ILP 4
+#endif
 
 enum CounterIdx : int {
     C_PENDING = 0,    // new keys handed to k_place
