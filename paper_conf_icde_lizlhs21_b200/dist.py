@@ -27,7 +27,13 @@ def _torch():
 
 
 class DistTable:
-    def __init__(self, shard, group=None, force_route: bool = False):
+    """Routes single-type batches to the owning shards.  The batch is split into
+    `chunks` pieces that are pipelined: the all-to-all of chunk c+1 (NCCL stream)
+    runs while the owner executes chunk c (compute stream), and the replies of
+    chunk c travel back while chunk c+1 executes.  Each rank must use the same
+    `chunks` (collectives are issued in the same order everywhere)."""
+
+    def __init__(self, shard, group=None, force_route: bool = False, chunks: int = 4):
         import torch.distributed as dist
         self.force_route = force_route
         self.dist = dist
@@ -35,35 +41,70 @@ class DistTable:
         self.world = dist.get_world_size(group)
         self.rank = dist.get_rank(group)
         self.shard = shard
+        self.chunks = max(1, int(chunks))
+        self.last_recv = 0
 
     # ------------------------------------------------------------ exchange
-    def _splits(self, counts) -> Tuple[List[int], List[int]]:
-        torch = _torch()
-        recv = torch.empty_like(counts)
-        self.dist.all_to_all_single(recv, counts, group=self.group)
-        both = torch.stack([counts, recv]).cpu()
-        return both[0].tolist(), both[1].tolist()
-
-    def _a2a(self, x, send_splits, recv_splits):
+    def _a2a(self, x, send_splits, recv_splits, async_op=False):
         torch = _torch()
         out = torch.empty(sum(recv_splits), dtype=x.dtype, device=x.device)
-        self.dist.all_to_all_single(out, x, recv_splits, send_splits, group=self.group)
-        return out
+        w = self.dist.all_to_all_single(out, x, recv_splits, send_splits, group=self.group, async_op=async_op)
+        return out, w
 
-    def _route(self, keys, values=None):
-        counts = self.shard.route_count(keys, self.world)
-        kout, vout, pos = self.shard.route_scatter(keys, values, self.world, counts)
-        send, recv = self._splits(counts)
-        self.last_recv = sum(recv)
-        rk = self._a2a(kout, send, recv)
-        rv = self._a2a(vout, send, recv) if values is not None else None
-        return rk, rv, pos, send, recv
-
-    def _reply(self, pos, send, recv, vals=None, status=None):
-        # replies travel back with the splits reversed
-        bv = self._a2a(vals, recv, send) if vals is not None else None
-        bs = self._a2a(status, recv, send) if status is not None else None
-        return self.shard.route_unpermute(pos, bv, bs)
+    def _run(self, op, keys, values=None, n_out=1):
+        """Pipelined route -> all-to-all -> owner op -> all-to-all back -> unpermute.
+        op(keys, values) returns a tuple of n_out per-op result tensors."""
+        torch = _torch()
+        n = keys.numel()
+        C, W = self.chunks, self.world
+        bounds = [n * c // C for c in range(C + 1)]
+        parts, counts = [], []
+        for c in range(C):
+            kc = keys[bounds[c]:bounds[c + 1]]
+            vc = values[bounds[c]:bounds[c + 1]] if values is not None else None
+            cnt = self.shard.route_count(kc, W)
+            parts.append(self.shard.route_scatter(kc, vc, W, cnt))
+            counts.append(cnt)
+        # one exchange of every chunk's per-destination counts (row w: counts for rank w)
+        send = torch.stack(counts).t().contiguous()
+        recv = torch.empty_like(send)
+        self.dist.all_to_all_single(recv, send, group=self.group)
+        both = torch.stack([send, recv]).cpu()
+        ssp = [both[0][:, c].tolist() for c in range(C)]
+        rsp = [both[1][:, c].tolist() for c in range(C)]
+        self.last_recv = int(both[1].sum())
+        fwd = []
+        for c in range(C):
+            kout, vout, _ = parts[c]
+            rk, wk = self._a2a(kout, ssp[c], rsp[c], async_op=True)
+            rv, wv = self._a2a(vout, ssp[c], rsp[c], async_op=True) if values is not None else (None, None)
+            fwd.append((rk, wk, rv, wv))
+        back = []
+        for c in range(C):
+            rk, wk, rv, wv = fwd[c]
+            wk.wait()
+            if wv is not None:
+                wv.wait()
+            res = op(rk, rv)
+            res = res if isinstance(res, tuple) else (res,)
+            back.append([self._a2a(r, rsp[c], ssp[c], async_op=True) for r in res])
+        outs = [None] * n_out
+        pieces = [[] for _ in range(n_out)]
+        for c in range(C):
+            for (r, w) in back[c]:
+                w.wait()
+            _, _, pos = parts[c]
+            got = [r for (r, _) in back[c]]
+            if n_out == 1:
+                _, s = self.shard.route_unpermute(pos, None, got[0])
+                pieces[0].append(s)
+            else:
+                v, s = self.shard.route_unpermute(pos, got[0], got[1])
+                pieces[0].append(v)
+                pieces[1].append(s)
+        for j in range(n_out):
+            outs[j] = pieces[j][0] if C == 1 else torch.cat(pieces[j])
+        return outs[0] if n_out == 1 else tuple(outs)
 
     # ------------------------------------------------------------ batches
     # With one rank there is nothing to exchange: the batch goes straight to the
@@ -73,28 +114,21 @@ class DistTable:
         if self.world == 1 and not self.force_route:
             self.last_recv = keys.numel()
             return self.shard.insert(keys, values)
-        rk, rv, pos, send, recv = self._route(keys, values)
-        st = self.shard.insert(rk, rv)
-        _, s = self._reply(pos, send, recv, status=st)
-        return s
+        return self._run(lambda k, v: self.shard.insert(k, v), keys, values, n_out=1)
 
     def find(self, keys):
         """Returns (values int32-as-uint32, found uint8) in request order."""
         if self.world == 1 and not self.force_route:
             self.last_recv = keys.numel()
             return self.shard.find(keys)
-        rk, _, pos, send, recv = self._route(keys)
-        v, f = self.shard.find(rk)
-        return self._reply(pos, send, recv, vals=v, status=f)
+        return self._run(lambda k, v: self.shard.find(k), keys, None, n_out=2)
 
     def delete(self, keys):
         """Returns (old values, status) in request order."""
         if self.world == 1 and not self.force_route:
             self.last_recv = keys.numel()
             return self.shard.delete(keys)
-        rk, _, pos, send, recv = self._route(keys)
-        v, s = self.shard.delete(rk)
-        return self._reply(pos, send, recv, vals=v, status=s)
+        return self._run(lambda k, v: self.shard.delete(k), keys, None, n_out=2)
 
     def stats(self):
         return self.shard.stats()

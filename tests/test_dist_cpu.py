@@ -81,12 +81,12 @@ def _batches(world, nb=6, per=200, seed=3):
     return out
 
 
-def _worker(rank, world, port, q):
+def _worker(rank, world, port, q, chunks):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     from paper_conf_icde_lizlhs21_b200.dist import DistTable
-    dt = DistTable(DictShard())
+    dt = DistTable(DictShard(), chunks=chunks)
     model = {}
     ok = True
     for op, ks, vs in _batches(world):
@@ -124,12 +124,12 @@ def _free_port():
     return p
 
 
-@pytest.mark.parametrize("world", [2])
-def test_router_orchestration_gloo(world):
+@pytest.mark.parametrize("world,chunks", [(2, 1), (2, 3), (3, 4)])
+def test_router_orchestration_gloo(world, chunks):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q, chunks)) for r in range(world)]
     for p in procs:
         p.start()
     res = dict(q.get(timeout=240) for _ in range(world))
