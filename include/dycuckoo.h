@@ -134,6 +134,21 @@ dyc_status dyc_destroy(dyc_table* t);
 dyc_status dyc_insert_batch(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_values,
                             uint8_t* d_status, uint64_t n, dyc_stream_t stream);
 
+/* One insert batch delivered in parts (e.g. as shards of it arrive over the
+ * network): dyc_insert_begin(n_total), then dyc_insert_part() for parts whose
+ * sizes sum to at most n_total, then dyc_insert_end().  Equivalent to one
+ * dyc_insert_batch over the concatenation of the parts: one resize decision, one
+ * alpha check.  The same for deletes.  No other call on the table
+ * may come between begin and end. */
+dyc_status dyc_insert_begin(dyc_table* t, uint64_t n_total, dyc_stream_t stream);
+dyc_status dyc_insert_part(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_values,
+                           uint8_t* d_status, uint64_t n, dyc_stream_t stream);
+dyc_status dyc_insert_end(dyc_table* t, dyc_stream_t stream);
+dyc_status dyc_delete_begin(dyc_table* t, uint64_t n_total, dyc_stream_t stream);
+dyc_status dyc_delete_part(dyc_table* t, const uint32_t* d_keys, uint32_t* d_values_out,
+                           uint8_t* d_status, uint64_t n, dyc_stream_t stream);
+dyc_status dyc_delete_end(dyc_table* t, dyc_stream_t stream);
+
 /* Batched find (§V-B "Find"): at most two bucket probes per key.
  * d_values_out[n]: the value, or DYC_NOT_FOUND on a miss ("NULL").
  * d_found[n] (nullable): DYC_OP_FOUND or DYC_OP_NONE.  Never synchronizes. */
@@ -229,7 +244,7 @@ dyc_status dyc_profile_read(dyc_table* t, double* ms, uint64_t* calls);
  * ------------------------------------------------------------------------- */
 
 /* Counts ops per destination shard: d_counts[world] (uint64, device) receives
- * the histogram.  `t` supplies the hash constants (all ranks use one seed). */
+ * the histogram (world in 1..1024).  `t` supplies the hash constants (all ranks use one seed). */
 dyc_status dyc_route_count(dyc_table* t, const uint32_t* d_keys, uint64_t n, uint32_t world,
                            uint64_t* d_counts, dyc_stream_t stream);
 

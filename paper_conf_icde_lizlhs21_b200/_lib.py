@@ -58,6 +58,12 @@ SIGNATURES = {
     "dyc_destroy": (_I, [_TP]),
     "dyc_insert_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
     "dyc_find_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
+    "dyc_insert_begin": (_I, [_TP, _U64, _P]),
+    "dyc_insert_part": (_I, [_TP, _P, _P, _P, _U64, _P]),
+    "dyc_insert_end": (_I, [_TP, _P]),
+    "dyc_delete_begin": (_I, [_TP, _U64, _P]),
+    "dyc_delete_part": (_I, [_TP, _P, _P, _P, _U64, _P]),
+    "dyc_delete_end": (_I, [_TP, _P]),
     "dyc_delete_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
     "dyc_mixed_batch": (_I, [_TP, _P, _P, _P, _P, _P, _U64, _P]),
     "dyc_resize": (_I, [_TP, _I, _I, _P]),

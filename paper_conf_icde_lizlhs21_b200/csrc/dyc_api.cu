@@ -80,6 +80,9 @@ struct dyc_table {
     void* stage = nullptr;                 // device staging for the host-buffer entry points
     uint64_t stage_cap = 0;
     cudaStream_t cp_in = nullptr, cp_out = nullptr;   // copy streams of the host-buffer path
+    int part_op = 0;                       // 1 insert / 2 delete batch open (dyc_*_begin)
+    bool part_fuse = false;
+    uint64_t part_left = 0;
     void* mix = nullptr;                   // scratch of dyc_mixed_batch
     uint64_t mix_cap = 0;
     uint64_t n_upsize = 0, n_downsize = 0, n_fail_upsize = 0, n_residual = 0, n_evict = 0, n_place_retry = 0;
@@ -851,6 +854,66 @@ dyc_status dyc_insert_batch(dyc_table* t, const uint32_t* d_keys, const uint32_t
     DISPATCH_B(t, insert_impl<B_>(t, d_keys, d_values, d_status, n, S(stream)));
 }
 
+dyc_status dyc_insert_begin(dyc_table* t, uint64_t n_total, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (t->part_op) return set_err(DYC_ERR_INVALID_ARG, "a batch is already open");
+    t->part_op = 1;
+    t->part_left = n_total;
+    bool fuse = false;
+    dyc_status s;
+    switch (t->cfg.bucket_slots) {
+        case 4: s = insert_begin<4>(t, n_total, S(stream), fuse); break;
+        case 8: s = insert_begin<8>(t, n_total, S(stream), fuse); break;
+        case 16: s = insert_begin<16>(t, n_total, S(stream), fuse); break;
+        default: s = insert_begin<32>(t, n_total, S(stream), fuse); break;
+    }
+    t->part_fuse = fuse;
+    if (s != DYC_OK) t->part_op = 0;
+    return s;
+}
+
+dyc_status dyc_insert_part(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_values, uint8_t* d_status,
+                           uint64_t n, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (t->part_op != 1) return set_err(DYC_ERR_INVALID_ARG, "no insert batch open");
+    if (n > t->part_left) return set_err(DYC_ERR_INVALID_ARG, "parts exceed n_total");
+    if (n == 0) return DYC_OK;
+    t->part_left -= n;
+    DISPATCH_B(t, insert_chunk<B_>(t, d_keys, d_values, d_status, n, t->part_fuse, S(stream)));
+}
+
+dyc_status dyc_insert_end(dyc_table* t, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (t->part_op != 1) return set_err(DYC_ERR_INVALID_ARG, "no insert batch open");
+    t->part_op = 0;
+    DISPATCH_B(t, insert_end<B_>(t, t->part_fuse, S(stream)));
+}
+
+dyc_status dyc_delete_begin(dyc_table* t, uint64_t n_total, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (t->part_op) return set_err(DYC_ERR_INVALID_ARG, "a batch is already open");
+    t->part_op = 2;
+    t->part_left = n_total;
+    return zero_one(t, C_REMOVED, S(stream));
+}
+
+dyc_status dyc_delete_part(dyc_table* t, const uint32_t* d_keys, uint32_t* d_values_out, uint8_t* d_status,
+                           uint64_t n, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (t->part_op != 2) return set_err(DYC_ERR_INVALID_ARG, "no delete batch open");
+    if (n > t->part_left) return set_err(DYC_ERR_INVALID_ARG, "parts exceed n_total");
+    if (n == 0) return DYC_OK;
+    t->part_left -= n;
+    DISPATCH_B(t, delete_chunk<B_>(t, d_keys, d_values_out, d_status, n, S(stream)));
+}
+
+dyc_status dyc_delete_end(dyc_table* t, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (t->part_op != 2) return set_err(DYC_ERR_INVALID_ARG, "no delete batch open");
+    t->part_op = 0;
+    DISPATCH_B(t, delete_end<B_>(t, S(stream)));
+}
+
 dyc_status dyc_find_batch(dyc_table* t, const uint32_t* d_keys, uint32_t* d_values_out, uint8_t* d_found, uint64_t n,
                           dyc_stream_t stream) {
     TRY(enter(t, stream));
@@ -893,7 +956,8 @@ dyc_status dyc_mixed_batch(dyc_table* t, const uint8_t* d_ops, const uint32_t* d
     {
         ProfScope ps(t, DYC_PROF_OTHER, st);
         const OpDest od{d_ops};
-        k_group_count<OpDest><<<std::min<unsigned>(grid_for(n, kThreads), t->num_sms * 8), kThreads, 4 * 4, st>>>(
+        k_group_count<OpDest><<<std::min<unsigned>(grid_for(n, kThreads * 4), t->num_sms * 8), kThreads,
+                                (kThreads / 32) * 4 * 4, st>>>(
             od, n, 4, cnt);
         k_route_offsets<<<1, 32, 0, st>>>(cnt, 4, cnt + 4);
         k_group_scatter<OpDest><<<grid_for(n, (uint64_t)kThreads * kTileItems), kThreads, 4 * 12, st>>>(
@@ -1031,14 +1095,15 @@ dyc_status dyc_profile_read(dyc_table* t, double* ms, uint64_t* calls) {
 dyc_status dyc_route_count(dyc_table* t, const uint32_t* d_keys, uint64_t n, uint32_t world, uint64_t* d_counts,
                            dyc_stream_t stream) {
     TRY(enter(t, stream));
-    if (world < 1 || world > 2048) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..2048");
+    if (world < 1 || world > 1024) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..1024");
     CU(cudaMemsetAsync(d_counts, 0, world * 8, S(stream)));
     if (n == 0) return DYC_OK;
     const uint32_t sh = t->cfg.d + 1;
     {
         ProfScope ps(t, DYC_PROF_OTHER, S(stream));
         const HashDest hd{t->a[sh], t->b[sh], world, fastmod_magic(world), d_keys};
-        k_group_count<HashDest><<<std::min<unsigned>(grid_for(n, kThreads), t->num_sms * 8), kThreads, world * 4,
+        k_group_count<HashDest><<<std::min<unsigned>(grid_for(n, kThreads * 4), t->num_sms * 8), kThreads,
+                                  (kThreads / 32) * world * 4,
                                   S(stream)>>>(hd, n, world, (unsigned long long*)d_counts);
     }
     CU(cudaGetLastError());
@@ -1049,7 +1114,7 @@ dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_
                              uint32_t world, const uint64_t* d_counts, uint64_t* d_cursor, uint32_t* d_keys_out,
                              uint32_t* d_vals_out, uint32_t* d_pos, dyc_stream_t stream) {
     TRY(enter(t, stream));
-    if (world < 1 || world > 2048) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..2048");
+    if (world < 1 || world > 1024) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..1024");
     if (n == 0) return DYC_OK;
     if (n > 0xFFFFFFFFull) return set_err(DYC_ERR_INVALID_ARG, "route batch must be < 2^32 ops");
     const uint32_t sh = t->cfg.d + 1;
@@ -1073,7 +1138,7 @@ dyc_status dyc_route_unpermute(const uint32_t* d_pos, uint64_t n, const uint32_t
                                const uint8_t* d_reply_status, uint32_t* d_vals, uint8_t* d_status,
                                dyc_stream_t stream) {
     if (n == 0) return DYC_OK;
-    k_route_unpermute<<<grid_for(n, kThreads), kThreads, 0, S(stream)>>>(d_pos, n, d_reply_vals, d_reply_status,
+    k_route_unpermute<<<grid_for(n, kThreads * 4), kThreads, 0, S(stream)>>>(d_pos, n, d_reply_vals, d_reply_status,
                                                                         d_vals, d_status);
     CU(cudaGetLastError());
     return DYC_OK;

@@ -687,33 +687,34 @@ struct OpDest {
     __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return ops[i] & 3u; }
 };
 
-// Lanes of a warp with the same destination are combined with __match_any_sync,
-// so shared-memory atomics (32-bit, native) see one update per (warp, dest).
-__device__ __forceinline__ unsigned warp_group_add(unsigned* ctr, uint32_t dest, bool valid) {
-    const unsigned peers = __match_any_sync(kFull, valid ? dest : 0xFFFFFFFFu);
-    const int leader = __ffs(peers) - 1;
-    unsigned b0 = 0;
-    if (valid && (int)(threadIdx.x & 31) == leader) b0 = atomicAdd(&ctr[dest], (unsigned)__popc(peers));
-    b0 = __shfl_sync(kFull, b0, leader);
-    return b0 + __popc(peers & lanemask_lt());
-}
-
+// Pass 1: per-warp shared histograms (32-bit shared atomics, low contention),
+// summed per block, one global atomic per (block, destination).
 template <class Dest>
 __global__ void __launch_bounds__(kThreads) k_group_count(Dest dest, uint64_t n, uint32_t world,
                                                           unsigned long long* __restrict__ counts) {
-    extern __shared__ unsigned hist32[];
-    for (uint32_t w = threadIdx.x; w < world; w += blockDim.x) hist32[w] = 0;
+    extern __shared__ unsigned hist32[];                    // [kThreads/32][world]
+    for (uint32_t x = threadIdx.x; x < (kThreads / 32) * world; x += blockDim.x) hist32[x] = 0;
     __syncthreads();
-    for (uint64_t base = (uint64_t)blockIdx.x * blockDim.x; base < n; base += (uint64_t)gridDim.x * blockDim.x) {
-        const uint64_t i = base + threadIdx.x;
-        const bool valid = i < n;
-        warp_group_add(hist32, valid ? dest(i) : 0u, valid);
+    unsigned* mine = hist32 + (threadIdx.x >> 5) * world;
+    constexpr int IT = 4;
+    for (uint64_t b0 = (uint64_t)blockIdx.x * kThreads * IT; b0 < n; b0 += (uint64_t)gridDim.x * kThreads * IT) {
+#pragma unroll
+        for (int j = 0; j < IT; j++) {
+            const uint64_t i = b0 + (uint64_t)j * kThreads + threadIdx.x;
+            if (i < n) atomicAdd(&mine[dest(i)], 1u);
+        }
     }
     __syncthreads();
-    for (uint32_t w = threadIdx.x; w < world; w += blockDim.x)
-        if (hist32[w]) atomicAdd(&counts[w], (unsigned long long)hist32[w]);
+    for (uint32_t w = threadIdx.x; w < world; w += blockDim.x) {
+        unsigned long long c = 0;
+        for (int q = 0; q < kThreads / 32; q++) c += hist32[q * world + w];
+        if (c) atomicAdd(&counts[w], c);
+    }
 }
 
+// Pass 2: each block bins a tile of kTileItems ops per thread in shared memory,
+// reserves its range per destination with ONE global atomic per (tile, dest),
+// then writes its ops (order inside a (tile, dest) range is unspecified).
 template <class Dest>
 __global__ void __launch_bounds__(kThreads) k_group_scatter(Dest dest, const uint32_t* __restrict__ keys,
                                                             const uint32_t* __restrict__ vals_in, uint64_t n,
@@ -731,9 +732,8 @@ __global__ void __launch_bounds__(kThreads) k_group_scatter(Dest dest, const uin
 #pragma unroll
         for (int j = 0; j < kTileItems; j++) {
             const uint64_t i = t0 + (uint64_t)j * kThreads + threadIdx.x;
-            const bool valid = i < n;
-            dd[j] = valid ? dest(i) : 0xFFFFFFFFu;
-            rk[j] = warp_group_add(cnt, dd[j], valid);      // rank of this op within (tile, dest)
+            dd[j] = i < n ? dest(i) : 0xFFFFFFFFu;
+            rk[j] = i < n ? atomicAdd(&cnt[dd[j]], 1u) : 0u;  // rank within (tile, dest)
         }
         __syncthreads();
         for (uint32_t w = threadIdx.x; w < world; w += blockDim.x)
@@ -769,10 +769,29 @@ __global__ void __launch_bounds__(kThreads) k_route_unpermute(const uint32_t* __
                                                               const uint32_t* __restrict__ rv,
                                                               const uint8_t* __restrict__ rs,
                                                               uint32_t* __restrict__ vals, uint8_t* __restrict__ st) {
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-        const uint32_t p = pos[i];
-        if (rv && vals) vals[i] = rv[p];
-        if (rs && st) st[i] = rs[p];
+    constexpr int IT = 4;                                   // 4 ops per thread, loads in flight together
+    for (uint64_t b0 = (uint64_t)blockIdx.x * kThreads * IT; b0 < n; b0 += (uint64_t)gridDim.x * kThreads * IT) {
+        uint32_t p[IT], v[IT];
+        uint8_t s8[IT];
+#pragma unroll
+        for (int j = 0; j < IT; j++) {
+            const uint64_t i = b0 + (uint64_t)j * kThreads + threadIdx.x;
+            p[j] = i < n ? pos[i] : 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < IT; j++) {
+            const uint64_t i = b0 + (uint64_t)j * kThreads + threadIdx.x;
+            v[j] = (i < n && rv && vals) ? rv[p[j]] : 0u;
+            s8[j] = (i < n && rs && st) ? rs[p[j]] : 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < IT; j++) {
+            const uint64_t i = b0 + (uint64_t)j * kThreads + threadIdx.x;
+            if (i < n) {
+                if (rv && vals) vals[i] = v[j];
+                if (rs && st) st[i] = s8[j];
+            }
+        }
     }
 }
 

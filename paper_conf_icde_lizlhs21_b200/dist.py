@@ -51,9 +51,11 @@ class DistTable:
         w = self.dist.all_to_all_single(out, x, recv_splits, send_splits, group=self.group, async_op=async_op)
         return out, w
 
-    def _run(self, op, keys, values=None, n_out=1):
+    def _run(self, op, keys, values=None, n_out=1, begin=None, end=None):
         """Pipelined route -> all-to-all -> owner op -> all-to-all back -> unpermute.
-        op(keys, values) returns a tuple of n_out per-op result tensors."""
+        op(keys, values) returns a tuple of n_out per-op result tensors.  begin(n)
+        / end() bracket the owner's parts so that they form ONE batch (one
+        resize decision, one alpha check: dyc_*_begin/_part/_end)."""
         torch = _torch()
         n = keys.numel()
         C, W = self.chunks, self.world
@@ -73,6 +75,8 @@ class DistTable:
         ssp = [both[0][:, c].tolist() for c in range(C)]
         rsp = [both[1][:, c].tolist() for c in range(C)]
         self.last_recv = int(both[1].sum())
+        if begin is not None:
+            begin(self.last_recv)
         fwd = []
         for c in range(C):
             kout, vout, _ = parts[c]
@@ -88,23 +92,24 @@ class DistTable:
             res = op(rk, rv)
             res = res if isinstance(res, tuple) else (res,)
             back.append([self._a2a(r, rsp[c], ssp[c], async_op=True) for r in res])
-        outs = [None] * n_out
-        pieces = [[] for _ in range(n_out)]
+        if end is not None:
+            end()
+        # results land directly in their slice of the batch result (request order)
+        out_s = torch.empty(n, dtype=torch.uint8, device=keys.device)
+        out_v = torch.empty(n, dtype=torch.int32, device=keys.device) if n_out == 2 else None
         for c in range(C):
             for (r, w) in back[c]:
                 w.wait()
             _, _, pos = parts[c]
             got = [r for (r, _) in back[c]]
+            lo, hi = bounds[c], bounds[c + 1]
+            if hi == lo:
+                continue
             if n_out == 1:
-                _, s = self.shard.route_unpermute(pos, None, got[0])
-                pieces[0].append(s)
+                self.shard.route_unpermute(pos, None, got[0], out_status=out_s[lo:hi])
             else:
-                v, s = self.shard.route_unpermute(pos, got[0], got[1])
-                pieces[0].append(v)
-                pieces[1].append(s)
-        for j in range(n_out):
-            outs[j] = pieces[j][0] if C == 1 else torch.cat(pieces[j])
-        return outs[0] if n_out == 1 else tuple(outs)
+                self.shard.route_unpermute(pos, got[0], got[1], out_vals=out_v[lo:hi], out_status=out_s[lo:hi])
+        return out_s if n_out == 1 else (out_v, out_s)
 
     # ------------------------------------------------------------ batches
     # With one rank there is nothing to exchange: the batch goes straight to the
@@ -114,7 +119,8 @@ class DistTable:
         if self.world == 1 and not self.force_route:
             self.last_recv = keys.numel()
             return self.shard.insert(keys, values)
-        return self._run(lambda k, v: self.shard.insert(k, v), keys, values, n_out=1)
+        return self._run(lambda k, v: self.shard.insert_part(k, v), keys, values, n_out=1,
+                         begin=self.shard.insert_begin, end=self.shard.insert_end)
 
     def find(self, keys):
         """Returns (values int32-as-uint32, found uint8) in request order."""
@@ -128,7 +134,8 @@ class DistTable:
         if self.world == 1 and not self.force_route:
             self.last_recv = keys.numel()
             return self.shard.delete(keys)
-        return self._run(lambda k, v: self.shard.delete(k), keys, None, n_out=2)
+        return self._run(lambda k, v: self.shard.delete_part(k), keys, None, n_out=2,
+                         begin=self.shard.delete_begin, end=self.shard.delete_end)
 
     def stats(self):
         return self.shard.stats()

@@ -116,6 +116,41 @@ class Table:
                 "dyc_delete_batch")
         return values_out, status
 
+    # one batch delivered in parts (dyc_*_begin / _part / _end)
+    def insert_begin(self, n_total: int, stream=None):
+        L.check(self._lib.dyc_insert_begin(self._h, n_total, _stream_ptr(stream)), "dyc_insert_begin")
+
+    def insert_part(self, keys, values, status=None, stream=None):
+        torch = _torch()
+        n = keys.numel()
+        if status is None:
+            status = torch.empty(n, dtype=torch.uint8, device=keys.device)
+        L.check(self._lib.dyc_insert_part(self._h, keys.data_ptr() if n else None, values.data_ptr() if n else None,
+                                          status.data_ptr() if n else None, n, _stream_ptr(stream)),
+                "dyc_insert_part")
+        return status
+
+    def insert_end(self, stream=None):
+        L.check(self._lib.dyc_insert_end(self._h, _stream_ptr(stream)), "dyc_insert_end")
+
+    def delete_begin(self, n_total: int, stream=None):
+        L.check(self._lib.dyc_delete_begin(self._h, n_total, _stream_ptr(stream)), "dyc_delete_begin")
+
+    def delete_part(self, keys, values_out=None, status=None, stream=None):
+        torch = _torch()
+        n = keys.numel()
+        if values_out is None:
+            values_out = torch.empty(n, dtype=torch.int32, device=keys.device)
+        if status is None:
+            status = torch.empty(n, dtype=torch.uint8, device=keys.device)
+        L.check(self._lib.dyc_delete_part(self._h, keys.data_ptr() if n else None,
+                                          values_out.data_ptr() if n else None, status.data_ptr() if n else None,
+                                          n, _stream_ptr(stream)), "dyc_delete_part")
+        return values_out, status
+
+    def delete_end(self, stream=None):
+        L.check(self._lib.dyc_delete_end(self._h, _stream_ptr(stream)), "dyc_delete_end")
+
     def mixed(self, ops, keys, values, values_out=None, status=None, stream=None):
         """Mixed batch (find=0, insert=1, delete=2; phases find -> insert -> delete, Q10)."""
         torch = _torch()
@@ -249,12 +284,16 @@ class Table:
                                             _stream_ptr(stream)), "dyc_route_scatter")
         return kout, vout, pos
 
-    def route_unpermute(self, pos, reply_vals=None, reply_status=None, stream=None):
-        """vals[i] = reply_vals[pos[i]], status[i] = reply_status[pos[i]]."""
+    def route_unpermute(self, pos, reply_vals=None, reply_status=None, stream=None, out_vals=None, out_status=None):
+        """vals[i] = reply_vals[pos[i]], status[i] = reply_status[pos[i]] (written
+        into out_vals / out_status when given, e.g. slices of the batch result)."""
         torch = _torch()
         n = pos.numel()
-        v = torch.empty(n, dtype=torch.int32, device=pos.device) if reply_vals is not None else None
-        s = torch.empty(n, dtype=torch.uint8, device=pos.device) if reply_status is not None else None
+        v = s = None
+        if reply_vals is not None:
+            v = out_vals if out_vals is not None else torch.empty(n, dtype=torch.int32, device=pos.device)
+        if reply_status is not None:
+            s = out_status if out_status is not None else torch.empty(n, dtype=torch.uint8, device=pos.device)
         L.check(self._lib.dyc_route_unpermute(pos.data_ptr(), n,
                                               reply_vals.data_ptr() if reply_vals is not None else None,
                                               reply_status.data_ptr() if reply_status is not None else None,

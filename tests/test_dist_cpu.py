@@ -34,9 +34,17 @@ class DictShard:
         vout = values[order].clone() if values is not None else None
         return kout, vout, pos.to(torch.int32)
 
-    def route_unpermute(self, pos, rv=None, rs=None):
+    def route_unpermute(self, pos, rv=None, rs=None, out_vals=None, out_status=None):
         p = pos.to(torch.int64)
-        return (rv[p] if rv is not None else None), (rs[p] if rs is not None else None)
+        v = rv[p] if rv is not None else None
+        s = rs[p] if rs is not None else None
+        if out_vals is not None and v is not None:
+            out_vals.copy_(v)
+            v = out_vals
+        if out_status is not None and s is not None:
+            out_status.copy_(s)
+            s = out_status
+        return v, s
 
     def insert(self, keys, vals):
         st = torch.zeros(keys.numel(), dtype=torch.uint8)
@@ -47,6 +55,25 @@ class DictShard:
             st[i] = 2 if k in self.m else 1
             self.m[k] = v
         return st
+
+    # one batch in parts: the stand-in applies each part immediately
+    def insert_begin(self, n):
+        pass
+
+    def insert_part(self, keys, vals):
+        return self.insert(keys, vals)
+
+    def insert_end(self):
+        pass
+
+    def delete_begin(self, n):
+        pass
+
+    def delete_part(self, keys):
+        return self.delete(keys)
+
+    def delete_end(self):
+        pass
 
     def find(self, keys):
         v = torch.full((keys.numel(),), -1, dtype=torch.int32)

@@ -354,3 +354,34 @@ def test_c4_zipf_mixed_parity(oracle_mod):
         assert g.stats()["buckets"] == o.stats()["buckets"]
     check_layout(g, o)
     assert g.stats()["n_downsize"] > 0
+
+
+def test_batch_in_parts_equals_one_batch(oracle_mod):
+    """dyc_insert_begin/_part/_end (and the delete analogue) form ONE batch: one
+    resize decision and one alpha check, so the statuses, contents and the resize
+    schedule equal the single-batch oracle's."""
+    wl = W.random_op_stream(777, n_batches=12, batch=20000, universe=40000, init_capacity=64)
+    g, o = make_pair(oracle_mod, wl, B=8)
+    for i, b in enumerate(wl.batches):
+        n = b.keys.size
+        cuts = [0, n // 3, n // 3, (2 * n) // 3, n]            # includes an empty part
+        kd = dev(b.keys)
+        if b.op == "insert":
+            vd = dev(b.values)
+            g.insert_begin(n)
+            st = [g.insert_part(kd[cuts[j]:cuts[j + 1]], vd[cuts[j]:cuts[j + 1]]) for j in range(4)]
+            g.insert_end()
+            np.testing.assert_array_equal(torch.cat(st).cpu().numpy(), o.insert(b.keys, b.values))
+        elif b.op == "delete":
+            g.delete_begin(n)
+            parts = [g.delete_part(kd[cuts[j]:cuts[j + 1]]) for j in range(4)]
+            g.delete_end()
+            ov, os_ = o.delete(b.keys)
+            np.testing.assert_array_equal(torch.cat([p[1] for p in parts]).cpu().numpy(), os_)
+            np.testing.assert_array_equal(host_u32(torch.cat([p[0] for p in parts])), ov)
+        else:
+            v, f = g.find(kd)
+            ov, of = o.find(b.keys)
+            np.testing.assert_array_equal(f.cpu().numpy(), of)
+        np.testing.assert_array_equal(g.sorted_kv(), o.sorted_kv())
+        assert g.stats()["buckets"] == o.stats()["buckets"], f"schedule diverged at batch {i}"
