@@ -63,6 +63,10 @@ def parse():
     ap.add_argument("--no-rehash", action="store_true")
     ap.add_argument("--profile-only", action="store_true", help="a few steps, no extras (for ncu)")
     ap.add_argument("--l2-fetch", type=int, default=None, help="set cudaLimitMaxL2FetchGranularity (bytes)")
+    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4"],
+                    help="c2 = the headline (BASELINE configs[1]); c1/c3/c4 = the other single-GPU configs")
+    ap.add_argument("--scale", type=float, default=1.0, help="c3: stream scale; c4: universe scale")
+    ap.add_argument("--shape", default=None, help="c3: TW|RE, c4: LINE|COM")
     ap.add_argument("--routed", action="store_true",
                     help="use the sharded router even at N=1 (exercises the N>1 code path)")
     return ap.parse_args()
@@ -295,6 +299,8 @@ def main():
     n = 1 << args.log2n
     if world > 1 or args.routed:
         return multi_gpu(args, rank, world, local, dist)
+    if args.config != "c2":
+        return emit(bench_stream(args, local))
     cap, k_ins, v_ins, k_find, k_del = W.c2_rand_static_torch(args.log2n, device="cuda")
 
     stream = torch.cuda.current_stream()
@@ -477,6 +483,134 @@ def main():
                   "pending_after_upsert": pend, "evictions": s_ins["last_insert_evictions"]},
     }
     emit(line)
+
+
+def bench_stream(args, local):
+    """Configs C1, C3 (TW/RE sliding window) and C4 (LINE/COM Zipf mixed): the
+    whole stream of batches, each batch timed with CUDA events; Mops/s per op
+    type and overall, the fill factor after every batch (Fig. `fig:track-stability`
+    analogue), memory held, resize counts."""
+    import numpy as np
+    import torch
+    from paper_conf_icde_lizlhs21_b200 import workload as W
+    from paper_conf_icde_lizlhs21_b200.table import Table
+
+    t0 = time.time()
+    if args.config == "c1":
+        wl = W.c1_rand_small()
+        batches, mixed = wl.batches, False
+        name = "C1 RAND small (BASELINE configs[0]): 65,536 keys, 8x8192 insert, find (50% hit), delete"
+    elif args.config == "c3":
+        shape = args.shape or "TW"
+        wl = W.c3_dynamic(scale=args.scale, shape=shape, batch=max(1000, int(1_000_000 * min(1.0, args.scale * 4))),
+                          cycles=2)
+        batches, mixed = wl.batches, False
+        name = (f"C3 {shape}-shaped dynamic stream x{args.scale:g}: sliding window of insert + find (50% hit) + "
+                "0.2x delete batches, swap pass, 2 cycles")
+    else:
+        shape = args.shape or "COM"
+        U, D = (4_583_941, 1_000_000) if shape == "COM" else (45_159_880, 4_000_000)
+        U, D = max(1000, int(U * args.scale)), max(100, int(D * args.scale))
+        wl, batches = W.c4_zipf_mixed(U=U, distinct=D, grow_batches=16, cycles=2)
+        mixed = True
+        name = (f"C4 {shape}-shaped Zipf(0.99) mixed 50/30/20 batches of {D} distinct keys over U={U}, "
+                "grow 16 batches then drain, 2 cycles")
+    gen_s = time.time() - t0
+    g = Table(d=wl.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=args.bucket_slots)
+    dev = lambda a: torch.from_numpy(np.ascontiguousarray(a, dtype=np.uint32).view(np.int32)).cuda()  # noqa: E731
+    staged = []
+    for b in batches:
+        if mixed:
+            staged.append(("mixed", torch.from_numpy(b.ops).cuda(), dev(b.keys), dev(b.values)))
+        else:
+            staged.append((b.op, None, dev(b.keys), dev(b.values) if b.values is not None else None))
+    stream = torch.cuda.current_stream()
+
+    def run():
+        g.clear()
+        for op, ops, k, v in staged:
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            if op == "insert":
+                g.insert(k, v)
+            elif op == "find":
+                g.find(k)
+            elif op == "delete":
+                g.delete(k)
+            else:
+                g.mixed(ops, k, v)
+            e1.record(stream)
+    # warm-up pass(es), then the timed pass (table rebuilt from empty each pass)
+    for _ in range(max(1, args.warmup)):
+        run()
+    torch.cuda.synchronize()
+    rec = []
+    g.profile(True)
+    g.launch_count(reset=True)
+    with ClockSampler(local) as clk:
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        g.clear()
+        a.record(stream)
+        for op, ops, k, v in staged:
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            if op == "insert":
+                g.insert(k, v)
+            elif op == "find":
+                g.find(k)
+            elif op == "delete":
+                g.delete(k)
+            else:
+                g.mixed(ops, k, v)
+            e1.record(stream)
+            rec.append((op, k.numel(), e0, e1, ops))
+        b.record(stream)
+        torch.cuda.synchronize()
+    total_ms = a.elapsed_time(b)
+    launches = g.launch_count()
+    prof = g.profile_read()
+    g.profile(False)
+    per = {"insert": [0, 0.0], "find": [0, 0.0], "delete": [0, 0.0], "mixed": [0, 0.0]}
+    for op, cnt, e0, e1, _ in rec:
+        per[op][0] += cnt
+        per[op][1] += e0.elapsed_time(e1)
+    # fill-factor track: replay untimed with a stats call after every batch
+    g.clear()
+    track, mem = [], []
+    for op, ops, k, v in staged:
+        if op == "insert":
+            g.insert(k, v)
+        elif op == "find":
+            g.find(k)
+        elif op == "delete":
+            g.delete(k)
+        else:
+            g.mixed(ops, k, v)
+        st = g.stats()
+        track.append(round(st["fill"], 4))
+        mem.append(st["N"] * 8)
+    st = g.stats()
+    n_ops = sum(c for _, c, _, _, _ in rec)
+    ops_line = {f"{k}_mops": (v[0] / v[1] / 1e3 if v[1] else None) for k, v in per.items() if v[0]}
+    return {
+        "metric": METRIC, "value": n_ops / total_ms / 1e3, "unit": "Mops/s", "n_gpus": 1, "steps": 1,
+        "warmup": args.warmup, "ms_per_step": total_ms, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": name, "d": wl.d, "alpha": wl.alpha, "beta": wl.beta,
+                   "bucket_slots": args.bucket_slots, "batches": len(staged), "ops": n_ops},
+        "ops": ops_line,
+        "fill_track": {"min_after_mutation": min(x for x, (op, *_r) in zip(track, staged) if op != "find"),
+                       "max": max(track), "final": track[-1], "every_batch": track if len(track) <= 400 else None},
+        "table_bytes": {"max": max(mem), "final": mem[-1]},
+        "resizes": {k: st[k] for k in ("n_upsize", "n_downsize", "n_fail_upsize", "n_residual")},
+        "kernel_ms": {k: round(v[0], 3) for k, v in prof.items() if v[1]},
+        "kernel_calls": {k: v[1] for k, v in prof.items() if v[1]},
+        "gpu_launches": launches, "clocks": clk.summary(), "generator_seconds": gen_s,
+        "roofline": None, "cpu_baseline": None, "e2e": None,
+    }
 
 
 def multi_gpu(args, rank, world, local, dist):

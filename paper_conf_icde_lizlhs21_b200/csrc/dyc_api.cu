@@ -232,23 +232,10 @@ dyc_status upsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
     return DYC_OK;
 }
 
-// Place list[src][0..cnt) (count given on host or in a device counter), settling
-// failures: first a plain retry pass, then failure-triggered upsizes.
+// Retries the nfail homeless pairs in list[cur]: first a plain retry pass, then
+// failure-triggered upsizes (Q17: nothing is ever dropped).
 template <int B>
-dyc_status place_and_settle(dyc_table* t, int src, const unsigned long long* d_count, uint64_t h_count,
-                            bool first_fit, cudaStream_t st) {
-    TRY(zero_one(t, C_FAIL, st));
-    TRY(zero_one(t, C_EVICT, st));
-    {
-        ProfScope ps(t, DYC_PROF_PLACE, st);
-        k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->list[src], d_count, h_count,
-                                                         t->list[1 - src], t->d_ctr, first_fit);
-    }
-    CU(cudaGetLastError());
-    TRY(read_ctr(t, st));
-    t->n_evict += t->h_ctr[C_EVICT];
-    uint64_t nfail = t->h_ctr[C_FAIL];
-    int cur = 1 - src;
+dyc_status settle(dyc_table* t, int cur, uint64_t nfail, cudaStream_t st) {
     int round = 0;
     while (nfail > 0) {
         if (round > 0) {
@@ -261,8 +248,8 @@ dyc_status place_and_settle(dyc_table* t, int src, const unsigned long long* d_c
         TRY(zero_one(t, C_EVICT, st));
         {
             ProfScope ps(t, DYC_PROF_PLACE, st);
-            k_place<B><<<grid_for(nfail, kThreads / (B / 4)), kThreads, 0, st>>>(t->view(), t->list[cur], nullptr, nfail,
-                                                                       t->list[1 - cur], t->d_ctr, true);
+            k_place<B><<<grid_for(nfail, kThreads / (B / 4)), kThreads, 0, st>>>(t->view(), t->list[cur], nullptr,
+                                                                              nfail, t->list[1 - cur], t->d_ctr, true);
         }
         CU(cudaGetLastError());
         TRY(read_ctr(t, st));
@@ -274,11 +261,39 @@ dyc_status place_and_settle(dyc_table* t, int src, const unsigned long long* d_c
     return DYC_OK;
 }
 
+// Launches k_place over list[src][0..cnt) (count on the host or in a device
+// counter); homeless pairs are appended to list[1-src] at the C_FAIL cursor.
 template <int B>
-dyc_status downsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
+dyc_status launch_place(dyc_table* t, int src, const unsigned long long* d_count, uint64_t h_count, bool first_fit,
+                        cudaStream_t st) {
+    ProfScope ps(t, DYC_PROF_PLACE, st);
+    k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->list[src], d_count, h_count, t->list[1 - src],
+                                                     t->d_ctr, first_fit);
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+// Place list[src][0..cnt) and settle failures.
+template <int B>
+dyc_status place_and_settle(dyc_table* t, int src, const unsigned long long* d_count, uint64_t h_count,
+                            bool first_fit, cudaStream_t st) {
+    TRY(zero_one(t, C_FAIL, st));
+    TRY(zero_one(t, C_EVICT, st));
+    TRY(launch_place<B>(t, src, d_count, h_count, first_fit, st));
+    TRY(read_ctr(t, st));
+    t->n_evict += t->h_ctr[C_EVICT];
+    return settle<B>(t, 1 - src, t->h_ctr[C_FAIL], st);
+}
+
+// Halves subtable ti: merge kernel, then residual placement into
+// the pairs' other tables (a separate kernel, so excluding t is not
+// needed for correctness, Q16).  Residual failures are appended to list[1] at
+// the C_FAIL cursor and settled by the caller (several downsizes of one alpha
+// loop share one host sync).
+template <int B>
+dyc_status downsize_launch(dyc_table* t, uint32_t ti, cudaStream_t st) {
     const uint64_t n_old = t->nb[ti], h = n_old / 2;
     if (n_old < 2 || (n_old & 1)) return set_err(DYC_ERR_INVALID_ARG, "subtable cannot be halved");
-    TRY(ensure_lists(t, h * B, st));
     void* p = nullptr;
     TRY(dev_alloc(t, &p, h * B * 8, st));
     TRY(zero_one(t, C_RESIDUAL, st));
@@ -291,33 +306,61 @@ dyc_status downsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
     CU(cudaFreeAsync(t->sub[ti], st));
     t->sub[ti] = (unsigned long long*)p;
     t->nb[ti] = h;
-    // residuals go to the other table of their pair; run as a
-    // separate kernel, so the exclusion of t is not needed for correctness (Q16)
-    TRY(place_and_settle<B>(t, 0, t->d_ctr + C_RESIDUAL, 0, true, st));
-    t->n_residual += t->h_ctr[C_RESIDUAL];
-    return DYC_OK;
+    return launch_place<B>(t, 0, t->d_ctr + C_RESIDUAL, 0, true, st);
 }
 
 template <int B>
+dyc_status downsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
+    TRY(ensure_lists(t, (t->nb[ti] / 2) * B, st));
+    TRY(zero_one(t, C_FAIL, st));
+    TRY(zero_one(t, C_EVICT, st));
+    TRY(zero_one(t, C_RES_TOTAL, st));
+    TRY(downsize_launch<B>(t, ti, st));
+    TRY(read_ctr(t, st));
+    t->n_evict += t->h_ctr[C_EVICT];
+    t->n_residual += t->h_ctr[C_RES_TOTAL];
+    return settle<B>(t, 1, t->h_ctr[C_FAIL], st);
+}
+
+// Lower bound (Q11-Q13): while m < alpha*N halve the largest
+// subtable (unless it is odd / a single bucket, or halving would exceed beta).
+// The halvings depend only on m and the sizes, so the whole sequence is planned
+// on the host and launched back to back; residual failures of all of them are
+// settled once at the end (Q17: retry, then failure-triggered upsizes).
+template <int B>
 dyc_status enforce_lower(dyc_table* t, cudaStream_t st) {
-    bool shrank = false;
+    uint64_t nb[DYC_MAX_D];
+    for (uint32_t i = 0; i < t->cfg.d; i++) nb[i] = t->nb[i];
+    std::vector<uint32_t> plan;
+    uint64_t res_bound = 0;
     for (;;) {
-        const uint64_t N = t->N();
+        uint64_t N = 0;
+        for (uint32_t i = 0; i < t->cfg.d; i++) N += nb[i] * B;
         if (!((double)t->m < t->cfg.alpha * (double)N)) break;
-        const int ti = t->largest();
-        if (t->nb[ti] < 2 || (t->nb[ti] & 1)) break;
-        const uint64_t N_after = N - (t->nb[ti] / 2) * B;
+        int ti = (int)t->cfg.d - 1;                                   // largest, ties -> highest (Q12)
+        for (int i = (int)t->cfg.d - 2; i >= 0; i--)
+            if (nb[i] > nb[ti]) ti = i;
+        if (nb[ti] < 2 || (nb[ti] & 1)) break;
+        const uint64_t N_after = N - (nb[ti] / 2) * B;
         if ((double)t->m > t->cfg.beta * (double)N_after) break;
-        const uint64_t fails = t->n_fail_upsize;
-        TRY(downsize_table<B>(t, (uint32_t)ti, st));
+        plan.push_back((uint32_t)ti);
+        res_bound += (nb[ti] / 2) * B;
+        nb[ti] /= 2;
+    }
+    if (plan.empty()) return DYC_OK;
+    TRY(ensure_lists(t, std::min<uint64_t>(res_bound, t->m + 1) + 1, st));
+    TRY(zero_one(t, C_FAIL, st));
+    TRY(zero_one(t, C_EVICT, st));
+    TRY(zero_one(t, C_RES_TOTAL, st));
+    for (uint32_t ti : plan) {
+        TRY(downsize_launch<B>(t, ti, st));
         t->n_downsize++;
-        shrank = true;
-        if (t->n_fail_upsize != fails) break;   // Q17b
     }
-    if (shrank) {
-        CU(cudaStreamSynchronize(st));
-        cudaMemPoolTrimTo(t->pool, 0);
-    }
+    TRY(read_ctr(t, st));
+    t->n_evict += t->h_ctr[C_EVICT];
+    t->n_residual += t->h_ctr[C_RES_TOTAL];
+    TRY(settle<B>(t, 1, t->h_ctr[C_FAIL], st));
+    cudaMemPoolTrimTo(t->pool, 0);
     return DYC_OK;
 }
 

@@ -52,6 +52,7 @@ enum CounterIdx : int {
     C_RESIDUAL = 6,   // downsize residuals
     C_DUMP = 7,       // dump cursor
     C_SECOND = 8,     // keys in their second-choice subtable (stats)
+    C_RES_TOTAL = 9,  // residuals over several downsizes of one alpha loop
     C_COUNT0 = 16,    // per-subtable live counts [16, 32)
     C_N = 32
 };
@@ -611,6 +612,8 @@ __global__ void __launch_bounds__(kThreads) k_downsize(const unsigned long long*
             }
             if (s >= ctot) new_s[bb + s] = kEmptySlot;
         }
+        const unsigned rm = __ballot_sync(kFull, res);
+        if (rm && (threadIdx.x & 31) == (unsigned)(__ffs(rm) - 1)) atomicAdd(ctr + C_RES_TOTAL, (unsigned long long)__popc(rm));
         warp_append(res, e2, residual, ctr + C_RESIDUAL);
     }
 }

@@ -253,78 +253,96 @@ def c3_dynamic(scale: float = 1.0, shape: str = "TW", batch: int = 1_000_000, r:
     (50% live / 50% never inserted), one delete batch of r*batch OLDEST live keys
     (sliding window; r = #delete/#insert, reading Q22).  After the
     stream is exhausted the batches are replayed with insert and delete key sets
-    swapped (reading Q27); `cycles` repeats the whole thing."""
+    swapped (reading Q27); `cycles` repeats forward stream + swap pass.
+    Vectorised (numpy) so the full-size stream is generated in seconds."""
     s = config_seed(3) if seed_cfg is None else seed_cfg
     rng = np.random.Generator(np.random.PCG64(s))
     total, uniq, mult = {"TW": (50_876_784, 44_523_684, 4), "RE": (48_104_875, 41_466_682, 2)}[shape]
     T, U = max(1, int(total * scale)), max(1, int(uniq * scale))
     batch = max(1, int(batch))
     keys = key_range(0, U, s)
-    # repeats: T-U extra occurrences of random keys, each key at most mult-1 times,
-    # each repeat in a strictly later batch than the key's previous occurrence
-    n_rep = T - U
-    rep_keys = rng.choice(U, size=min(n_rep, U * (mult - 1)), replace=True)
-    cnt = np.bincount(rep_keys, minlength=U)
-    cnt = np.minimum(cnt, mult - 1)
-    first_batch = np.arange(U) // batch
     n_batches = (U + batch - 1) // batch
-    rep_slots = [[] for _ in range(n_batches + 4 * mult)]
-    ids = np.nonzero(cnt)[0]
-    for kid in ids:
-        b = int(first_batch[kid])
-        for j in range(int(cnt[kid])):
-            b += 1 + int(rng.integers(0, 3))
-            if b < len(rep_slots):
-                rep_slots[b].append(int(kid))
+    # repeats: T-U extra occurrences, each key at most mult-1 times, each in a
+    # strictly later batch than the key's previous occurrence
+    rep = rng.choice(U, size=min(T - U, U * (mult - 1)), replace=True)
+    cnt = np.minimum(np.bincount(rep, minlength=U), mult - 1)
+    rep_ids, rep_batch = [], []
+    cur = np.arange(U) // batch
+    for j in range(mult - 1):
+        sel = np.nonzero(cnt > j)[0]
+        cur_sel = cur[sel] + 1 + rng.integers(0, 3, size=sel.size)
+        cur[sel] = cur_sel
+        rep_ids.append(sel)
+        rep_batch.append(cur_sel)
+    rep_ids = np.concatenate(rep_ids) if rep_ids else np.zeros(0, np.int64)
+    rep_batch = np.concatenate(rep_batch) if rep_batch else np.zeros(0, np.int64)
+    nb_total = int(max(n_batches, rep_batch.max() + 1 if rep_batch.size else 0))
+    order_rb = np.argsort(rep_batch, kind="stable")
+    rep_ids, rep_batch = rep_ids[order_rb], rep_batch[order_rb]
+    rep_bounds = np.searchsorted(rep_batch, np.arange(nb_total + 1))
     w = Workload(f"C3-{shape}-x{scale:g}", 4, 0.3, 0.85, init_capacity)
-    ins_batches = []
-    for b in range(len(rep_slots)):
-        fresh = np.arange(b * batch, min((b + 1) * batch, U)) if b < n_batches else np.zeros(0, np.int64)
-        ids_b = np.concatenate([fresh, np.array(rep_slots[b], dtype=np.int64)])
-        if ids_b.size:
-            ins_batches.append(np.unique(ids_b))          # distinct within the batch
-    live = {}                                              # key id -> insertion order (FIFO)
-    order = 0
+    # FIFO of live keys by insertion time: order[] holds key ids, live_pos[kid]
+    # the position of the key's current life (-1 when not live)
+    order = np.empty(T + 1, dtype=np.int64)
+    tail = head = 0
+    live_pos = np.full(U, -1, dtype=np.int64)
+    nlive = 0
+    ins_batches, del_batches = [], []
     miss_ctr = 0
-    del_batches = []
-    for b, ids_b in enumerate(ins_batches):
-        ver = b + 1
-        w.batches.append(Batch("insert", keys[ids_b], val_of(keys[ids_b], ver)))
-        for kid in ids_b.tolist():
-            if kid not in live:
-                live[kid] = order
-                order += 1
-        nf = batch
-        lv = np.fromiter(live.keys(), dtype=np.int64, count=len(live))
-        hits = keys[rng.choice(lv, size=min(nf // 2, lv.size), replace=False)] if lv.size else np.zeros(0, np.uint32)
-        miss = key_range(MISS_BASE + miss_ctr, nf - hits.size, s)
-        miss_ctr += nf - hits.size
-        q = np.concatenate([hits, miss])
+    for b in range(nb_total):
+        fresh = np.arange(b * batch, min((b + 1) * batch, U)) if b < n_batches else np.zeros(0, np.int64)
+        ids_b = np.unique(np.concatenate([fresh, rep_ids[rep_bounds[b]:rep_bounds[b + 1]]]))
+        if ids_b.size == 0:
+            continue
+        ins_batches.append(ids_b)
+        w.batches.append(Batch("insert", keys[ids_b], val_of(keys[ids_b], b + 1)))
+        new = ids_b[live_pos[ids_b] < 0]                   # first life or re-insert after delete
+        order[tail:tail + new.size] = new
+        live_pos[new] = np.arange(tail, tail + new.size)
+        tail += new.size
+        nlive += new.size
+        # finds: half live (sampled), half never inserted
+        nh = min(batch // 2, nlive)
+        hits = np.zeros(0, np.int64)
+        while hits.size < nh:
+            cand_pos = rng.integers(head, tail, size=2 * (nh - hits.size) + 16)
+            cand = order[cand_pos]
+            ok = live_pos[cand] == cand_pos
+            hits = np.unique(np.concatenate([hits, cand[ok]]))[:nh] if hits.size else np.unique(cand[ok])[:nh]
+        miss = key_range(MISS_BASE + miss_ctr, batch - hits.size, s)
+        miss_ctr += batch - hits.size
+        q = np.concatenate([keys[hits], miss])
         rng.shuffle(q)
         w.batches.append(Batch("find", q))
-        nd = int(r * batch)
-        oldest = sorted(live, key=live.get)[:nd]
-        for kid in oldest:
-            del live[kid]
-        del_ids = np.array(oldest, dtype=np.int64)
-        del_batches.append(del_ids)
-        w.batches.append(Batch("delete", keys[del_ids]))
+        # deletes: the r*batch oldest live keys
+        nd = min(int(r * batch), nlive)
+        got = []
+        need = nd
+        while need > 0:
+            seg = order[head:min(tail, head + 2 * need + 64)]
+            pos = np.arange(head, head + seg.size)
+            ok = live_pos[seg] == pos
+            take = np.nonzero(ok)[0][:need]
+            if take.size:
+                got.append(seg[take])
+                head = pos[take[-1]] + 1
+                need -= take.size
+            else:
+                head += seg.size
+        dl = np.concatenate(got) if got else np.zeros(0, np.int64)
+        live_pos[dl] = -1
+        nlive -= dl.size
+        del_batches.append(dl)
+        w.batches.append(Batch("delete", keys[dl]))
     base = list(w.batches)
     for c in range(cycles):
-        if c == 0:
-            # swap pass of the first cycle
-            for b, ids_b in enumerate(ins_batches):
-                d_ids = del_batches[b]
-                w.batches.append(Batch("insert", keys[d_ids], val_of(keys[d_ids], 1000 + b)))
-                w.batches.append(Batch("delete", keys[ids_b]))
-        else:
-            # later cycles replay the forward stream, then the swap pass again
-            for bt in base:
+        if c > 0:
+            for bt in base:       # replay the forward stream
                 w.batches.append(Batch(bt.op, bt.keys.copy(), None if bt.values is None else bt.values.copy()))
-            for b, ids_b in enumerate(ins_batches):
-                d_ids = del_batches[b]
-                w.batches.append(Batch("insert", keys[d_ids], val_of(keys[d_ids], 2000 + b)))
-                w.batches.append(Batch("delete", keys[ids_b]))
+        for b, ids_b in enumerate(ins_batches):                # swap pass (P:L734)
+            d_ids = del_batches[b]
+            w.batches.append(Batch("insert", keys[d_ids], val_of(keys[d_ids], 1000 * (c + 1) + b)))
+            w.batches.append(Batch("delete", keys[ids_b]))
     return w
 
 
@@ -337,24 +355,30 @@ class MixedBatch:
     values: np.ndarray   # uint32
 
 
-def zipf_distinct(rng, cdf: np.ndarray, count: int, exclude=None) -> np.ndarray:
-    """Draw Zipf ranks (inverse CDF) until `count` distinct ranks are collected."""
+def zipf_distinct(rng, cdf: np.ndarray, count: int, exclude: Optional[np.ndarray] = None) -> np.ndarray:
+    """Draw Zipf ranks (inverse CDF) until `count` distinct ranks are collected,
+    in first-draw order (vectorised with a seen-mask over the universe)."""
+    seen = np.zeros(cdf.size + 1, dtype=bool)
+    if exclude is not None and len(exclude):
+        seen[np.asarray(exclude, dtype=np.int64)] = True
     got = []
-    seen = set() if exclude is None else set(exclude)
-    while len(got) < count:
-        draw = np.searchsorted(cdf, rng.random(max(1024, 2 * (count - len(got)))), side="right")
-        for x in draw.tolist():
-            if x not in seen:
-                seen.add(x)
-                got.append(x)
-                if len(got) == count:
-                    break
-    return np.array(got, dtype=np.int64)
+    have = 0
+    while have < count:
+        draw = np.searchsorted(cdf, rng.random(max(4096, 2 * (count - have))), side="right")
+        draw = draw[~seen[draw]]
+        if draw.size == 0:
+            continue
+        _, first = np.unique(draw, return_index=True)
+        new = draw[np.sort(first)][:count - have]
+        seen[new] = True
+        got.append(new)
+        have += new.size
+    return np.concatenate(got).astype(np.int64)
 
 
 def c4_zipf_mixed(U: int = 45_159_880, distinct: int = 4_000_000, grow_batches: int = 16, cycles: int = 2,
                   exponent: float = 0.99, seed_cfg: Optional[int] = None, init_capacity: int = 1 << 20,
-                  drain_floor: float = 0.10):
+                  drain_floor: float = 0.10, max_drain: int = 64):
     """Mixed 50/30/20 find/insert/delete batches over Zipf(0.99) ranks of a
     universe of U keys (LINE-shaped: U = 45,159,880; COM-shaped: U = 4,583,941
     with 1M-distinct batches).  Grow phase: `grow_batches` batches; drain phase:
@@ -364,14 +388,22 @@ def c4_zipf_mixed(U: int = 45_159_880, distinct: int = 4_000_000, grow_batches: 
     s = config_seed(4) if seed_cfg is None else seed_cfg
     rng = np.random.Generator(np.random.PCG64(s))
     ranks = np.arange(1, U + 1, dtype=np.float64)
-    pmf = ranks ** (-exponent)
-    cdf = np.cumsum(pmf)
+    cdf = np.cumsum(ranks ** (-exponent))
     cdf /= cdf[-1]
     keys_of = lambda r: key_of(np.asarray(r, dtype=np.uint64), s)  # noqa: E731  (rank -> key, a bijection)
     meta = Workload(f"C4-zipf-U{U}", 4, 0.3, 0.85, init_capacity)
     out = []
-    live = set()
+    live = np.zeros(U + 1, dtype=bool)
+    nlive = 0
     ver = 0
+
+    def apply(r, ops):
+        nonlocal nlive
+        ins, dl = r[ops == 1], r[ops == 2]
+        nlive += int((~live[ins]).sum()) - int(live[dl].sum())
+        live[ins] = True
+        live[dl] = False
+
     for c in range(cycles):
         for b in range(grow_batches):
             ver += 1
@@ -380,17 +412,16 @@ def c4_zipf_mixed(U: int = 45_159_880, distinct: int = 4_000_000, grow_batches: 
             ops = np.where(u < 0.5, 0, np.where(u < 0.8, 1, 2)).astype(np.uint8)
             k = keys_of(r)
             out.append(MixedBatch(ops, k, val_of(k, ver)))
-            for rr, op in zip(r.tolist(), ops.tolist()):
-                if op == 1:
-                    live.add(rr)
-                elif op == 2:
-                    live.discard(rr)
-        peak = len(live)
-        while len(live) > drain_floor * peak and live:
+            apply(r, ops)
+        peak = nlive
+        for _ in range(max_drain):
+            if nlive <= drain_floor * peak or nlive == 0:
+                break
             ver += 1
-            nd = min(len(live), int(0.45 * distinct))
-            dl = rng.choice(np.fromiter(live, dtype=np.int64, count=len(live)), size=nd, replace=False)
-            rest = zipf_distinct(rng, cdf, distinct - nd, exclude=dl.tolist())
+            nd = min(nlive, int(0.45 * distinct))
+            lv = np.nonzero(live)[0]
+            dl = rng.choice(lv, size=nd, replace=False)
+            rest = zipf_distinct(rng, cdf, distinct - nd, exclude=dl)
             u = rng.random(rest.size)
             ops_rest = np.where(u < 0.5 / 0.55, 0, 1).astype(np.uint8)      # 50 find : 5 insert
             r = np.concatenate([dl, rest])
@@ -399,9 +430,5 @@ def c4_zipf_mixed(U: int = 45_159_880, distinct: int = 4_000_000, grow_batches: 
             r, ops = r[perm], ops[perm]
             k = keys_of(r)
             out.append(MixedBatch(ops, k, val_of(k, ver)))
-            for rr, op in zip(r.tolist(), ops.tolist()):
-                if op == 1:
-                    live.add(rr)
-                elif op == 2:
-                    live.discard(rr)
+            apply(r, ops)
     return meta, out
