@@ -63,9 +63,10 @@ def parse():
     ap.add_argument("--no-rehash", action="store_true")
     ap.add_argument("--profile-only", action="store_true", help="a few steps, no extras (for ncu)")
     ap.add_argument("--l2-fetch", type=int, default=None, help="set cudaLimitMaxL2FetchGranularity (bytes)")
-    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4"],
+    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4", "c5"],
                     help="c2 = the headline (BASELINE configs[1]); c1/c3/c4 = the other single-GPU configs")
     ap.add_argument("--scale", type=float, default=1.0, help="c3: stream scale; c4: universe scale")
+    ap.add_argument("--c5-log2keys", type=int, default=31, help="c5: log2 of the total key count")
     ap.add_argument("--shape", default=None, help="c3: TW|RE, c4: LINE|COM")
     ap.add_argument("--routed", action="store_true",
                     help="use the sharded router even at N=1 (exercises the N>1 code path)")
@@ -297,6 +298,21 @@ def main():
     if args.l2_fetch is not None:
         L.check(L.dyc_set_l2_fetch_granularity(args.l2_fetch), "dyc_set_l2_fetch_granularity")
     n = 1 << args.log2n
+    if args.config == "c5":
+        if dist is None and world == 1:
+            import torch.distributed as dist
+            os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+            os.environ.setdefault("MASTER_PORT", "29541")
+            os.environ.setdefault("RANK", "0")
+            os.environ.setdefault("WORLD_SIZE", "1")
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        from paper_conf_icde_lizlhs21_b200.dist import bench_c5
+        line = bench_c5(args, rank, world, local, METRIC, ClockSampler)
+        if rank == 0:
+            emit(line)
+        dist.barrier()
+        dist.destroy_process_group()
+        return
     if world > 1 or args.routed:
         return multi_gpu(args, rank, world, local, dist)
     if args.config != "c2":

@@ -108,6 +108,7 @@ typedef struct {
     uint64_t last_insert_new;         /* new keys of the last insert batch               */
     uint64_t last_insert_pending;     /* ... of which needed the eviction kernel (k_place) */
     uint64_t last_insert_evictions;   /* eviction hops of the last insert batch          */
+    uint64_t bytes_cached;            /* released buffers kept for reuse (dyc_trim frees them) */
 } dyc_stats_t;
 
 /* Fills *cfg with the defaults: d=4, B=8, alpha=0.3, beta=0.85 (Table
@@ -185,6 +186,11 @@ dyc_status dyc_mixed_batch(dyc_table* t, const uint8_t* d_ops, const uint32_t* d
 dyc_status dyc_resize(dyc_table* t, int direction, int subtable, dyc_stream_t stream);
 dyc_status dyc_resize_ex(dyc_table* t, int direction, int subtable, int method, dyc_stream_t stream);
 
+/* Returns the buffers the table keeps for reuse (released subtables after a
+ * resize, old scratch) to the device.  Resizing frees a subtable's old buffer
+ * into this cache, so up/down cycles do not pay cudaMalloc each time. */
+dyc_status dyc_trim(dyc_table* t);
+
 /* Empties the table without resizing (all slots EMPTY, m = 0). */
 dyc_status dyc_clear(dyc_table* t, dyc_stream_t stream);
 
@@ -253,13 +259,14 @@ dyc_status dyc_route_count(dyc_table* t, const uint32_t* d_keys, uint64_t n, uin
  * where offset is the exclusive prefix sum of d_counts[world] (the histogram
  * from dyc_route_count, computed on the device here).  d_cursor[world]
  * (uint64, device) is scratch.  d_vals_in and d_vals_out may be NULL
- * (finds/deletes).  d_pos[i] (uint32) receives op i's position in the send
+ * (finds/deletes).  d_tags_in / d_tags_out (nullable) carry a uint8 per op (the op
+ * code of a mixed batch).  d_pos[i] (uint32) receives op i's position in the send
  * buffer, for dyc_route_unpermute.  Positions within one destination are in
  * unspecified order. */
 dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_vals_in,
-                             uint64_t n, uint32_t world, const uint64_t* d_counts, uint64_t* d_cursor,
-                             uint32_t* d_keys_out, uint32_t* d_vals_out, uint32_t* d_pos,
-                             dyc_stream_t stream);
+                             const uint8_t* d_tags_in, uint64_t n, uint32_t world, const uint64_t* d_counts,
+                             uint64_t* d_cursor, uint32_t* d_keys_out, uint32_t* d_vals_out,
+                             uint8_t* d_tags_out, uint32_t* d_pos, dyc_stream_t stream);
 
 /* Gathers replies back into request order: d_vals[i] = d_reply_vals[d_pos[i]],
  * d_status[i] = d_reply_status[d_pos[i]] (either pair may be NULL). */

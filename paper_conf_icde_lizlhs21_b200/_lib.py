@@ -37,7 +37,8 @@ class dyc_stats_t(C.Structure):
                 ("n_fail_upsize", C.c_uint64), ("n_residual", C.c_uint64), ("n_evict", C.c_uint64),
                 ("n_place_retry", C.c_uint64), ("n_second_table", C.c_uint64),
                 ("bytes_allocated", C.c_uint64), ("last_insert_new", C.c_uint64),
-                ("last_insert_pending", C.c_uint64), ("last_insert_evictions", C.c_uint64)]
+                ("last_insert_pending", C.c_uint64), ("last_insert_evictions", C.c_uint64),
+                ("bytes_cached", C.c_uint64)]
 
 
 class DycError(RuntimeError):
@@ -69,6 +70,7 @@ SIGNATURES = {
     "dyc_resize": (_I, [_TP, _I, _I, _P]),
     "dyc_resize_ex": (_I, [_TP, _I, _I, _I, _P]),
     "dyc_clear": (_I, [_TP, _P]),
+    "dyc_trim": (_I, [_TP]),
     "dyc_stats": (_I, [_TP, C.POINTER(dyc_stats_t), _P]),
     "dyc_dump": (_I, [_TP, _P, _P, _P, _U64, C.POINTER(_U64), _P]),
     "dyc_hash_params": (_I, [_TP, _P, _P]),
@@ -80,7 +82,7 @@ SIGNATURES = {
     "dyc_profile_enable": (_I, [_TP, _I]),
     "dyc_profile_read": (_I, [_TP, _P, _P]),
     "dyc_route_count": (_I, [_TP, _P, _U64, _U32, _P, _P]),
-    "dyc_route_scatter": (_I, [_TP, _P, _P, _U64, _U32, _P, _P, _P, _P, _P, _P]),
+    "dyc_route_scatter": (_I, [_TP, _P, _P, _P, _U64, _U32, _P, _P, _P, _P, _P, _P, _P]),
     "dyc_route_unpermute": (_I, [_P, _U64, _P, _P, _P, _P, _P]),
     "dyc_bench_gather": (_I, [_P, _U64, _U64, _U32, _U64, _P, _P]),
     "dyc_set_l2_fetch_granularity": (_I, [_U32]),

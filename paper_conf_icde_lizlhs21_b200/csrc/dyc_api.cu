@@ -14,6 +14,7 @@
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <unordered_map>
 #include <vector>
 
 #include <cuda_runtime.h>
@@ -68,7 +69,13 @@ struct dyc_table {
     int device = 0;
     int num_sms = 148;
     int place_blocks = 148 * 8;            // persistent grid of k_place
-    cudaMemPool_t pool = nullptr;
+    // device memory: cudaMalloc plus a per-table cache of released buffers
+    // (stream-ordered pool growth measured 10-30 GB/s on B200 vs ~1 ms/GB for
+    // cudaMalloc; profiles/r1_memory_model.md)
+    struct CachedBuf { void* p; uint64_t bytes; cudaEvent_t ev; };
+    std::vector<CachedBuf> cache;
+    uint64_t cache_bytes = 0;
+    std::unordered_map<void*, uint64_t> live;   // pointer -> bytes of live allocations
     unsigned long long* sub[DYC_MAX_D] = {};
     uint64_t nb[DYC_MAX_D] = {};
     uint32_t a[DYC_MAX_D + 2] = {}, b[DYC_MAX_D + 2] = {};
@@ -166,15 +173,70 @@ unsigned grid_for(uint64_t work, uint64_t per_block) {
     return (unsigned)g;
 }
 
+void trim_cache(dyc_table* t) {
+    for (auto& c : t->cache) {
+        cudaFree(c.p);                       // synchronizes the device
+        if (c.ev) t->ev_pool.push_back(c.ev);
+    }
+    t->cache.clear();
+    t->cache_bytes = 0;
+}
+
+// Allocation: an exact-size buffer released earlier by this table is reused (the
+// stream first waits for the work that used it); otherwise cudaMalloc.  On OOM
+// the cache is flushed and the allocation retried once.
 dyc_status dev_alloc(dyc_table* t, void** p, uint64_t bytes, cudaStream_t st) {
-    cudaError_t e = cudaMallocFromPoolAsync(p, std::max<uint64_t>(bytes, 8), t->pool, st);
+    bytes = std::max<uint64_t>(bytes, 256);
+    for (size_t i = 0; i < t->cache.size(); i++) {
+        if (t->cache[i].bytes == bytes) {
+            dyc_table::CachedBuf c = t->cache[i];
+            t->cache.erase(t->cache.begin() + (long)i);
+            t->cache_bytes -= c.bytes;
+            if (c.ev) {
+                cudaStreamWaitEvent(st, c.ev, 0);
+                t->ev_pool.push_back(c.ev);
+            }
+            *p = c.p;
+            t->live[c.p] = bytes;
+            return DYC_OK;
+        }
+    }
+    cudaError_t e = cudaMalloc(p, bytes);
+    if (e == cudaErrorMemoryAllocation && !t->cache.empty()) {
+        cudaGetLastError();
+        trim_cache(t);
+        e = cudaMalloc(p, bytes);
+    }
     if (e != cudaSuccess) {
         cudaGetLastError();
         *p = nullptr;
         return set_err(DYC_ERR_OOM, std::string("device allocation of ") + std::to_string(bytes) + " bytes failed: " +
                                         cudaGetErrorString(e));
     }
+    t->live[*p] = bytes;
     return DYC_OK;
+}
+
+// Release: the buffer goes to the cache, tagged with an event on `st` so that a
+// later reuse waits for the work still using it.
+void dev_free(dyc_table* t, void* p, cudaStream_t st) {
+    if (!p) return;
+    auto it = t->live.find(p);
+    const uint64_t bytes = it == t->live.end() ? 0 : it->second;
+    if (it != t->live.end()) t->live.erase(it);
+    cudaEvent_t ev = t->ev();
+    cudaEventRecord(ev, st);
+    t->cache.push_back({p, bytes, ev});
+    t->cache_bytes += bytes;
+    uint64_t cap = 256ull << 20;
+    for (uint32_t i = 0; i < t->cfg.d; i++) cap += t->nb[i] * t->cfg.bucket_slots * 8;
+    while (t->cache_bytes > cap && !t->cache.empty()) {      // oldest first
+        cudaEventSynchronize(t->cache.front().ev);
+        cudaFree(t->cache.front().p);
+        t->ev_pool.push_back(t->cache.front().ev);
+        t->cache_bytes -= t->cache.front().bytes;
+        t->cache.erase(t->cache.begin());
+    }
 }
 
 dyc_status read_ctr(dyc_table* t, cudaStream_t st) {
@@ -201,11 +263,11 @@ dyc_status ensure_lists(dyc_table* t, uint64_t n, cudaStream_t st) {
     TRY(dev_alloc(t, &l0, cap * 8, st));
     dyc_status s = dev_alloc(t, &l1, cap * 8, st);
     if (s != DYC_OK) {
-        cudaFreeAsync(l0, st);
+        dev_free(t, l0, st);
         return s;
     }
-    if (t->list[0]) cudaFreeAsync(t->list[0], st);
-    if (t->list[1]) cudaFreeAsync(t->list[1], st);
+    dev_free(t, t->list[0], st);
+    dev_free(t, t->list[1], st);
     t->list[0] = (unsigned long long*)l0;
     t->list[1] = (unsigned long long*)l1;
     t->list_cap = cap;
@@ -226,7 +288,7 @@ dyc_status upsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
             (uint32_t)n_new);
     }
     CU(cudaGetLastError());
-    CU(cudaFreeAsync(t->sub[ti], st));
+    dev_free(t, t->sub[ti], st);
     t->sub[ti] = (unsigned long long*)p;
     t->nb[ti] = n_new;
     return DYC_OK;
@@ -303,7 +365,7 @@ dyc_status downsize_launch(dyc_table* t, uint32_t ti, cudaStream_t st) {
                                                                        (uint32_t)h, t->list[0], t->d_ctr);
     }
     CU(cudaGetLastError());
-    CU(cudaFreeAsync(t->sub[ti], st));
+    dev_free(t, t->sub[ti], st);
     t->sub[ti] = (unsigned long long*)p;
     t->nb[ti] = h;
     return launch_place<B>(t, 0, t->d_ctr + C_RESIDUAL, 0, true, st);
@@ -360,7 +422,6 @@ dyc_status enforce_lower(dyc_table* t, cudaStream_t st) {
     t->n_evict += t->h_ctr[C_EVICT];
     t->n_residual += t->h_ctr[C_RES_TOTAL];
     TRY(settle<B>(t, 1, t->h_ctr[C_FAIL], st));
-    cudaMemPoolTrimTo(t->pool, 0);
     return DYC_OK;
 }
 
@@ -630,7 +691,7 @@ dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaSt
     t->n_evict += t->h_ctr[C_EVICT];
     const uint64_t nfail = t->h_ctr[C_FAIL];
     for (uint32_t i = 0; i < d; i++)
-        if (touched[i]) CU(cudaFreeAsync(old[i], st));
+        if (touched[i]) dev_free(t, old[i], st);
     if (nfail) TRY(place_and_settle<B>(t, 1, nullptr, nfail, true, st));
     return DYC_OK;
 }
@@ -699,6 +760,7 @@ dyc_status stats_impl(dyc_table* t, dyc_stats_t* out, cudaStream_t st) {
     out->n_place_retry = t->n_place_retry;
     out->n_second_table = t->h_ctr[C_SECOND];
     out->bytes_allocated = out->N * 8 + 2 * t->list_cap * 8 + t->stage_cap + C_N * 8;
+    out->bytes_cached = t->cache_bytes;
     out->last_insert_new = t->last_new;
     out->last_insert_pending = t->last_pending;
     out->last_insert_evictions = t->last_evict;
@@ -729,9 +791,9 @@ dyc_status dump_impl(dyc_table* t, uint64_t* h_kv, uint32_t* h_tab, uint64_t* h_
         if (h_tab) CU(cudaMemcpyAsync(h_tab, tb, ncopy * 4, cudaMemcpyDeviceToHost, st));
         if (h_bkt) CU(cudaMemcpyAsync(h_bkt, bk, ncopy * 8, cudaMemcpyDeviceToHost, st));
     }
-    CU(cudaFreeAsync(kv, st));
-    CU(cudaFreeAsync(tb, st));
-    CU(cudaFreeAsync(bk, st));
+    dev_free(t, kv, st);
+    dev_free(t, tb, st);
+    dev_free(t, bk, st);
     CU(cudaStreamSynchronize(st));
     if (n_out) *n_out = cnt;
     if (cnt != m) return set_err(DYC_ERR_CUDA, "dump found " + std::to_string(cnt) + " live slots, expected " +
@@ -762,7 +824,7 @@ dyc_status enter(dyc_table* t, dyc_stream_t s) {
 
 dyc_status ensure_stage(dyc_table* t, uint64_t bytes, cudaStream_t st) {
     if (bytes <= t->stage_cap) return DYC_OK;
-    if (t->stage) CU(cudaFreeAsync(t->stage, st));
+    if (t->stage) dev_free(t, t->stage, st);
     t->stage = nullptr;
     t->stage_cap = 0;
     TRY(dev_alloc(t, &t->stage, bytes, st));
@@ -819,17 +881,6 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
         t->a[s] = (uint32_t)(1 + splitmix64(st) % (kP - 1));   // a_s in [1, p)
         t->b[s] = (uint32_t)(splitmix64(st) % kP);             // b_s in [0, p)
     }
-    cudaMemPoolProps props{};
-    props.allocType = cudaMemAllocationTypePinned;
-    props.location.type = cudaMemLocationTypeDevice;
-    props.location.id = t->device;
-    cudaError_t e = cudaMemPoolCreate(&t->pool, &props);
-    if (e != cudaSuccess) {
-        delete t;
-        return cuda_err(e, "cudaMemPoolCreate");
-    }
-    uint64_t thr = ~0ull;
-    cudaMemPoolSetAttribute(t->pool, cudaMemPoolAttrReleaseThreshold, &thr);
     uint64_t per = (cfg->init_capacity + (uint64_t)d * B - 1) / ((uint64_t)d * B);   // Q13
     if (per < 1) per = 1;
     if (per > 0xFFFFFFFFull) {
@@ -871,18 +922,14 @@ dyc_status dyc_destroy(dyc_table* t) {
     if (!t) return DYC_OK;
     cudaSetDevice(t->device);
     cudaDeviceSynchronize();
-    for (uint32_t i = 0; i < t->cfg.d; i++)
-        if (t->sub[i]) cudaFree(t->sub[i]);
-    for (int i = 0; i < 2; i++)
-        if (t->list[i]) cudaFree(t->list[i]);
-    if (t->stage) cudaFree(t->stage);
-    if (t->mix) cudaFree(t->mix);
-    if (t->cp_in) cudaStreamDestroy(t->cp_in);
-    if (t->cp_out) cudaStreamDestroy(t->cp_out);
+    for (auto& kv : t->live) cudaFree(kv.first);   // subtables, lists, staging, scratch
+    t->live.clear();
+    trim_cache(t);
     if (t->d_ctr) cudaFree(t->d_ctr);
     if (t->h_ctr) cudaFreeHost(t->h_ctr);
+    if (t->cp_in) cudaStreamDestroy(t->cp_in);
+    if (t->cp_out) cudaStreamDestroy(t->cp_out);
     cudaDeviceSynchronize();
-    if (t->pool) cudaMemPoolDestroy(t->pool);
     for (auto& r : t->recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
     for (auto e : t->ev_pool) cudaEventDestroy(e);
     delete t;
@@ -983,7 +1030,7 @@ dyc_status dyc_mixed_batch(dyc_table* t, const uint8_t* d_ops, const uint32_t* d
     // scratch: keys, values, out values (u32 x n each), pos (u32 x n), status (u8 x n), 8 counters
     const uint64_t need = n * 17 + 128;
     if (need > t->mix_cap) {
-        if (t->mix) CU(cudaFreeAsync(t->mix, st));
+        if (t->mix) dev_free(t, t->mix, st);
         t->mix = nullptr;
         t->mix_cap = 0;
         TRY(dev_alloc(t, &t->mix, need, st));
@@ -1040,6 +1087,13 @@ dyc_status dyc_clear(dyc_table* t, dyc_stream_t stream) {
     for (uint32_t i = 0; i < t->cfg.d; i++)
         CU(cudaMemsetAsync(t->sub[i], 0xFF, t->nb[i] * t->cfg.bucket_slots * 8, S(stream)));
     t->m = 0;
+    return DYC_OK;
+}
+
+dyc_status dyc_trim(dyc_table* t) {
+    TRY(check_table(t));
+    CU(cudaSetDevice(t->device));
+    trim_cache(t);
     return DYC_OK;
 }
 
@@ -1153,9 +1207,10 @@ dyc_status dyc_route_count(dyc_table* t, const uint32_t* d_keys, uint64_t n, uin
     return DYC_OK;
 }
 
-dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_vals_in, uint64_t n,
-                             uint32_t world, const uint64_t* d_counts, uint64_t* d_cursor, uint32_t* d_keys_out,
-                             uint32_t* d_vals_out, uint32_t* d_pos, dyc_stream_t stream) {
+dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_vals_in,
+                             const uint8_t* d_tags_in, uint64_t n, uint32_t world, const uint64_t* d_counts,
+                             uint64_t* d_cursor, uint32_t* d_keys_out, uint32_t* d_vals_out, uint8_t* d_tags_out,
+                             uint32_t* d_pos, dyc_stream_t stream) {
     TRY(enter(t, stream));
     if (world < 1 || world > 1024) return set_err(DYC_ERR_INVALID_ARG, "world must be 1..1024");
     if (n == 0) return DYC_OK;
@@ -1171,7 +1226,8 @@ dyc_status dyc_route_scatter(dyc_table* t, const uint32_t* d_keys, const uint32_
         const HashDest hd{t->a[sh], t->b[sh], world, fastmod_magic(world), d_keys};
         k_group_scatter<HashDest><<<grid_for(n, (uint64_t)kThreads * kTileItems), kThreads, world * 12,
                                     S(stream)>>>(hd, d_keys, d_vals_in, n, world, (unsigned long long*)d_cursor,
-                                                 d_keys_out, d_vals_out, d_pos);
+                                                 d_keys_out, d_vals_out, d_pos, d_tags_in,
+                                                 d_tags_in ? d_tags_out : nullptr);
     }
     CU(cudaGetLastError());
     return DYC_OK;

@@ -724,7 +724,9 @@ __global__ void __launch_bounds__(kThreads) k_group_scatter(Dest dest, const uin
                                                             uint32_t world, unsigned long long* __restrict__ cursor,
                                                             uint32_t* __restrict__ keys_out,
                                                             uint32_t* __restrict__ vals_out,
-                                                            uint32_t* __restrict__ pos_out) {
+                                                            uint32_t* __restrict__ pos_out,
+                                                            const uint8_t* __restrict__ tags_in = nullptr,
+                                                            uint8_t* __restrict__ tags_out = nullptr) {
     extern __shared__ unsigned long long base[];            // per-destination global base of this tile
     unsigned* cnt = (unsigned*)(base + world);              // per-destination count / running rank
     const uint64_t tile = (uint64_t)kThreads * kTileItems;
@@ -749,6 +751,7 @@ __global__ void __launch_bounds__(kThreads) k_group_scatter(Dest dest, const uin
                 const uint64_t pos = base[dd[j]] + rk[j];
                 keys_out[pos] = keys[i];
                 if (vals_out) vals_out[pos] = vals_in ? vals_in[i] : 0u;
+                if (tags_out) tags_out[pos] = tags_in[i];
                 pos_out[i] = (uint32_t)pos;
             }
         }

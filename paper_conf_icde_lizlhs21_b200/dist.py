@@ -51,7 +51,7 @@ class DistTable:
         w = self.dist.all_to_all_single(out, x, recv_splits, send_splits, group=self.group, async_op=async_op)
         return out, w
 
-    def _run(self, op, keys, values=None, n_out=1, begin=None, end=None):
+    def _run(self, op, keys, values=None, n_out=1, begin=None, end=None, tags=None):
         """Pipelined route -> all-to-all -> owner op -> all-to-all back -> unpermute.
         op(keys, values) returns a tuple of n_out per-op result tensors.  begin(n)
         / end() bracket the owner's parts so that they form ONE batch (one
@@ -65,7 +65,12 @@ class DistTable:
             kc = keys[bounds[c]:bounds[c + 1]]
             vc = values[bounds[c]:bounds[c + 1]] if values is not None else None
             cnt = self.shard.route_count(kc, W)
-            parts.append(self.shard.route_scatter(kc, vc, W, cnt))
+            if tags is None:
+                kout, vout, pos = self.shard.route_scatter(kc, vc, W, cnt)
+                tout = None
+            else:
+                kout, vout, pos, tout = self.shard.route_scatter(kc, vc, W, cnt, tags=tags[bounds[c]:bounds[c + 1]])
+            parts.append((kout, vout, pos, tout))
             counts.append(cnt)
         # one exchange of every chunk's per-destination counts (row w: counts for rank w)
         send = torch.stack(counts).t().contiguous()
@@ -79,17 +84,18 @@ class DistTable:
             begin(self.last_recv)
         fwd = []
         for c in range(C):
-            kout, vout, _ = parts[c]
+            kout, vout, _, tout = parts[c]
             rk, wk = self._a2a(kout, ssp[c], rsp[c], async_op=True)
             rv, wv = self._a2a(vout, ssp[c], rsp[c], async_op=True) if values is not None else (None, None)
-            fwd.append((rk, wk, rv, wv))
+            rt, wt = self._a2a(tout, ssp[c], rsp[c], async_op=True) if tags is not None else (None, None)
+            fwd.append((rk, wk, rv, wv, rt, wt))
         back = []
         for c in range(C):
-            rk, wk, rv, wv = fwd[c]
-            wk.wait()
-            if wv is not None:
-                wv.wait()
-            res = op(rk, rv)
+            rk, wk, rv, wv, rt, wt = fwd[c]
+            for w_ in (wk, wv, wt):
+                if w_ is not None:
+                    w_.wait()
+            res = op(rk, rv) if tags is None else op(rk, rv, rt)
             res = res if isinstance(res, tuple) else (res,)
             back.append([self._a2a(r, rsp[c], ssp[c], async_op=True) for r in res])
         if end is not None:
@@ -100,7 +106,7 @@ class DistTable:
         for c in range(C):
             for (r, w) in back[c]:
                 w.wait()
-            _, _, pos = parts[c]
+            pos = parts[c][2]
             got = [r for (r, _) in back[c]]
             lo, hi = bounds[c], bounds[c + 1]
             if hi == lo:
@@ -136,6 +142,16 @@ class DistTable:
             return self.shard.delete(keys)
         return self._run(lambda k, v: self.shard.delete_part(k), keys, None, n_out=2,
                          begin=self.shard.delete_begin, end=self.shard.delete_end)
+
+    def mixed(self, ops, keys, values):
+        """Mixed batch (op codes 0 find / 1 insert / 2 delete, reading Q10).  The op
+        codes travel with the keys; each owner runs its part as a mixed batch.
+        Keys are distinct within the batch, so splitting it into chunks and
+        shards changes no result.  Returns (values, status) in request order."""
+        if self.world == 1 and not self.force_route:
+            self.last_recv = keys.numel()
+            return self.shard.mixed(ops, keys, values)
+        return self._run(lambda k, v, t: self.shard.mixed(t, k, v), keys, values, n_out=2, tags=ops)
 
     def stats(self):
         return self.shard.stats()
@@ -269,4 +285,77 @@ def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_pea
         "gpu_launches": launches,
         "clocks": clk.summary(),
         "roofline": roofline, "cpu_baseline": None, "e2e": e2e,
+    }
+
+
+# ---------------------------------------------------------------- config C5
+def bench_c5(args, rank, world, local, metric, ClockSampler):
+    """Config C5 (BASELINE.json configs[4]): 2^31 RAND keys hash-partitioned over
+    G shards.  Fill: global batches of 16M inserts of key(0 .. 2^31-1); then 32
+    mixed 50/30/20 global batches of 16M ops.  Rank r issues ops [r*16M/G,
+    (r+1)*16M/G) of every global batch; each shard starts at 1M slots and
+    resizes on its own.  Time = max over ranks, per phase."""
+    import torch
+    import torch.distributed as dist
+    from . import workload as W
+    from .table import Table
+
+    log2k = getattr(args, "c5_log2keys", 31)
+    batch = 1 << min(24, log2k - 3)
+    shard = Table(d=4, init_capacity=1 << 20, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
+    dt = DistTable(shard, force_route=getattr(args, "routed", False))
+    stream = torch.cuda.current_stream()
+    gen = W.c5_batches_torch(rank, world, device="cuda", log2_keys=log2k, batch=batch, mixed_batches=32)
+    fill, mixed = [], []
+    for item in gen:                      # materialise this rank's slices up front (inputs resident in HBM)
+        (fill if item[0] == "insert" else mixed).append(item)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    checks = torch.zeros(4, dtype=torch.int64, device="cuda")
+    shard.profile(True)
+    with ClockSampler(local) as clk:
+        a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+        a.record(stream)
+        for _, k, v in fill:
+            st = dt.insert(k, v)
+            checks[0] += (st == 1).sum()
+        b.record(stream)
+        for _, ops, k, v in mixed:
+            vals, st = dt.mixed(ops, k, v)
+            checks[1] += ((ops == 0) & (st == 1)).sum()
+            checks[2] += ((ops == 1) & (st == 1)).sum()
+            checks[3] += ((ops == 2) & (st == 1)).sum()
+        c.record(stream)
+        torch.cuda.synchronize()
+    t = torch.tensor([a.elapsed_time(b), b.elapsed_time(c)], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(checks)
+    prof = shard.profile_read()
+    shard.profile(False)
+    st = shard.stats()
+    fill_ms, mixed_ms = float(t[0]), float(t[1])
+    n_fill, n_mixed = len(fill) * batch, len(mixed) * batch
+    if rank != 0:
+        return None
+    return {
+        "metric": metric, "value": (n_fill + n_mixed) / ((fill_ms + mixed_ms) * 1e-3) / 1e6, "unit": "Mops/s",
+        "n_gpus": world, "steps": 1, "warmup": 0, "ms_per_step": fill_ms + mixed_ms, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": f"C5 RAND 2^{log2k} keys hash-partitioned over {world} shard(s): {len(fill)} global "
+                               f"insert batches of {batch}, then {len(mixed)} mixed 50/30/20 batches of {batch}",
+                   "d": 4, "alpha": 0.3, "beta": 0.85, "bucket_slots": args.bucket_slots,
+                   "parallelism": f"shard{world}", "init_capacity_per_shard": 1 << 20},
+        "phases": {"fill_ms": fill_ms, "fill_mops": n_fill / fill_ms / 1e3,
+                   "mixed_ms": mixed_ms, "mixed_mops": n_mixed / mixed_ms / 1e3},
+        "check": {"inserted_fill": int(checks[0]), "expected_fill": n_fill,
+                  "found_in_mixed": int(checks[1]), "expected_found": len(mixed) * (batch // 4),
+                  "inserted_in_mixed": int(checks[2]), "deleted_in_mixed": int(checks[3])},
+        "shard0": {"fill": st["fill"], "buckets": st["buckets"], "m": st["m"], "n_upsize": st["n_upsize"],
+                   "n_downsize": st["n_downsize"], "bytes": st["bytes_allocated"]},
+        "kernel_ms_rank0": {k: round(v[0], 2) for k, v in prof.items() if v[1]},
+        "kernel_calls_rank0": {k: v[1] for k, v in prof.items() if v[1]},
+        "clocks": clk.summary(), "gpu_launches": sum(v[1] for v in prof.values()), "roofline": None,
+        "cpu_baseline": None, "e2e": None,
     }

@@ -201,6 +201,10 @@ class Table:
         L.check(self._lib.dyc_resize_ex(self._h, direction, subtable, method, _stream_ptr(stream)),
                 "dyc_resize_ex")
 
+    def trim(self):
+        """Return cached (released) device buffers to the device."""
+        L.check(self._lib.dyc_trim(self._h), "dyc_trim")
+
     def clear(self, stream=None):
         L.check(self._lib.dyc_clear(self._h, _stream_ptr(stream)), "dyc_clear")
 
@@ -214,7 +218,7 @@ class Table:
                     n_place_retry=s.n_place_retry, n_second_table=s.n_second_table,
                     bytes_allocated=s.bytes_allocated, last_insert_new=s.last_insert_new,
                     last_insert_pending=s.last_insert_pending,
-                    last_insert_evictions=s.last_insert_evictions)
+                    last_insert_evictions=s.last_insert_evictions, bytes_cached=s.bytes_cached)
 
     def dump(self, stream=None):
         """(kv uint64, table uint32, bucket uint64) host arrays, unspecified order."""
@@ -269,20 +273,24 @@ class Table:
                                           _stream_ptr(stream)), "dyc_route_count")
         return counts
 
-    def route_scatter(self, keys, values, world: int, counts, stream=None):
-        """Groups ops by destination shard; returns (keys_out, values_out|None, pos)."""
+    def route_scatter(self, keys, values, world: int, counts, stream=None, tags=None):
+        """Groups ops by destination shard; returns (keys_out, values_out|None, pos)
+        or, with a uint8 `tags` tensor, (keys_out, values_out|None, pos, tags_out)."""
         torch = _torch()
         _check_u32(keys, "keys")
         n = keys.numel()
         kout = torch.empty(n, dtype=torch.int32, device=keys.device)
         vout = torch.empty(n, dtype=torch.int32, device=keys.device) if values is not None else None
+        tout = torch.empty(n, dtype=torch.uint8, device=keys.device) if tags is not None else None
         pos = torch.empty(n, dtype=torch.int32, device=keys.device)
         cursor = torch.empty(world, dtype=torch.int64, device=keys.device)
         L.check(self._lib.dyc_route_scatter(self._h, keys.data_ptr(), values.data_ptr() if values is not None else None,
-                                            n, world, counts.data_ptr(), cursor.data_ptr(), kout.data_ptr(),
-                                            vout.data_ptr() if vout is not None else None, pos.data_ptr(),
+                                            tags.data_ptr() if tags is not None else None, n, world,
+                                            counts.data_ptr(), cursor.data_ptr(), kout.data_ptr(),
+                                            vout.data_ptr() if vout is not None else None,
+                                            tout.data_ptr() if tout is not None else None, pos.data_ptr(),
                                             _stream_ptr(stream)), "dyc_route_scatter")
-        return kout, vout, pos
+        return (kout, vout, pos) if tags is None else (kout, vout, pos, tout)
 
     def route_unpermute(self, pos, reply_vals=None, reply_status=None, stream=None, out_vals=None, out_status=None):
         """vals[i] = reply_vals[pos[i]], status[i] = reply_status[pos[i]] (written

@@ -432,3 +432,42 @@ def c4_zipf_mixed(U: int = 45_159_880, distinct: int = 4_000_000, grow_batches: 
             out.append(MixedBatch(ops, k, val_of(k, ver)))
             apply(r, ops)
     return meta, out
+
+
+# ---------------------------------------------------------------------------
+# Config C5: RAND 2^31 keys hash-partitioned across G GPUs.
+def c5_batches_torch(rank: int, world: int, device="cuda", log2_keys: int = 31, batch: int = 1 << 24,
+                     fill_batches: Optional[int] = None, mixed_batches: int = 32, seed_cfg: Optional[int] = None):
+    """Generator of this rank's slice of every global batch (rank r issues ops
+    [r*batch/G, (r+1)*batch/G) of each).  Fill: key(0 .. 2^log2_keys - 1) in
+    global batches of `batch` inserts.  Then mixed 50/30/20 global batches:
+    finds = half live keys key(2^(log2_keys-1) + perm(j)) (a range no mixed batch
+    deletes) and half never-inserted misses; inserts = new keys from the index
+    range above the fill; deletes = distinct live keys key(b*0.2*batch + j).
+    Keys are distinct within every global batch.  Yields (op, keys, values)
+    int32 tensors; op in {"insert", "mixed"}; a mixed batch is (ops u8, keys, vals)."""
+    import torch
+    s = config_seed(5) if seed_cfg is None else seed_cfg
+    n_keys = 1 << log2_keys
+    fb = fill_batches if fill_batches is not None else n_keys // batch
+    lo, hi = rank * batch // world, (rank + 1) * batch // world
+    loc = torch.arange(lo, hi, dtype=torch.int64, device=device)
+    for j in range(fb):
+        k = _key_of_t(j * batch + loc, s)
+        yield "insert", _as_i32(k), _as_i32(_lowbias32_t(k ^ 0x9E3779B9))
+    nf, ni = batch // 2, (batch * 3) // 10
+    nd = batch - nf - ni
+    half = n_keys >> 1
+    for b in range(mixed_batches):
+        g = loc                                               # this rank's positions in the global batch
+        is_f, is_i = g < nf, (g >= nf) & (g < nf + ni)
+        # finds: even positions live (from [half, n_keys)), odd positions misses
+        live_idx = half + (_perm_pow2_t(g, log2_keys - 1, s ^ (b * 7919 + 1)) & (half - 1))
+        miss_idx = n_keys + (1 << 30) + b * batch + g
+        f_idx = torch.where(g % 2 == 0, live_idx, miss_idx)
+        i_idx = n_keys + b * ni + (g - nf)                    # new keys above the fill range
+        d_idx = b * nd + (g - nf - ni)                        # distinct live keys below `half`
+        idx = torch.where(is_f, f_idx, torch.where(is_i, i_idx, d_idx))
+        k = _key_of_t(idx, s)
+        ops = torch.where(is_f, 0, torch.where(is_i, 1, 2)).to(torch.uint8)
+        yield "mixed", ops, _as_i32(k), _as_i32(_lowbias32_t(k ^ (0x9E3779B9 * (b + 2) & 0xFFFFFFFF)))

@@ -24,7 +24,7 @@ class DictShard:
         k = keys.to(torch.int64) & 0xFFFFFFFF
         return torch.bincount(k % world, minlength=world).to(torch.int64)
 
-    def route_scatter(self, keys, values, world, counts):
+    def route_scatter(self, keys, values, world, counts, tags=None):
         k = keys.to(torch.int64) & 0xFFFFFFFF
         dest = k % world
         order = torch.argsort(dest, stable=True)
@@ -32,7 +32,24 @@ class DictShard:
         pos[order] = torch.arange(order.numel())
         kout = keys[order].clone()
         vout = values[order].clone() if values is not None else None
+        if tags is not None:
+            return kout, vout, pos.to(torch.int32), tags[order].clone()
         return kout, vout, pos.to(torch.int32)
+
+    def mixed(self, ops, keys, vals):
+        v = torch.full((keys.numel(),), -1, dtype=torch.int32)
+        s = torch.zeros(keys.numel(), dtype=torch.uint8)
+        for op in (0, 1, 2):
+            sel = torch.nonzero(ops == op).flatten()
+            if sel.numel() == 0:
+                continue
+            if op == 0:
+                v[sel], s[sel] = self.find(keys[sel])
+            elif op == 1:
+                s[sel] = self.insert(keys[sel], vals[sel])
+            else:
+                v[sel], s[sel] = self.delete(keys[sel])
+        return v, s
 
     def route_unpermute(self, pos, rv=None, rs=None, out_vals=None, out_status=None):
         p = pos.to(torch.int64)
@@ -135,6 +152,27 @@ def _worker(rank, world, port, q, chunks):
             for r in range(world):
                 for k in ks[r]:
                     model.pop(int(k), None)
+    # one mixed batch (find -> insert -> delete, reading Q10), keys distinct across ranks
+    rng = np.random.Generator(np.random.PCG64(99))
+    allk = rng.choice(np.arange(1, 1 << 20), size=300 * world, replace=False)
+    allops = rng.integers(0, 3, size=allk.size)
+    mk = torch.tensor(allk[rank * 300:(rank + 1) * 300], dtype=torch.int32)
+    mo = torch.tensor(allops[rank * 300:(rank + 1) * 300], dtype=torch.uint8)
+    mv = torch.arange(300, dtype=torch.int32) + 7
+    v, s = dt.mixed(mo, mk, mv)
+    for i, (k, op) in enumerate(zip(mk.tolist(), mo.tolist())):
+        if op == 0:
+            ok &= (int(s[i]) == (1 if k in model else 0)) and (int(s[i]) == 0 or int(v[i]) == model[k])
+        elif op == 1:
+            ok &= int(s[i]) == (2 if k in model else 1)
+        else:
+            ok &= int(s[i]) == (1 if k in model else 0)
+    for r in range(world):
+        for k, op, j in zip(allk[r * 300:(r + 1) * 300], allops[r * 300:(r + 1) * 300], range(300)):
+            if op == 1:
+                model[int(k)] = j + 7
+            elif op == 2:
+                model.pop(int(k), None)
     # union of the shards == the single-table model
     sizes = [None] * world
     dist.all_gather_object(sizes, len(dt.shard.m))

@@ -74,3 +74,28 @@ def test_dist_table_nccl_world1(oracle_mod):
         np.testing.assert_array_equal(shard.sorted_kv(), o.sorted_kv())
     finally:
         dist.destroy_process_group()
+
+
+def test_dist_table_mixed_routed_world1(oracle_mod):
+    """DistTable.mixed through the CUDA routing kernels (op codes travel with the
+    keys) equals the oracle's mixed batch (reading Q10)."""
+    import torch.distributed as dist
+    from paper_conf_icde_lizlhs21_b200.dist import DistTable
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1)
+    try:
+        meta, batches = W.c4_zipf_mixed(U=50000, distinct=5000, grow_batches=4, cycles=1, init_capacity=1024)
+        shard = Table(d=4, init_capacity=1024, alpha=meta.alpha, beta=meta.beta, bucket_slots=8)
+        o = oracle_mod.OracleTable(d=4, init_capacity=1024, alpha=meta.alpha, beta=meta.beta, bucket_slots=8)
+        dt = DistTable(shard, force_route=True, chunks=3)
+        for b in batches:
+            v, st = dt.mixed(torch.from_numpy(b.ops).cuda(), dev(b.keys), dev(b.values))
+            ov, os_ = o.mixed(b.ops, b.keys, b.values)
+            np.testing.assert_array_equal(st.cpu().numpy(), os_)
+            np.testing.assert_array_equal(v.cpu().numpy().view(np.uint32), ov)
+            np.testing.assert_array_equal(shard.sorted_kv(), o.sorted_kv())
+    finally:
+        dist.destroy_process_group()
