@@ -67,6 +67,11 @@ def parse():
                     help="c2 = the headline (BASELINE configs[1]); c1/c3/c4 = the other single-GPU configs")
     ap.add_argument("--scale", type=float, default=1.0, help="c3: stream scale; c4: universe scale")
     ap.add_argument("--c5-log2keys", type=int, default=31, help="c5: log2 of the total key count")
+    ap.add_argument("--d", type=int, default=4, help="number of subtables (paper default 4, P:L804)")
+    ap.add_argument("--alpha", type=float, default=None, help="lower fill bound (c3/c4 sweeps, Table tbl:parameters)")
+    ap.add_argument("--beta", type=float, default=None, help="upper fill bound (sweeps; c2 fill target)")
+    ap.add_argument("--r", type=float, default=0.2, help="c3: deletes per insert (P:L732-733)")
+    ap.add_argument("--batch", type=int, default=None, help="c3: batch size (Table tbl:parameters: 2e5..1e6)")
     ap.add_argument("--shape", default=None, help="c3: TW|RE, c4: LINE|COM")
     ap.add_argument("--routed", action="store_true",
                     help="use the sharded router even at N=1 (exercises the N>1 code path)")
@@ -317,10 +322,12 @@ def main():
         return multi_gpu(args, rank, world, local, dist)
     if args.config != "c2":
         return emit(bench_stream(args, local))
-    cap, k_ins, v_ins, k_find, k_del = W.c2_rand_static_torch(args.log2n, device="cuda")
+    beta = args.beta or 0.85
+    cap, k_ins, v_ins, k_find, k_del = W.c2_rand_static_torch(args.log2n, device="cuda", beta=beta)
 
     stream = torch.cuda.current_stream()
-    g = Table(d=4, init_capacity=cap, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
+    g = Table(d=args.d, init_capacity=cap, alpha=0.3 if args.alpha is None else args.alpha,
+              beta=min(0.99, beta + 1e-6) if beta > 0.85 else 0.85, bucket_slots=args.bucket_slots)
     st_ins = torch.empty(n, dtype=torch.uint8, device="cuda")
     v_out = torch.empty(n, dtype=torch.int32, device="cuda")
     f_out = torch.empty(n, dtype=torch.uint8, device="cuda")
@@ -343,7 +350,10 @@ def main():
         if evs: evs[4].record(stream)
         g.delete(k_del, dv_out, ds_out)
         if evs: evs[5].record(stream)
-        g.resize(-1)
+        try:
+            g.resize(-1)
+        except L.DycError:
+            pass          # the delete's own alpha check already halved it back (small d / low fill)
         if evs:
             evs[6].record(stream)
             record.append(evs)
@@ -361,7 +371,10 @@ def main():
     assert int(ds_out.sum().item()) == n // 2
     s_del_before = g.stats()
     phi_after_up = s_del_before["n_second_table"] / max(1, s_del_before["m"])
-    g.resize(-1)
+    try:
+        g.resize(-1)
+    except L.DycError:
+        pass
 
     for _ in range(args.warmup):
         step()
@@ -483,7 +496,7 @@ def main():
         "config": {"workload": f"C2 RAND static (BASELINE.json configs[1]): 2^{args.log2n} inserts to fill 0.85, "
                                f"2^{args.log2n} finds (50% hit), one subtable upsize, 2^{args.log2n - 1} deletes, "
                                "one subtable downsize",
-                   "d": 4, "alpha": 0.3, "beta": 0.85, "bucket_slots": args.bucket_slots,
+                   "d": args.d, "alpha": 0.3, "beta": beta, "bucket_slots": args.bucket_slots,
                    "table_bytes": int(s_ins["N"] * 8),
                    "l2": "inputs and table larger than L2 (126 MB); no flush needed"},
         "phase_ms": phase_ms,
@@ -518,11 +531,15 @@ def bench_stream(args, local):
         name = "C1 RAND small (BASELINE configs[0]): 65,536 keys, 8x8192 insert, find (50% hit), delete"
     elif args.config == "c3":
         shape = args.shape or "TW"
-        wl = W.c3_dynamic(scale=args.scale, shape=shape, batch=max(1000, int(1_000_000 * min(1.0, args.scale * 4))),
-                          cycles=2)
+        bsz = args.batch or max(1000, int(1_000_000 * min(1.0, args.scale * 4)))
+        wl = W.c3_dynamic(scale=args.scale, shape=shape, batch=bsz, r=args.r, cycles=2)
+        if args.alpha is not None:
+            wl.alpha = args.alpha
+        if args.beta is not None:
+            wl.beta = args.beta
         batches, mixed = wl.batches, False
-        name = (f"C3 {shape}-shaped dynamic stream x{args.scale:g}: sliding window of insert + find (50% hit) + "
-                "0.2x delete batches, swap pass, 2 cycles")
+        name = (f"C3 {shape}-shaped dynamic stream x{args.scale:g}: sliding window of {bsz} inserts + find (50% hit)"
+                f" + {args.r:g}x delete batches, swap pass, 2 cycles, alpha {wl.alpha:g} beta {wl.beta:g}")
     else:
         shape = args.shape or "COM"
         U, D = (4_583_941, 1_000_000) if shape == "COM" else (45_159_880, 4_000_000)
@@ -532,7 +549,7 @@ def bench_stream(args, local):
         name = (f"C4 {shape}-shaped Zipf(0.99) mixed 50/30/20 batches of {D} distinct keys over U={U}, "
                 "grow 16 batches then drain, 2 cycles")
     gen_s = time.time() - t0
-    g = Table(d=wl.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=args.bucket_slots)
+    g = Table(d=args.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=args.bucket_slots)
     dev = lambda a: torch.from_numpy(np.ascontiguousarray(a, dtype=np.uint32).view(np.int32)).cuda()  # noqa: E731
     staged = []
     for b in batches:
@@ -615,7 +632,7 @@ def bench_stream(args, local):
         "metric": METRIC, "value": n_ops / total_ms / 1e3, "unit": "Mops/s", "n_gpus": 1, "steps": 1,
         "warmup": args.warmup, "ms_per_step": total_ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": name, "d": wl.d, "alpha": wl.alpha, "beta": wl.beta,
+        "config": {"workload": name, "d": args.d, "alpha": wl.alpha, "beta": wl.beta,
                    "bucket_slots": args.bucket_slots, "batches": len(staged), "ops": n_ops},
         "ops": ops_line,
         "fill_track": {"min_after_mutation": min(x for x, (op, *_r) in zip(track, staged) if op != "find"),
