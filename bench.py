@@ -447,6 +447,68 @@ def main():
             resize[f"{name}_downsize_ms"] = timed(lambda: t2.resize(-1, -1, method))
             t2.close()
             del t2
+        # resize under live traffic (NEXT-1): the split/merge runs on a
+        # second stream while a 2^k find batch runs on this one (dyc_resize_begin/commit)
+        rs = torch.cuda.Stream()
+        for direction, fill in ((+1, 0.85), (-1, 0.30)):
+            tag = "upsize" if direction > 0 else "downsize"
+            t2 = Table(d=4, init_capacity=cap, alpha=0.05, beta=0.85, bucket_slots=args.bucket_slots)
+            if direction < 0:
+                t2.resize(+1)
+            m_fill = min(n, int(fill * t2.stats()["N"]))
+            t2.insert(k_ins[:m_fill], v_ins[:m_fill], st_ins[:m_fill])
+
+            def seq():
+                t2.resize(direction)
+                t2.find(k_find, v_out, f_out)
+
+            def live():
+                t2.resize_begin(direction, resize_stream=rs)
+                t2.find(k_find, v_out, f_out)
+                t2.resize_commit()
+
+            t2.find(k_find, v_out, f_out)
+            hits0 = int(f_out.sum().item())
+            res = {}
+            for name, fn in (("sequential", seq), ("live", live), ("sequential", seq), ("live", live)):
+                ms = timed(fn)                         # second pass of each is the warm one
+                assert int(f_out.sum().item()) == hits0, "find during a live resize lost keys"
+                res[name] = ms
+                t2.resize(-direction)                  # back to the starting shape
+            res["find_alone"] = timed(lambda: t2.find(k_find, v_out, f_out))
+
+            # latency of a small find batch that arrives when the resize starts:
+            # behind a blocking resize vs. beside a live one (availability)
+            ns = min(n, 1 << 20)
+
+            def small_find_latency(live_mode):
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                torch.cuda.synchronize()
+                a.record(stream)
+                if live_mode:
+                    t2.resize_begin(direction, resize_stream=rs)
+                else:
+                    t2.resize(direction)
+                t2.find(k_find[:ns], v_out[:ns], f_out[:ns])
+                b.record(stream)
+                if live_mode:
+                    t2.resize_commit()
+                torch.cuda.synchronize()
+                t2.resize(-direction)
+                return a.elapsed_time(b)
+
+            for live_mode in (False, True, False, True):
+                res[f"lat_{live_mode}"] = small_find_latency(live_mode)
+            resize[f"small_find_latency_ms_behind_blocking_{tag}"] = res["lat_False"]
+            resize[f"small_find_latency_ms_during_live_{tag}"] = res["lat_True"]
+            resize["small_find_keys"] = ns
+            resize[f"live_{tag}_plus_find_ms"] = res["live"]
+            resize[f"sequential_{tag}_then_find_ms"] = res["sequential"]
+            resize[f"find_alone_ms_at_{tag}_fill"] = res["find_alone"]
+            t2.close()
+            del t2
+        resize["live_note"] = ("live_* = dyc_resize_begin on a second stream + a 2^k find batch on the caller's "
+                               "stream + dyc_resize_commit; sequential_* = dyc_resize then the same find batch")
         resize["speedup_upsize_vs_rehash_all"] = resize["rehash_all_upsize_ms"] / resize["split_upsize_ms"]
         resize["speedup_upsize_vs_reinsert_subtable"] = (resize["reinsert_subtable_upsize_ms"]
                                                          / resize["split_upsize_ms"])

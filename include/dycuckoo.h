@@ -109,6 +109,8 @@ typedef struct {
     uint64_t last_insert_pending;     /* ... of which needed the eviction kernel (k_place) */
     uint64_t last_insert_evictions;   /* eviction hops of the last insert batch          */
     uint64_t bytes_cached;            /* released buffers kept for reuse (dyc_trim frees them) */
+    uint64_t n_live_resize;           /* resizes committed through dyc_resize_begin/commit */
+    uint64_t n_deferred;              /* ops deferred because their subtable was being resized */
 } dyc_stats_t;
 
 /* Fills *cfg with the defaults: d=4, B=8, alpha=0.3, beta=0.85 (Table
@@ -185,6 +187,40 @@ dyc_status dyc_mixed_batch(dyc_table* t, const uint8_t* d_ops, const uint32_t* d
  * DYC_ERR_INVALID_ARG.  dyc_resize_ex selects the method (DYC_RESIZE_*). */
 dyc_status dyc_resize(dyc_table* t, int direction, int subtable, dyc_stream_t stream);
 dyc_status dyc_resize_ex(dyc_table* t, int direction, int subtable, int method, dyc_stream_t stream);
+
+/* Resize under live traffic ("we do not need
+ * to lock all hash tables and only to resize one", "it only locks the
+ * subtable being resized and supports concurrent updates for the remaining
+ * subtables").
+ *
+ * dyc_resize_begin enqueues the split (direction +1) or merge
+ * (direction -1) of one subtable (-1 = the policy's choice; the
+ * same shape rules as dyc_resize) on `resize_stream`, ordered after the work
+ * already enqueued on `stream`, and returns without waiting.  The resize is
+ * then "in flight" until it is committed:
+ *   - find batches run concurrently with it and see every key (they read the
+ *     subtable's old buffer, which nothing writes while it is being copied);
+ *   - insert and delete batches run against the old buffer too, with the
+ *     resized subtable locked: ops that need to write it (an update or delete
+ *     of a key stored there, a new key whose other candidate bucket is full) are
+ *     deferred; if a batch has any, it commits the resize at its end and then
+ *     applies them, so every batch's statuses, values and the table contents
+ *     are exactly those of the sequential order "resize, then the batches";
+ *   - every resize decision (Q11) is taken against the post-resize
+ *     size; one that has to act commits first;
+ *   - dyc_resize*, dyc_stats, dyc_dump and dyc_clear commit first.
+ * dyc_resize_commit makes `stream` wait for the resize kernel and installs the
+ * new buffer (a downsize then places its residuals); it is a no-op
+ * when nothing is in flight.  All batches of the window must be issued on one
+ * stream (`stream`), or ordered by the caller.  Errors: DYC_ERR_INVALID_ARG if
+ * a resize is already in flight, a part batch is open, or the shape rules
+ * forbid the resize; DYC_ERR_OOM. */
+dyc_status dyc_resize_begin(dyc_table* t, int direction, int subtable, dyc_stream_t stream,
+                            dyc_stream_t resize_stream);
+dyc_status dyc_resize_commit(dyc_table* t, dyc_stream_t stream);
+/* *in_flight = 1 while a resize is uncommitted; *kernel_done = 1 once its
+ * kernel has finished on the device (either pointer may be NULL). */
+dyc_status dyc_resize_query(const dyc_table* t, int* in_flight, int* kernel_done);
 
 /* Returns the buffers the table keeps for reuse (released subtables after a
  * resize, old scratch) to the device.  Resizing frees a subtable's old buffer

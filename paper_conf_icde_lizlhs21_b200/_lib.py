@@ -38,7 +38,7 @@ class dyc_stats_t(C.Structure):
                 ("n_place_retry", C.c_uint64), ("n_second_table", C.c_uint64),
                 ("bytes_allocated", C.c_uint64), ("last_insert_new", C.c_uint64),
                 ("last_insert_pending", C.c_uint64), ("last_insert_evictions", C.c_uint64),
-                ("bytes_cached", C.c_uint64)]
+                ("bytes_cached", C.c_uint64), ("n_live_resize", C.c_uint64), ("n_deferred", C.c_uint64)]
 
 
 class DycError(RuntimeError):
@@ -69,6 +69,9 @@ SIGNATURES = {
     "dyc_mixed_batch": (_I, [_TP, _P, _P, _P, _P, _P, _U64, _P]),
     "dyc_resize": (_I, [_TP, _I, _I, _P]),
     "dyc_resize_ex": (_I, [_TP, _I, _I, _I, _P]),
+    "dyc_resize_begin": (_I, [_TP, _I, _I, _P, _P]),
+    "dyc_resize_commit": (_I, [_TP, _P]),
+    "dyc_resize_query": (_I, [_TP, C.POINTER(_I), C.POINTER(_I)]),
     "dyc_clear": (_I, [_TP, _P]),
     "dyc_trim": (_I, [_TP]),
     "dyc_stats": (_I, [_TP, C.POINTER(dyc_stats_t), _P]),

@@ -96,6 +96,21 @@ struct dyc_table {
     uint64_t launches = 0;
     uint64_t last_new = 0, last_pending = 0, last_evict = 0;
     cudaStream_t last = nullptr;
+    // resize under live traffic (dyc_resize_begin / dyc_resize_commit, NEXT-1):
+    // the split / merge kernel of subtable `ti` runs on the caller's resize
+    // stream into `nbuf` while batches keep using the old buffer of ti
+    // (read-only for them: the LK kernel variants defer any write to ti).
+    struct Live {
+        bool active = false;
+        int dir = 0;
+        uint32_t ti = 0;
+        unsigned long long* nbuf = nullptr;
+        uint64_t nnb = 0;
+        unsigned long long* res[2] = {nullptr, nullptr};   // downsize residuals / their failures
+        unsigned long long* ctr = nullptr;                  // counters of the resize stream (C_N)
+        cudaEvent_t start = nullptr, done = nullptr;
+    } rz;
+    uint64_t n_live_resize = 0, n_deferred = 0;
     // per-kernel event profiling (dyc_profile_*)
     bool prof = false;
     struct Rec { int kind; cudaEvent_t a, b; };
@@ -115,6 +130,11 @@ struct dyc_table {
         uint64_t s = 0;
         for (uint32_t t = 0; t < cfg.d; t++) s += nb[t] * cfg.bucket_slots;
         return s;
+    }
+    // N once the resize in flight (if any) is committed: the size every resize
+    // decision is taken against, as if the resize had completed first
+    uint64_t N_after() const {
+        return rz.active ? N() - nb[rz.ti] * cfg.bucket_slots + rz.nnb * cfg.bucket_slots : N();
     }
     int smallest() const {      // ties -> lowest index (Q12)
         int best = 0;
@@ -297,7 +317,8 @@ dyc_status upsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
 // Retries the nfail homeless pairs in list[cur]: first a plain retry pass, then
 // failure-triggered upsizes (Q17: nothing is ever dropped).
 template <int B>
-dyc_status settle(dyc_table* t, int cur, uint64_t nfail, cudaStream_t st) {
+dyc_status settle(dyc_table* t, int cur, uint64_t nfail, cudaStream_t st, unsigned long long* const* lists = nullptr) {
+    unsigned long long* const* L = lists ? lists : t->list;
     int round = 0;
     while (nfail > 0) {
         if (round > 0) {
@@ -310,8 +331,8 @@ dyc_status settle(dyc_table* t, int cur, uint64_t nfail, cudaStream_t st) {
         TRY(zero_one(t, C_EVICT, st));
         {
             ProfScope ps(t, DYC_PROF_PLACE, st);
-            k_place<B><<<grid_for(nfail, kThreads / (B / 4)), kThreads, 0, st>>>(t->view(), t->list[cur], nullptr,
-                                                                              nfail, t->list[1 - cur], t->d_ctr, true);
+            k_place<B><<<grid_for(nfail, kThreads / (B / 4)), kThreads, 0, st>>>(t->view(), L[cur], nullptr, nfail,
+                                                                              L[1 - cur], t->d_ctr, true);
         }
         CU(cudaGetLastError());
         TRY(read_ctr(t, st));
@@ -425,16 +446,151 @@ dyc_status enforce_lower(dyc_table* t, cudaStream_t st) {
     return DYC_OK;
 }
 
+// ------------------------------------------------ resize under live traffic (NEXT-1)
+// Commits the resize in flight: the caller's stream waits for the split/merge
+// kernel, the new buffer replaces the old one (released after the batches that
+// still read it), and a downsize's residuals are placed into their pairs' other
+// tables and settled like any placement failure (Q17).
+template <int B>
+dyc_status live_commit(dyc_table* t, cudaStream_t st) {
+    auto& r = t->rz;
+    if (!r.active) return DYC_OK;
+    CU(cudaStreamWaitEvent(st, r.done, 0));
+    const uint32_t ti = r.ti;
+    dev_free(t, t->sub[ti], st);
+    t->sub[ti] = r.nbuf;
+    t->nb[ti] = r.nnb;
+    r.active = false;
+    r.nbuf = nullptr;
+    t->n_live_resize++;
+    if (r.dir > 0) {
+        t->n_upsize++;
+        return DYC_OK;
+    }
+    t->n_downsize++;
+    TRY(zero_one(t, C_FAIL, st));
+    TRY(zero_one(t, C_EVICT, st));
+    {
+        ProfScope ps(t, DYC_PROF_PLACE, st);
+        k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), r.res[0], r.ctr + C_RESIDUAL, 0, r.res[1],
+                                                         t->d_ctr, true);
+    }
+    CU(cudaGetLastError());
+    CU(cudaMemcpyAsync(t->d_ctr + C_RES_TOTAL, r.ctr + C_RES_TOTAL, 8, cudaMemcpyDeviceToDevice, st));
+    TRY(read_ctr(t, st));
+    t->n_evict += t->h_ctr[C_EVICT];
+    t->n_residual += t->h_ctr[C_RES_TOTAL];
+    TRY(settle<B>(t, 1, t->h_ctr[C_FAIL], st, r.res));
+    dev_free(t, r.res[0], st);
+    dev_free(t, r.res[1], st);
+    r.res[0] = r.res[1] = nullptr;
+    return DYC_OK;
+}
+
+// Checks a resize request against the policy's shape rules and
+// resolves subtable -1 to the policy's choice.
+dyc_status pick_resize(const dyc_table* t, int direction, int subtable, int& ti) {
+    ti = subtable;
+    if (direction > 0) {
+        if (ti < 0) ti = t->smallest();
+        if (ti >= (int)t->cfg.d || t->nb[ti] != t->nb[t->smallest()])
+            return set_err(DYC_ERR_INVALID_ARG, "only a smallest subtable may be doubled (P:L311-312)");
+        if (2 * t->nb[ti] > 0xFFFFFFFFull) return set_err(DYC_ERR_OOM, "subtable would exceed 2^32 buckets");
+    } else {
+        if (ti < 0) ti = t->largest();
+        if (ti >= (int)t->cfg.d || t->nb[ti] != t->nb[t->largest()])
+            return set_err(DYC_ERR_INVALID_ARG, "only a largest subtable may be halved (P:L311-312)");
+        if (t->nb[ti] < 2 || (t->nb[ti] & 1)) return set_err(DYC_ERR_INVALID_ARG, "subtable cannot be halved");
+    }
+    return DYC_OK;
+}
+
+// Starts the split or merge of one subtable on
+// `rs`, after the work already enqueued on `st`, and returns; see dyc_resize_begin.
+template <int B>
+dyc_status live_begin(dyc_table* t, int direction, int subtable, cudaStream_t st, cudaStream_t rs) {
+    auto& r = t->rz;
+    if (r.active) return set_err(DYC_ERR_INVALID_ARG, "a resize is already in flight (dyc_resize_commit first)");
+    if (t->part_op) return set_err(DYC_ERR_INVALID_ARG, "a batch is open (dyc_*_end first)");
+    int ti = -1;
+    TRY(pick_resize(t, direction, subtable, ti));
+    if (!r.start) CU(cudaEventCreateWithFlags(&r.start, cudaEventDisableTiming));
+    if (!r.done) CU(cudaEventCreateWithFlags(&r.done, cudaEventDisableTiming));
+    if (!r.ctr) CU(cudaMalloc(&r.ctr, C_N * 8));
+    CU(cudaEventRecord(r.start, st));
+    CU(cudaStreamWaitEvent(rs, r.start, 0));
+    const uint64_t n_old = t->nb[ti];
+    const uint64_t nn = direction > 0 ? 2 * n_old : n_old / 2;
+    void* p = nullptr;
+    TRY(dev_alloc(t, &p, nn * B * 8, rs));
+    if (direction > 0) {
+        ProfScope ps(t, DYC_PROF_UPSIZE, rs);
+        k_upsize<B><<<grid_for(n_old * B, kThreads), kThreads, 0, rs>>>(t->sub[ti], (unsigned long long*)p,
+                                                                        (uint32_t)n_old, t->a[ti + 1], t->b[ti + 1],
+                                                                        fastmod_magic(nn), (uint32_t)nn);
+    } else {
+        void* r0 = nullptr;
+        void* r1 = nullptr;
+        dyc_status s = dev_alloc(t, &r0, nn * B * 8, rs);
+        if (s == DYC_OK) s = dev_alloc(t, &r1, nn * B * 8, rs);
+        if (s != DYC_OK) {
+            dev_free(t, p, rs);
+            dev_free(t, r0, rs);
+            return s;
+        }
+        r.res[0] = (unsigned long long*)r0;
+        r.res[1] = (unsigned long long*)r1;
+        CU(cudaMemsetAsync(r.ctr, 0, C_N * 8, rs));
+        ProfScope ps(t, DYC_PROF_DOWNSIZE, rs);
+        k_downsize<B><<<grid_for(nn * B, kThreads), kThreads, 0, rs>>>(t->sub[ti], (unsigned long long*)p,
+                                                                       (uint32_t)nn, r.res[0], r.ctr);
+    }
+    CU(cudaGetLastError());
+    CU(cudaEventRecord(r.done, rs));
+    r.active = true;
+    r.dir = direction;
+    r.ti = (uint32_t)ti;
+    r.nbuf = (unsigned long long*)p;
+    r.nnb = nn;
+    return DYC_OK;
+}
+
+// After a mutating batch: the alpha loop (Q11), taken against the size
+// the table has once the resize in flight is committed; it commits first when
+// it has to act.
+template <int B>
+dyc_status policy_lower(dyc_table* t, cudaStream_t st) {
+    if (t->rz.active) {
+        if (!((double)t->m < t->cfg.alpha * (double)t->N_after())) return DYC_OK;
+        TRY(live_commit<B>(t, st));
+    }
+    return enforce_lower<B>(t, st);
+}
+
+template <int B>
+dyc_status launch_apply(dyc_table* t, const unsigned long long* list, bool del, uint64_t n, cudaStream_t st) {
+    ProfScope ps(t, DYC_PROF_OTHER, st);
+    k_apply<B><<<grid_for(n, kThreads / (B / 4)), kThreads, 0, st>>>(t->view(), list, t->d_ctr + C_DEFER, del);
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
 // insert = begin (scratch, counters, FUSE decision) + one k_upsert per chunk of
 // the batch + end (resize decision, placement, failures, alpha loop).  Splitting
 // the upsert into chunks is invisible to the semantics: every chunk only probes,
 // updates and CASes into free slots (or queues to the pending list), and all
 // placement with evictions happens once, in insert_end.
+//
+// While a resize is in flight (NEXT-1) a batch that could need an upsize
+// ((m+n) > beta*N_after) commits it first; any other runs the LK upsert against
+// the old buffer of the locked subtable and commits only if some of its ops
+// need that subtable (deferred updates, keys with no free non-locked slot).
 template <int B>
 dyc_status insert_begin(dyc_table* t, uint64_t n, cudaStream_t st, bool& fuse) {
+    if (t->rz.active && (double)(t->m + n) > t->cfg.beta * (double)t->N_after()) TRY(live_commit<B>(t, st));
     TRY(ensure_lists(t, n, st));
     TRY(zero_ctr(t, st));
-    fuse = (double)(t->m + n) <= t->cfg.beta * (double)t->N();
+    fuse = t->rz.active || (double)(t->m + n) <= t->cfg.beta * (double)t->N();
     return DYC_OK;
 }
 
@@ -445,7 +601,10 @@ dyc_status insert_chunk(dyc_table* t, const uint32_t* keys, const uint32_t* vals
     const unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
     {
         ProfScope ps(t, DYC_PROF_UPSERT, st);
-        if (fuse)
+        if (t->rz.active)
+            k_upsert<B, true, U, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0],
+                                                                  t->d_ctr, t->rz.ti, t->list[1]);
+        else if (fuse)
             k_upsert<B, true, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
         else
             k_upsert<B, false, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
@@ -456,6 +615,22 @@ dyc_status insert_chunk(dyc_table* t, const uint32_t* keys, const uint32_t* vals
 
 template <int B>
 dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
+    if (t->rz.active) {
+        TRY(read_ctr(t, st));
+        const uint64_t ins = t->h_ctr[C_INSERTED], pend = t->h_ctr[C_PENDING], dfr = t->h_ctr[C_DEFER];
+        t->n_deferred += dfr;
+        const uint64_t ev0 = t->n_evict;
+        if (pend || dfr) {
+            TRY(live_commit<B>(t, st));
+            if (dfr) TRY(launch_apply<B>(t, t->list[1], false, dfr, st));
+            if (pend) TRY(place_and_settle<B>(t, 0, t->d_ctr + C_PENDING, 0, true, st));
+        }
+        t->m += ins;
+        t->last_new = ins;
+        t->last_pending = pend;
+        t->last_evict = t->n_evict - ev0;
+        return policy_lower<B>(t, st);
+    }
     if (!fuse) {
         // the resize decision needs n_new before any placement (Q11)
         TRY(read_ctr(t, st));
@@ -497,14 +672,30 @@ dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t
     return DYC_OK;
 }
 
+// delete = prep (counters; with a resize in flight also the deferred list) +
+// one k_delete per chunk + end (m, deferred removals, alpha loop).
+template <int B>
+dyc_status delete_prep(dyc_table* t, uint64_t n, cudaStream_t st) {
+    TRY(zero_one(t, C_REMOVED, st));
+    if (t->rz.active) {
+        TRY(ensure_lists(t, n, st));
+        TRY(zero_one(t, C_DEFER, st));
+    }
+    return DYC_OK;
+}
+
 template <int B>
 dyc_status delete_chunk(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
                         cudaStream_t st) {
     {
         ProfScope ps(t, DYC_PROF_DELETE, st);
         constexpr int U = DYC_DELETE_U;
-        k_delete<B, U><<<grid_for(n, (uint64_t)(kThreads / (B / 4)) * U), kThreads, 0, st>>>(t->view(), keys, vals,
-                                                                                            status, n, t->d_ctr);
+        const unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
+        if (t->rz.active)
+            k_delete<B, U, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, t->rz.ti,
+                                                            t->list[0]);
+        else
+            k_delete<B, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr);
     }
     CU(cudaGetLastError());
     return DYC_OK;
@@ -514,13 +705,19 @@ template <int B>
 dyc_status delete_end(dyc_table* t, cudaStream_t st) {
     TRY(read_ctr(t, st));
     t->m -= t->h_ctr[C_REMOVED];
-    return enforce_lower<B>(t, st);
+    if (t->rz.active && t->h_ctr[C_DEFER]) {
+        const uint64_t dfr = t->h_ctr[C_DEFER];
+        t->n_deferred += dfr;
+        TRY(live_commit<B>(t, st));
+        TRY(launch_apply<B>(t, t->list[0], true, dfr, st));
+    }
+    return policy_lower<B>(t, st);
 }
 
 template <int B>
 dyc_status delete_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
                        cudaStream_t st) {
-    TRY(zero_one(t, C_REMOVED, st));
+    TRY(delete_prep<B>(t, n, st));
     TRY(delete_chunk<B>(t, keys, vals, status, n, st));
     return delete_end<B>(t, st);
 }
@@ -636,7 +833,7 @@ dyc_status delete_host_impl(dyc_table* t, const uint32_t* hk, uint32_t* hv, uint
     uint32_t* v = k + n;
     uint8_t* s = (uint8_t*)(v + n);
     HostPipe P{t, st, {}};
-    TRY(zero_one(t, C_REMOVED, st));
+    TRY(delete_prep<B>(t, n, st));
     for (uint64_t off = 0; off < n; off += kChunk) {
         const uint64_t len = std::min(kChunk, n - off);
         void* d_in[1] = {k};
@@ -698,6 +895,7 @@ dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaSt
 
 template <int B>
 dyc_status resize_impl(dyc_table* t, int direction, int subtable, int method, cudaStream_t st) {
+    TRY(live_commit<B>(t, st));
     if (direction == 0) {
         while ((double)t->m > t->cfg.beta * (double)t->N()) {
             TRY(upsize_table<B>(t, (uint32_t)t->smallest(), st));
@@ -710,17 +908,8 @@ dyc_status resize_impl(dyc_table* t, int direction, int subtable, int method, cu
         if (direction > 0) t->n_upsize++; else t->n_downsize++;
         return DYC_OK;
     }
-    int ti = subtable;
-    if (direction > 0) {
-        if (ti < 0) ti = t->smallest();
-        if (ti >= (int)t->cfg.d || t->nb[ti] != t->nb[t->smallest()])
-            return set_err(DYC_ERR_INVALID_ARG, "only a smallest subtable may be doubled (P:L311-312)");
-    } else {
-        if (ti < 0) ti = t->largest();
-        if (ti >= (int)t->cfg.d || t->nb[ti] != t->nb[t->largest()])
-            return set_err(DYC_ERR_INVALID_ARG, "only a largest subtable may be halved (P:L311-312)");
-        if (t->nb[ti] < 2 || (t->nb[ti] & 1)) return set_err(DYC_ERR_INVALID_ARG, "subtable cannot be halved");
-    }
+    int ti = -1;
+    TRY(pick_resize(t, direction, subtable, ti));
     if (method == DYC_RESIZE_REINSERT_SUBTABLE) {
         TRY(reinsert_resize<B>(t, direction, ti, false, st));
     } else if (direction > 0) {
@@ -734,6 +923,7 @@ dyc_status resize_impl(dyc_table* t, int direction, int subtable, int method, cu
 
 template <int B>
 dyc_status stats_impl(dyc_table* t, dyc_stats_t* out, cudaStream_t st) {
+    TRY(live_commit<B>(t, st));
     TRY(zero_ctr(t, st));
     const TableView tv = t->view();
     for (uint32_t i = 0; i < t->cfg.d; i++) {
@@ -764,12 +954,15 @@ dyc_status stats_impl(dyc_table* t, dyc_stats_t* out, cudaStream_t st) {
     out->last_insert_new = t->last_new;
     out->last_insert_pending = t->last_pending;
     out->last_insert_evictions = t->last_evict;
+    out->n_live_resize = t->n_live_resize;
+    out->n_deferred = t->n_deferred;
     return DYC_OK;
 }
 
 template <int B>
 dyc_status dump_impl(dyc_table* t, uint64_t* h_kv, uint32_t* h_tab, uint64_t* h_bkt, uint64_t cap, uint64_t* n_out,
                      cudaStream_t st) {
+    TRY(live_commit<B>(t, st));
     const uint64_t m = t->m;
     void *kv = nullptr, *tb = nullptr, *bk = nullptr;
     TRY(dev_alloc(t, &kv, m * 8, st));
@@ -809,6 +1002,8 @@ dyc_status dump_impl(dyc_table* t, uint64_t* h_kv, uint32_t* h_tab, uint64_t* h_
         case 32: { constexpr int B_ = 32; return CALL; }                           \
         default: return set_err(DYC_ERR_INVALID_ARG, "unsupported bucket_slots");  \
     }
+
+dyc_status live_commit_any(dyc_table* t, cudaStream_t st) { DISPATCH_B(t, live_commit<B_>(t, st)); }
 
 dyc_status check_table(const dyc_table* t) {
     if (!t) return set_err(DYC_ERR_INVALID_ARG, "null table");
@@ -926,6 +1121,9 @@ dyc_status dyc_destroy(dyc_table* t) {
     t->live.clear();
     trim_cache(t);
     if (t->d_ctr) cudaFree(t->d_ctr);
+    if (t->rz.ctr) cudaFree(t->rz.ctr);
+    if (t->rz.start) cudaEventDestroy(t->rz.start);
+    if (t->rz.done) cudaEventDestroy(t->rz.done);
     if (t->h_ctr) cudaFreeHost(t->h_ctr);
     if (t->cp_in) cudaStreamDestroy(t->cp_in);
     if (t->cp_out) cudaStreamDestroy(t->cp_out);
@@ -984,7 +1182,7 @@ dyc_status dyc_delete_begin(dyc_table* t, uint64_t n_total, dyc_stream_t stream)
     if (t->part_op) return set_err(DYC_ERR_INVALID_ARG, "a batch is already open");
     t->part_op = 2;
     t->part_left = n_total;
-    return zero_one(t, C_REMOVED, S(stream));
+    DISPATCH_B(t, delete_prep<B_>(t, n_total, S(stream)));
 }
 
 dyc_status dyc_delete_part(dyc_table* t, const uint32_t* d_keys, uint32_t* d_values_out, uint8_t* d_status,
@@ -1082,8 +1280,36 @@ dyc_status dyc_resize(dyc_table* t, int direction, int subtable, dyc_stream_t st
     return dyc_resize_ex(t, direction, subtable, DYC_RESIZE_SPLIT, stream);
 }
 
+dyc_status dyc_resize_begin(dyc_table* t, int direction, int subtable, dyc_stream_t stream,
+                            dyc_stream_t resize_stream) {
+    TRY(enter(t, stream));
+    if (direction != 1 && direction != -1) return set_err(DYC_ERR_INVALID_ARG, "direction must be +1 or -1");
+    DISPATCH_B(t, live_begin<B_>(t, direction, subtable, S(stream), S(resize_stream)));
+}
+
+dyc_status dyc_resize_commit(dyc_table* t, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (t->part_op) return set_err(DYC_ERR_INVALID_ARG, "a batch is open (dyc_*_end first)");
+    DISPATCH_B(t, live_commit<B_>(t, S(stream)));
+}
+
+dyc_status dyc_resize_query(const dyc_table* t, int* in_flight, int* kernel_done) {
+    TRY(check_table(t));
+    if (in_flight) *in_flight = t->rz.active ? 1 : 0;
+    if (kernel_done) {
+        *kernel_done = 1;
+        if (t->rz.active) {
+            const cudaError_t e = cudaEventQuery(t->rz.done);
+            if (e == cudaErrorNotReady) *kernel_done = 0;
+            else if (e != cudaSuccess) return cuda_err(e, "cudaEventQuery");
+        }
+    }
+    return DYC_OK;
+}
+
 dyc_status dyc_clear(dyc_table* t, dyc_stream_t stream) {
     TRY(enter(t, stream));
+    if (t->rz.active) TRY(live_commit_any(t, S(stream)));
     for (uint32_t i = 0; i < t->cfg.d; i++)
         CU(cudaMemsetAsync(t->sub[i], 0xFF, t->nb[i] * t->cfg.bucket_slots * 8, S(stream)));
     t->m = 0;

@@ -53,6 +53,7 @@ enum CounterIdx : int {
     C_DUMP = 7,       // dump cursor
     C_SECOND = 8,     // keys in their second-choice subtable (stats)
     C_RES_TOTAL = 9,  // residuals over several downsizes of one alpha loop
+    C_DEFER = 10,     // ops on a subtable locked by a resize in flight (NEXT-1)
     C_COUNT0 = 16,    // per-subtable live counts [16, 32)
     C_N = 32
 };
@@ -278,12 +279,21 @@ __device__ __forceinline__ unsigned empty_mask(const unsigned long long (&s)[4])
 // exact; FUSE is only used when no upsize can be needed ((m+n) <= beta*N).
 // Each group carries U ops whose probes are issued together (memory-level
 // parallelism: the kernel is bound by random line requests).
-template <int B, bool FUSE, int U>
+//
+// LK (resize under live traffic, NEXT-1): subtable `locked` is
+// being resized by a concurrent kernel, so its (old, read-only) buffer may be
+// probed but not written.  An existing key found there keeps status UPDATED but
+// its new value is appended to `defer` (applied by k_apply after the resize is
+// committed); a new key may only take a free slot of its OTHER candidate bucket,
+// else it is pending (placed after the commit).
+template <int B, bool FUSE, int U, bool LK = false>
 __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView tv, const uint32_t* __restrict__ keys,
                                                      const uint32_t* __restrict__ vals,
                                                      uint8_t* __restrict__ status, uint64_t n,
                                                      unsigned long long* __restrict__ pending,
-                                                     unsigned long long* __restrict__ ctr) {
+                                                     unsigned long long* __restrict__ ctr,
+                                                     uint32_t locked = 0xFFFFFFFFu,
+                                                     unsigned long long* __restrict__ defer = nullptr) {
     constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
@@ -303,6 +313,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
         unsigned h1[U], h2[U], em1[U], em2[U];
         bool need2[U], isnew[U], placed[U];
         int j1[U], j2[U];
+        bool lk1[U], lk2[U];
         {
             unsigned long long s1[U][4];
 #pragma unroll
@@ -312,6 +323,8 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                 k[u] = valid ? __ldg(keys + i[u]) : kEmptyKey;
                 kv[u] = make_kv(k[u], valid ? __ldg(vals + i[u]) : 0u);
                 const Pair p = pair_of(tv, k[u]);
+                lk1[u] = LK && p.t1 == locked;
+                lk2[u] = LK && p.t2 == locked;
                 b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
                 b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
                 probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
@@ -319,7 +332,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
 #pragma unroll
             for (int u = 0; u < U; u++) {
                 j1[u] = match_slot<4>(s1[u], k[u]);
-                em1[u] = empty_mask(s1[u]);
+                em1[u] = lk1[u] ? 0u : empty_mask(s1[u]);
             }
         }
         {
@@ -336,14 +349,15 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
 #pragma unroll
             for (int u = 0; u < U; u++) {
                 j2[u] = match_slot<4>(s2[u], k[u]);
-                em2[u] = empty_mask(s2[u]);
+                em2[u] = lk2[u] ? 0u : empty_mask(s2[u]);
             }
         }
 #pragma unroll
         for (int u = 0; u < U; u++) {
             h2[u] = g.ballot(need2[u] && j2[u] >= 0);
-            if (h1[u] && g.sub == first_lane(h1[u])) st_u64_cg(b1[u] + 4 * g.sub + j1[u], kv[u]);
-            if (h2[u] && g.sub == first_lane(h2[u])) st_u64_cg(b2[u] + 4 * g.sub + j2[u], kv[u]);
+            if (h1[u] && !lk1[u] && g.sub == first_lane(h1[u])) st_u64_cg(b1[u] + 4 * g.sub + j1[u], kv[u]);
+            if (h2[u] && !lk2[u] && g.sub == first_lane(h2[u])) st_u64_cg(b2[u] + 4 * g.sub + j2[u], kv[u]);
+            if (LK) warp_append(g.sub == 0 && ((h1[u] && lk1[u]) || (h2[u] && lk2[u])), kv[u], defer, ctr + C_DEFER);
             isnew[u] = need2[u] && h2[u] == 0;
             placed[u] = false;
         }
@@ -478,11 +492,16 @@ __global__ void __launch_bounds__(kThreads) k_reinsert(TableView tv, const unsig
 // ------------------------------------------------------------- delete (S4)
 // Probe t1 then t2; the lane holding the key overwrites its slot with EMPTY (no
 // lock: keys in a batch are distinct).  U ops per group in flight.
-template <int B, int U>
+// LK: a key found in the `locked` subtable (being resized concurrently) is
+// reported DELETED with its old value, and its removal is appended to `defer`
+// (applied by k_apply after the resize is committed).
+template <int B, int U, bool LK = false>
 __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView tv, const uint32_t* __restrict__ keys,
                                                      uint32_t* __restrict__ old_vals,
                                                      uint8_t* __restrict__ status, uint64_t n,
-                                                     unsigned long long* __restrict__ ctr) {
+                                                     unsigned long long* __restrict__ ctr,
+                                                     uint32_t locked = 0xFFFFFFFFu,
+                                                     unsigned long long* __restrict__ defer = nullptr) {
     constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
@@ -498,13 +517,15 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
         unsigned long long* b1[U];
         unsigned long long* b2[U];
         unsigned h1[U];
-        bool need2[U];
+        bool need2[U], lk1[U], lk2[U];
         int j1[U];
 #pragma unroll
         for (int u = 0; u < U; u++) {
             i[u] = base + (uint64_t)u * QPW + grp;
             k[u] = i[u] < n ? __ldg(keys + i[u]) : kEmptyKey;
             const Pair p = pair_of(tv, k[u]);
+            lk1[u] = LK && p.t1 == locked;
+            lk2[u] = LK && p.t2 == locked;
             b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
             b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
             probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
@@ -526,8 +547,9 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
             lookup_slot<4>(s2[u], k[u], lv2);
             const int j2 = need2[u] ? match_slot<4>(s2[u], k[u]) : -1;
             const unsigned h2 = g.ballot(j2 >= 0);
-            if (h1[u] && g.sub == first_lane(h1[u])) st_u64_cg(b1[u] + 4 * g.sub + j1[u], kEmptySlot);
-            if (h2 && g.sub == first_lane(h2)) st_u64_cg(b2[u] + 4 * g.sub + j2, kEmptySlot);
+            if (h1[u] && !lk1[u] && g.sub == first_lane(h1[u])) st_u64_cg(b1[u] + 4 * g.sub + j1[u], kEmptySlot);
+            if (h2 && !lk2[u] && g.sub == first_lane(h2)) st_u64_cg(b2[u] + 4 * g.sub + j2, kEmptySlot);
+            if (LK) warp_append(g.sub == 0 && ((h1[u] && lk1[u]) || (h2 && lk2[u])), make_kv(k[u], 0u), defer, ctr + C_DEFER);
             const uint32_t o1 = g.bcast32(lv1, first_lane(h1[u]));
             const uint32_t o2 = g.bcast32(lv2, first_lane(h2));
             const bool hit = (h1[u] | h2) != 0;
@@ -539,6 +561,39 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
         }
     }
     block_add<kThreads>(ctr + C_REMOVED, removed);
+}
+
+// Applies the deferred ops of a batch that ran while a subtable was locked by a
+// resize (NEXT-1), once the resize is committed: each listed key is present in
+// one of its two candidate buckets; `del` removes it, otherwise its value is
+// replaced by the listed one.  One lane group per entry.
+template <int B>
+__global__ void __launch_bounds__(kThreads) k_apply(TableView tv, const unsigned long long* __restrict__ list,
+                                                    const unsigned long long* __restrict__ count_ptr, bool del) {
+    constexpr int G = B / 4, QPW = 32 / G;
+    __shared__ SmemView sv;
+    load_view(tv, sv);
+    const Grp<G> g;
+    const unsigned grp = g.lane / G;
+    const uint64_t cnt = *count_ptr;
+    const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
+    const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
+    for (uint64_t base = w * QPW; base < cnt; base += nwarps * QPW) {
+        const uint64_t i = base + grp;
+        const unsigned long long kv = i < cnt ? list[i] : kEmptySlot;
+        const uint32_t k = key_of(kv);
+        const Pair p = pair_of(tv, k);
+        const unsigned long long new_e = del ? kEmptySlot : kv;
+#pragma unroll
+        for (int h = 0; h < 2; h++) {
+            unsigned long long* bp = bucket_ptr(sv, h ? p.t2 : p.t1, bucket_of(sv, h ? p.t2 : p.t1, k), B);
+            unsigned long long s[4];
+            probe_cg<B>(bp + 4 * g.sub, s);
+            const int j = k != kEmptyKey ? match_slot<4>(s, k) : -1;
+            const unsigned hb = g.ballot(j >= 0);
+            if (hb && g.sub == first_lane(hb)) st_u64_cg(bp + 4 * g.sub + j, new_e);
+        }
+    }
 }
 
 // ------------------------------------------------------------- upsize (S8)

@@ -201,6 +201,24 @@ class Table:
         L.check(self._lib.dyc_resize_ex(self._h, direction, subtable, method, _stream_ptr(stream)),
                 "dyc_resize_ex")
 
+    def resize_begin(self, direction: int, subtable: int = -1, stream=None, resize_stream=None):
+        """Start a one-subtable resize on `resize_stream` and return at once
+        (dyc_resize_begin; NEXT-1).  Batches issued on `stream`
+        before dyc_resize_commit run concurrently with it."""
+        if resize_stream is None:
+            raise ValueError("resize_begin needs a resize_stream (a torch.cuda.Stream)")
+        L.check(self._lib.dyc_resize_begin(self._h, direction, subtable, _stream_ptr(stream),
+                                           _stream_ptr(resize_stream)), "dyc_resize_begin")
+
+    def resize_commit(self, stream=None):
+        L.check(self._lib.dyc_resize_commit(self._h, _stream_ptr(stream)), "dyc_resize_commit")
+
+    def resize_query(self):
+        """(in_flight, kernel_done) of the resize started by resize_begin."""
+        a, b = C.c_int(), C.c_int()
+        L.check(self._lib.dyc_resize_query(self._h, C.byref(a), C.byref(b)), "dyc_resize_query")
+        return bool(a.value), bool(b.value)
+
     def trim(self):
         """Return cached (released) device buffers to the device."""
         L.check(self._lib.dyc_trim(self._h), "dyc_trim")
@@ -218,7 +236,8 @@ class Table:
                     n_place_retry=s.n_place_retry, n_second_table=s.n_second_table,
                     bytes_allocated=s.bytes_allocated, last_insert_new=s.last_insert_new,
                     last_insert_pending=s.last_insert_pending,
-                    last_insert_evictions=s.last_insert_evictions, bytes_cached=s.bytes_cached)
+                    last_insert_evictions=s.last_insert_evictions, bytes_cached=s.bytes_cached,
+                    n_live_resize=s.n_live_resize, n_deferred=s.n_deferred)
 
     def dump(self, stream=None):
         """(kv uint64, table uint32, bucket uint64) host arrays, unspecified order."""
