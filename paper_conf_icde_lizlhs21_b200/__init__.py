@@ -6,5 +6,6 @@ C ABI of include/dycuckoo.h (libdyc.so).  Importing this package does not load
 the library; ``Table`` does, and fails loudly if it is missing.
 """
 from .table import Table  # noqa: F401
+from .wide import WideTable  # noqa: F401
 
-__all__ = ["Table"]
+__all__ = ["Table", "WideTable"]

@@ -41,6 +41,24 @@ class dyc_stats_t(C.Structure):
                 ("bytes_cached", C.c_uint64), ("n_live_resize", C.c_uint64), ("n_deferred", C.c_uint64)]
 
 
+class dyw_config(C.Structure):
+    _fields_ = [("d", C.c_uint32), ("value_words", C.c_uint32), ("mode", C.c_uint32), ("max_hops", C.c_uint32),
+                ("alpha", C.c_double), ("beta", C.c_double), ("init_capacity", C.c_uint64), ("seed", C.c_uint64)]
+
+
+class dyw_stats_t(C.Structure):
+    _fields_ = [("m", C.c_uint64), ("N", C.c_uint64), ("d", C.c_uint32), ("B", C.c_uint32),
+                ("W", C.c_uint32), ("mode", C.c_uint32),
+                ("buckets", C.c_uint64 * DYC_MAX_D), ("count", C.c_uint64 * DYC_MAX_D),
+                ("fill", C.c_double), ("n_upsize", C.c_uint64), ("n_downsize", C.c_uint64),
+                ("n_fail_upsize", C.c_uint64), ("n_residual", C.c_uint64), ("n_evict", C.c_uint64),
+                ("n_lock_fail", C.c_uint64), ("last_insert_new", C.c_uint64),
+                ("last_insert_pending", C.c_uint64), ("bytes_allocated", C.c_uint64)]
+
+
+DYW_MODE_VOTER, DYW_MODE_GROUPED, DYW_MODE_LOCKFREE = 0, 1, 2
+
+
 class DycError(RuntimeError):
     def __init__(self, code: int, fn: str, msg: str):
         name = _STATUS_NAMES[code] if 0 <= code < len(_STATUS_NAMES) else str(code)
@@ -70,6 +88,19 @@ SIGNATURES = {
     "dyc_resize": (_I, [_TP, _I, _I, _P]),
     "dyc_resize_ex": (_I, [_TP, _I, _I, _I, _P]),
     "dyc_resize_begin": (_I, [_TP, _I, _I, _P, _P]),
+    # wide-key table (include/dycuckoo_wide.h, NEXT-3)
+    "dyw_config_default": (_I, [C.POINTER(dyw_config)]),
+    "dyw_create": (_I, [C.POINTER(dyw_config), C.POINTER(_TP)]),
+    "dyw_destroy": (_I, [_TP]),
+    "dyw_insert_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
+    "dyw_find_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
+    "dyw_delete_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
+    "dyw_resize": (_I, [_TP, _I, _I, _P]),
+    "dyw_clear": (_I, [_TP, _P]),
+    "dyw_stats": (_I, [_TP, C.POINTER(dyw_stats_t), _P]),
+    "dyw_dump": (_I, [_TP, _P, _P, _P, _P, _U64, C.POINTER(_U64), _P]),
+    "dyw_hash_probe": (_I, [_TP, _P, _U64, _P, _P, _P]),
+    "dyw_launch_count": (_U64, [_TP, _I]),
     "dyc_resize_commit": (_I, [_TP, _P]),
     "dyc_resize_query": (_I, [_TP, C.POINTER(_I), C.POINTER(_I)]),
     "dyc_clear": (_I, [_TP, _P]),

@@ -14,7 +14,7 @@ CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libdyc.so")
 SOURCES = ["dyc_api.cu"]
-DEPS = ["dyc_api.cu", "dyc_kernels.cuh", "dyc_device.cuh"]
+DEPS = ["dyc_api.cu", "dyc_kernels.cuh", "dyc_device.cuh", "dyw_api.cuh", "dyw_kernels.cuh"]
 
 NVCC_FLAGS = [
     "-O3", "-std=c++17", "-lineinfo",
@@ -34,7 +34,7 @@ def needs_build() -> bool:
     if not os.path.exists(LIB):
         return True
     t = os.path.getmtime(LIB)
-    files = [os.path.join(CSRC, f) for f in DEPS] + [os.path.join(INCLUDE, "dycuckoo.h")]
+    files = [os.path.join(CSRC, f) for f in DEPS] + [os.path.join(INCLUDE, h) for h in ("dycuckoo.h", "dycuckoo_wide.h")]
     return any(os.path.getmtime(f) > t for f in files)
 
 

@@ -1505,3 +1505,6 @@ dyc_status dyc_bench_gather(const void* d_buf, uint64_t buf_bytes, uint64_t n_re
 }
 
 }  // extern "C"
+
+// ---------------------------------------------------------------- wide-key table (NEXT-3)
+#include "dyw_api.cuh"

@@ -18,7 +18,7 @@ def declared_functions():
     for h in glob.glob(os.path.join(INCLUDE, "*.h")):
         text = open(h).read()
         text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
-        for m in re.finditer(r"^\s*[A-Za-z_][\w\s\*]*?\b(dyc_\w+)\s*\(", text, flags=re.M):
+        for m in re.finditer(r"^\s*[A-Za-z_][\w\s\*]*?\b(dy[cw]_\w+)\s*\(", text, flags=re.M):
             names.add(m.group(1))
     return names
 
