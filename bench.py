@@ -63,7 +63,7 @@ def parse():
     ap.add_argument("--no-rehash", action="store_true")
     ap.add_argument("--profile-only", action="store_true", help="a few steps, no extras (for ncu)")
     ap.add_argument("--l2-fetch", type=int, default=None, help="set cudaLimitMaxL2FetchGranularity (bytes)")
-    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4", "c5"],
+    ap.add_argument("--config", default="c2", choices=["c1", "c2", "c3", "c4", "c5", "wide"],
                     help="c2 = the headline (BASELINE configs[1]); c1/c3/c4 = the other single-GPU configs")
     ap.add_argument("--scale", type=float, default=1.0, help="c3: stream scale; c4: universe scale")
     ap.add_argument("--c5-log2keys", type=int, default=31, help="c5: log2 of the total key count")
@@ -73,6 +73,7 @@ def parse():
     ap.add_argument("--r", type=float, default=0.2, help="c3: deletes per insert (P:L732-733)")
     ap.add_argument("--batch", type=int, default=None, help="c3: batch size (Table tbl:parameters: 2e5..1e6)")
     ap.add_argument("--shape", default=None, help="c3: TW|RE, c4: LINE|COM")
+    ap.add_argument("--wide-modes", default=None, help="--config wide: comma list of voter_W2,grouped_W2,...")
     ap.add_argument("--routed", action="store_true",
                     help="use the sharded router even at N=1 (exercises the N>1 code path)")
     return ap.parse_args()
@@ -320,6 +321,8 @@ def main():
         return
     if world > 1 or args.routed:
         return multi_gpu(args, rank, world, local, dist)
+    if args.config == "wide":
+        return emit(bench_wide(args, local))
     if args.config != "c2":
         return emit(bench_stream(args, local))
     beta = args.beta or 0.85
@@ -449,7 +452,8 @@ def main():
             del t2
         # resize under live traffic (NEXT-1): the split/merge runs on a
         # second stream while a 2^k find batch runs on this one (dyc_resize_begin/commit)
-        rs = torch.cuda.Stream()
+        rs = torch.cuda.Stream(priority=100)       # resize work: lowest priority
+        hs = torch.cuda.Stream(priority=-100)      # the batch stream of the latency probe: highest
         for direction, fill in ((+1, 0.85), (-1, 0.30)):
             tag = "upsize" if direction > 0 else "downsize"
             t2 = Table(d=4, init_capacity=cap, alpha=0.05, beta=0.85, bucket_slots=args.bucket_slots)
@@ -482,17 +486,19 @@ def main():
             ns = min(n, 1 << 20)
 
             def small_find_latency(live_mode):
+                # batches on a high-priority stream, the live resize on a low-priority
+                # one: the find's blocks are scheduled ahead of the resize's
                 a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 torch.cuda.synchronize()
-                a.record(stream)
+                a.record(hs)
                 if live_mode:
-                    t2.resize_begin(direction, resize_stream=rs)
+                    t2.resize_begin(direction, stream=hs, resize_stream=rs)
                 else:
-                    t2.resize(direction)
-                t2.find(k_find[:ns], v_out[:ns], f_out[:ns])
-                b.record(stream)
+                    t2.resize(direction, stream=hs)
+                t2.find(k_find[:ns], v_out[:ns], f_out[:ns], stream=hs)
+                b.record(hs)
                 if live_mode:
-                    t2.resize_commit()
+                    t2.resize_commit(stream=hs)
                 torch.cuda.synchronize()
                 t2.resize(-direction)
                 return a.elapsed_time(b)
@@ -574,6 +580,86 @@ def main():
                   "pending_after_upsert": pend, "evictions": s_ins["last_insert_evictions"]},
     }
     emit(line)
+
+
+def bench_wide(args, local):
+    """NEXT-3: the wide-key table (u64 keys, W-word values) on C2's shape at
+    2^log2n keys, in each placement mode: VOTER (Alg. 1 bucket locks),
+    GROUPED (per-lane try-locks) and LOCKFREE (128-bit atomics, W = 1).  A step is
+    clear + insert (fill 0.85) + find (50% hit) + delete (half the keys)."""
+    import torch
+    from paper_conf_icde_lizlhs21_b200 import workload as W
+    from paper_conf_icde_lizlhs21_b200.wide import WideTable
+    log2n = min(args.log2n, 26)
+    n = 1 << log2n
+    stream = torch.cuda.current_stream()
+    results = {}
+    combos = (("voter", 2), ("grouped", 2), ("voter", 1), ("grouped", 1), ("lockfree", 1))
+    if args.wide_modes:
+        combos = [c for c in combos if f"{c[0]}_W{c[1]}" in args.wide_modes.split(",")]
+    for mode, Wd in combos:
+        cap, k, v, q, dk = W.wide_static_torch(log2n, Wd)
+        g = WideTable(d=4, init_capacity=cap, alpha=0.1, beta=0.85, value_words=Wd, mode=mode)
+        st = torch.empty(n, dtype=torch.uint8, device="cuda")
+        vo = torch.empty((n, Wd), dtype=torch.int64, device="cuda")
+        fo = torch.empty(n, dtype=torch.uint8, device="cuda")
+        do = torch.empty((n // 2, Wd), dtype=torch.int64, device="cuda")
+        ds = torch.empty(n // 2, dtype=torch.uint8, device="cuda")
+
+        def step(rec=None):
+            ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)] if rec is not None else None
+            g.clear()
+            if ev: ev[0].record(stream)
+            g.insert(k, v, st)
+            if ev: ev[1].record(stream)
+            g.find(q, vo, fo)
+            if ev: ev[2].record(stream)
+            g.delete(dk, do, ds)
+            if ev:
+                ev[3].record(stream)
+                rec.append(ev)
+
+        step()
+        torch.cuda.synchronize()
+        s_ins = None
+        assert int(fo.sum().item()) == n // 2 and bool(ds.bool().all().item()), mode
+        for _ in range(max(1, args.warmup - 1)):
+            step()
+        g.launch_count(reset=True)
+        rec = []
+        for _ in range(args.steps):
+            step(rec)
+        torch.cuda.synchronize()
+        ins = statistics.median(r[0].elapsed_time(r[1]) for r in rec)
+        fnd = statistics.median(r[1].elapsed_time(r[2]) for r in rec)
+        dele = statistics.median(r[2].elapsed_time(r[3]) for r in rec)
+        g.clear()
+        s0 = g.stats()
+        g.insert(k, v, st)
+        s_ins = g.stats()
+        s_ins["n_evict"] -= s0["n_evict"]
+        s_ins["n_lock_fail"] -= s0["n_lock_fail"]
+        results[f"{mode}_W{Wd}"] = {
+            "insert_mops": n / ins / 1e3, "find_mops": n / fnd / 1e3, "delete_mops": (n // 2) / dele / 1e3,
+            "insert_ms": ins, "find_ms": fnd, "delete_ms": dele,
+            "step_mops": (2 * n + n // 2) / (ins + fnd + dele) / 1e3,
+            "fill": s_ins["fill"], "evictions_per_insert_batch": s_ins["n_evict"],
+            "lock_failures_per_insert_batch": s_ins["n_lock_fail"],
+            "pending_after_upsert": s_ins["last_insert_pending"], "launches_per_step": g.launch_count() / args.steps,
+            "bucket_slots": s_ins["B"], "table_bytes": s_ins["bytes_allocated"],
+        }
+        g.close()
+        del g, k, v, q, dk
+        torch.cuda.empty_cache()
+    best = max(r["step_mops"] for r in results.values())
+    return {
+        "metric": METRIC + " (wide-key variant, NEXT-3)", "value": best, "unit": "Mops/s", "n_gpus": 1,
+        "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "config": {"workload": f"wide-key C2 shape: 2^{log2n} u64 keys inserted to fill 0.85, 2^{log2n} finds "
+                               f"(50% hit), 2^{log2n - 1} deletes; d=4", "modes": list(results)},
+        "modes": results,
+    }
 
 
 def bench_stream(args, local):

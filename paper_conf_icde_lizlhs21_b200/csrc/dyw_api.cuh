@@ -5,6 +5,13 @@
 #include "dycuckoo_wide.h"
 #include "dyw_kernels.cuh"
 
+#ifndef DYW_U
+#define DYW_U 4   // ops per lane group in flight in find / upsert / delete
+#endif
+#ifndef DYW_U_CAS
+#define DYW_U_CAS 2   // ... in the LOCKFREE upsert, whose CAS128 rounds lose to more in flight (measured U = 1/2/4)
+#endif
+
 struct dyw_table {
     dyw_config cfg{};
     int L = dyw::SEP;     // layout
@@ -215,13 +222,20 @@ dyc_status w_insert(dyw_table* t, const u64* keys, const u64* vals, uint8_t* sta
     TRY(w_ensure_lists(t, n, st));
     TRY(w_zero(t, 0, dyw::W_N, st));
     const bool fuse = L == dyw::PACK && (double)(t->m + n) <= t->cfg.beta * (double)t->N();
-    constexpr int QPW = 32 / dyw::Lay<L>::B;
-    const unsigned grid = grid_for(n, (uint64_t)(dyw::kThreads / 32) * QPW);
+    constexpr int QPW = 32 / dyw::Lay<L>::B, U = L == dyw::PACK ? DYW_U_CAS : DYW_U;
+    const unsigned grid = grid_for(n, (uint64_t)(dyw::kThreads / 32) * QPW * U);
     t->launches++;
-    if (fuse)
-        dyw::k_wupsert<L, W, true><<<grid, dyw::kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
-    else
-        dyw::k_wupsert<L, W, false><<<grid, dyw::kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
+    if constexpr (L == dyw::PACK) {
+        if (fuse)
+            dyw::k_wupsert<L, W, true, U><<<grid, dyw::kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0],
+                                                                          t->d_ctr);
+        else
+            dyw::k_wupsert<L, W, false, U><<<grid, dyw::kThreads, 0, st>>>(t->view(), keys, vals, status, n,
+                                                                           t->list[0], t->d_ctr);
+    } else {                                      // lock modes: every new key goes through placement
+        dyw::k_wupsert<L, W, false, U><<<grid, dyw::kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0],
+                                                                       t->d_ctr);
+    }
     CU(cudaGetLastError());
     TRY(w_read_ctr(t, st));
     const uint64_t n_new = t->h_ctr[dyw::W_INSERTED], pend = t->h_ctr[dyw::W_PENDING];
@@ -246,20 +260,20 @@ dyc_status w_insert(dyw_table* t, const u64* keys, const u64* vals, uint8_t* sta
 
 template <int L, int W>
 dyc_status w_find(dyw_table* t, const u64* keys, u64* out, uint8_t* found, uint64_t n, cudaStream_t st) {
-    constexpr int QPW = 32 / dyw::Lay<L>::B;
+    constexpr int QPW = 32 / dyw::Lay<L>::B, U = DYW_U;
     t->launches++;
-    dyw::k_wfind<L, W><<<grid_for(n, (uint64_t)(dyw::kThreads / 32) * QPW), dyw::kThreads, 0, st>>>(t->view(), keys,
-                                                                                                  out, found, n);
+    dyw::k_wfind<L, W, U><<<grid_for(n, (uint64_t)(dyw::kThreads / 32) * QPW * U), dyw::kThreads, 0, st>>>(
+        t->view(), keys, out, found, n);
     CU(cudaGetLastError());
     return DYC_OK;
 }
 
 template <int L, int W>
 dyc_status w_delete(dyw_table* t, const u64* keys, u64* out, uint8_t* status, uint64_t n, cudaStream_t st) {
-    constexpr int QPW = 32 / dyw::Lay<L>::B;
+    constexpr int QPW = 32 / dyw::Lay<L>::B, U = DYW_U;
     TRY(w_zero(t, dyw::W_REMOVED, 1, st));
     t->launches++;
-    dyw::k_wdelete<L, W><<<grid_for(n, (uint64_t)(dyw::kThreads / 32) * QPW), dyw::kThreads, 0, st>>>(
+    dyw::k_wdelete<L, W, U><<<grid_for(n, (uint64_t)(dyw::kThreads / 32) * QPW * U), dyw::kThreads, 0, st>>>(
         t->view(), keys, out, status, n, t->d_ctr);
     CU(cudaGetLastError());
     TRY(w_read_ctr(t, st));

@@ -207,6 +207,45 @@ __device__ __forceinline__ void kv_append(bool pred, u64 k, const u64 (&v)[W], K
     }
 }
 
+// Block-aggregated append of up to R records per thread: ONE global atomic per
+// block per call (a single list cursor hit by every warp serializes at the L2
+// atomic unit; measured ~1 G atomics/s).  Every thread of the block must call it.
+template <int W, int R>
+__device__ __forceinline__ void block_append(const bool (&pred)[R], const u64 (&k)[R], const u64 (&v)[R][W],
+                                             KVList l, u64* counter) {
+    __shared__ unsigned s_cnt;
+    __shared__ u64 s_base;
+    const unsigned lane = threadIdx.x & 31;
+    unsigned c = 0;
+#pragma unroll
+    for (int r = 0; r < R; r++) c += pred[r] ? 1u : 0u;
+    unsigned inc = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned y = __shfl_up_sync(kFull, inc, o);
+        if (lane >= (unsigned)o) inc += y;
+    }
+    const unsigned wtot = __shfl_sync(kFull, inc, 31);
+    if (threadIdx.x == 0) s_cnt = 0;
+    __syncthreads();
+    unsigned woff = 0;
+    if (lane == 31 && wtot) woff = atomicAdd(&s_cnt, wtot);
+    woff = __shfl_sync(kFull, woff, 31);
+    __syncthreads();
+    if (threadIdx.x == 0) s_base = s_cnt ? atomicAdd(counter, (u64)s_cnt) : 0ull;
+    __syncthreads();
+    u64 at = s_base + woff + (inc - c);
+#pragma unroll
+    for (int r = 0; r < R; r++) {
+        if (pred[r]) {
+            l.keys[at] = k[r];
+#pragma unroll
+            for (int q = 0; q < W; q++) l.vals[at * W + q] = v[r][q];
+            at++;
+        }
+    }
+}
+
 template <int NT>
 __device__ __forceinline__ void wblock_add(u64* dst, u64 v) {
 #pragma unroll
@@ -257,8 +296,75 @@ __device__ __forceinline__ void probe_slot(const WSmem& sv, uint32_t t, uint32_t
     }
 }
 
+// Both probes of U ops of a lane group, all loads of a round issued together
+// (memory-level parallelism: the kernels are bound by random line requests).
+// Per op: the hit (group-relative lane mask, table, bucket; PACK: the value
+// word the hit lane read) and, for the upsert, the EMPTY masks of both buckets.
+template <int L, int U>
+struct Probe2 {
+    u64 k[U];
+    bool act[U];
+    WPair p[U];
+    uint32_t b1[U], b2[U];
+    unsigned hb[U], em1[U], em2[U];
+    uint32_t ht[U], hbk[U];
+    u64 hv[U];
+
+    template <int G>
+    __device__ __forceinline__ void run(const WView& tv, const WSmem& sv, const WGrp<G>& g, const u64* keys,
+                                        uint64_t n, uint64_t base, unsigned grp, bool nc) {
+        constexpr int QPW = 32 / G;
+        static_assert(U <= G, "one hashing lane per op");
+        // the three hashes of op u are computed once, by lane u of the group, and
+        // broadcast (computing them on all G lanes made the kernels ALU-bound)
+        u64 mk = kE;
+        uint32_t mt = 0, m1 = 0, m2 = 0;
+        if (g.sub < (unsigned)U) {
+            const uint64_t i = base + (uint64_t)g.sub * QPW + grp;
+            mk = i < n ? __ldg(keys + i) : kE;
+            const WPair mp = wpair(tv, mk);
+            mt = mp.t1 | (mp.t2 << 16);
+            m1 = wbucket(sv, mp.t1, mk);
+            m2 = wbucket(sv, mp.t2, mk);
+        }
+        u64 sk[U], sval[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            k[u] = g.bcast(mk, u);
+            const uint32_t tt = __shfl_sync(kFull, mt, g.base + u);
+            p[u] = WPair{tt & 0xFFFFu, tt >> 16};
+            b1[u] = __shfl_sync(kFull, m1, g.base + u);
+            b2[u] = __shfl_sync(kFull, m2, g.base + u);
+            act[u] = k[u] != kE;
+            probe_slot<L>(sv, p[u].t1, b1[u], g.sub, nc, act[u], sk[u], sval[u]);
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            hb[u] = g.ballot(act[u] && sk[u] == k[u]);
+            em1[u] = g.ballot(act[u] && sk[u] == kE);
+            ht[u] = p[u].t1;
+            hbk[u] = b1[u];
+            hv[u] = sval[u];
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) probe_slot<L>(sv, p[u].t2, b2[u], g.sub, nc, act[u] && !hb[u], sk[u], sval[u]);
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const bool need = act[u] && !hb[u];
+            const unsigned h2 = g.ballot(need && sk[u] == k[u]);
+            em2[u] = g.ballot(need && sk[u] == kE);
+            if (need && h2) {
+                hb[u] = h2;
+                ht[u] = p[u].t2;
+                hbk[u] = b2[u];
+                hv[u] = sval[u];
+            }
+        }
+    }
+};
+
 // ------------------------------------------------------------------ find (S3)
-template <int L, int W>
+template <int L, int W, int U>
 __global__ void __launch_bounds__(kThreads) k_wfind(WView tv, const u64* __restrict__ keys, u64* __restrict__ out,
                                                     uint8_t* __restrict__ found, uint64_t n) {
     constexpr int G = Lay<L>::B, QPW = 32 / G;
@@ -268,37 +374,33 @@ __global__ void __launch_bounds__(kThreads) k_wfind(WView tv, const u64* __restr
     const unsigned grp = g.lane / G;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
-    for (uint64_t base = w * QPW; base < n; base += nwarps * QPW) {
-        const uint64_t i = base + grp;
-        const u64 k = i < n ? __ldg(keys + i) : kE;
-        const bool act = k != kE;
-        const WPair p = wpair(tv, k);
-        bool hit = false;
-        u64 v[W];
+    for (uint64_t base = w * QPW * U; base < n; base += nwarps * QPW * U) {
+        Probe2<L, U> pr;
+        pr.run(tv, sv, g, keys, n, base, grp, true);
+        u64 v[U][W];
 #pragma unroll
-        for (int q = 0; q < W; q++) v[q] = kE;
+        for (int u = 0; u < U; u++) {
+            const bool mine = pr.hb[u] && g.sub == lowest(pr.hb[u]);
 #pragma unroll
-        for (int h = 0; h < 2; h++) {
-            const uint32_t t = h ? p.t2 : p.t1;
-            const uint32_t b = wbucket(sv, t, k);
-            u64 sk, sval;
-            probe_slot<L>(sv, t, b, g.sub, true, act && !hit, sk, sval);
-            const unsigned hb = g.ballot(act && !hit && sk == k);
-            if (hb && g.sub == lowest(hb)) {
-                if (L == SEP) ld_vals<W>(sv.sub[t].vals + ((uint64_t)b * G + g.sub) * W, v, true);
-                else v[0] = sval;
+            for (int q = 0; q < W; q++) v[u][q] = kE;
+            if (L == SEP) {
+                if (mine) ld_vals<W>(sv.sub[pr.ht[u]].vals + ((uint64_t)pr.hbk[u] * G + g.sub) * W, v[u], true);
+            } else {
+                v[u][0] = pr.hv[u];
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const uint64_t i = base + (uint64_t)u * QPW + grp;
+            if (i >= n) continue;
+            const bool hit = pr.hb[u] != 0;
+            const bool writer = hit ? g.sub == lowest(pr.hb[u]) : g.sub == 0;
+            if (writer) {
                 if (out) {
 #pragma unroll
-                    for (int q = 0; q < W; q++) out[i * W + q] = v[q];
+                    for (int q = 0; q < W; q++) out[i * W + q] = hit ? v[u][q] : kE;
                 }
-            }
-            hit |= hb != 0;
-        }
-        if (g.sub == 0 && i < n) {
-            if (found) found[i] = hit ? 1 : 0;
-            if (!hit && out) {
-#pragma unroll
-                for (int q = 0; q < W; q++) out[i * W + q] = kE;
+                if (found) found[i] = hit ? 1 : 0;
             }
         }
     }
@@ -310,7 +412,7 @@ __global__ void __launch_bounds__(kThreads) k_wfind(WView tv, const u64* __restr
 // move during this kernel and keys in a batch are distinct).  A new key
 // (status INSERTED) is, with FUSE (PACK only), CAS-ed into a free slot of its
 // first-fit bucket; otherwise it is appended to `pending` for placement.
-template <int L, int W, bool FUSE>
+template <int L, int W, bool FUSE, int U>
 __global__ void __launch_bounds__(kThreads) k_wupsert(WView tv, const u64* __restrict__ keys,
                                                       const u64* __restrict__ vals, uint8_t* __restrict__ status,
                                                       uint64_t n, KVList pending, u64* __restrict__ ctr) {
@@ -322,59 +424,78 @@ __global__ void __launch_bounds__(kThreads) k_wupsert(WView tv, const u64* __res
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     u64 n_ins = 0, n_upd = 0;
-    for (uint64_t base = w * QPW; base < n; base += nwarps * QPW) {
-        const uint64_t i = base + grp;
-        const u64 k = i < n ? __ldg(keys + i) : kE;
-        const bool act = k != kE;
-        u64 v[W];
+    constexpr uint64_t per_block = (uint64_t)(kThreads / 32) * QPW * U;
+    (void)w;
+    (void)nwarps;
+    for (uint64_t bbase = (uint64_t)blockIdx.x * per_block; bbase < n; bbase += (uint64_t)gridDim.x * per_block) {
+        const uint64_t base = bbase + (uint64_t)(threadIdx.x >> 5) * QPW * U;   // block-uniform trip count
+        Probe2<L, U> pr;
+        pr.run(tv, sv, g, keys, n, base, grp, false);
+        u64 v[U][W];
+        bool isnew[U], placed[U];
 #pragma unroll
-        for (int q = 0; q < W; q++) v[q] = act ? __ldg(vals + i * W + q) : 0ull;
-        const WPair p = wpair(tv, k);
-        bool hit = false, placed = false;
-        unsigned em[2] = {0u, 0u};
-        uint32_t bk[2];
+        for (int u = 0; u < U; u++) {
+            const uint64_t i = base + (uint64_t)u * QPW + grp;
 #pragma unroll
-        for (int h = 0; h < 2; h++) {
-            const uint32_t t = h ? p.t2 : p.t1;
-            bk[h] = wbucket(sv, t, k);
-            u64 sk, sval;
-            probe_slot<L>(sv, t, bk[h], g.sub, false, act && !hit, sk, sval);
-            const unsigned hb = g.ballot(act && !hit && sk == k);
-            em[h] = g.ballot(act && !hit && sk == kE);
-            if (hb && g.sub == lowest(hb)) {
-                if (L == SEP) st_vals<W>(sv.sub[t].vals + ((uint64_t)bk[h] * G + g.sub) * W, v);
-                else st_cg(sv.sub[t].keys + ((uint64_t)bk[h] * G + g.sub) * 2 + 1, v[0]);
+            for (int q = 0; q < W; q++) v[u][q] = pr.act[u] ? __ldg(vals + i * W + q) : 0ull;
+            if (pr.hb[u] && g.sub == lowest(pr.hb[u])) {
+                if (L == SEP) st_vals<W>(sv.sub[pr.ht[u]].vals + ((uint64_t)pr.hbk[u] * G + g.sub) * W, v[u]);
+                else st_cg(sv.sub[pr.ht[u]].keys + ((uint64_t)pr.hbk[u] * G + g.sub) * 2 + 1, v[u][0]);
             }
-            hit |= hb != 0;
+            isnew[u] = pr.act[u] && !pr.hb[u];
+            placed[u] = false;
         }
-        const bool isnew = act && !hit;
         if (FUSE && L == PACK) {
+            // first-fit CAS128 into the free pairs of t1, then t2; every round the
+            // U ops of the group each issue one CAS, so their round trips overlap
 #pragma unroll
             for (int h = 0; h < 2; h++) {
-                const uint32_t t = h ? p.t2 : p.t1;
-                unsigned e = isnew ? em[h] : 0u;
+                unsigned e[U];
+#pragma unroll
+                for (int u = 0; u < U; u++) e[u] = isnew[u] ? (h ? pr.em2[u] : pr.em1[u]) : 0u;
                 for (;;) {
-                    const unsigned cand = g.ballot(!placed && e != 0);
-                    if (!__any_sync(kFull, cand != 0)) break;
-                    bool ok = false;
-                    if (cand && g.sub == lowest(e)) {
-                        u64 ok_, ov_;
-                        cas128(sv.sub[t].keys + ((uint64_t)bk[h] * G + g.sub) * 2, kE, kE, k, v[0], ok_, ov_);
-                        ok = ok_ == kE && ov_ == kE;
+                    unsigned cand[U];
+                    bool any = false;
+#pragma unroll
+                    for (int u = 0; u < U; u++) {
+                        cand[u] = g.ballot(!placed[u] && e[u] != 0);
+                        any |= cand[u] != 0;
                     }
-                    const unsigned okb = g.ballot(ok);
-                    if (cand) {
-                        if (okb) placed = true;
-                        else e &= ~(1u << lowest(e));
+                    if (!__any_sync(kFull, any)) break;
+                    bool ok[U];
+#pragma unroll
+                    for (int u = 0; u < U; u++) {
+                        ok[u] = false;
+                        if (cand[u] && g.sub == lowest(e[u])) {
+                            const uint32_t t = h ? pr.p[u].t2 : pr.p[u].t1;
+                            const uint32_t bb = h ? pr.b2[u] : pr.b1[u];
+                            u64 ok_, ov_;
+                            cas128(sv.sub[t].keys + ((uint64_t)bb * G + g.sub) * 2, kE, kE, pr.k[u], v[u][0], ok_, ov_);
+                            ok[u] = ok_ == kE && ov_ == kE;
+                        }
+                    }
+#pragma unroll
+                    for (int u = 0; u < U; u++) {
+                        const unsigned okb = g.ballot(ok[u]);
+                        if (cand[u]) {
+                            if (okb) placed[u] = true;
+                            else e[u] &= ~(1u << lowest(e[u]));
+                        }
                     }
                 }
             }
         }
         const bool lead = g.sub == 0;
-        if (lead && i < n && status) status[i] = act ? (hit ? 2 : 1) : 0;
-        kv_append<W>(lead && isnew && !placed, k, v, pending, ctr + W_PENDING);
-        n_ins += lead && isnew;
-        n_upd += lead && act && hit;
+        bool app[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const uint64_t i = base + (uint64_t)u * QPW + grp;
+            if (lead && i < n && status) status[i] = pr.act[u] ? (pr.hb[u] ? 2 : 1) : 0;
+            app[u] = lead && isnew[u] && !placed[u];
+            n_ins += lead && isnew[u];
+            n_upd += lead && pr.act[u] && pr.hb[u];
+        }
+        block_append<W, U>(app, pr.k, v, pending, ctr + W_PENDING);
     }
     wblock_add<kThreads>(ctr + W_INSERTED, n_ins);
     wblock_add<kThreads>(ctr + W_UPDATED, n_upd);
@@ -673,7 +794,7 @@ __global__ void __launch_bounds__(kThreads) k_wplace_lockfree(WView tv, KVList s
 // ------------------------------------------------------------------ delete (S4)
 // Lock-free in every mode ("does not require locking"): the lane holding
 // the key overwrites it with EMPTY (PACK: the whole pair).
-template <int L, int W>
+template <int L, int W, int U>
 __global__ void __launch_bounds__(kThreads) k_wdelete(WView tv, const u64* __restrict__ keys, u64* __restrict__ old,
                                                       uint8_t* __restrict__ status, uint64_t n, u64* __restrict__ ctr) {
     constexpr int G = Lay<L>::B, QPW = 32 / G;
@@ -684,42 +805,39 @@ __global__ void __launch_bounds__(kThreads) k_wdelete(WView tv, const u64* __res
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     u64 removed = 0;
-    for (uint64_t base = w * QPW; base < n; base += nwarps * QPW) {
-        const uint64_t i = base + grp;
-        const u64 k = i < n ? __ldg(keys + i) : kE;
-        const bool act = k != kE;
-        const WPair p = wpair(tv, k);
-        bool hit = false;
+    for (uint64_t base = w * QPW * U; base < n; base += nwarps * QPW * U) {
+        Probe2<L, U> pr;
+        pr.run(tv, sv, g, keys, n, base, grp, false);
+        u64 v[U][W];
 #pragma unroll
-        for (int h = 0; h < 2; h++) {
-            const uint32_t t = h ? p.t2 : p.t1;
-            const uint32_t b = wbucket(sv, t, k);
-            u64 sk, sval;
-            probe_slot<L>(sv, t, b, g.sub, false, act && !hit, sk, sval);
-            const unsigned hb = g.ballot(act && !hit && sk == k);
-            if (hb && g.sub == lowest(hb)) {
-                u64 v[W];
+        for (int u = 0; u < U; u++) {
+            const bool mine = pr.hb[u] && g.sub == lowest(pr.hb[u]);
+#pragma unroll
+            for (int q = 0; q < W; q++) v[u][q] = kE;
+            if (mine) {
                 if (L == SEP) {
-                    if (old) ld_vals<W>(sv.sub[t].vals + ((uint64_t)b * G + g.sub) * W, v, false);
-                    st_cg(sv.sub[t].keys + (uint64_t)b * G + g.sub, kE);
+                    if (old) ld_vals<W>(sv.sub[pr.ht[u]].vals + ((uint64_t)pr.hbk[u] * G + g.sub) * W, v[u], false);
+                    st_cg(sv.sub[pr.ht[u]].keys + (uint64_t)pr.hbk[u] * G + g.sub, kE);
                 } else {
-                    v[0] = sval;
-                    st_pair(sv.sub[t].keys + ((uint64_t)b * G + g.sub) * 2, kE, kE);
+                    v[u][0] = pr.hv[u];
+                    st_pair(sv.sub[pr.ht[u]].keys + ((uint64_t)pr.hbk[u] * G + g.sub) * 2, kE, kE);
                 }
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const uint64_t i = base + (uint64_t)u * QPW + grp;
+            if (i >= n) continue;
+            const bool hit = pr.hb[u] != 0;
+            const bool writer = hit ? g.sub == lowest(pr.hb[u]) : g.sub == 0;
+            if (writer) {
                 if (old) {
 #pragma unroll
-                    for (int q = 0; q < W; q++) old[i * W + q] = v[q];
+                    for (int q = 0; q < W; q++) old[i * W + q] = hit ? v[u][q] : kE;
                 }
+                if (status) status[i] = hit ? 1 : 0;
+                removed += hit;
             }
-            hit |= hb != 0;
-        }
-        if (g.sub == 0 && i < n) {
-            if (status) status[i] = hit ? 1 : 0;
-            if (!hit && old) {
-#pragma unroll
-                for (int q = 0; q < W; q++) old[i * W + q] = kE;
-            }
-            removed += hit;
         }
     }
     wblock_add<kThreads>(ctr + W_REMOVED, removed);

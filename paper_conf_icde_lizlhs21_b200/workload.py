@@ -242,6 +242,25 @@ def c2_rand_static_torch(log2_n: int = 27, device="cuda", seed_cfg: Optional[int
     return cap, _as_i32(k), _as_i32(v), _as_i32(q), _as_i32(dk)
 
 
+def wide_static_torch(log2_n: int = 26, value_words: int = 2, device="cuda", beta: float = 0.85):
+    """C2's shape for the wide-key table (NEXT-3): 64-bit keys whose low half is
+    C2's key (distinct, so the 64-bit keys are distinct and misses stay misses)
+    and whose high half is a second mix of it; values of W words.  Returns
+    (init_capacity, keys i64[n], values i64[n, W], find_keys i64[n] (50% hit),
+    del_keys i64[n/2])."""
+    import torch
+    cap, k, _, q, dk = c2_rand_static_torch(log2_n, device=device, beta=beta)
+
+    def widen(x32):
+        lo = x32.to(torch.int64) & 0xFFFFFFFF
+        hi = _lowbias32_t(lo ^ 0x6A09E667)
+        return (hi << 32) | lo                       # int64 bit pattern of the u64 key
+
+    kw = widen(k)
+    vals = torch.stack([kw * (2 * w + 3) + w for w in range(value_words)], dim=1).contiguous()
+    return cap, kw, vals, widen(q), widen(dk)
+
+
 # ---------------------------------------------------------------------------
 # Config C3: TW/RE-shaped dynamic stream (PAPER.md §VI-A "Dynamic Hashing
 # Comparison", P:L729-737; datasets Table `table:exp_data_sets` P:L671-672).
