@@ -19,7 +19,8 @@ DYC_NOT_FOUND = 0xFFFFFFFF
 DYC_OK, DYC_ERR_INVALID_ARG, DYC_ERR_OOM, DYC_ERR_CUDA, DYC_ERR_INSERT_FAILED, DYC_ERR_NO_DEVICE = range(6)
 DYC_RESIZE_SPLIT, DYC_RESIZE_REINSERT_SUBTABLE, DYC_RESIZE_REHASH_ALL = range(3)
 DYC_PROF_KINDS = 16
-PROF_NAMES = ["k_find", "k_upsert", "k_place", "k_delete", "k_upsize", "k_downsize", "k_reinsert", "other"]
+PROF_NAMES = ["k_find", "k_upsert", "k_place", "k_delete", "k_upsize", "k_downsize", "k_reinsert", "other",
+              "bin_group", "bin_find", "bin_ins", "bin_place", "bin_delete", "bin_out"]
 _STATUS_NAMES = ["DYC_OK", "DYC_ERR_INVALID_ARG", "DYC_ERR_OOM", "DYC_ERR_CUDA",
                  "DYC_ERR_INSERT_FAILED", "DYC_ERR_NO_DEVICE"]
 
@@ -113,6 +114,8 @@ SIGNATURES = {
     "dyc_find_batch_host": (_I, [_TP, _P, _P, _P, _U64, _P]),
     "dyc_delete_batch_host": (_I, [_TP, _P, _P, _P, _U64, _P]),
     "dyc_launch_count": (_U64, [_TP, _I]),
+    "dyc_set_binning": (_I, [_TP, _I, _I, _I]),
+    "dyc_get_binning": (_I, [_TP, C.POINTER(_U64), C.POINTER(_U32)]),
     "dyc_profile_enable": (_I, [_TP, _I]),
     "dyc_profile_read": (_I, [_TP, _P, _P]),
     "dyc_route_count": (_I, [_TP, _P, _U64, _U32, _P, _P]),

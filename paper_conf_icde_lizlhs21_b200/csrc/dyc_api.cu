@@ -22,6 +22,7 @@
 #include "dycuckoo.h"
 #include "dyc_device.cuh"
 #include "dyc_kernels.cuh"
+#include "dyc_binned.cuh"
 
 using namespace dyc;
 
@@ -111,6 +112,15 @@ struct dyc_table {
         cudaEvent_t start = nullptr, done = nullptr;
     } rz;
     uint64_t n_live_resize = 0, n_deferred = 0;
+    // region-binned execution of large batches (dyc_binned.cuh, dyc_set_binning)
+    int bin_mode = 0;                      // 0 off (direct kernels), 1 binned whenever eligible
+    int bin_rlog2 = 0;                     // log2 buckets per region (0: ~16 MB regions)
+    int bin_olog2 = 20;                    // log2 ops per result group
+    uint32_t* bin_buf = nullptr;           // per-op record streams (u32 words)
+    uint64_t bin_cap = 0;                  // words
+    uint32_t* bin_small = nullptr;         // hist / offsets / cursors
+    uint64_t n_binned = 0;                 // batches run binned
+    uint32_t last_regions = 0;
     // per-kernel event profiling (dyc_profile_*)
     bool prof = false;
     struct Rec { int kind; cudaEvent_t a, b; };
@@ -575,6 +585,166 @@ dyc_status launch_apply(dyc_table* t, const unsigned long long* list, bool del, 
     return DYC_OK;
 }
 
+// ------------------------------------------------------------------ binned path
+// Region-binned execution (dyc_binned.cuh) of batches much larger than L2:
+// opt-in (dyc_set_binning mode 1).  Measured on B200 at config C2 it reaches
+// the L2 locality it aims for (every table line fetched once per pass) but its
+// passes are latency-bound (per-block rank / reserve / write chains), so it is
+// slower than the direct kernels there (profiles/r1g_binned.md) and is not the
+// default.  Eligible: no resize in flight, n < 2^30 ops.
+constexpr uint32_t kSmallWords = 2 * kMaxBins + 2 * (kMaxBins + 1) + 4 * kMaxBins + kMaxBins;
+
+bool bin_plan(dyc_table* t, uint64_t n, BinCtx& bc) {
+    if (t->bin_mode != 1 || t->rz.active || n == 0 || n >= (1ull << 30)) return false;
+    uint64_t NB = 0;
+    for (uint32_t i = 0; i < t->cfg.d; i++) NB += t->nb[i];
+    const uint64_t bucket_bytes = (uint64_t)t->cfg.bucket_slots * 8;
+    uint32_t rl = (uint32_t)t->bin_rlog2;
+    if (rl == 0) {
+        rl = 0;
+        while ((bucket_bytes << (rl + 1)) <= (16ull << 20)) rl++;
+    }
+    while (((NB + (1ull << rl) - 1) >> rl) > kMaxBins) rl++;
+    uint32_t ol = (uint32_t)std::max(1, t->bin_olog2);
+    while (((n + (1ull << ol) - 1) >> ol) > kMaxBins) ol++;
+    memset(&bc, 0, sizeof(bc));
+    uint64_t acc = 0;
+    for (uint32_t i = 0; i < t->cfg.d; i++) { bc.gbase[i] = acc; acc += t->nb[i]; }
+    bc.rshift = rl;
+    bc.R = (uint32_t)((NB + (1ull << rl) - 1) >> rl);
+    bc.ishift = ol;
+    bc.Rout = (uint32_t)((n + (1ull << ol) - 1) >> ol);
+    return true;
+}
+
+dyc_status bin_ensure(dyc_table* t, uint64_t words, cudaStream_t st) {
+    if (!t->bin_small) TRY(dev_alloc(t, (void**)&t->bin_small, kSmallWords * 4, st));
+    if (words <= t->bin_cap) return DYC_OK;
+    if (t->bin_buf) dev_free(t, t->bin_buf, st);
+    t->bin_buf = nullptr;
+    t->bin_cap = 0;
+    TRY(dev_alloc(t, (void**)&t->bin_buf, words * 4, st));
+    t->bin_cap = words;
+    return DYC_OK;
+}
+
+struct BinSmall {
+    uint32_t *hist, *off, *cur, *rcur;
+};
+
+// Region counts, bin offsets and cursors, then the grouping of the batch by the
+// region of h^{t1} into (ok, ov, oi).
+dyc_status bin_group(dyc_table* t, const BinCtx& bc, const uint32_t* keys, const uint32_t* vals, uint64_t n,
+                     uint32_t* ok, uint32_t* ov, uint32_t* oi, uint32_t* rv_out, uint8_t* rs_out, BinSmall& bs,
+                     cudaStream_t st) {
+    bs.hist = t->bin_small;
+    bs.off = bs.hist + 2 * kMaxBins;
+    bs.cur = bs.off + 2 * (kMaxBins + 1);
+    bs.rcur = bs.cur + 4 * kMaxBins;
+    CU(cudaMemsetAsync(bs.hist, 0, 2 * bc.R * 4, st));
+    const TableView tv = t->view();
+    ProfScope ps(t, DYC_PROF_BIN_GROUP, st);
+    k_bin_hist<<<grid_for(n, kThreads * 16), kThreads, 2 * bc.R * 4, st>>>(tv, bc, keys, n, bs.hist);
+    k_bin_offsets<<<1, 1024, 0, st>>>(bs.hist, bc.R, bc.Rout, bc.ishift, bs.off, bs.cur, bs.rcur);
+    k_bin_scatter<<<grid_for(n, (uint64_t)kThreads * kScatterItems), kThreads, bc.R * 4, st>>>(
+        tv, bc, keys, vals, n, bs.cur, ok, ov, oi, rv_out, rs_out);
+    t->launches += 2;
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+template <int B, int U>
+unsigned pass_grid(uint64_t n) { return grid_for(n, (uint64_t)(kThreads / (B / 4)) * U); }
+
+inline size_t pass_smem(const BinCtx& bc) { return (size_t)pass_smem_words(bc.R, bc.Rout) * 4; }
+
+// find (DEL = false) / delete (DEL = true): group by t1 region, F1/D1, F2/D2,
+// results back in request order.
+template <int B, bool DEL>
+dyc_status binned_fd(dyc_table* t, const BinCtx& bc, const uint32_t* keys, uint32_t* vals, uint8_t* flag, uint64_t n,
+                     cudaStream_t st) {
+    constexpr int U = 4;
+    TRY(bin_ensure(t, 6 * n, st));
+    uint32_t* Ak = t->bin_buf;
+    uint32_t* Ai = Ak + n;
+    uint32_t* Bk = Ai + n;
+    uint32_t* Bi = Bk + n;
+    uint32_t* Ri = Bi + n;
+    uint32_t* Rv = Ri + n;
+    BinSmall sm{};
+    TRY(bin_group(t, bc, keys, nullptr, n, Ak, nullptr, Ai, vals, flag, sm, st));
+    const TableView tv = t->view();
+    const uint32_t R = bc.R;
+    {
+        ProfScope ps(t, DEL ? DYC_PROF_BIN_DELETE : DYC_PROF_BIN_FIND, st);
+        PassIO io1{sm.off, sm.cur, Ak, nullptr, Ai, Bk, nullptr, Bi, sm.cur + R, Ri, Rv, sm.rcur};
+        k_bin_fd<B, U, DEL, false><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io1, t->d_ctr);
+        PassIO io2{sm.off + R + 1, sm.cur + R, Bk, nullptr, Bi, nullptr, nullptr, nullptr, nullptr, Ri, Rv, sm.rcur};
+        k_bin_fd<B, U, DEL, true><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io2, t->d_ctr);
+        t->launches++;
+    }
+    CU(cudaGetLastError());
+    if (vals || flag) {
+        ProfScope ps(t, DYC_PROF_BIN_OUT, st);
+        k_bin_out<<<grid_for(n, (uint64_t)kThreads * kOutItems), kThreads, 0, st>>>(Ri, Rv, sm.rcur, bc.ishift, n,
+                                                                                   vals, flag);
+    }
+    CU(cudaGetLastError());
+    t->n_binned++;
+    t->last_regions = bc.R;
+    return DYC_OK;
+}
+
+// insert (FUSE case): group by t1 region, I1 (t1 existence), I2 (t2 existence,
+// t2 placement of keys whose t1 bucket was full), I3 (t1 placement), I4 (t2
+// placement of the overflow); pending keys are then placed by insert_end.
+template <int B>
+dyc_status binned_ins(dyc_table* t, const BinCtx& bc, const uint32_t* keys, const uint32_t* vals, uint8_t* status,
+                      uint64_t n, cudaStream_t st) {
+    constexpr int U = 4;
+    TRY(bin_ensure(t, 7 * n, st));
+    uint32_t* Ak = t->bin_buf;
+    uint32_t* Av = Ak + n;
+    uint32_t* Ai = Av + n;
+    uint32_t* Bk = Ai + n;
+    uint32_t* Bv = Bk + n;
+    uint32_t* Bi = Bv + n;
+    uint32_t* Ri = status ? Bi + n : nullptr;
+    BinSmall sm{};
+    TRY(bin_group(t, bc, keys, vals, n, Ak, Av, Ai, nullptr, status, sm, st));
+    const TableView tv = t->view();
+    const uint32_t R = bc.R;
+    unsigned long long* pend = t->list[0];
+    {
+        ProfScope ps(t, DYC_PROF_BIN_INS, st);
+        PassIO io1{sm.off, sm.cur, Ak, Av, Ai, Bk, Bv, Bi, sm.cur + R, Ri, nullptr, sm.rcur};
+        k_bin_ins<B, U, false><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io1, pend, t->d_ctr);
+        PassIO io2{sm.off + R + 1, sm.cur + R, Bk, Bv, Bi, Ak, Av, nullptr, sm.cur + 2 * R, Ri, nullptr, sm.rcur};
+        k_bin_ins<B, U, true><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io2, pend, t->d_ctr);
+        t->launches++;
+    }
+    CU(cudaGetLastError());
+    {
+        ProfScope ps(t, DYC_PROF_BIN_PLACE, st);
+        PassIO io3{sm.off, sm.cur + 2 * R, Ak, Av, nullptr, Bk, Bv, nullptr, sm.cur + 3 * R, nullptr, nullptr, sm.rcur};
+        k_bin_place<B, U, false><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io3, pend, t->d_ctr);
+        PassIO io4{sm.off + R + 1, sm.cur + 3 * R, Bk, Bv, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr,
+                   nullptr, sm.rcur};
+        k_bin_place<B, U, true><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io4, pend, t->d_ctr);
+        t->launches++;
+    }
+    CU(cudaGetLastError());
+    if (status) {
+        ProfScope ps(t, DYC_PROF_BIN_OUT, st);
+        k_bin_out<<<grid_for(n, (uint64_t)kThreads * kOutItems), kThreads, 0, st>>>(Ri, nullptr, sm.rcur, bc.ishift,
+                                                                                   n, nullptr, status);
+    }
+    CU(cudaGetLastError());
+    t->n_binned++;
+    t->last_regions = bc.R;
+    return DYC_OK;
+}
+
 // insert = begin (scratch, counters, FUSE decision) + one k_upsert per chunk of
 // the batch + end (resize decision, placement, failures, alpha loop).  Splitting
 // the upsert into chunks is invisible to the semantics: every chunk only probes,
@@ -655,7 +825,9 @@ dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals,
                        cudaStream_t st) {
     bool fuse = false;
     TRY(insert_begin<B>(t, n, st, fuse));
-    TRY(insert_chunk<B>(t, keys, vals, status, n, fuse, st));
+    BinCtx bc;
+    if (fuse && bin_plan(t, n, bc)) TRY(binned_ins<B>(t, bc, keys, vals, status, n, st));
+    else TRY(insert_chunk<B>(t, keys, vals, status, n, fuse, st));
     return insert_end<B>(t, fuse, st);
 }
 
@@ -664,6 +836,8 @@ dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t
                      cudaStream_t st) {
     constexpr int ILP = (B <= 16) ? DYC_FIND_ILP : 2;
     constexpr uint64_t per_block = (uint64_t)(kThreads / (B / 4)) * ILP;   // queries per block per pass
+    BinCtx bc;
+    if (bin_plan(t, n, bc)) return binned_fd<B, false>(t, bc, keys, vals, found, n, st);
     {
         ProfScope ps(t, DYC_PROF_FIND, st);
         k_find<B, ILP><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n);
@@ -718,7 +892,9 @@ template <int B>
 dyc_status delete_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
                        cudaStream_t st) {
     TRY(delete_prep<B>(t, n, st));
-    TRY(delete_chunk<B>(t, keys, vals, status, n, st));
+    BinCtx bc;
+    if (bin_plan(t, n, bc)) TRY((binned_fd<B, true>(t, bc, keys, vals, status, n, st)));
+    else TRY(delete_chunk<B>(t, keys, vals, status, n, st));
     return delete_end<B>(t, st);
 }
 
@@ -1378,6 +1554,23 @@ dyc_status dyc_delete_batch_host(dyc_table* t, const uint32_t* h_keys, uint32_t*
     if (n == 0) return DYC_OK;
     if (!h_keys) return set_err(DYC_ERR_INVALID_ARG, "null keys");
     DISPATCH_B(t, delete_host_impl<B_>(t, h_keys, h_values_out, h_status, n, S(stream)));
+}
+
+dyc_status dyc_set_binning(dyc_table* t, int mode, int region_log2, int out_log2) {
+    TRY(check_table(t));
+    if (mode < 0 || mode > 1 || region_log2 < 0 || region_log2 > 31 || out_log2 < 0 || out_log2 > 29)
+        return set_err(DYC_ERR_INVALID_ARG, "dyc_set_binning: mode 0..1, region_log2 0..31, out_log2 0..29");
+    t->bin_mode = mode;
+    t->bin_rlog2 = region_log2;
+    t->bin_olog2 = out_log2 ? out_log2 : 20;
+    return DYC_OK;
+}
+
+dyc_status dyc_get_binning(const dyc_table* t, uint64_t* n_binned_batches, uint32_t* last_regions) {
+    TRY(check_table(t));
+    if (n_binned_batches) *n_binned_batches = t->n_binned;
+    if (last_regions) *last_regions = t->last_regions;
+    return DYC_OK;
 }
 
 uint64_t dyc_launch_count(const dyc_table* t, int reset) {
