@@ -275,7 +275,7 @@ dyc_status dyc_delete_batch_host(dyc_table* t, const uint32_t* h_keys, uint32_t*
  * Eligible: n < 2^30, no resize in flight, and for inserts no upsize needed
  * before placement ((m + n) <= beta*N).  Measured on B200 (DESIGN.md §5,
  * profiles/r1g_binned.md) it is slower than the direct kernels at config C2, so
- * it is opt-in.  region_log2 = 0 picks ~16 MB regions; out_log2 = 0 picks 2^20
+ * it is opt-in.  region_log2 = 0 picks ~32 MB regions; out_log2 = 0 picks 2^20
  * ops; both are raised as needed to keep at most 1024 bins.  Scratch: up to 32
  * bytes per op, owned by the table.  Errors: DYC_ERR_INVALID_ARG for mode
  * outside 0..1, region_log2 > 31 or out_log2 > 29. */

@@ -114,11 +114,10 @@ struct dyc_table {
     uint64_t n_live_resize = 0, n_deferred = 0;
     // region-binned execution of large batches (dyc_binned.cuh, dyc_set_binning)
     int bin_mode = 0;                      // 0 off (direct kernels), 1 binned whenever eligible
-    int bin_rlog2 = 0;                     // log2 buckets per region (0: ~16 MB regions)
+    int bin_rlog2 = 0;                     // log2 buckets per region (0: ~32 MB regions)
     int bin_olog2 = 20;                    // log2 ops per result group
     uint32_t* bin_buf = nullptr;           // per-op record streams (u32 words)
     uint64_t bin_cap = 0;                  // words
-    uint32_t* bin_small = nullptr;         // hist / offsets / cursors
     uint64_t n_binned = 0;                 // batches run binned
     uint32_t last_regions = 0;
     // per-kernel event profiling (dyc_profile_*)
@@ -587,107 +586,168 @@ dyc_status launch_apply(dyc_table* t, const unsigned long long* list, bool del, 
 
 // ------------------------------------------------------------------ binned path
 // Region-binned execution (dyc_binned.cuh) of batches much larger than L2:
-// opt-in (dyc_set_binning mode 1).  Measured on B200 at config C2 it reaches
-// the L2 locality it aims for (every table line fetched once per pass) but its
-// passes are latency-bound (per-block rank / reserve / write chains), so it is
-// slower than the direct kernels there (profiles/r1g_binned.md) and is not the
-// default.  Eligible: no resize in flight, n < 2^30 ops.
-constexpr uint32_t kSmallWords = 2 * kMaxBins + 2 * (kMaxBins + 1) + 4 * kMaxBins + kMaxBins;
-
+// opt-in (dyc_set_binning mode 1); see profiles/r1g_binned.md for its
+// measurements against the direct kernels.  Eligible: no resize in flight,
+// n < 2^30 ops.
 bool bin_plan(dyc_table* t, uint64_t n, BinCtx& bc) {
     if (t->bin_mode != 1 || t->rz.active || n == 0 || n >= (1ull << 30)) return false;
-    uint64_t NB = 0;
-    for (uint32_t i = 0; i < t->cfg.d; i++) NB += t->nb[i];
     const uint64_t bucket_bytes = (uint64_t)t->cfg.bucket_slots * 8;
     uint32_t rl = (uint32_t)t->bin_rlog2;
-    if (rl == 0) {
-        rl = 0;
-        while ((bucket_bytes << (rl + 1)) <= (16ull << 20)) rl++;
-    }
-    while (((NB + (1ull << rl) - 1) >> rl) > kMaxBins) rl++;
-    uint32_t ol = (uint32_t)std::max(1, t->bin_olog2);
+    if (rl == 0)
+        while ((bucket_bytes << (rl + 1)) <= (32ull << 20)) rl++;     // 32 MB regions (measured best)
+    auto regions = [&](uint32_t r) {
+        uint64_t R = 0;
+        for (uint32_t i = 0; i < t->cfg.d; i++) R += (t->nb[i] + (1ull << r) - 1) >> r;
+        return R;
+    };
+    while (regions(rl) > kMaxBins) rl++;
+    uint32_t ol = std::max<uint32_t>(kChunkShift, (uint32_t)t->bin_olog2);
     while (((n + (1ull << ol) - 1) >> ol) > kMaxBins) ol++;
     memset(&bc, 0, sizeof(bc));
     uint64_t acc = 0;
-    for (uint32_t i = 0; i < t->cfg.d; i++) { bc.gbase[i] = acc; acc += t->nb[i]; }
+    for (uint32_t i = 0; i < t->cfg.d; i++) {       // subtables start on region boundaries
+        bc.gbase[i] = acc;
+        acc += ((t->nb[i] + (1ull << rl) - 1) >> rl) << rl;
+    }
+    if (acc > 0xFFFFFFFFull) return false;          // global bucket indices are 32-bit
     bc.rshift = rl;
-    bc.R = (uint32_t)((NB + (1ull << rl) - 1) >> rl);
+    bc.R = (uint32_t)(acc >> rl);
     bc.ishift = ol;
     bc.Rout = (uint32_t)((n + (1ull << ol) - 1) >> ol);
+    bc.P = (uint32_t)(t->num_sms * kBinBPS);
     return true;
 }
 
-dyc_status bin_ensure(dyc_table* t, uint64_t words, cudaStream_t st) {
-    if (!t->bin_small) TRY(dev_alloc(t, (void**)&t->bin_small, kSmallWords * 4, st));
-    if (words <= t->bin_cap) return DYC_OK;
-    if (t->bin_buf) dev_free(t, t->bin_buf, st);
-    t->bin_buf = nullptr;
-    t->bin_cap = 0;
-    TRY(dev_alloc(t, (void**)&t->bin_buf, words * 4, st));
-    t->bin_cap = words;
+// Scratch of one binned batch.  Region streams A (t1 regions) and Bq (t2
+// regions) of uint4 records, the result stream (uint2 find/delete, uint32
+// insert); each with per-chunk fills, bin bases and cursors (dyc_binned.cuh).
+struct BinPlan {
+    uint32_t chA, chR;                   // chunks allocated per region stream / result stream
+    uint32_t *baseA, *ctrA, *baseB, *ctrB, *baseR, *ctrR, *tiles;
+    uint32_t *fillA, *fillB, *fillR;
+    uint4 *A, *Bq;
+    void* Res;
+};
+
+// Chunks of a region stream: the bins' expected capacities (the same integer
+// formula as k_bin_init_regions), rounded to kPoolAlign, plus a worst-case pool.
+uint32_t region_stream_chunks(const dyc_table* t, const BinCtx& bc, uint64_t n, uint32_t passes) {
+    uint64_t area = 0;
+    for (uint32_t r = 0; r < bc.R; r++) {
+        const uint64_t g0 = (uint64_t)r << bc.rshift;
+        uint32_t ti = 0;
+        for (uint32_t u = 1; u < t->cfg.d; u++)
+            if (bc.gbase[u] <= g0) ti = u;
+        const uint64_t lo = g0 - bc.gbase[ti];
+        const uint64_t hi = std::min<uint64_t>(t->nb[ti], lo + (1ull << bc.rshift));
+        area += bin_cap_chunks(region_expect(n, t->cfg.d, t->nb[ti], hi > lo ? hi - lo : 0), bc.P, passes);
+    }
+    area = (area + kPoolAlign - 1) / kPoolAlign * kPoolAlign;
+    const uint64_t pool = (n + kChunk - 1) / kChunk + (uint64_t)passes * bc.P * bc.R + kPoolAlign;
+    return (uint32_t)(area + pool);
+}
+
+dyc_status bin_alloc(dyc_table* t, const BinCtx& bc, uint64_t n, BinPlan& pl, cudaStream_t st) {
+    pl.chA = region_stream_chunks(t, bc, n, 1);
+    pl.chR = bc.Rout * (((1u << bc.ishift) >> kChunkShift) + 2 * (bc.P + 1));
+    const uint64_t small = 6ull * (kMaxBins + 1) + kTileCtrs;
+    const uint64_t words = small + 2ull * pl.chA + pl.chR + 8          // counters, fills (+ align)
+                           + 2ull * pl.chA * kChunk * 4                // A, Bq records (4 words each)
+                           + (uint64_t)pl.chR * kChunk * 2;            // results (<= 2 words each)
+    if (words > t->bin_cap) {
+        if (t->bin_buf) dev_free(t, t->bin_buf, st);
+        t->bin_buf = nullptr;
+        t->bin_cap = 0;
+        TRY(dev_alloc(t, (void**)&t->bin_buf, words * 4, st));
+        t->bin_cap = words;
+    }
+    uint32_t* w = t->bin_buf;
+    pl.baseA = w; w += kMaxBins + 1;
+    pl.ctrA = w;  w += kMaxBins + 1;
+    pl.baseB = w; w += kMaxBins + 1;
+    pl.ctrB = w;  w += kMaxBins + 1;
+    pl.baseR = w; w += kMaxBins + 1;
+    pl.ctrR = w;  w += kMaxBins + 1;
+    pl.tiles = w; w += kTileCtrs;
+    pl.fillA = w; w += pl.chA;
+    pl.fillB = w; w += pl.chA;
+    pl.fillR = w; w += pl.chR;
+    w = (uint32_t*)(((uintptr_t)w + 15) & ~(uintptr_t)15);
+    pl.A = (uint4*)w;  w += (uint64_t)pl.chA * kChunk * 4;
+    pl.Bq = (uint4*)w; w += (uint64_t)pl.chA * kChunk * 4;
+    pl.Res = w;
     return DYC_OK;
 }
 
-struct BinSmall {
-    uint32_t *hist, *off, *cur, *rcur;
-};
+template <class Rec>
+Stream<Rec> stream_of(Rec* rec, uint32_t* fill, uint32_t* ctr, const uint32_t* base, uint32_t nbins, uint32_t nch) {
+    return Stream<Rec>{rec, fill, ctr, base, nbins, nch};
+}
 
-// Region counts, bin offsets and cursors, then the grouping of the batch by the
-// region of h^{t1} into (ok, ov, oi).
+// Emptying a region stream before a kernel fills it: chunk fills to 0 and the
+// bin ranges / cursors from the expected counts.
+dyc_status region_reset(dyc_table* t, const BinCtx& bc, uint64_t n, uint32_t* fill, uint32_t nch, uint32_t* base,
+                        uint32_t* ctr, cudaStream_t st) {
+    CU(cudaMemsetAsync(fill, 0, (size_t)nch * 4, st));
+    k_bin_init_regions<<<1, 1024, 0, st>>>(t->view(), bc, n, 1, base, ctr);
+    t->launches++;
+    return DYC_OK;
+}
+
+template <class K>
+void allow_smem(K kernel) {
+    cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024);
+}
+
+// Bin ranges of streams A and R, tile counters, then the grouping of the batch
+// by the region of h^{t1} into stream A.
 dyc_status bin_group(dyc_table* t, const BinCtx& bc, const uint32_t* keys, const uint32_t* vals, uint64_t n,
-                     uint32_t* ok, uint32_t* ov, uint32_t* oi, uint32_t* rv_out, uint8_t* rs_out, BinSmall& bs,
-                     cudaStream_t st) {
-    bs.hist = t->bin_small;
-    bs.off = bs.hist + 2 * kMaxBins;
-    bs.cur = bs.off + 2 * (kMaxBins + 1);
-    bs.rcur = bs.cur + 4 * kMaxBins;
-    CU(cudaMemsetAsync(bs.hist, 0, 2 * bc.R * 4, st));
+                     uint32_t* rv_out, uint8_t* rs_out, BinPlan& pl, cudaStream_t st) {
     const TableView tv = t->view();
     ProfScope ps(t, DYC_PROF_BIN_GROUP, st);
-    k_bin_hist<<<grid_for(n, kThreads * 16), kThreads, 2 * bc.R * 4, st>>>(tv, bc, keys, n, bs.hist);
-    k_bin_offsets<<<1, 1024, 0, st>>>(bs.hist, bc.R, bc.Rout, bc.ishift, bs.off, bs.cur, bs.rcur);
-    k_bin_scatter<<<grid_for(n, (uint64_t)kThreads * kScatterItems), kThreads, bc.R * 4, st>>>(
-        tv, bc, keys, vals, n, bs.cur, ok, ov, oi, rv_out, rs_out);
-    t->launches += 2;
+    TRY(region_reset(t, bc, n, pl.fillA, pl.chA, pl.baseA, pl.ctrA, st));
+    CU(cudaMemsetAsync(pl.fillR, 0, (size_t)pl.chR * 4, st));
+    k_bin_init_results<<<1, 1024, 0, st>>>(bc, 2, pl.baseR, pl.ctrR, pl.tiles);
+    allow_smem(k_bin_scatter);
+    const Stream<uint4> A = stream_of(pl.A, pl.fillA, pl.ctrA, pl.baseA, bc.R, pl.chA);
+    k_bin_scatter<<<bc.P, kThreads, 6 * bc.R * 4, st>>>(tv, bc, keys, vals, n, A, rv_out, rs_out);
+    t->launches++;
     CU(cudaGetLastError());
     return DYC_OK;
 }
 
-template <int B, int U>
-unsigned pass_grid(uint64_t n) { return grid_for(n, (uint64_t)(kThreads / (B / 4)) * U); }
-
-inline size_t pass_smem(const BinCtx& bc) { return (size_t)pass_smem_words(bc.R, bc.Rout) * 4; }
+template <int B>
+constexpr int bin_U() { return B <= 8 ? DYC_BIN_U : (B == 16 ? 2 : 1); }
 
 // find (DEL = false) / delete (DEL = true): group by t1 region, F1/D1, F2/D2,
 // results back in request order.
 template <int B, bool DEL>
 dyc_status binned_fd(dyc_table* t, const BinCtx& bc, const uint32_t* keys, uint32_t* vals, uint8_t* flag, uint64_t n,
                      cudaStream_t st) {
-    constexpr int U = 4;
-    TRY(bin_ensure(t, 6 * n, st));
-    uint32_t* Ak = t->bin_buf;
-    uint32_t* Ai = Ak + n;
-    uint32_t* Bk = Ai + n;
-    uint32_t* Bi = Bk + n;
-    uint32_t* Ri = Bi + n;
-    uint32_t* Rv = Ri + n;
-    BinSmall sm{};
-    TRY(bin_group(t, bc, keys, nullptr, n, Ak, nullptr, Ai, vals, flag, sm, st));
+    constexpr int U = bin_U<B>();
+    BinPlan pl{};
+    TRY(bin_alloc(t, bc, n, pl, st));
+    TRY(bin_group(t, bc, keys, nullptr, n, vals, flag, pl, st));
+    TRY(region_reset(t, bc, n, pl.fillB, pl.chA, pl.baseB, pl.ctrB, st));
     const TableView tv = t->view();
-    const uint32_t R = bc.R;
+    const Stream<uint4> A = stream_of(pl.A, pl.fillA, pl.ctrA, pl.baseA, bc.R, pl.chA);
+    const Stream<uint4> Bs = stream_of(pl.Bq, pl.fillB, pl.ctrB, pl.baseB, bc.R, pl.chA);
+    const Stream<uint2> Rs = stream_of((uint2*)pl.Res, pl.fillR, pl.ctrR, pl.baseR, bc.Rout, pl.chR);
     {
         ProfScope ps(t, DEL ? DYC_PROF_BIN_DELETE : DYC_PROF_BIN_FIND, st);
-        PassIO io1{sm.off, sm.cur, Ak, nullptr, Ai, Bk, nullptr, Bi, sm.cur + R, Ri, Rv, sm.rcur};
-        k_bin_fd<B, U, DEL, false><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io1, t->d_ctr);
-        PassIO io2{sm.off + R + 1, sm.cur + R, Bk, nullptr, Bi, nullptr, nullptr, nullptr, nullptr, Ri, Rv, sm.rcur};
-        k_bin_fd<B, U, DEL, true><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io2, t->d_ctr);
+        allow_smem(k_bin_fd<B, U, DEL, false>);
+        allow_smem(k_bin_fd<B, U, DEL, true>);
+        k_bin_fd<B, U, DEL, false><<<bc.P, kThreads, 6 * (bc.R + bc.Rout) * 4, st>>>(tv, bc, A, Bs, Rs, pl.tiles,
+                                                                                     t->d_ctr);
+        k_bin_fd<B, U, DEL, true><<<bc.P, kThreads, 6 * bc.Rout * 4, st>>>(tv, bc, Bs, Bs, Rs, pl.tiles + 1,
+                                                                           t->d_ctr);
         t->launches++;
     }
     CU(cudaGetLastError());
     if (vals || flag) {
         ProfScope ps(t, DYC_PROF_BIN_OUT, st);
-        k_bin_out<<<grid_for(n, (uint64_t)kThreads * kOutItems), kThreads, 0, st>>>(Ri, Rv, sm.rcur, bc.ishift, n,
-                                                                                   vals, flag);
+        k_bin_out<uint2><<<grid_for((uint64_t)pl.chR * kChunk, (uint64_t)kThreads * 8), kThreads, 0, st>>>(Rs, vals,
+                                                                                                      flag);
     }
     CU(cudaGetLastError());
     t->n_binned++;
@@ -695,49 +755,40 @@ dyc_status binned_fd(dyc_table* t, const BinCtx& bc, const uint32_t* keys, uint3
     return DYC_OK;
 }
 
-// insert (FUSE case): group by t1 region, I1 (t1 existence), I2 (t2 existence,
-// t2 placement of keys whose t1 bucket was full), I3 (t1 placement), I4 (t2
-// placement of the overflow); pending keys are then placed by insert_end.
+// insert (FUSE case): group by t1 region, I1 (t1 existence + tentative t1
+// placement), I2 (t2 existence, t2 placement), I3 (cleanup of tentative copies
+// of keys that existed in t2); pending keys are then placed by insert_end.
 template <int B>
 dyc_status binned_ins(dyc_table* t, const BinCtx& bc, const uint32_t* keys, const uint32_t* vals, uint8_t* status,
                       uint64_t n, cudaStream_t st) {
-    constexpr int U = 4;
-    TRY(bin_ensure(t, 7 * n, st));
-    uint32_t* Ak = t->bin_buf;
-    uint32_t* Av = Ak + n;
-    uint32_t* Ai = Av + n;
-    uint32_t* Bk = Ai + n;
-    uint32_t* Bv = Bk + n;
-    uint32_t* Bi = Bv + n;
-    uint32_t* Ri = status ? Bi + n : nullptr;
-    BinSmall sm{};
-    TRY(bin_group(t, bc, keys, vals, n, Ak, Av, Ai, nullptr, status, sm, st));
+    constexpr int U = bin_U<B>();
+    BinPlan pl{};
+    TRY(bin_alloc(t, bc, n, pl, st));
+    TRY(bin_group(t, bc, keys, vals, n, nullptr, status, pl, st));
     const TableView tv = t->view();
-    const uint32_t R = bc.R;
+    const Stream<uint4> A = stream_of(pl.A, pl.fillA, pl.ctrA, pl.baseA, bc.R, pl.chA);
+    const Stream<uint4> Bs = stream_of(pl.Bq, pl.fillB, pl.ctrB, pl.baseB, bc.R, pl.chA);
+    const Stream<uint32_t> Rs = stream_of(status ? (uint32_t*)pl.Res : (uint32_t*)nullptr, pl.fillR, pl.ctrR,
+                                          pl.baseR, bc.Rout, pl.chR);
     unsigned long long* pend = t->list[0];
     {
         ProfScope ps(t, DYC_PROF_BIN_INS, st);
-        PassIO io1{sm.off, sm.cur, Ak, Av, Ai, Bk, Bv, Bi, sm.cur + R, Ri, nullptr, sm.rcur};
-        k_bin_ins<B, U, false><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io1, pend, t->d_ctr);
-        PassIO io2{sm.off + R + 1, sm.cur + R, Bk, Bv, Bi, Ak, Av, nullptr, sm.cur + 2 * R, Ri, nullptr, sm.rcur};
-        k_bin_ins<B, U, true><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io2, pend, t->d_ctr);
-        t->launches++;
-    }
-    CU(cudaGetLastError());
-    {
-        ProfScope ps(t, DYC_PROF_BIN_PLACE, st);
-        PassIO io3{sm.off, sm.cur + 2 * R, Ak, Av, nullptr, Bk, Bv, nullptr, sm.cur + 3 * R, nullptr, nullptr, sm.rcur};
-        k_bin_place<B, U, false><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io3, pend, t->d_ctr);
-        PassIO io4{sm.off + R + 1, sm.cur + 3 * R, Bk, Bv, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr,
-                   nullptr, sm.rcur};
-        k_bin_place<B, U, true><<<pass_grid<B, U>(n), kThreads, pass_smem(bc), st>>>(tv, bc, io4, pend, t->d_ctr);
-        t->launches++;
+        allow_smem(k_bin_ins<B, U, false>);
+        allow_smem(k_bin_ins<B, U, true>);
+        TRY(region_reset(t, bc, n, pl.fillB, pl.chA, pl.baseB, pl.ctrB, st));
+        k_bin_ins<B, U, false><<<bc.P, kThreads, 6 * (bc.R + bc.Rout) * 4, st>>>(tv, bc, A, Bs, Rs, pend, pl.tiles,
+                                                                                 t->d_ctr);
+        TRY(region_reset(t, bc, n, pl.fillA, pl.chA, pl.baseA, pl.ctrA, st));
+        k_bin_ins<B, U, true><<<bc.P, kThreads, 6 * (bc.R + bc.Rout) * 4, st>>>(tv, bc, Bs, A, Rs, pend,
+                                                                                pl.tiles + 1, t->d_ctr);
+        k_bin_cleanup<B, U><<<bc.P, kThreads, 0, st>>>(tv, bc, A, pl.tiles + 2, t->d_ctr);
+        t->launches += 2;
     }
     CU(cudaGetLastError());
     if (status) {
         ProfScope ps(t, DYC_PROF_BIN_OUT, st);
-        k_bin_out<<<grid_for(n, (uint64_t)kThreads * kOutItems), kThreads, 0, st>>>(Ri, nullptr, sm.rcur, bc.ishift,
-                                                                                   n, nullptr, status);
+        k_bin_out<uint32_t><<<grid_for((uint64_t)pl.chR * kChunk, (uint64_t)kThreads * 8), kThreads, 0, st>>>(
+            Rs, nullptr, status);
     }
     CU(cudaGetLastError());
     t->n_binned++;

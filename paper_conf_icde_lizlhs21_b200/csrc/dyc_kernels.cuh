@@ -38,6 +38,9 @@ constexpr int kThreads = 256;
 #ifndef DYC_DELETE_U
 #define DYC_DELETE_U 2
 #endif
+#ifndef DYC_UPSERT_SPEC
+#define DYC_UPSERT_SPEC 0
+#endif
 #ifndef DYC_FIND_ILP
 #define DYC_FIND_ILP 4
 #endif
@@ -54,6 +57,7 @@ enum CounterIdx : int {
     C_SECOND = 8,     // keys in their second-choice subtable (stats)
     C_RES_TOTAL = 9,  // residuals over several downsizes of one alpha loop
     C_DEFER = 10,     // ops on a subtable locked by a resize in flight (NEXT-1)
+    C_CLEANUP = 11,   // binned insert: keys placed in t1 by I1 that turned out to live in t2
     C_COUNT0 = 16,    // per-subtable live counts [16, 32)
     C_N = 32
 };
@@ -314,6 +318,39 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
         bool need2[U], isnew[U], placed[U];
         int j1[U], j2[U];
         bool lk1[U], lk2[U];
+#if DYC_UPSERT_SPEC
+        // speculative: both candidate buckets are read together (one round trip);
+        // the t2 read is wasted only for keys found in t1 (updates)
+        {
+            unsigned long long s1[U][4], s2[U][4];
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                i[u] = base + (uint64_t)u * QPW + grp;
+                const bool valid = i[u] < n;
+                k[u] = valid ? __ldg(keys + i[u]) : kEmptyKey;
+                kv[u] = make_kv(k[u], valid ? __ldg(vals + i[u]) : 0u);
+                const Pair p = pair_of(tv, k[u]);
+                lk1[u] = LK && p.t1 == locked;
+                lk2[u] = LK && p.t2 == locked;
+                b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
+                b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
+                probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
+#pragma unroll
+                for (int q = 0; q < 4; q++) s2[u][q] = kEmptySlot;
+                probe_cg_pred<B>(b2[u] + 4 * g.sub, s2[u], k[u] != kEmptyKey);
+            }
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                const bool active = k[u] != kEmptyKey;
+                j1[u] = match_slot<4>(s1[u], k[u]);
+                em1[u] = lk1[u] ? 0u : empty_mask(s1[u]);
+                h1[u] = g.ballot(active && j1[u] >= 0);
+                need2[u] = active && h1[u] == 0;
+                j2[u] = need2[u] ? match_slot<4>(s2[u], k[u]) : -1;
+                em2[u] = (lk2[u] || !need2[u]) ? 0u : empty_mask(s2[u]);
+            }
+        }
+#else
         {
             unsigned long long s1[U][4];
 #pragma unroll
@@ -352,6 +389,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                 em2[u] = lk2[u] ? 0u : empty_mask(s2[u]);
             }
         }
+#endif
 #pragma unroll
         for (int u = 0; u < U; u++) {
             h2[u] = g.ballot(need2[u] && j2[u] >= 0);
