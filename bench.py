@@ -251,7 +251,9 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
     traffic, traffic_src = None, None
     pdir = os.path.join(ROOT, "profiles")
     tr_files = sorted(f for f in os.listdir(pdir) if f.endswith("_traffic.json")) if os.path.isdir(pdir) else []
-    if tr_files and args.log2n == 27 and args.bucket_slots == 8 and n_ins == (1 << 27):
+    # the captured traffic is per launch of the unchunked C2 kernel: only comparable
+    # when the timed path launches the dominant kernel once per step (not routed)
+    if tr_files and args.log2n == 27 and args.bucket_slots == 8 and n_ins == (1 << 27) and calls == 1:
         tr = json.load(open(os.path.join(pdir, tr_files[-1])))
         if dom in tr:
             traffic, traffic_src = tr[dom], f"profiles/{tr_files[-1]} (ncu --set full, dram read+write per launch)"
