@@ -247,7 +247,33 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
     torch.cuda.synchronize()
     gather_ms = e0.elapsed_time(e1)
     gather_gbs = nreads * bkt / (gather_ms * 1e-3) / 1e9
+    # the same reads, each followed by an 8-byte store into the bucket read (the
+    # probe-then-write pattern of insert/delete: a read plus a dirty-line write-back)
+    for seed in (17, 18):
+        if seed == 18:
+            e2, e3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e2.record(stream)
+        L.check(L.dyc_bench_gather_ex(buf.data_ptr(), buf.numel(), nreads, bkt, seed, L.DYC_GATHER_WRITE,
+                                      sink.data_ptr(), stream.cuda_stream), "dyc_bench_gather_ex")
+    e3.record(stream)
+    torch.cuda.synchronize()
+    rw_ms = e2.elapsed_time(e3)
     del buf
+    # Linear cost model of random accesses from the two measurements: a bucket
+    # read costs 1/R, a write-back cw = 1/M - 1/R (M = read+write ops/s).  A
+    # kernel doing r reads and w write-backs per op then peaks at 1/(r/R + w*cw)
+    # ops/s; frac_of_access_ceiling = its ops/s over that.
+    R = nreads / (gather_ms * 1e-3)
+    M = nreads / (rw_ms * 1e-3)
+    cw = max(0.0, 1.0 / M - 1.0 / R)
+    placed = (n_ins - pend) / max(1, n_ins)
+    acc_model = {"k_find": (probes_find, 0.0, n_find), "k_upsert": (2.0, placed, n_ins),
+                 "k_delete": (1.0 + phi_del, 1.0, n_del)}
+    acc_frac = {}
+    for k, (r_, w_, units) in acc_model.items():
+        if k in kern and kern[k] > 0:
+            ceiling = 1.0 / (r_ / R + w_ * cw)
+            acc_frac[k] = round(units / (kern[k] * 1e-3) / ceiling, 4)
     traffic, traffic_src = None, None
     pdir = os.path.join(ROOT, "profiles")
     tr_files = sorted(f for f in os.listdir(pdir) if f.endswith("_traffic.json")) if os.path.isdir(pdir) else []
@@ -267,6 +293,12 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
                                   "gprobes_per_s": nreads / (gather_ms * 1e-3) / 1e9,
                                   "what": "dyc_bench_gather: random bucket reads, probe access pattern only"},
         "frac_of_random_ceiling": achieved / gather_gbs,
+        "access_ceiling": {"read_gaccess_per_s": R / 1e9, "read_then_write_gops_per_s": M / 1e9,
+                           "write_back_ns": cw * 1e9,
+                           "model_reads_writes_per_op": {k: [round(v[0], 4), round(v[1], 4)] for k, v in acc_model.items()},
+                           "what": "dyc_bench_gather(_ex): random bucket reads, and reads each followed by a store "
+                                   "into the bucket; ceiling(kernel) = 1/(reads/R + writes*(1/M - 1/R))"},
+        "frac_of_access_ceiling": acc_frac,
         "kernel_ms_per_step": {k: round(v, 4) for k, v in kern.items()},
         "other_kernels_ms_per_step": round(prof["other"][0] / args.steps, 4),
         "model": {"phi": phi, "hit_rate": hit_rate, "evictions_per_insert": E, "probes_per_find": probes_find,

@@ -350,6 +350,15 @@ dyc_status dyc_bench_gather(const void* d_buf, uint64_t buf_bytes, uint64_t n_re
                             uint32_t bytes_per_read, uint64_t seed, uint64_t* d_sink,
                             dyc_stream_t stream);
 
+/* dyc_bench_gather with flags: DYC_GATHER_WRITE (1) makes every read followed
+ * by an 8-byte store into the bucket just read (the probe-then-write pattern of
+ * insert and delete: one random read plus one dirty-line write-back per op), so
+ * d_buf is overwritten.  Errors: DYC_ERR_INVALID_ARG for other flag bits or
+ * sizes as in dyc_bench_gather. */
+#define DYC_GATHER_WRITE 1u
+dyc_status dyc_bench_gather_ex(void* d_buf, uint64_t buf_bytes, uint64_t n_reads, uint32_t bytes_per_read,
+                               uint64_t seed, uint32_t flags, uint64_t* d_sink, dyc_stream_t stream);
+
 /* Device-wide L2 fetch granularity (cudaLimitMaxL2FetchGranularity, bytes in
  * 0..128, a hint) for the current device: how much the L2 pulls from HBM on a
  * sector miss.  Random 32-byte bucket probes want 32. */

@@ -19,6 +19,7 @@ DYC_NOT_FOUND = 0xFFFFFFFF
 DYC_OK, DYC_ERR_INVALID_ARG, DYC_ERR_OOM, DYC_ERR_CUDA, DYC_ERR_INSERT_FAILED, DYC_ERR_NO_DEVICE = range(6)
 DYC_RESIZE_SPLIT, DYC_RESIZE_REINSERT_SUBTABLE, DYC_RESIZE_REHASH_ALL = range(3)
 DYC_PROF_KINDS = 16
+DYC_GATHER_WRITE = 1
 PROF_NAMES = ["k_find", "k_upsert", "k_place", "k_delete", "k_upsize", "k_downsize", "k_reinsert", "other",
               "bin_group", "bin_find", "bin_ins", "bin_place", "bin_delete", "bin_out"]
 _STATUS_NAMES = ["DYC_OK", "DYC_ERR_INVALID_ARG", "DYC_ERR_OOM", "DYC_ERR_CUDA",
@@ -122,6 +123,7 @@ SIGNATURES = {
     "dyc_route_scatter": (_I, [_TP, _P, _P, _P, _U64, _U32, _P, _P, _P, _P, _P, _P, _P]),
     "dyc_route_unpermute": (_I, [_P, _U64, _P, _P, _P, _P, _P]),
     "dyc_bench_gather": (_I, [_P, _U64, _U64, _U32, _U64, _P, _P]),
+    "dyc_bench_gather_ex": (_I, [_P, _U64, _U64, _U32, _U64, _U32, _P, _P]),
     "dyc_set_l2_fetch_granularity": (_I, [_U32]),
     "dyc_get_l2_fetch_granularity": (_I, [C.POINTER(_U32)]),
     "dyc_last_error": (C.c_char_p, []),

@@ -1726,26 +1726,36 @@ dyc_status dyc_get_l2_fetch_granularity(uint32_t* bytes) {
     return DYC_OK;
 }
 
-dyc_status dyc_bench_gather(const void* d_buf, uint64_t buf_bytes, uint64_t n_reads, uint32_t bytes_per_read,
-                            uint64_t seed, uint64_t* d_sink, dyc_stream_t stream) {
+dyc_status dyc_bench_gather_ex(void* d_buf, uint64_t buf_bytes, uint64_t n_reads, uint32_t bytes_per_read,
+                               uint64_t seed, uint32_t flags, uint64_t* d_sink, dyc_stream_t stream) {
     if (bytes_per_read != 32 && bytes_per_read != 64 && bytes_per_read != 128 && bytes_per_read != 256)
         return set_err(DYC_ERR_INVALID_ARG, "bytes_per_read must be 32, 64, 128 or 256");
+    if (flags & ~1u) return set_err(DYC_ERR_INVALID_ARG, "flags: only DYC_GATHER_WRITE (1) is defined");
     const uint64_t units = buf_bytes / bytes_per_read;
     if (units == 0) return set_err(DYC_ERR_INVALID_ARG, "buffer too small");
     const uint64_t lanes_per_read = bytes_per_read / 32;
     const unsigned grid = grid_for(n_reads * lanes_per_read, (uint64_t)kThreads * 4);
-    const unsigned long long* buf = (const unsigned long long*)d_buf;
+    unsigned long long* buf = (unsigned long long*)d_buf;
     unsigned long long* sink = (unsigned long long*)d_sink;
-    for (uint64_t s_ = 0; s_ < 1; s_++) {
-        switch (bytes_per_read) {
-            case 32: k_gather<4><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
-            case 64: k_gather<8><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
-            case 128: k_gather<16><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
-            default: k_gather<32><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break;
-        }
+    const bool wr = flags & 1u;
+#define DYC_GATHER(BB)                                                                               \
+    (wr ? k_gather<BB, true><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink)      \
+        : k_gather<BB, false><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink))
+    switch (bytes_per_read) {
+        case 32: DYC_GATHER(4); break;
+        case 64: DYC_GATHER(8); break;
+        case 128: DYC_GATHER(16); break;
+        default: DYC_GATHER(32); break;
     }
+#undef DYC_GATHER
     CU(cudaGetLastError());
     return DYC_OK;
+}
+
+dyc_status dyc_bench_gather(const void* d_buf, uint64_t buf_bytes, uint64_t n_reads, uint32_t bytes_per_read,
+                            uint64_t seed, uint64_t* d_sink, dyc_stream_t stream) {
+    return dyc_bench_gather_ex(const_cast<void*>(d_buf), buf_bytes, n_reads, bytes_per_read, seed, 0, d_sink,
+                               stream);
 }
 
 }  // extern "C"

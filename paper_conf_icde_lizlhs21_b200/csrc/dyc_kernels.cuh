@@ -899,8 +899,11 @@ __global__ void __launch_bounds__(kThreads) k_route_unpermute(const uint32_t* __
 // uniformly random bucket-aligned offsets, by a G = B/4 lane group with the same
 // 256-bit loads and L2 prefetch size as k_find.  Its rate is the random-access
 // ceiling the probe kernels are compared with.
-template <int B>
-__global__ void __launch_bounds__(kThreads) k_gather(const unsigned long long* __restrict__ buf, uint64_t n_units,
+// WRITE: after its read, each group also stores one 8-byte slot into the bucket
+// it read (the probe-then-write pattern of an insert or delete: one read plus
+// one dirty-line write-back per op); the stored word depends on the data read.
+template <int B, bool WRITE = false>
+__global__ void __launch_bounds__(kThreads) k_gather(unsigned long long* __restrict__ buf, uint64_t n_units,
                                                      uint64_t n_reads, uint64_t seed,
                                                      unsigned long long* __restrict__ sink) {
     constexpr int G = B / 4, QPW = 32 / G, ILP = 4;
@@ -911,6 +914,7 @@ __global__ void __launch_bounds__(kThreads) k_gather(const unsigned long long* _
     unsigned long long acc = 0;
     for (uint64_t base = w * QPW * ILP; base < n_reads; base += nwarps * QPW * ILP) {
         unsigned long long s[ILP][4];
+        unsigned long long* wp[ILP];
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
             const uint64_t i = base + (uint64_t)j * QPW + grp;
@@ -918,11 +922,21 @@ __global__ void __launch_bounds__(kThreads) k_gather(const unsigned long long* _
             h ^= h >> 29;
             h *= 0xBF58476D1CE4E5B9ull;
             h ^= h >> 32;
-            const unsigned long long* p = buf + __umul64hi(h, n_units) * B + 4 * g.sub;
-            probe_nc_pred<B>(p, s[j], i < n_reads);
+            unsigned long long* p = buf + __umul64hi(h, n_units) * B + 4 * g.sub;
+            if (WRITE) {
+                probe_cg_pred<B>(p, s[j], i < n_reads);
+                wp[j] = i < n_reads ? p : nullptr;
+            } else {
+                probe_nc_pred<B>(p, s[j], i < n_reads);
+            }
         }
 #pragma unroll
         for (int j = 0; j < ILP; j++) acc ^= s[j][0] ^ s[j][1] ^ s[j][2] ^ s[j][3];
+        if (WRITE) {
+#pragma unroll
+            for (int j = 0; j < ILP; j++)
+                if (g.sub == 0 && wp[j]) st_u64_cg(wp[j] + (acc & 3), s[j][0] + 1);
+        }
     }
     if (acc == 0x0123456789ABCDEFull) *sink = acc;   // keeps the loads alive
 }
