@@ -57,7 +57,7 @@ namespace dyc {
 #define DYC_BIN_BPS 4
 #endif
 #ifndef DYC_BIN_U
-#define DYC_BIN_U 2
+#define DYC_BIN_U 1
 #endif
 constexpr uint32_t kMaxBins = 1024;   // regions per bin set; result groups per batch
 constexpr uint32_t kChunk = 128;      // records per chunk
@@ -103,7 +103,7 @@ __host__ __device__ __forceinline__ uint64_t region_expect(uint64_t n, uint32_t 
 struct BinSmem {
     uint64_t gbase[kMaxD];
     uint8_t t_of_r[kMaxBins];           // subtable of region r
-    uint32_t tile;                      // tile handed to the block
+    uint32_t tile, tile2;               // tiles handed to the block (current / next)
 };
 
 __device__ __forceinline__ void load_bins(const TableView& tv, const BinCtx& bc, BinSmem& bs) {
@@ -347,7 +347,7 @@ _Pragma("unroll")
 _Pragma("unroll")
         for (int u = 0; u < U; u++) {
             j[u] = todo[u] ? (uint32_t)(__ffs(free[u]) - 1) : 0u;
-            old[u] = todo[u] ? cas_slot(bp[u] + j[u], kEmptySlot, kv[u]) : 0ull;
+            old[u] = cas_slot_pred(bp[u] + j[u], kEmptySlot, kv[u], todo[u], 0ull);
         }
 _Pragma("unroll")
         for (int u = 0; u < U; u++) {
@@ -363,41 +363,69 @@ __device__ __forceinline__ uint32_t gbucket(const BinSmem& bs, const SmemView& s
     return (uint32_t)(bs.gbase[t] + bucket_of(sv, t, k));
 }
 
-// Loads record u of this lane in the tile at chunk c0, hashes its bucket in the
-// subtable of its region and issues the probe.  Returns whether the position
-// holds a record.
-template <int B, int U, bool NC>
-__device__ __forceinline__ bool load_probe(const Stream<uint4>& in, const BinSmem& bs, const SmemView& sv,
-                                           uint32_t c0, int u, uint4& r, uint32_t& cur,
-                                           unsigned long long*& bp, unsigned long long (&s)[B]) {
-    uint32_t p = 0, bin = 0;
-    const bool has = tile_rec<U>(in.fill, c0, in.pool_end, u, p, bin);
-    r = has ? __ldcs(in.rec + p) : make_uint4(kEmptyKey, 0, 0, 0);
+// Loads the U records of this lane in the tile at chunk c0 (kNone: none), with
+// whether each position holds a record and its bin.  Issued one tile ahead of
+// its use (see DYC_BIN_TILE_LOOP), so the stream latency overlaps the probes
+// and appends of the tile before.
+template <int U>
+__device__ __forceinline__ void load_recs(const Stream<uint4>& in, uint32_t c0, uint4 (&r)[U], bool (&has)[U],
+                                          uint32_t (&bin)[U]) {
+_Pragma("unroll")
+    for (int u = 0; u < U; u++) {
+        uint32_t p = 0;
+        bin[u] = 0;
+        has[u] = c0 != kNone && tile_rec<U>(in.fill, c0, in.pool_end, u, p, bin[u]);
+        r[u] = has[u] ? __ldcs(in.rec + p) : make_uint4(kEmptyKey, 0, 0, 0);
+    }
+}
+
+// Hashes a record's bucket in the subtable of its region and issues the probe.
+template <int B, bool NC>
+__device__ __forceinline__ void probe_rec(const BinSmem& bs, const SmemView& sv, const uint4& r, bool has,
+                                          uint32_t bin, uint32_t& cur, unsigned long long*& bp,
+                                          unsigned long long (&s)[B]) {
     const uint32_t t = bs.t_of_r[has ? bin : 0];
     const uint32_t b = has ? bucket_of(sv, t, r.x) : 0u;
     cur = (uint32_t)(bs.gbase[t] + b);
     bp = bucket_ptr(sv, t, b, B);
     probe_lane<B, NC>(bp, s, has);
-    return has;
 }
 
-// Tile loop of a persistent consumer: BODY runs for every tile (chunk c0); the
-// next tile index is fetched by thread 0 before the body (its latency overlaps).
-#define DYC_BIN_TILE_LOOP(WK, BS, ...)                                                   \
-    {                                                                                    \
-        if (threadIdx.x == 0) (BS).tile = atomicAdd((WK).counter, 1u);                   \
-        __syncthreads();                                                                 \
-        uint32_t tile_ = (BS).tile;                                                      \
-        while (tile_ < (WK).total()) {                                                   \
-            __syncthreads();                                                             \
-            uint32_t nxt_ = 0;                                                           \
-            if (threadIdx.x == 0) nxt_ = atomicAdd((WK).counter, 1u);                    \
-            const uint32_t c0 = (WK).chunk0(tile_);                                      \
-            __VA_ARGS__                                                                  \
-            if (threadIdx.x == 0) (BS).tile = nxt_;                                      \
-            __syncthreads();                                                             \
-            tile_ = (BS).tile;                                                           \
-        }                                                                                \
+// Tile loop of a persistent consumer of stream IN: the body runs for every tile
+// with the tile's records prefetched in pr/ph/pb (record, present, bin); the
+// records of the next tile are loaded before the body, and thread 0 fetches the
+// index of the tile after that, so neither latency sits on the body's chain.
+#define DYC_BIN_TILE_LOOP(U_, IN, WK, BS, ...)                                              \
+    {                                                                                       \
+        if (threadIdx.x == 0) {                                                             \
+            (BS).tile = atomicAdd((WK).counter, 1u);                                        \
+            (BS).tile2 = atomicAdd((WK).counter, 1u);                                       \
+        }                                                                                   \
+        __syncthreads();                                                                    \
+        uint32_t tile_ = (BS).tile, next_ = (BS).tile2;                                     \
+        uint4 pr[U_];                                                                       \
+        bool ph[U_];                                                                        \
+        uint32_t pb[U_];                                                                    \
+        load_recs<U_>(IN, tile_ < (WK).total() ? (WK).chunk0(tile_) : kNone, pr, ph, pb);   \
+        while (tile_ < (WK).total()) {                                                      \
+            __syncthreads();                                                                \
+            uint32_t nn_ = 0;                                                               \
+            if (threadIdx.x == 0) nn_ = atomicAdd((WK).counter, 1u);                        \
+            uint4 qr[U_];                                                                   \
+            bool qh[U_];                                                                    \
+            uint32_t qb[U_];                                                                \
+            load_recs<U_>(IN, next_ < (WK).total() ? (WK).chunk0(next_) : kNone, qr, qh, qb); \
+            __VA_ARGS__                                                                     \
+            _Pragma("unroll") for (int u_ = 0; u_ < U_; u_++) {                             \
+                pr[u_] = qr[u_];                                                            \
+                ph[u_] = qh[u_];                                                            \
+                pb[u_] = qb[u_];                                                            \
+            }                                                                               \
+            if (threadIdx.x == 0) (BS).tile = nn_;                                          \
+            __syncthreads();                                                                \
+            tile_ = next_;                                                                  \
+            next_ = (BS).tile;                                                              \
+        }                                                                                   \
     }
 
 // ------------------------------------------------------- grouping by region
@@ -477,7 +505,7 @@ __global__ void __launch_bounds__(kThreads, kBinBPS) k_bin_fd(TableView tv, BinC
     load_view(tv, sv);
     const Walker<U> wk = make_walker<U>(in, tiles);
     unsigned long long removed = 0;
-    DYC_BIN_TILE_LOOP(wk, bs, {
+    DYC_BIN_TILE_LOOP(U, in, wk, bs, {
         uint4 r[U];
         bool has[U], hit[U];
         uint32_t v[U], ob[U], rk[U], cur[U];
@@ -485,7 +513,11 @@ __global__ void __launch_bounds__(kThreads, kBinBPS) k_bin_fd(TableView tv, BinC
             unsigned long long s[U][B];
             unsigned long long* bp[U];
 _Pragma("unroll")
-            for (int u = 0; u < U; u++) has[u] = load_probe<B, U, !DEL>(in, bs, sv, c0, u, r[u], cur[u], bp[u], s[u]);
+            for (int u = 0; u < U; u++) {
+                r[u] = pr[u];
+                has[u] = ph[u];
+                probe_rec<B, !DEL>(bs, sv, r[u], has[u], pb[u], cur[u], bp[u], s[u]);
+            }
 _Pragma("unroll")
             for (int u = 0; u < U; u++) {
                 const int j = has[u] ? lane_match<B>(s[u], r[u].x) : -1;
@@ -550,7 +582,7 @@ __global__ void __launch_bounds__(kThreads, kBinBPS) k_bin_ins(TableView tv, Bin
     load_view(tv, sv);
     const Walker<U> wk = make_walker<U>(in, tiles);
     unsigned long long n_ins = 0, n_upd = 0, n_clean = 0;
-    DYC_BIN_TILE_LOOP(wk, bs, {
+    DYC_BIN_TILE_LOOP(U, in, wk, bs, {
         uint4 r[U];
         bool has[U], hit[U], fwd[U];
         uint32_t nb_[U], nrk[U], rb[U], rrk[U], cur[U];
@@ -558,7 +590,11 @@ __global__ void __launch_bounds__(kThreads, kBinBPS) k_bin_ins(TableView tv, Bin
             unsigned long long s[U][B];
             unsigned long long* bp[U];
 _Pragma("unroll")
-            for (int u = 0; u < U; u++) has[u] = load_probe<B, U, false>(in, bs, sv, c0, u, r[u], cur[u], bp[u], s[u]);
+            for (int u = 0; u < U; u++) {
+                r[u] = pr[u];
+                has[u] = ph[u];
+                probe_rec<B, false>(bs, sv, r[u], has[u], pb[u], cur[u], bp[u], s[u]);
+            }
             unsigned long long kv[U];
             uint32_t fm[U];
             bool want[U], placed[U];
@@ -639,14 +675,18 @@ __global__ void __launch_bounds__(kThreads, kBinBPS) k_bin_cleanup(TableView tv,
     load_bins(tv, bc, bs);
     load_view(tv, sv);
     const Walker<U> wk = make_walker<U>(in, tiles);
-    DYC_BIN_TILE_LOOP(wk, bs, {
+    DYC_BIN_TILE_LOOP(U, in, wk, bs, {
         unsigned long long s[U][B];
         unsigned long long* bp[U];
         uint4 r[U];
         bool has[U];
         uint32_t cur[U];
 _Pragma("unroll")
-        for (int u = 0; u < U; u++) has[u] = load_probe<B, U, false>(in, bs, sv, c0, u, r[u], cur[u], bp[u], s[u]);
+        for (int u = 0; u < U; u++) {
+            r[u] = pr[u];
+            has[u] = ph[u];
+            probe_rec<B, false>(bs, sv, r[u], has[u], pb[u], cur[u], bp[u], s[u]);
+        }
 _Pragma("unroll")
         for (int u = 0; u < U; u++) {
             const int j = has[u] ? lane_match<B>(s[u], r[u].x) : -1;

@@ -192,6 +192,17 @@ __device__ __forceinline__ unsigned long long cas_slot(unsigned long long* p, un
     asm volatile("atom.global.cas.b64 %0, [%1], %2, %3;" : "=l"(old) : "l"(p), "l"(cmp), "l"(v) : "memory");
     return old;
 }
+// Predicated CAS (no branch around it, so several can be in flight at once);
+// returns `dflt` when pred is false.
+__device__ __forceinline__ unsigned long long cas_slot_pred(unsigned long long* p, unsigned long long cmp,
+                                                            unsigned long long v, bool pred,
+                                                            unsigned long long dflt) {
+    unsigned long long old = dflt;
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %4, 0;\n\t"
+                 "@q atom.global.cas.b64 %0, [%1], %2, %3;\n\t}"
+                 : "+l"(old) : "l"(p), "l"(cmp), "l"(v), "r"((unsigned)pred) : "memory");
+    return old;
+}
 __device__ __forceinline__ unsigned long long exch_slot(unsigned long long* p, unsigned long long v) {
     unsigned long long old;
     asm volatile("atom.global.exch.b64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
