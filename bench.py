@@ -196,12 +196,17 @@ def reference_arm(args, rank, world):
     emit(line)
 
 
-def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi_del, cap, stream):
+def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi_del, cap, stream, probes=None):
     """Roofline of the dominant kernel.  Algorithmic bytes: every
     probe reads one whole bucket (8*B bytes, the unit the method compares), every
     slot write costs one 32-byte sector, plus the streamed keys/values/status.
     achieved = algorithmic bytes per launch / mean launch time (CUDA events
-    recorded by libdyc.so on the launching stream over the timed region)."""
+    recorded by libdyc.so on the launching stream over the timed region).
+    `probes` = the kernels' own probe counts from the calibration pass
+    (dyc_probe_count_*): {kind: (ops, second probes)}.  With the first-choice-
+    full invariant a find miss or a new key in a non-full
+    first-choice bucket reads one bucket, not two, so the bytes a launch really
+    needs come from these counts, not from a phi model."""
     import torch
     from paper_conf_icde_lizlhs21_b200 import _lib as L
     peak, peak_src = measured_peaks()
@@ -211,17 +216,23 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
     bkt = 8 * args.bucket_slots
     sec = 32
     probes_find = hit_rate * (1 + phi) + (1 - hit_rate) * 2
+    reads_upsert, reads_delete = 2.0, 1.0 + phi_del
+    if probes:
+        probes_find = 1.0 + probes["find"][1] / max(1, probes["find"][0])
+        reads_upsert = 1.0 + probes["upsert"][1] / max(1, probes["upsert"][0])
+        reads_delete = 1.0 + probes["delete"][1] / max(1, probes["delete"][0])
     slots_sub = (cap // 4 // args.bucket_slots + 1) * args.bucket_slots     # slots of one subtable
     bytes_alg = {
         # find: first-choice bucket, then the second one unless hit; + key, value, flag
         "k_find": n_find * (probes_find * bkt + 9),
-        # upsert of new keys: both candidate buckets read (existence check), one
-        # sector written for each key placed here; + key, value, status
-        "k_upsert": n_ins * (2 * bkt + 9) + (n_ins - pend) * sec,
+        # upsert of new keys: the first-choice bucket, and the second one unless
+        # the invariant rules it out (existence check); one sector written for
+        # each key placed here; + key, value, status
+        "k_upsert": n_ins * (reads_upsert * bkt + 9) + (n_ins - pend) * sec,
         # eviction kernel: per pending key one write; per hop one bucket read + one exchange
         "k_place": pend * sec + ev * (bkt + sec),
         # delete (all hits): 1+φ bucket reads, one sector written; + key, old value, status
-        "k_delete": n_del * ((1 + phi_del) * bkt + sec + 9),
+        "k_delete": n_del * (reads_delete * bkt + sec + 9),
         # upsize: stream the subtable in (8 B/slot) and twice its size out (16 B/slot)
         "k_upsize": slots_sub * 24,
         # downsize: stream twice the new size in, the new size out
@@ -267,8 +278,8 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
     M = nreads / (rw_ms * 1e-3)
     cw = max(0.0, 1.0 / M - 1.0 / R)
     placed = (n_ins - pend) / max(1, n_ins)
-    acc_model = {"k_find": (probes_find, 0.0, n_find), "k_upsert": (2.0, placed, n_ins),
-                 "k_delete": (1.0 + phi_del, 1.0, n_del)}
+    acc_model = {"k_find": (probes_find, 0.0, n_find), "k_upsert": (reads_upsert, placed, n_ins),
+                 "k_delete": (reads_delete, 1.0, n_del)}
     acc_frac = {}
     for k, (r_, w_, units) in acc_model.items():
         if k in kern and kern[k] > 0:
@@ -302,6 +313,9 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
         "kernel_ms_per_step": {k: round(v, 4) for k, v in kern.items()},
         "other_kernels_ms_per_step": round(prof["other"][0] / args.steps, 4),
         "model": {"phi": phi, "hit_rate": hit_rate, "evictions_per_insert": E, "probes_per_find": probes_find,
+                  "reads_per_upsert": reads_upsert, "reads_per_delete": reads_delete,
+                  "probe_counts": probes, "probe_source": "measured (dyc_probe_count_read, calibration pass)"
+                  if probes else "model (phi, hit rate)",
                   "pending_keys": pend, "bucket_bytes": bkt, "sector_bytes": sec},
     }
 
@@ -397,14 +411,19 @@ def main():
 
     # calibration pass (untimed): correctness spot checks + per-phase statistics
     g.clear()
+    g.probe_count(True)
     g.insert(k_ins, v_ins, st_ins)
+    probes = {"upsert": g.probe_count_read()["upsert"]}
     s_ins = g.stats()
     assert s_ins["m"] == n and s_ins["n_upsize"] == 0, s_ins
     g.find(k_find, v_out, f_out)
+    probes["find"] = g.probe_count_read()["find"]
     hit_rate = float(f_out.float().mean().item())
     phi = s_ins["n_second_table"] / max(1, s_ins["m"])
     g.resize(+1)
     g.delete(k_del, dv_out, ds_out)
+    probes["delete"] = g.probe_count_read()["delete"]
+    g.probe_count(False)
     assert int(ds_out.sum().item()) == n // 2
     s_del_before = g.stats()
     phi_after_up = s_del_before["n_second_table"] / max(1, s_del_before["m"])
@@ -439,7 +458,7 @@ def main():
 
     # --------------------------------------------------------- roofline
     roofline = compute_roofline(args, prof, n_ins=n, n_find=n, n_del=n // 2, s_ins=s_ins, hit_rate=hit_rate,
-                                phi=phi, phi_del=phi_after_up, cap=cap, stream=stream)
+                                phi=phi, phi_del=phi_after_up, cap=cap, stream=stream, probes=probes)
     pend = s_ins["last_insert_pending"]
 
     # --------------------------------------------------------- resize baselines

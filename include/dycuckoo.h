@@ -305,6 +305,30 @@ enum {
 dyc_status dyc_profile_enable(dyc_table* t, int enable);
 dyc_status dyc_profile_read(dyc_table* t, double* ms, uint64_t* calls);
 
+/* Probe accounting (measurement only; off by default, costs one extra atomic
+ * per block).  While enabled, k_find, k_upsert and k_delete count the ops they
+ * process and the second-bucket probes they issue.  dyc_probe_count_read
+ * synchronizes the device, writes out6[6] = {find ops, find second probes,
+ * upsert ops, upsert second probes, delete ops, delete second probes} (host
+ * memory) and resets the counts.  The bench derives its algorithmic bytes per
+ * op from these instead of from a model. */
+dyc_status dyc_probe_count_enable(dyc_table* t, int enable);
+dyc_status dyc_probe_count_read(dyc_table* t, uint64_t* out6);
+
+/* The first-choice-full invariant (FFI; not in the paper): bit t
+ * of *mask is set while every stored key whose first-choice subtable is t but
+ * which lives in its second choice has a FULL bucket in t.  While it holds, a
+ * key absent from a non-full first-choice bucket in t is absent from the
+ * table, so find and the existence check of insert skip the second probe
+ * (still <= 2 probes).  Set for every t by dyc_create / dyc_clear;
+ * cleared for t by an upsize or a live resize of t, and for all t by a batch
+ * that removed keys, a binned insert or a reinsert baseline (dyc_resize_ex
+ * methods 1, 2).  Downsizes and placements preserve it.  Results never depend
+ * on it, only the probe count does.  Batches on one table must not overlap in
+ * time (one stream, or ordered by events): a delete running concurrently with
+ * a find could make a bucket non-full under it. */
+dyc_status dyc_clean_mask(const dyc_table* t, uint32_t* mask);
+
 /* ---------------------------------------------------------------------------
  * Hash-partitioned sharding across G GPUs (build component C1).
  * shard(k) = x_{d+1}(k) mod G, independent of the pair and bucket hashes.

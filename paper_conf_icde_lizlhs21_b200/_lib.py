@@ -119,6 +119,9 @@ SIGNATURES = {
     "dyc_get_binning": (_I, [_TP, C.POINTER(_U64), C.POINTER(_U32)]),
     "dyc_profile_enable": (_I, [_TP, _I]),
     "dyc_profile_read": (_I, [_TP, _P, _P]),
+    "dyc_probe_count_enable": (_I, [_TP, _I]),
+    "dyc_probe_count_read": (_I, [_TP, _P]),
+    "dyc_clean_mask": (_I, [_TP, C.POINTER(_U32)]),
     "dyc_route_count": (_I, [_TP, _P, _U64, _U32, _P, _P]),
     "dyc_route_scatter": (_I, [_TP, _P, _P, _P, _U64, _U32, _P, _P, _P, _P, _P, _P, _P]),
     "dyc_route_unpermute": (_I, [_P, _U64, _P, _P, _P, _P, _P]),

@@ -81,6 +81,15 @@ struct dyc_table {
     uint64_t nb[DYC_MAX_D] = {};
     uint32_t a[DYC_MAX_D + 2] = {}, b[DYC_MAX_D + 2] = {};
     uint64_t m = 0;
+    // first-choice-full invariant per subtable (TableView::clean):
+    // set for all on create / clear; an upsize of t (split buckets are no longer
+    // full) or a live resize of t clears bit t; a batch that removed keys, a
+    // binned insert (its cleanup pass removes tentative copies) or a reinsert
+    // baseline clears all.  Downsizes and placements (first-fit, evictions)
+    // preserve it.
+    uint32_t clean = 0;
+    bool count_probes = false;             // dyc_probe_count_enable (measurement)
+    unsigned long long* d_probe = nullptr; // {ops, second probes} x {find, upsert, delete}
     unsigned long long* list[2] = {nullptr, nullptr};
     uint64_t list_cap = 0;
     unsigned long long* d_ctr = nullptr;   // C_N device counters
@@ -171,6 +180,8 @@ struct dyc_table {
         v.dm1 = cfg.d - 1;
         v.recip_dm1 = (65536u + v.dm1 - 1) / v.dm1;
         v.max_hops = cfg.max_hops;
+        v.clean = rz.active ? (clean & ~(1u << rz.ti)) : clean;
+        v.probe = count_probes ? d_probe : nullptr;
         return v;
     }
 };
@@ -312,7 +323,7 @@ dyc_status upsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
     const uint64_t slots = n_old * B;
     {
         ProfScope ps(t, DYC_PROF_UPSIZE, st);
-        k_upsize<B><<<grid_for(slots, kThreads), kThreads, 0, st>>>(
+        k_upsize<B><<<grid_for(slots, kThreads * kResU), kThreads, 0, st>>>(
             t->sub[ti], (unsigned long long*)p, (uint32_t)n_old, t->a[ti + 1], t->b[ti + 1], fastmod_magic(n_new),
             (uint32_t)n_new);
     }
@@ -320,6 +331,7 @@ dyc_status upsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
     dev_free(t, t->sub[ti], st);
     t->sub[ti] = (unsigned long long*)p;
     t->nb[ti] = n_new;
+    t->clean &= ~(1u << ti);        // split buckets are no longer full
     return DYC_OK;
 }
 
@@ -391,7 +403,7 @@ dyc_status downsize_launch(dyc_table* t, uint32_t ti, cudaStream_t st) {
     TRY(zero_one(t, C_RESIDUAL, st));
     {
         ProfScope ps(t, DYC_PROF_DOWNSIZE, st);
-        k_downsize<B><<<grid_for(h * B, kThreads), kThreads, 0, st>>>(t->sub[ti], (unsigned long long*)p,
+        k_downsize<B><<<grid_for(h * B, kThreads * kResU), kThreads, 0, st>>>(t->sub[ti], (unsigned long long*)p,
                                                                        (uint32_t)h, t->list[0], t->d_ctr);
     }
     CU(cudaGetLastError());
@@ -534,7 +546,7 @@ dyc_status live_begin(dyc_table* t, int direction, int subtable, cudaStream_t st
     TRY(dev_alloc(t, &p, nn * B * 8, rs));
     if (direction > 0) {
         ProfScope ps(t, DYC_PROF_UPSIZE, rs);
-        k_upsize<B><<<grid_for(n_old * B, kThreads), kThreads, 0, rs>>>(t->sub[ti], (unsigned long long*)p,
+        k_upsize<B><<<grid_for(n_old * B, kThreads * kResU), kThreads, 0, rs>>>(t->sub[ti], (unsigned long long*)p,
                                                                         (uint32_t)n_old, t->a[ti + 1], t->b[ti + 1],
                                                                         fastmod_magic(nn), (uint32_t)nn);
     } else {
@@ -551,11 +563,12 @@ dyc_status live_begin(dyc_table* t, int direction, int subtable, cudaStream_t st
         r.res[1] = (unsigned long long*)r1;
         CU(cudaMemsetAsync(r.ctr, 0, C_N * 8, rs));
         ProfScope ps(t, DYC_PROF_DOWNSIZE, rs);
-        k_downsize<B><<<grid_for(nn * B, kThreads), kThreads, 0, rs>>>(t->sub[ti], (unsigned long long*)p,
+        k_downsize<B><<<grid_for(nn * B, kThreads * kResU), kThreads, 0, rs>>>(t->sub[ti], (unsigned long long*)p,
                                                                        (uint32_t)nn, r.res[0], r.ctr);
     }
     CU(cudaGetLastError());
     CU(cudaEventRecord(r.done, rs));
+    t->clean &= ~(1u << ti);        // LK batches may bypass ti's (old) buckets
     r.active = true;
     r.dir = direction;
     r.ti = (uint32_t)ti;
@@ -877,7 +890,10 @@ dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals,
     bool fuse = false;
     TRY(insert_begin<B>(t, n, st, fuse));
     BinCtx bc;
-    if (fuse && bin_plan(t, n, bc)) TRY(binned_ins<B>(t, bc, keys, vals, status, n, st));
+    if (fuse && bin_plan(t, n, bc)) {
+        t->clean = 0;               // its cleanup pass removes tentative t1 copies
+        TRY(binned_ins<B>(t, bc, keys, vals, status, n, st));
+    }
     else TRY(insert_chunk<B>(t, keys, vals, status, n, fuse, st));
     return insert_end<B>(t, fuse, st);
 }
@@ -930,6 +946,7 @@ template <int B>
 dyc_status delete_end(dyc_table* t, cudaStream_t st) {
     TRY(read_ctr(t, st));
     t->m -= t->h_ctr[C_REMOVED];
+    if (t->h_ctr[C_REMOVED]) t->clean = 0;   // emptied slots break the invariant
     if (t->rz.active && t->h_ctr[C_DEFER]) {
         const uint64_t dfr = t->h_ctr[C_DEFER];
         t->n_deferred += dfr;
@@ -1117,6 +1134,7 @@ dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaSt
     for (uint32_t i = 0; i < d; i++)
         if (touched[i]) dev_free(t, old[i], st);
     if (nfail) TRY(place_and_settle<B>(t, 1, nullptr, nfail, true, st));
+    t->clean = 0;
     return DYC_OK;
 }
 
@@ -1320,6 +1338,9 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
         }
     }
     if (s == DYC_OK && cudaMalloc(&t->d_ctr, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMalloc");
+    if (s == DYC_OK && cudaMalloc(&t->d_probe, 6 * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMalloc");
+    if (s == DYC_OK && cudaMemset(t->d_probe, 0, 6 * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMemset");
+    t->clean = (1u << d) - 1u;      // an empty table satisfies the invariant
     if (s == DYC_OK && cudaMallocHost(&t->h_ctr, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMallocHost");
     if (s == DYC_OK && cudaDeviceSynchronize() != cudaSuccess) s = cuda_err(cudaGetLastError(), "create");
     if (s != DYC_OK) {
@@ -1348,6 +1369,7 @@ dyc_status dyc_destroy(dyc_table* t) {
     t->live.clear();
     trim_cache(t);
     if (t->d_ctr) cudaFree(t->d_ctr);
+    if (t->d_probe) cudaFree(t->d_probe);
     if (t->rz.ctr) cudaFree(t->rz.ctr);
     if (t->rz.start) cudaEventDestroy(t->rz.start);
     if (t->rz.done) cudaEventDestroy(t->rz.done);
@@ -1540,6 +1562,7 @@ dyc_status dyc_clear(dyc_table* t, dyc_stream_t stream) {
     for (uint32_t i = 0; i < t->cfg.d; i++)
         CU(cudaMemsetAsync(t->sub[i], 0xFF, t->nb[i] * t->cfg.bucket_slots * 8, S(stream)));
     t->m = 0;
+    t->clean = (1u << t->cfg.d) - 1u;
     return DYC_OK;
 }
 
@@ -1637,6 +1660,31 @@ dyc_status dyc_profile_enable(dyc_table* t, int enable) {
     t->recs.clear();
     for (int k = 0; k < DYC_PROF_KINDS; k++) { t->prof_ms[k] = 0; t->prof_calls[k] = 0; }
     t->prof = enable != 0;
+    return DYC_OK;
+}
+
+dyc_status dyc_probe_count_enable(dyc_table* t, int enable) {
+    TRY(check_table(t));
+    CU(cudaSetDevice(t->device));
+    CU(cudaMemset(t->d_probe, 0, 6 * 8));
+    t->count_probes = enable != 0;
+    return DYC_OK;
+}
+
+dyc_status dyc_probe_count_read(dyc_table* t, uint64_t* out6) {
+    TRY(check_table(t));
+    if (!out6) return set_err(DYC_ERR_INVALID_ARG, "null out");
+    CU(cudaSetDevice(t->device));
+    CU(cudaDeviceSynchronize());
+    CU(cudaMemcpy(out6, t->d_probe, 6 * 8, cudaMemcpyDeviceToHost));
+    CU(cudaMemset(t->d_probe, 0, 6 * 8));
+    return DYC_OK;
+}
+
+dyc_status dyc_clean_mask(const dyc_table* t, uint32_t* mask) {
+    TRY(check_table(t));
+    if (!mask) return set_err(DYC_ERR_INVALID_ARG, "null out");
+    *mask = t->rz.active ? (t->clean & ~(1u << t->rz.ti)) : t->clean;
     return DYC_OK;
 }
 

@@ -44,7 +44,15 @@ struct TableView {
     uint32_t dm1;                // d-1
     uint32_t recip_dm1;          // ceil(2^16/(d-1)): q div (d-1) = (q*recip)>>16 for q < 2^8
     uint32_t max_hops;
-    uint32_t pad;
+    // bit t set <=> subtable t satisfies the first-choice-full invariant (FFI,
+    // DESIGN.md §5): every stored key whose FIRST choice is t but which lives in
+    // its second-choice subtable has a FULL bucket h_t(k).  Then a key absent
+    // from a non-full first-choice bucket of such a t is absent from the table,
+    // and the second probe can be skipped.  Maintained by the host (dyc_api.cu).
+    uint32_t clean;
+    // measurement only (dyc_probe_count_enable): {ops, second probes} per kernel
+    // kind (find, upsert, delete); nullptr in normal operation
+    unsigned long long* probe;
 };
 
 // Shared-memory copy of the per-subtable fields, indexed by a lane-varying t.

@@ -21,7 +21,7 @@ namespace dyc {
 constexpr int kThreads = 256;
 // minimum resident blocks per SM requested from ptxas (register budget) per kernel family
 #ifndef DYC_FIND_MINB
-#define DYC_FIND_MINB 1
+#define DYC_FIND_MINB 3
 #endif
 #ifndef DYC_UPSERT_MINB
 #define DYC_UPSERT_MINB 1
@@ -125,9 +125,19 @@ __device__ __forceinline__ bool coop_cas_empty(const Grp<G>& g, unsigned long lo
     return placed;
 }
 
+__device__ __forceinline__ unsigned empty_mask(const unsigned long long (&s)[4]) {
+    unsigned m = 0;
+#pragma unroll
+    for (int j = 0; j < 4; j++)
+        if (s[j] == kEmptySlot) m |= 1u << j;
+    return m;
+}
+
 // ----------------------------------------------------------------- find (S3)
 // ILP queries per group; all first probes are issued back to back, then the
 // second probes (predicated, only after a first-probe miss: <= 2 lookups).
+// A miss in a non-full first-choice bucket of a subtable that holds the
+// first-choice-full invariant (TableView::clean) is final: no second probe.
 template <int B, int ILP>
 __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, const uint32_t* __restrict__ keys,
                                                    uint32_t* __restrict__ vals, uint8_t* __restrict__ found,
@@ -140,9 +150,10 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
     const uint64_t wtile = (uint64_t)QPW * ILP;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
+    unsigned long long n_ops = 0, n_p2 = 0;
     for (uint64_t base = w * wtile; base < n; base += nwarps * wtile) {
         uint32_t k[ILP], v[ILP];
-        bool f[ILP];
+        bool f[ILP], c1[ILP];
         const unsigned long long* p2[ILP];
         unsigned long long s[ILP][4];
 #pragma unroll
@@ -153,23 +164,29 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
             const Pair p = pair_of(tv, k[j]);
+            c1[j] = (tv.clean >> p.t1) & 1u;
             p2[j] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[j]), B) + 4 * g.sub;
             probe_nc<B>(bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[j]), B) + 4 * g.sub, s[j]);
         }
+        bool need2[ILP];
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
             uint32_t lv = 0;
             const bool lh = lookup_slot<4>(s[j], k[j], lv) && k[j] != kEmptyKey;
             const unsigned hb = g.ballot(lh);
+            const unsigned eb = g.ballot(empty_mask(s[j]) != 0);
             f[j] = hb != 0;
             v[j] = g.bcast32(lv, first_lane(hb));
+            need2[j] = !f[j] && k[j] != kEmptyKey && !(c1[j] && eb != 0);
+            n_ops += g.sub == 0 && k[j] != kEmptyKey;
+            n_p2 += g.sub == 0 && need2[j];
         }
 #pragma unroll
-        for (int j = 0; j < ILP; j++) probe_nc_pred<B>(p2[j], s[j], !f[j] && k[j] != kEmptyKey);
+        for (int j = 0; j < ILP; j++) probe_nc_pred<B>(p2[j], s[j], need2[j]);
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
             uint32_t lv = 0;
-            const bool lh = !f[j] && k[j] != kEmptyKey && lookup_slot<4>(s[j], k[j], lv);
+            const bool lh = need2[j] && lookup_slot<4>(s[j], k[j], lv);
             const unsigned hb = g.ballot(lh);
             const uint32_t v2 = g.bcast32(lv, first_lane(hb));
             if (hb) { f[j] = true; v[j] = v2; }
@@ -179,6 +196,10 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
                 if (found) found[i] = f[j] ? 1 : 0;
             }
         }
+    }
+    if (tv.probe) {
+        block_add<kThreads>(tv.probe + 0, n_ops);
+        block_add<kThreads>(tv.probe + 1, n_p2);
     }
 }
 
@@ -266,14 +287,6 @@ __device__ __forceinline__ void coop_cas_multi(const Grp<G>& g, unsigned long lo
     }
 }
 
-__device__ __forceinline__ unsigned empty_mask(const unsigned long long (&s)[4]) {
-    unsigned m = 0;
-#pragma unroll
-    for (int j = 0; j < 4; j++)
-        if (s[j] == kEmptySlot) m |= 1u << j;
-    return m;
-}
-
 // ------------------------------------------------------ insert phase 1 (S5)
 // Upsert: probe t1's bucket, then t2's; an existing key gets its value replaced
 // (Alg. 1, status UPDATED).  A new key (status INSERTED) is, with FUSE,
@@ -305,7 +318,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
     const unsigned grp = g.lane / G;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
-    unsigned long long n_ins = 0, n_upd = 0;
+    unsigned long long n_ins = 0, n_upd = 0, n_ops = 0, n_p2 = 0;
     for (uint64_t base = w * (QPW * U); base < n; base += nwarps * (QPW * U)) {
         // per op only the match position and the free-slot mask of each bucket
         // are kept, not the 4-slot snapshots (register budget -> more ops in flight)
@@ -353,6 +366,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
 #else
         {
             unsigned long long s1[U][4];
+            bool c1[U];
 #pragma unroll
             for (int u = 0; u < U; u++) {
                 i[u] = base + (uint64_t)u * QPW + grp;
@@ -362,23 +376,31 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                 const Pair p = pair_of(tv, k[u]);
                 lk1[u] = LK && p.t1 == locked;
                 lk2[u] = LK && p.t2 == locked;
+                c1[u] = ((tv.clean >> p.t1) & 1u) && !lk1[u];
                 b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
                 b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
                 probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
             }
 #pragma unroll
             for (int u = 0; u < U; u++) {
+                const bool active = k[u] != kEmptyKey;
                 j1[u] = match_slot<4>(s1[u], k[u]);
-                em1[u] = lk1[u] ? 0u : empty_mask(s1[u]);
+                const unsigned e = empty_mask(s1[u]);
+                em1[u] = lk1[u] ? 0u : e;
+                h1[u] = g.ballot(active && j1[u] >= 0);
+                // first-choice-full invariant: absent from a non-full first-choice
+                // bucket of a clean subtable => absent from the table (no t2 probe)
+                const unsigned eb = g.ballot(e != 0);   // every lane votes (no short circuit)
+                const bool skip = c1[u] && eb != 0;
+                need2[u] = active && h1[u] == 0 && !skip;
+                n_ops += g.sub == 0 && active;
+                n_p2 += g.sub == 0 && need2[u];
             }
         }
         {
             unsigned long long s2[U][4];
 #pragma unroll
             for (int u = 0; u < U; u++) {
-                const bool active = k[u] != kEmptyKey;
-                h1[u] = g.ballot(active && j1[u] >= 0);
-                need2[u] = active && h1[u] == 0;
 #pragma unroll
                 for (int q = 0; q < 4; q++) s2[u][q] = kEmptySlot;
                 probe_cg_pred<B>(b2[u] + 4 * g.sub, s2[u], need2[u]);
@@ -386,7 +408,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
 #pragma unroll
             for (int u = 0; u < U; u++) {
                 j2[u] = match_slot<4>(s2[u], k[u]);
-                em2[u] = lk2[u] ? 0u : empty_mask(s2[u]);
+                em2[u] = (lk2[u] || !need2[u]) ? 0u : empty_mask(s2[u]);
             }
         }
 #endif
@@ -396,7 +418,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
             if (h1[u] && !lk1[u] && g.sub == first_lane(h1[u])) st_u64_cg(b1[u] + 4 * g.sub + j1[u], kv[u]);
             if (h2[u] && !lk2[u] && g.sub == first_lane(h2[u])) st_u64_cg(b2[u] + 4 * g.sub + j2[u], kv[u]);
             if (LK) warp_append(g.sub == 0 && ((h1[u] && lk1[u]) || (h2[u] && lk2[u])), kv[u], defer, ctr + C_DEFER);
-            isnew[u] = need2[u] && h2[u] == 0;
+            isnew[u] = k[u] != kEmptyKey && h1[u] == 0 && h2[u] == 0;
             placed[u] = false;
         }
         if (FUSE) {
@@ -415,6 +437,10 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
     }
     block_add<kThreads>(ctr + C_INSERTED, n_ins);
     block_add<kThreads>(ctr + C_UPDATED, n_upd);
+    if (tv.probe) {
+        block_add<kThreads>(tv.probe + 2, n_ops);
+        block_add<kThreads>(tv.probe + 3, n_p2);
+    }
 }
 
 // ------------------------------------------------------ insert phase 2 (S7)
@@ -424,7 +450,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
 // range as soon as their current chain ends, so a long eviction chain does not
 // hold the other groups of the warp idle.  Per group a small state machine:
 //   phase 0/1 : first-fit probe of t1 / t2 (reading Q3; skipped when
-//               first_fit = false, i.e. the upsert already found both full),
+//               first_fit = false, i.e. the upsert already found t1 full),
 //   phase 2   : eviction hops: probe for a free slot (after the first hop), else
 //               exchange a pseudo-random victim (Q5) and carry it to the other
 //               table of ITS pair; after max_hops (Q6) the
@@ -458,7 +484,11 @@ __global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv
             k = key_of(kv);
             const Pair p = pair_of(tv, k);
             phase = first_fit ? 0 : 2;
-            t = first_fit ? p.t1 : ((mix32(k) & 1u) ? p.t2 : p.t1);
+            // without first-fit, hop 0 evicts from t1 without a probe: k_upsert
+            // saw that bucket full; its t2 bucket may be unread (first-choice-full
+            // shortcut) and evicting from a non-full bucket would break the
+            // invariant for the victim
+            t = p.t1;
             hop = 0;
         }
         if (!__any_sync(kFull, phase >= 0)) break;
@@ -547,7 +577,7 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
     const unsigned grp = g.lane / G;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
-    unsigned long long removed = 0;
+    unsigned long long removed = 0, n_ops = 0, n_p2 = 0;
     for (uint64_t base = w * (QPW * U); base < n; base += nwarps * (QPW * U)) {
         uint64_t i[U];
         uint32_t k[U];
@@ -573,7 +603,11 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
             const bool active = k[u] != kEmptyKey;
             j1[u] = active ? match_slot<4>(s1[u], k[u]) : -1;
             h1[u] = g.ballot(j1[u] >= 0);
+            // no first-choice-full shortcut here (unlike k_find / k_upsert): the
+            // deletes of this same batch make buckets non-full while it runs
             need2[u] = active && h1[u] == 0;
+            n_ops += g.sub == 0 && active;
+            n_p2 += g.sub == 0 && need2[u];
 #pragma unroll
             for (int q = 0; q < 4; q++) s2[u][q] = kEmptySlot;
             probe_cg_pred<B>(b2[u] + 4 * g.sub, s2[u], need2[u]);
@@ -599,6 +633,10 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
         }
     }
     block_add<kThreads>(ctr + C_REMOVED, removed);
+    if (tv.probe) {
+        block_add<kThreads>(tv.probe + 4, n_ops);
+        block_add<kThreads>(tv.probe + 5, n_p2);
+    }
 }
 
 // Applies the deferred ops of a batch that ran while a subtable was locked by a
@@ -639,32 +677,52 @@ __global__ void __launch_bounds__(kThreads) k_apply(TableView tv, const unsigned
 // ballot (the warp-cooperative bucket pass of P:L379-380).  New bucket b gets the
 // entries that stay, b+n_old the ones that move; unused slots are written EMPTY,
 // so the new buffer needs no memset.  Streams: read 8 B, write 16 B per old slot.
+// Streaming layout: each thread loads kResU slots up front (bytes in flight for
+// HBM), the two new buckets are assembled in a per-warp shared-memory tile, and
+// lane s then writes slot s of both, so every store instruction of a warp covers
+// 256 contiguous bytes.
+constexpr int kResU = 4;
+
 template <int B>
 __global__ void __launch_bounds__(kThreads) k_upsize(const unsigned long long* __restrict__ old_s,
                                                      unsigned long long* __restrict__ new_s, uint32_t n_old,
                                                      uint32_t a, uint32_t b, uint64_t magic2, uint32_t n2) {
     static_assert(B <= 32 && (32 % B) == 0, "bucket must divide a warp");
+    __shared__ unsigned long long tile[kThreads / 32][2][32];
     const uint64_t total = (uint64_t)n_old * B;
-    const unsigned lane = threadIdx.x & 31;
-    const unsigned gmask = (B == 32) ? kFull : (((1u << B) - 1u) << (lane & ~(unsigned)(B - 1)));
+    const unsigned lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const unsigned gbase = lane & ~(unsigned)(B - 1);
+    const unsigned gmask = (B == 32) ? kFull : (((1u << B) - 1u) << gbase);
     const unsigned lt = lanemask_lt() & gmask;
-    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < total; base += (uint64_t)gridDim.x * kThreads) {
-        const uint64_t g = base + threadIdx.x;
-        const bool valid = g < total;
-        const unsigned long long e = valid ? __ldcs(old_s + g) : kEmptySlot;
-        const uint32_t bucket = (uint32_t)(g / B);
-        const uint32_t s = (uint32_t)(g % B);
-        const bool occ = key_of(e) != kEmptyKey;
-        bool hi = false;
-        if (occ) hi = fastmod(hx(a, b, key_of(e)), magic2, n2) != bucket;
-        const unsigned hb = __ballot_sync(kFull, occ && hi) & gmask;
-        const unsigned lb = __ballot_sync(kFull, occ && !hi) & gmask;
-        if (valid) {
-            const uint64_t lo_base = (uint64_t)bucket * B;
-            const uint64_t hi_base = ((uint64_t)bucket + n_old) * B;
-            if (occ) new_s[(hi ? hi_base : lo_base) + __popc((hi ? hb : lb) & lt)] = e;
-            if (s >= (uint32_t)__popc(lb)) new_s[lo_base + s] = kEmptySlot;
-            if (s >= (uint32_t)__popc(hb)) new_s[hi_base + s] = kEmptySlot;
+    const unsigned s = lane & (B - 1);
+    for (uint64_t base = (uint64_t)blockIdx.x * kThreads * kResU; base < total;
+         base += (uint64_t)gridDim.x * kThreads * kResU) {
+        unsigned long long e[kResU];
+#pragma unroll
+        for (int u = 0; u < kResU; u++) {
+            const uint64_t g = base + (uint64_t)u * kThreads + threadIdx.x;
+            e[u] = g < total ? __ldcs(old_s + g) : kEmptySlot;
+        }
+#pragma unroll
+        for (int u = 0; u < kResU; u++) {
+            const uint64_t g = base + (uint64_t)u * kThreads + threadIdx.x;
+            const uint32_t bucket = (uint32_t)(g / B);
+            const bool occ = key_of(e[u]) != kEmptyKey;
+            bool hi = false;
+            if (occ) hi = fastmod(hx(a, b, key_of(e[u])), magic2, n2) != bucket;
+            const unsigned hb = __ballot_sync(kFull, occ && hi) & gmask;
+            const unsigned lb = __ballot_sync(kFull, occ && !hi) & gmask;
+            tile[w][0][lane] = kEmptySlot;
+            tile[w][1][lane] = kEmptySlot;
+            __syncwarp();
+            if (occ) tile[w][hi ? 1 : 0][gbase + __popc((hi ? hb : lb) & lt)] = e[u];
+            __syncwarp();
+            const unsigned long long lo_v = tile[w][0][lane], hi_v = tile[w][1][lane];
+            __syncwarp();
+            if (g < total) {
+                __stcs(new_s + (uint64_t)bucket * B + s, lo_v);
+                __stcs(new_s + ((uint64_t)bucket + n_old) * B + s, hi_v);
+            }
         }
     }
 }
@@ -673,42 +731,52 @@ __global__ void __launch_bounds__(kThreads) k_upsize(const unsigned long long* _
 // One lane per slot of the halved table: new bucket b' takes old b' then old
 // b'+h in slot order, keeps the first B (reading Q18) and appends the rest to
 // the residual list, which k_place then inserts into the pairs' other tables
-// (P:L392-393).  Streams: read 16 B, write 8 B per new slot.
+// (P:L392-393).  Streams: read 16 B, write 8 B per new slot.  Same streaming
+// layout as k_upsize (kResU slots per thread, per-warp tile, coalesced stores).
 template <int B>
 __global__ void __launch_bounds__(kThreads) k_downsize(const unsigned long long* __restrict__ old_s,
                                                        unsigned long long* __restrict__ new_s, uint32_t h,
                                                        unsigned long long* __restrict__ residual,
                                                        unsigned long long* __restrict__ ctr) {
     static_assert(B <= 32 && (32 % B) == 0, "bucket must divide a warp");
+    __shared__ unsigned long long tile[kThreads / 32][32];
     const uint64_t total = (uint64_t)h * B;
-    const unsigned lane = threadIdx.x & 31;
-    const unsigned gmask = (B == 32) ? kFull : (((1u << B) - 1u) << (lane & ~(unsigned)(B - 1)));
+    const unsigned lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const unsigned gbase = lane & ~(unsigned)(B - 1);
+    const unsigned gmask = (B == 32) ? kFull : (((1u << B) - 1u) << gbase);
     const unsigned lt = lanemask_lt() & gmask;
-    for (uint64_t base = (uint64_t)blockIdx.x * kThreads; base < total; base += (uint64_t)gridDim.x * kThreads) {
-        const uint64_t g = base + threadIdx.x;
-        const bool valid = g < total;
-        const unsigned long long e1 = valid ? __ldcs(old_s + g) : kEmptySlot;
-        const unsigned long long e2 = valid ? __ldcs(old_s + g + total) : kEmptySlot;
-        const bool o1 = key_of(e1) != kEmptyKey, o2 = key_of(e2) != kEmptyKey;
-        const unsigned m1 = __ballot_sync(kFull, o1) & gmask;
-        const unsigned m2 = __ballot_sync(kFull, o2) & gmask;
-        const uint32_t c1 = __popc(m1), ctot = c1 + __popc(m2);
-        const uint32_t r1 = __popc(m1 & lt), r2 = c1 + __popc(m2 & lt);
-        const uint64_t bb = (g / B) * B;
-        const uint32_t s = (uint32_t)(g % B);
-        bool res = false;
-        if (valid) {
-            if (o1) new_s[bb + r1] = e1;                 // r1 < c1 <= B always fits
-            if (o2) {
-                if (r2 < (uint32_t)B) new_s[bb + r2] = e2;
-                else res = true;
-            }
-            if (s >= ctot) new_s[bb + s] = kEmptySlot;
+    unsigned long long nres = 0;
+    for (uint64_t base = (uint64_t)blockIdx.x * kThreads * kResU; base < total;
+         base += (uint64_t)gridDim.x * kThreads * kResU) {
+        unsigned long long e1[kResU], e2[kResU];
+#pragma unroll
+        for (int u = 0; u < kResU; u++) {
+            const uint64_t g = base + (uint64_t)u * kThreads + threadIdx.x;
+            e1[u] = g < total ? __ldcs(old_s + g) : kEmptySlot;
+            e2[u] = g < total ? __ldcs(old_s + g + total) : kEmptySlot;
         }
-        const unsigned rm = __ballot_sync(kFull, res);
-        if (rm && (threadIdx.x & 31) == (unsigned)(__ffs(rm) - 1)) atomicAdd(ctr + C_RES_TOTAL, (unsigned long long)__popc(rm));
-        warp_append(res, e2, residual, ctr + C_RESIDUAL);
+#pragma unroll
+        for (int u = 0; u < kResU; u++) {
+            const uint64_t g = base + (uint64_t)u * kThreads + threadIdx.x;
+            const bool o1 = key_of(e1[u]) != kEmptyKey, o2 = key_of(e2[u]) != kEmptyKey;
+            const unsigned m1 = __ballot_sync(kFull, o1) & gmask;
+            const unsigned m2 = __ballot_sync(kFull, o2) & gmask;
+            const uint32_t c1 = __popc(m1);
+            const uint32_t r1 = __popc(m1 & lt), r2 = c1 + __popc(m2 & lt);
+            tile[w][lane] = kEmptySlot;
+            __syncwarp();
+            if (o1) tile[w][gbase + r1] = e1[u];                  // r1 < c1 <= B always fits
+            const bool res = o2 && r2 >= (uint32_t)B;
+            if (o2 && !res) tile[w][gbase + r2] = e2[u];
+            __syncwarp();
+            const unsigned long long v = tile[w][lane];
+            __syncwarp();
+            if (g < total) __stcs(new_s + g, v);
+            nres += res;
+            warp_append(res, e2[u], residual, ctr + C_RESIDUAL);
+        }
     }
+    block_add<kThreads>(ctr + C_RES_TOTAL, nres);
 }
 
 // ---------------------------------------------------------- stats / dump (S10)

@@ -296,6 +296,22 @@ class Table:
         L.check(self._lib.dyc_profile_read(self._h, ms.ctypes.data, calls.ctypes.data), "dyc_profile_read")
         return {name: (float(ms[i]), int(calls[i])) for i, name in enumerate(L.PROF_NAMES)}
 
+    def probe_count(self, enable: bool = True) -> None:
+        """Count ops and second-bucket probes in k_find / k_upsert / k_delete (measurement)."""
+        L.check(self._lib.dyc_probe_count_enable(self._h, 1 if enable else 0), "dyc_probe_count_enable")
+
+    def probe_count_read(self) -> Dict[str, Tuple[int, int]]:
+        """{kind: (ops, second probes)} since the last read; resets the counts."""
+        out = np.zeros(6, dtype=np.uint64)
+        L.check(self._lib.dyc_probe_count_read(self._h, out.ctypes.data), "dyc_probe_count_read")
+        return {k: (int(out[2 * i]), int(out[2 * i + 1])) for i, k in enumerate(("find", "upsert", "delete"))}
+
+    def clean_mask(self) -> int:
+        """Bit t: subtable t holds the first-choice-full invariant (dyc_clean_mask)."""
+        m = C.c_uint32()
+        L.check(self._lib.dyc_clean_mask(self._h, C.byref(m)), "dyc_clean_mask")
+        return int(m.value)
+
     # ------------------------------------------------------------ routing (S11)
     def route_count(self, keys, world: int, counts=None, stream=None):
         """Per-shard histogram (uint64 -> int64 tensor of length world)."""
