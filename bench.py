@@ -600,10 +600,41 @@ def main():
             e2e_step()
             torch.cuda.synchronize()
             ts.append(time.perf_counter() - t0)
+        # PCIe ceiling of the same transfers: pinned copies alone (H2D, D2H, both at
+        # once on two streams), then the per-phase bound max(H2D/h, D2H/d) summed over
+        # the phases (each phase's results depend on its inputs; phases are ordered)
+        pbuf = torch.empty(1 << 30, dtype=torch.uint8, pin_memory=True)
+        dbuf = torch.empty(1 << 30, dtype=torch.uint8, device="cuda")
+        dbuf2 = torch.empty(1 << 30, dtype=torch.uint8, device="cuda")
+        pbuf2 = torch.empty(1 << 30, dtype=torch.uint8, pin_memory=True)
+        s_in, s_out = torch.cuda.Stream(), torch.cuda.Stream()
+
+        def copy_rate(h2d, d2h):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            for _ in range(2):
+                if h2d:
+                    with torch.cuda.stream(s_in):
+                        dbuf.copy_(pbuf, non_blocking=True)
+                if d2h:
+                    with torch.cuda.stream(s_out):
+                        pbuf2.copy_(dbuf2, non_blocking=True)
+            torch.cuda.synchronize()
+            return 2 * (1 << 30) / (time.perf_counter() - t0) / 1e9
+        copy_rate(True, True)
+        h2d_gbs, d2h_gbs, duplex_gbs = copy_rate(True, False), copy_rate(False, True), copy_rate(True, True)
+        del pbuf, pbuf2, dbuf, dbuf2
+        phase_bytes = [(8 * n, n), (4 * n, 5 * n), (4 * (n // 2), 5 * (n // 2))]   # insert, find, delete
+        bound_s = sum(max(hb / (duplex_gbs * 1e9), db / (duplex_gbs * 1e9)) for hb, db in phase_bytes)
         e2e = {"value": n_ops / statistics.mean(ts) / 1e6, "unit": "Mops/s",
                "h2d_bytes_per_step": 4 * n + 4 * n + 4 * n + 4 * (n // 2),
                "d2h_bytes_per_step": n + 5 * n + 5 * (n // 2),
                "ms_per_step": 1e3 * statistics.mean(ts),
+               "pcie": {"h2d_gbs": h2d_gbs, "d2h_gbs": d2h_gbs, "duplex_gbs_per_direction": duplex_gbs,
+                        "bound_ms_per_step": bound_s * 1e3,
+                        "frac_of_pcie_bound": bound_s / statistics.mean(ts),
+                        "what": "pinned 1 GiB copies alone; bound = sum over phases of max(H2D, D2H) bytes at "
+                                "the duplex per-direction rate"},
                "path": "dyc_{insert,find,delete}_batch_host (pinned host buffers, copies inside)"}
 
     cpu = None
