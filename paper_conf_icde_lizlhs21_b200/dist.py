@@ -301,7 +301,9 @@ def bench_c5(args, rank, world, local, metric, ClockSampler):
     from .table import Table
 
     log2k = getattr(args, "c5_log2keys", 31)
-    batch = 1 << min(24, log2k - 3)
+    # 128 fill batches at every scale (2^31 keys: 16M per batch, the config);
+    # keeps the 32 mixed batches' deletes below the live-find range at any scale
+    batch = 1 << min(24, log2k - 7)
     shard = Table(d=4, init_capacity=1 << 20, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
     dt = DistTable(shard, force_route=getattr(args, "routed", False))
     stream = torch.cuda.current_stream()
@@ -313,6 +315,13 @@ def bench_c5(args, rank, world, local, metric, ClockSampler):
     if world > 1:
         dist.barrier()
     checks = torch.zeros(4, dtype=torch.int64, device="cuda")
+    # key(i) is a bijection of u32, so exactly one index maps to the reserved
+    # EMPTY key (reading Q25: rejected with status INVALID, never stored)
+    reserved = sum(int((k == -1).sum()) for _, k, _ in fill)
+    exp_mixed = torch.zeros(2, dtype=torch.int64, device="cuda")   # valid (non-reserved) inserts, deletes
+    for _, ops, k, _ in mixed:
+        exp_mixed[0] += ((ops == 1) & (k != -1)).sum()
+        exp_mixed[1] += ((ops == 2) & (k != -1)).sum()
     shard.profile(True)
     with ClockSampler(local) as clk:
         a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
@@ -336,6 +345,11 @@ def bench_c5(args, rank, world, local, metric, ClockSampler):
     shard.profile(False)
     st = shard.stats()
     fill_ms, mixed_ms = float(t[0]), float(t[1])
+    r_t = torch.tensor([reserved], dtype=torch.int64, device="cuda")
+    if world > 1:
+        dist.all_reduce(r_t)
+        dist.all_reduce(exp_mixed)
+    reserved_all = int(r_t.item())
     n_fill, n_mixed = len(fill) * batch, len(mixed) * batch
     if rank != 0:
         return None
@@ -349,9 +363,11 @@ def bench_c5(args, rank, world, local, metric, ClockSampler):
                    "parallelism": f"shard{world}", "init_capacity_per_shard": 1 << 20},
         "phases": {"fill_ms": fill_ms, "fill_mops": n_fill / fill_ms / 1e3,
                    "mixed_ms": mixed_ms, "mixed_mops": n_mixed / mixed_ms / 1e3},
-        "check": {"inserted_fill": int(checks[0]), "expected_fill": n_fill,
+        "check": {"inserted_fill": int(checks[0]), "expected_fill": n_fill - reserved_all,
+                  "reserved_key_in_fill": reserved_all,
                   "found_in_mixed": int(checks[1]), "expected_found": len(mixed) * (batch // 4),
-                  "inserted_in_mixed": int(checks[2]), "deleted_in_mixed": int(checks[3])},
+                  "inserted_in_mixed": int(checks[2]), "expected_inserted_in_mixed": int(exp_mixed[0]),
+                  "deleted_in_mixed": int(checks[3]), "expected_deleted_in_mixed": int(exp_mixed[1])},
         "shard0": {"fill": st["fill"], "buckets": st["buckets"], "m": st["m"], "n_upsize": st["n_upsize"],
                    "n_downsize": st["n_downsize"], "bytes": st["bytes_allocated"]},
         "kernel_ms_rank0": {k: round(v[0], 2) for k, v in prof.items() if v[1]},

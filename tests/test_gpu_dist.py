@@ -99,3 +99,42 @@ def test_dist_table_mixed_routed_world1(oracle_mod):
             np.testing.assert_array_equal(shard.sorted_kv(), o.sorted_kv())
     finally:
         dist.destroy_process_group()
+
+
+def test_bench_c5_small_checks(oracle_mod):
+    """bench_c5 (config C5) at 2^20 keys on one shard: every fill key except the
+    reserved one is INSERTED (reading Q25: key(i) is a bijection of u32, so one
+    index maps to EMPTY), every live find hits, and the mixed inserts/deletes
+    succeed exactly for the non-reserved keys."""
+    import types
+    import torch.distributed as dist
+    from paper_conf_icde_lizlhs21_b200.dist import bench_c5
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+
+    class NoClock:
+        def __init__(self, *a):
+            pass
+
+        def __enter__(self):
+            return self
+
+        def __exit__(self, *a):
+            return False
+
+        def summary(self):
+            return {}
+
+    dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1)
+    try:
+        args = types.SimpleNamespace(c5_log2keys=20, bucket_slots=8, routed=True, steps=1, warmup=0)
+        out = bench_c5(args, 0, 1, 0, "m", NoClock)
+    finally:
+        dist.destroy_process_group()
+    c = out["check"]
+    assert c["inserted_fill"] == c["expected_fill"] == (1 << 20) - c["reserved_key_in_fill"]
+    assert c["found_in_mixed"] == c["expected_found"]
+    assert c["inserted_in_mixed"] == c["expected_inserted_in_mixed"]
+    assert c["deleted_in_mixed"] == c["expected_deleted_in_mixed"]
