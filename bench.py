@@ -76,7 +76,12 @@ def parse():
     ap.add_argument("--wide-modes", default=None, help="--config wide: comma list of voter_W2,grouped_W2,...")
     ap.add_argument("--routed", action="store_true",
                     help="use the sharded router even at N=1 (exercises the N>1 code path)")
-    return ap.parse_args()
+    ap.add_argument("--p2p", action="store_true",
+                    help="route through the fused peer-memory dispatch/combine kernels (CUDA IPC) "
+                         "instead of NCCL all-to-all")
+    args = ap.parse_args()
+    args.routed = args.routed or args.p2p
+    return args
 
 
 # ---------------------------------------------------------------- clocks

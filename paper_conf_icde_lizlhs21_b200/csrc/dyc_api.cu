@@ -1761,6 +1761,108 @@ dyc_status dyc_route_unpermute(const uint32_t* d_pos, uint64_t n, const uint32_t
     return DYC_OK;
 }
 
+// ---------------------------------------------- peer-memory routing (fused)
+dyc_status dyc_ipc_alloc(uint64_t bytes, void** d_ptr) {
+    if (!d_ptr || bytes == 0) return set_err(DYC_ERR_INVALID_ARG, "dyc_ipc_alloc: null out pointer or 0 bytes");
+    *d_ptr = nullptr;
+    cudaError_t e = cudaMalloc(d_ptr, bytes);
+    if (e == cudaErrorMemoryAllocation) {
+        cudaGetLastError();
+        return set_err(DYC_ERR_OOM, "dyc_ipc_alloc: out of device memory");
+    }
+    CU(e);
+    CU(cudaMemset(*d_ptr, 0, bytes));
+    return DYC_OK;
+}
+
+dyc_status dyc_ipc_free(void* d_ptr) {
+    if (d_ptr) CU(cudaFree(d_ptr));
+    return DYC_OK;
+}
+
+dyc_status dyc_ipc_get_handle(void* d_ptr, void* handle64) {
+    if (!d_ptr || !handle64) return set_err(DYC_ERR_INVALID_ARG, "dyc_ipc_get_handle: null pointer");
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "CUDA IPC handle is 64 bytes");
+    cudaIpcMemHandle_t h;
+    CU(cudaIpcGetMemHandle(&h, d_ptr));
+    memcpy(handle64, &h, 64);
+    return DYC_OK;
+}
+
+dyc_status dyc_ipc_open(const void* handle64, void** d_ptr) {
+    if (!d_ptr || !handle64) return set_err(DYC_ERR_INVALID_ARG, "dyc_ipc_open: null pointer");
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle64, 64);
+    CU(cudaIpcOpenMemHandle(d_ptr, h, cudaIpcMemLazyEnablePeerAccess));
+    return DYC_OK;
+}
+
+dyc_status dyc_ipc_close(void* d_ptr) {
+    if (d_ptr) CU(cudaIpcCloseMemHandle(d_ptr));
+    return DYC_OK;
+}
+
+dyc_status dyc_route_push(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_vals, const uint8_t* d_tags,
+                          uint64_t n, uint32_t world, uint32_t src_rank, void* const* d_recv,
+                          uint64_t* const* d_recv_count, uint64_t recv_cap, dyc_stream_t stream) {
+    TRY(enter(t, stream));
+    if (world < 1 || world > kMaxPeers) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_push: world must be 1..64");
+    if (src_rank >= world) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_push: src_rank >= world");
+    if (!d_recv || !d_recv_count) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_push: null peer arrays");
+    if (n > 0xFFFFFFFFull) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_push: batch must be < 2^32 ops");
+    if (n == 0) return DYC_OK;
+    PeerPtrs rp{}, cp{};
+    for (uint32_t w = 0; w < world; w++) {
+        if (!d_recv[w] || !d_recv_count[w]) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_push: null peer pointer");
+        rp.p[w] = d_recv[w];
+        cp.p[w] = d_recv_count[w];
+    }
+    const uint32_t sh = t->cfg.d + 1;
+    {
+        ProfScope ps(t, DYC_PROF_OTHER, S(stream));
+        const HashDest hd{t->a[sh], t->b[sh], world, fastmod_magic(world), d_keys};
+        k_route_push<<<std::min<unsigned>(grid_for(n, (uint64_t)kThreads * kTileItems), t->num_sms * 8), kThreads,
+                       world * 12, S(stream)>>>(hd, d_vals, d_tags, n, world, src_rank, rp, cp, recv_cap);
+    }
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+dyc_status dyc_route_unpack(const void* d_recs, uint64_t n, uint32_t* d_keys, uint32_t* d_vals, uint8_t* d_tags,
+                            dyc_stream_t stream) {
+    if (n == 0) return DYC_OK;
+    if (!d_recs || !d_keys) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_unpack: null pointer");
+    k_route_unpack<<<grid_for(n, kThreads * 4), kThreads, 0, S(stream)>>>((const uint4*)d_recs, n, d_keys, d_vals,
+                                                                       d_tags);
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
+dyc_status dyc_route_reply(const void* d_recs, uint64_t n, const uint32_t* d_vals, const uint8_t* d_status,
+                           uint32_t world, uint32_t* const* d_out_vals, uint8_t* const* d_out_status,
+                           dyc_stream_t stream) {
+    if (world < 1 || world > kMaxPeers) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_reply: world must be 1..64");
+    if (n == 0) return DYC_OK;
+    if (!d_recs) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_reply: null records");
+    if ((d_vals == nullptr) != (d_out_vals == nullptr) || (d_status == nullptr) != (d_out_status == nullptr))
+        return set_err(DYC_ERR_INVALID_ARG, "dyc_route_reply: a result array and its destinations must both be given");
+    PeerPtrs vp{}, sp{};
+    for (uint32_t w = 0; w < world; w++) {
+        if (d_out_vals) {
+            if (!d_out_vals[w]) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_reply: null peer pointer");
+            vp.p[w] = d_out_vals[w];
+        }
+        if (d_out_status) {
+            if (!d_out_status[w]) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_reply: null peer pointer");
+            sp.p[w] = d_out_status[w];
+        }
+    }
+    k_route_reply<<<grid_for(n, kThreads * 4), kThreads, 0, S(stream)>>>((const uint4*)d_recs, n, d_vals, d_status,
+                                                                      vp, sp);
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
 dyc_status dyc_set_l2_fetch_granularity(uint32_t bytes) {
     if (bytes > 128) return set_err(DYC_ERR_INVALID_ARG, "granularity must be 0..128");
     CU(cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, bytes));

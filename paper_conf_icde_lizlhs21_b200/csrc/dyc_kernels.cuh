@@ -962,6 +962,106 @@ __global__ void __launch_bounds__(kThreads) k_route_unpermute(const uint32_t* __
     }
 }
 
+// ------------------------------------- peer-memory routing (S11, fused path)
+// Dispatch and combine written straight into the owners' / requesters' memory
+// (NVLink peer pointers from CUDA IPC; local pointers when G shards share one
+// GPU).  Replaces route_count + count exchange + route_scatter + all-to-all
+// (dispatch) and all-to-all + route_unpermute (combine): the shard hash, the
+// reservation of the destination range and the transfer are one kernel, and a
+// reply lands at its op's index in the requester's result.  A record is 16 B:
+// {key, value, src_index, src_rank << 8 | tag}.
+constexpr uint32_t kMaxPeers = 64;
+struct PeerPtrs {
+    void* p[kMaxPeers];
+};
+
+// Each block bins a tile of kTileItems ops per thread by destination shard in
+// shared memory, reserves its range in every destination's receive buffer with
+// ONE system-scope atomic on that shard's counter (so the atomics crossing
+// NVLink scale with tiles, not ops), then stores one 16-B record per op.
+// Records past `cap` are not stored (the owner sees count > cap and fails).
+__global__ void __launch_bounds__(kThreads) k_route_push(HashDest dest, const uint32_t* __restrict__ vals,
+                                                         const uint8_t* __restrict__ tags, uint64_t n,
+                                                         uint32_t world, uint32_t src_rank, PeerPtrs recv,
+                                                         PeerPtrs recv_count, uint64_t cap) {
+    extern __shared__ unsigned long long base[];            // per-destination base of this tile
+    unsigned* cnt = (unsigned*)(base + world);
+    const uint64_t tile = (uint64_t)kThreads * kTileItems;
+    for (uint64_t t0 = (uint64_t)blockIdx.x * tile; t0 < n; t0 += (uint64_t)gridDim.x * tile) {
+        for (uint32_t w = threadIdx.x; w < world; w += blockDim.x) cnt[w] = 0;
+        __syncthreads();
+        uint32_t dd[kTileItems], rk[kTileItems];
+#pragma unroll
+        for (int j = 0; j < kTileItems; j++) {
+            const uint64_t i = t0 + (uint64_t)j * kThreads + threadIdx.x;
+            dd[j] = i < n ? dest(i) : 0xFFFFFFFFu;
+            rk[j] = i < n ? atomicAdd(&cnt[dd[j]], 1u) : 0u;
+        }
+        __syncthreads();
+        for (uint32_t w = threadIdx.x; w < world; w += blockDim.x)
+            base[w] = cnt[w] ? atomicAdd_system((unsigned long long*)recv_count.p[w], (unsigned long long)cnt[w])
+                             : 0ull;
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < kTileItems; j++) {
+            const uint64_t i = t0 + (uint64_t)j * kThreads + threadIdx.x;
+            if (dd[j] != 0xFFFFFFFFu) {
+                const uint64_t pos = base[dd[j]] + rk[j];
+                if (pos < cap) {
+                    const uint4 r = make_uint4(dest.keys[i], vals ? vals[i] : 0u, (uint32_t)i,
+                                               (src_rank << 8) | (tags ? tags[i] : 0u));
+                    reinterpret_cast<uint4*>(recv.p[dd[j]])[pos] = r;
+                }
+            }
+        }
+        __syncthreads();
+    }
+    __threadfence_system();
+}
+
+// Owner side: records -> the key / value / tag arrays the batch kernels read.
+__global__ void __launch_bounds__(kThreads) k_route_unpack(const uint4* __restrict__ recs, uint64_t n,
+                                                           uint32_t* __restrict__ keys, uint32_t* __restrict__ vals,
+                                                           uint8_t* __restrict__ tags) {
+    for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n; i += (uint64_t)gridDim.x * kThreads) {
+        const uint4 r = recs[i];
+        keys[i] = r.x;
+        if (vals) vals[i] = r.y;
+        if (tags) tags[i] = (uint8_t)(r.w & 0xFFu);
+    }
+}
+
+// Combine: the result of record j goes to index src_index of its requester's
+// result arrays (peer pointers), i.e. straight into request order.
+__global__ void __launch_bounds__(kThreads) k_route_reply(const uint4* __restrict__ recs, uint64_t n,
+                                                          const uint32_t* __restrict__ rv,
+                                                          const uint8_t* __restrict__ rs, PeerPtrs out_vals,
+                                                          PeerPtrs out_status) {
+    constexpr int IT = 4;
+    for (uint64_t b0 = (uint64_t)blockIdx.x * kThreads * IT; b0 < n; b0 += (uint64_t)gridDim.x * kThreads * IT) {
+        uint4 r[IT];
+        uint32_t v[IT];
+        uint8_t s8[IT];
+#pragma unroll
+        for (int j = 0; j < IT; j++) {
+            const uint64_t i = b0 + (uint64_t)j * kThreads + threadIdx.x;
+            r[j] = i < n ? recs[i] : make_uint4(0, 0, 0, 0);
+            v[j] = (i < n && rv) ? rv[i] : 0u;
+            s8[j] = (i < n && rs) ? rs[i] : 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < IT; j++) {
+            const uint64_t i = b0 + (uint64_t)j * kThreads + threadIdx.x;
+            if (i < n) {
+                const uint32_t src = r[j].w >> 8;
+                if (rv) reinterpret_cast<uint32_t*>(out_vals.p[src])[r[j].z] = v[j];
+                if (rs) reinterpret_cast<uint8_t*>(out_status.p[src])[r[j].z] = s8[j];
+            }
+        }
+    }
+    __threadfence_system();
+}
+
 // ------------------------------------------------------ random-gather ceiling
 // The probe access pattern with no table logic: reads of one B-slot bucket at
 // uniformly random bucket-aligned offsets, by a G = B/4 lane group with the same

@@ -33,7 +33,8 @@ class DistTable:
     chunk c travel back while chunk c+1 executes.  Each rank must use the same
     `chunks` (collectives are issued in the same order everywhere)."""
 
-    def __init__(self, shard, group=None, force_route: bool = False, chunks: int = 4):
+    def __init__(self, shard, group=None, force_route: bool = False, chunks: int = 4, p2p: bool = False,
+                 max_ops: Optional[int] = None):
         import torch.distributed as dist
         self.force_route = force_route
         self.dist = dist
@@ -43,6 +44,11 @@ class DistTable:
         self.shard = shard
         self.chunks = max(1, int(chunks))
         self.last_recv = 0
+        self.p2p = None
+        if p2p:
+            if not max_ops:
+                raise ValueError("p2p routing needs max_ops (the largest batch any rank issues)")
+            self.p2p = PeerRouter(self, int(max_ops))
 
     # ------------------------------------------------------------ exchange
     def _a2a(self, x, send_splits, recv_splits, async_op=False):
@@ -52,6 +58,11 @@ class DistTable:
         return out, w
 
     def _run(self, op, keys, values=None, n_out=1, begin=None, end=None, tags=None):
+        if self.p2p is not None:
+            return self.p2p.run(op, keys, values, n_out, begin, end, tags)
+        return self._run_a2a(op, keys, values, n_out, begin, end, tags)
+
+    def _run_a2a(self, op, keys, values=None, n_out=1, begin=None, end=None, tags=None):
         """Pipelined route -> all-to-all -> owner op -> all-to-all back -> unpermute.
         op(keys, values) returns a tuple of n_out per-op result tensors.  begin(n)
         / end() bracket the owner's parts so that they form ONE batch (one
@@ -157,6 +168,89 @@ class DistTable:
         return self.shard.stats()
 
 
+class PeerRouter:
+    """Fused dispatch / combine over peer memory (dyc_route_push / dyc_route_reply;
+    DESIGN.md §7).  Each rank owns, in plain cudaMalloc buffers shared through
+    CUDA IPC: a receive buffer of world * max_ops 16-B records, its uint64
+    receive counter, and its result arrays (u32 values, u8 status) for up to
+    max_ops ops.  A batch is
+
+        push (every rank: hash, reserve, store records into the owners' buffers)
+        -> barrier -> owner: unpack, ONE local batch, reply (results stored at
+        the op's index in the requester's result arrays), reset counter
+        -> barrier -> results are in request order.
+
+    No counts are exchanged, nothing is unpermuted, and no NCCL data movement is
+    used; the barriers are host barriers of the process group after a stream
+    sync (they order the peer stores, which complete with their kernels)."""
+
+    def __init__(self, dt, max_ops: int):
+        import torch
+        from .table import PeerBuffer
+        self.dt, self.max_ops = dt, max_ops
+        W, r = dt.world, dt.rank
+        self.cap = W * max_ops
+        self.recv = PeerBuffer(16 * self.cap)
+        self.cnt = PeerBuffer(8)
+        self.rv = PeerBuffer(4 * max_ops)
+        self.rs = PeerBuffer(max_ops)
+        bufs = (self.recv, self.cnt, self.rv, self.rs)
+        mine = [b.handle() for b in bufs]
+        allh = [None] * W
+        dt.dist.all_gather_object(allh, mine, group=dt.group)
+        ptrs = [[b.ptr for b in bufs] if w == r else [b.open(h) for b, h in zip(bufs, allh[w])] for w in range(W)]
+        self.recv_p, self.cnt_p, self.rv_p, self.rs_p = ([p[i] for p in ptrs] for i in range(4))
+        dev = torch.device("cuda", torch.cuda.current_device())
+        self.k = torch.empty(self.cap, dtype=torch.int32, device=dev)
+        self.v = torch.empty(self.cap, dtype=torch.int32, device=dev)
+        self.t = torch.empty(self.cap, dtype=torch.uint8, device=dev)
+        self.count = self.cnt.tensor(1, torch.int64)
+        self.out_v = self.rv.tensor(max_ops, torch.int32)
+        self.out_s = self.rs.tensor(max_ops, torch.uint8)
+        self._barrier()
+
+    def _barrier(self):
+        import torch
+        torch.cuda.current_stream().synchronize()
+        self.dt.dist.barrier(group=self.dt.group)
+
+    def run(self, op, keys, values, n_out, begin, end, tags):
+        from .table import Table
+        dt = self.dt
+        n = keys.numel()
+        if n > self.max_ops:
+            raise ValueError(f"batch of {n} ops exceeds the router's max_ops {self.max_ops}")
+        dt.shard.route_push(keys, values, dt.world, dt.rank, self.recv_p, self.cnt_p, self.cap, tags=tags)
+        self._barrier()
+        m = int(self.count.item())
+        if m > self.cap:
+            raise RuntimeError(f"receive buffer overflow: {m} records > {self.cap}")
+        dt.last_recv = m
+        k = self.k[:m]
+        v = self.v[:m] if values is not None else None
+        t = self.t[:m] if tags is not None else None
+        Table.route_unpack(self.recv.ptr, m, k, v, t)
+        if begin is not None:
+            begin(m)
+        res = op(k, v) if tags is None else op(k, v, t)
+        res = res if isinstance(res, tuple) else (res,)
+        if end is not None:
+            end()
+        if n_out == 1:
+            Table.route_reply(self.recv.ptr, m, dt.world, status=res[0], out_status_ptrs=self.rs_p)
+        else:
+            Table.route_reply(self.recv.ptr, m, dt.world, vals=res[0], status=res[1], out_val_ptrs=self.rv_p,
+                              out_status_ptrs=self.rs_p)
+        self.count.zero_()
+        self._barrier()
+        out_s = self.out_s[:n].clone()
+        return out_s if n_out == 1 else (self.out_v[:n].clone(), out_s)
+
+    def close(self):
+        for b in (self.recv, self.cnt, self.rv, self.rs):
+            b.close()
+
+
 # ---------------------------------------------------------------- bench (N > 1)
 def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_peaks, run_oracle_sample,
                     compute_roofline=None):
@@ -175,7 +269,8 @@ def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_pea
     cap, k_ins, v_ins, k_find, k_del = W.c2_rand_static_torch(args.log2n, device="cuda", key_base=rank * n,
                                                               miss_base=rank * n)
     shard = Table(d=4, init_capacity=cap, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
-    dt = DistTable(shard, force_route=True)      # exercise the router even at N=1 (--routed)
+    p2p = getattr(args, "p2p", False)
+    dt = DistTable(shard, force_route=True, p2p=p2p, max_ops=n if p2p else None)  # router even at N=1
     stream = torch.cuda.current_stream()
 
     def step(evs=None):
@@ -277,6 +372,7 @@ def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_pea
                                f"2^{args.log2n - 1} deletes), hash-partitioned over {world} shards, "
                                "NCCL all-to-all routing", "d": 4, "alpha": 0.3, "beta": 0.85,
                    "bucket_slots": args.bucket_slots, "parallelism": f"shard{world}",
+                   "routing": "p2p (fused push/reply over peer memory)" if p2p else "nccl all-to-all",
                    "l2": "inputs and tables larger than L2; no flush needed"},
         "phase_ms_rank0": phases,
         "check": {"all_inserted_ranks": int(ok[0].item()), "found_total": int(ok[1].item()),
@@ -305,7 +401,9 @@ def bench_c5(args, rank, world, local, metric, ClockSampler):
     # keeps the 32 mixed batches' deletes below the live-find range at any scale
     batch = 1 << min(24, log2k - 7)
     shard = Table(d=4, init_capacity=1 << 20, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
-    dt = DistTable(shard, force_route=getattr(args, "routed", False))
+    p2p = getattr(args, "p2p", False)
+    dt = DistTable(shard, force_route=getattr(args, "routed", False) or p2p, p2p=p2p,
+                   max_ops=(batch + world - 1) // world if p2p else None)
     stream = torch.cuda.current_stream()
     gen = W.c5_batches_torch(rank, world, device="cuda", log2_keys=log2k, batch=batch, mixed_batches=32)
     fill, mixed = [], []
@@ -360,7 +458,9 @@ def bench_c5(args, rank, world, local, metric, ClockSampler):
         "config": {"workload": f"C5 RAND 2^{log2k} keys hash-partitioned over {world} shard(s): {len(fill)} global "
                                f"insert batches of {batch}, then {len(mixed)} mixed 50/30/20 batches of {batch}",
                    "d": 4, "alpha": 0.3, "beta": 0.85, "bucket_slots": args.bucket_slots,
-                   "parallelism": f"shard{world}", "init_capacity_per_shard": 1 << 20},
+                   "parallelism": f"shard{world}", "init_capacity_per_shard": 1 << 20,
+                   "routing": "p2p (fused push/reply over peer memory)" if p2p else
+                   ("nccl all-to-all" if (world > 1 or getattr(args, "routed", False)) else "local")},
         "phases": {"fill_ms": fill_ms, "fill_mops": n_fill / fill_ms / 1e3,
                    "mixed_ms": mixed_ms, "mixed_mops": n_mixed / mixed_ms / 1e3},
         "check": {"inserted_fill": int(checks[0]), "expected_fill": n_fill - reserved_all,

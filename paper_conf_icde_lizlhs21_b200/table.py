@@ -37,6 +37,63 @@ def _stream_ptr(stream) -> int:
     return int(s.cuda_stream)
 
 
+def _ptr_array(ptrs, world: int):
+    if len(ptrs) != world:
+        raise ValueError(f"expected {world} device pointers, got {len(ptrs)}")
+    return C.cast((C.c_void_p * world)(*[int(p) for p in ptrs]), C.c_void_p)
+
+
+class PeerBuffer:
+    """A device buffer from dyc_ipc_alloc (plain cudaMalloc, zero-filled) that
+    other processes map through CUDA IPC (dyc_ipc_get_handle / dyc_ipc_open).
+    `ptr` is the local address; `handle()` the 64-byte IPC handle; `open(h)`
+    maps a peer's handle and returns its address here (closed by close())."""
+
+    def __init__(self, nbytes: int):
+        p = C.c_void_p()
+        L.check(L.load_library().dyc_ipc_alloc(int(nbytes), C.byref(p)), "dyc_ipc_alloc")
+        self.ptr, self.nbytes, self._opened = int(p.value), int(nbytes), []
+
+    def handle(self) -> bytes:
+        h = (C.c_char * 64)()
+        L.check(L.load_library().dyc_ipc_get_handle(self.ptr, h), "dyc_ipc_get_handle")
+        return bytes(h.raw)
+
+    def open(self, handle: bytes) -> int:
+        p = C.c_void_p()
+        L.check(L.load_library().dyc_ipc_open(C.create_string_buffer(handle, 64), C.byref(p)), "dyc_ipc_open")
+        self._opened.append(int(p.value))
+        return int(p.value)
+
+    def tensor(self, n: int, dtype):
+        """Zero-copy torch view of the first n elements (__cuda_array_interface__)."""
+        torch = _torch()
+        typestr = {torch.int32: "<i4", torch.uint8: "|u1", torch.int64: "<i8"}[dtype]
+        size = n * torch.tensor([], dtype=dtype).element_size()
+        if size > self.nbytes:
+            raise ValueError("view larger than the buffer")
+
+        class _View:
+            __cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (self.ptr, False), "version": 3,
+                                        "strides": None, "stream": None}
+        return torch.as_tensor(_View(), device="cuda")
+
+    def close(self):
+        lib = L.load_library()
+        for p in self._opened:
+            lib.dyc_ipc_close(p)
+        self._opened = []
+        if self.ptr:
+            lib.dyc_ipc_free(self.ptr)
+            self.ptr = 0
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # noqa: BLE001
+            pass
+
+
 class Table:
     """A DyCuckoo table (two-layer cuckoo hash, d subtables; see include/dycuckoo.h)."""
 
@@ -359,6 +416,38 @@ class Table:
                                               s.data_ptr() if s is not None else None, _stream_ptr(stream)),
                 "dyc_route_unpermute")
         return v, s
+
+    # ------------------------------------------- fused routing over peer memory
+    def route_push(self, keys, values, world: int, src_rank: int, recv_ptrs, count_ptrs, recv_cap: int,
+                   tags=None, stream=None):
+        """Dispatch (dyc_route_push): every op is stored as a 16-B record in its
+        shard's receive buffer.  recv_ptrs / count_ptrs: `world` device
+        addresses (ints; peer pointers from PeerBuffer.open or local ones)."""
+        _check_u32(keys, "keys")
+        L.check(self._lib.dyc_route_push(self._h, keys.data_ptr(), values.data_ptr() if values is not None else None,
+                                         tags.data_ptr() if tags is not None else None, keys.numel(), world,
+                                         src_rank, _ptr_array(recv_ptrs, world), _ptr_array(count_ptrs, world),
+                                         recv_cap, _stream_ptr(stream)), "dyc_route_push")
+
+    @staticmethod
+    def route_unpack(recs_ptr: int, n: int, keys, values=None, tags=None, stream=None):
+        """Records at device address recs_ptr -> keys[:n] (and values / tags)."""
+        L.check(L.load_library().dyc_route_unpack(recs_ptr, n, keys.data_ptr(),
+                                                  values.data_ptr() if values is not None else None,
+                                                  tags.data_ptr() if tags is not None else None,
+                                                  _stream_ptr(stream)), "dyc_route_unpack")
+
+    @staticmethod
+    def route_reply(recs_ptr: int, n: int, world: int, vals=None, status=None, out_val_ptrs=None,
+                    out_status_ptrs=None, stream=None):
+        """Combine (dyc_route_reply): result j goes to its requester's result
+        arrays (device addresses per rank) at the op's index."""
+        L.check(L.load_library().dyc_route_reply(
+            recs_ptr, n, vals.data_ptr() if vals is not None else None,
+            status.data_ptr() if status is not None else None, world,
+            _ptr_array(out_val_ptrs, world) if vals is not None else None,
+            _ptr_array(out_status_ptrs, world) if status is not None else None,
+            _stream_ptr(stream)), "dyc_route_reply")
 
     def launch_count(self, reset: bool = False) -> int:
         return int(self._lib.dyc_launch_count(self._h, 1 if reset else 0))
