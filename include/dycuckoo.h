@@ -370,15 +370,15 @@ dyc_status dyc_route_unpermute(const uint32_t* d_pos, uint64_t n, const uint32_t
  * result at its op's index in the requester's result arrays.  Peer buffers are
  * plain cudaMalloc allocations shared through CUDA IPC (NVLink peer pointers
  * between GPUs of one node; the same calls work between processes on one GPU).
- * A receive record is 16 bytes, dyc_route_rec below.  The caller orders the
- * phases across ranks (dispatch on every rank, barrier, owner batch + combine,
+ * A receive buffer of capacity `cap` ops is structure-of-arrays, so the owner
+ * runs its batch on the keys / values / op codes in place:
+ *     keys u32[cap] at byte 0, values u32[cap] at 4*cap,
+ *     meta u64[cap] at 8*cap (src_index | src_rank << 32), tags u8[cap] at 16*cap
+ * (DYC_ROUTE_RECV_BYTES(cap) = 17*cap bytes).  The caller orders the phases
+ * across ranks (dispatch on every rank, barrier, owner batch + combine,
  * barrier) and resets its receive counter between batches.
  * ------------------------------------------------------------------------- */
-typedef struct {
-    uint32_t key, value;
-    uint32_t src_index;               /* op index in the requester's batch      */
-    uint32_t src_tag;                 /* requester rank << 8 | tag (op code)    */
-} dyc_route_rec;
+#define DYC_ROUTE_RECV_BYTES(cap) (17ull * (uint64_t)(cap))
 
 /* Device buffer for IPC sharing: cudaMalloc of `bytes`, zero-filled (so a
  * receive counter starts at 0).  Owned by the caller; release with
@@ -394,33 +394,29 @@ dyc_status dyc_ipc_open(const void* handle64, void** d_ptr);
 dyc_status dyc_ipc_close(void* d_ptr);
 
 /* Dispatch: op i (d_keys[i], d_vals[i] or 0, d_tags[i] or 0) goes to shard
- * s = x_{d+1}(k) mod world (same hash as dyc_route_count): it is stored as a
- * dyc_route_rec {key, value, i, src_rank << 8 | tag} at position
- * atomicAdd_system(d_recv_count[s], ...) of d_recv[s].  d_recv and
- * d_recv_count are HOST arrays of `world` device pointers (peer or local):
- * d_recv[s] holds recv_cap records, *d_recv_count[s] is a uint64 counter in
- * shard s's memory.  Records past recv_cap are dropped; the owner detects
- * *count > recv_cap and must treat the batch as failed.  Order within a
- * shard's buffer is unspecified.  d_vals, d_tags nullable.  world 1..64,
- * src_rank < world, n < 2^32; else DYC_ERR_INVALID_ARG.  `t` supplies the
- * hash constants (all ranks use one seed). */
+ * s = x_{d+1}(k) mod world (same hash as dyc_route_count): at position
+ * g = atomicAdd_system(d_recv_count[s], ...) of receive buffer d_recv[s]
+ * (layout above) it stores keys[g] = key, values[g] (if d_vals), meta[g] =
+ * i | src_rank << 32, tags[g] (if d_tags).  d_recv and d_recv_count are HOST
+ * arrays of `world` device pointers (peer or local): d_recv[s] holds recv_cap
+ * ops, *d_recv_count[s] is a uint64 counter in shard s's memory.  Ops past
+ * recv_cap are dropped; the owner detects *count > recv_cap and must treat the
+ * batch as failed.  Order within a shard's buffer is unspecified.  d_vals,
+ * d_tags nullable.  world 1..64, src_rank < world, n < 2^32; else
+ * DYC_ERR_INVALID_ARG.  `t` supplies the hash constants (all ranks use one seed). */
 dyc_status dyc_route_push(dyc_table* t, const uint32_t* d_keys, const uint32_t* d_vals, const uint8_t* d_tags,
                           uint64_t n, uint32_t world, uint32_t src_rank, void* const* d_recv,
                           uint64_t* const* d_recv_count, uint64_t recv_cap, dyc_stream_t stream);
 
-/* Owner side: splits n records (device) into d_keys[n] and, when non-NULL,
- * d_vals[n] / d_tags[n] (the op code carried in the low byte of src_tag). */
-dyc_status dyc_route_unpack(const void* d_recs, uint64_t n, uint32_t* d_keys, uint32_t* d_vals, uint8_t* d_tags,
-                            dyc_stream_t stream);
-
-/* Combine: for record j of d_recs[n] with requester r = src_tag >> 8 and index
- * i = src_index, stores d_vals[j] into d_out_vals[r][i] and d_status[j] into
- * d_out_status[r][i].  d_out_vals / d_out_status are HOST arrays of `world`
- * device pointers (the requesters' result arrays, peer or local); each pair
- * (d_vals, d_out_vals), (d_status, d_out_status) is both NULL or both given. */
-dyc_status dyc_route_reply(const void* d_recs, uint64_t n, const uint32_t* d_vals, const uint8_t* d_status,
-                           uint32_t world, uint32_t* const* d_out_vals, uint8_t* const* d_out_status,
-                           dyc_stream_t stream);
+/* Combine: for received op j < n of the local buffer d_recv (capacity
+ * recv_cap, layout above) with meta[j] = i | r << 32, stores d_vals[j] into
+ * d_out_vals[r][i] and d_status[j] into d_out_status[r][i].  d_out_vals /
+ * d_out_status are HOST arrays of `world` device pointers (the requesters'
+ * result arrays, peer or local); each pair (d_vals, d_out_vals), (d_status,
+ * d_out_status) is both NULL or both given.  n <= recv_cap. */
+dyc_status dyc_route_reply(const void* d_recv, uint64_t recv_cap, uint64_t n, const uint32_t* d_vals,
+                           const uint8_t* d_status, uint32_t world, uint32_t* const* d_out_vals,
+                           uint8_t* const* d_out_status, dyc_stream_t stream);
 
 /* ---------------------------------------------------------------------------
  * Measurement helpers (bench.py; not part of the method).

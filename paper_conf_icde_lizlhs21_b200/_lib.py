@@ -131,8 +131,7 @@ SIGNATURES = {
     "dyc_ipc_open": (_I, [_P, C.POINTER(C.c_void_p)]),
     "dyc_ipc_close": (_I, [_P]),
     "dyc_route_push": (_I, [_TP, _P, _P, _P, _U64, _U32, _U32, _P, _P, _U64, _P]),
-    "dyc_route_unpack": (_I, [_P, _U64, _P, _P, _P, _P]),
-    "dyc_route_reply": (_I, [_P, _U64, _P, _P, _U32, _P, _P, _P]),
+    "dyc_route_reply": (_I, [_P, _U64, _U64, _P, _P, _U32, _P, _P, _P]),
     "dyc_bench_gather": (_I, [_P, _U64, _U64, _U32, _U64, _P, _P]),
     "dyc_bench_gather_ex": (_I, [_P, _U64, _U64, _U32, _U64, _U32, _P, _P]),
     "dyc_set_l2_fetch_granularity": (_I, [_U32]),

@@ -1821,29 +1821,20 @@ dyc_status dyc_route_push(dyc_table* t, const uint32_t* d_keys, const uint32_t* 
     {
         ProfScope ps(t, DYC_PROF_OTHER, S(stream));
         const HashDest hd{t->a[sh], t->b[sh], world, fastmod_magic(world), d_keys};
-        k_route_push<<<std::min<unsigned>(grid_for(n, (uint64_t)kThreads * kTileItems), t->num_sms * 8), kThreads,
-                       world * 12, S(stream)>>>(hd, d_vals, d_tags, n, world, src_rank, rp, cp, recv_cap);
+        k_route_push<<<std::min<unsigned>(grid_for(n, (uint64_t)kThreads * kPushItems), t->num_sms * 4), kThreads,
+                       0, S(stream)>>>(hd, d_vals, d_tags, n, world, src_rank, rp, cp, recv_cap);
     }
     CU(cudaGetLastError());
     return DYC_OK;
 }
 
-dyc_status dyc_route_unpack(const void* d_recs, uint64_t n, uint32_t* d_keys, uint32_t* d_vals, uint8_t* d_tags,
-                            dyc_stream_t stream) {
-    if (n == 0) return DYC_OK;
-    if (!d_recs || !d_keys) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_unpack: null pointer");
-    k_route_unpack<<<grid_for(n, kThreads * 4), kThreads, 0, S(stream)>>>((const uint4*)d_recs, n, d_keys, d_vals,
-                                                                       d_tags);
-    CU(cudaGetLastError());
-    return DYC_OK;
-}
-
-dyc_status dyc_route_reply(const void* d_recs, uint64_t n, const uint32_t* d_vals, const uint8_t* d_status,
-                           uint32_t world, uint32_t* const* d_out_vals, uint8_t* const* d_out_status,
-                           dyc_stream_t stream) {
+dyc_status dyc_route_reply(const void* d_recv, uint64_t recv_cap, uint64_t n, const uint32_t* d_vals,
+                           const uint8_t* d_status, uint32_t world, uint32_t* const* d_out_vals,
+                           uint8_t* const* d_out_status, dyc_stream_t stream) {
     if (world < 1 || world > kMaxPeers) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_reply: world must be 1..64");
     if (n == 0) return DYC_OK;
-    if (!d_recs) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_reply: null records");
+    if (!d_recv) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_reply: null receive buffer");
+    if (n > recv_cap) return set_err(DYC_ERR_INVALID_ARG, "dyc_route_reply: n > recv_cap");
     if ((d_vals == nullptr) != (d_out_vals == nullptr) || (d_status == nullptr) != (d_out_status == nullptr))
         return set_err(DYC_ERR_INVALID_ARG, "dyc_route_reply: a result array and its destinations must both be given");
     PeerPtrs vp{}, sp{};
@@ -1857,8 +1848,8 @@ dyc_status dyc_route_reply(const void* d_recs, uint64_t n, const uint32_t* d_val
             sp.p[w] = d_out_status[w];
         }
     }
-    k_route_reply<<<grid_for(n, kThreads * 4), kThreads, 0, S(stream)>>>((const uint4*)d_recs, n, d_vals, d_status,
-                                                                      vp, sp);
+    const unsigned long long* meta = (const unsigned long long*)((const char*)d_recv + 8 * recv_cap);
+    k_route_reply<<<grid_for(n, kThreads * 4), kThreads, 0, S(stream)>>>(meta, n, d_vals, d_status, vp, sp);
     CU(cudaGetLastError());
     return DYC_OK;
 }

@@ -968,50 +968,79 @@ __global__ void __launch_bounds__(kThreads) k_route_unpermute(const uint32_t* __
 // GPU).  Replaces route_count + count exchange + route_scatter + all-to-all
 // (dispatch) and all-to-all + route_unpermute (combine): the shard hash, the
 // reservation of the destination range and the transfer are one kernel, and a
-// reply lands at its op's index in the requester's result.  A record is 16 B:
-// {key, value, src_index, src_rank << 8 | tag}.
+// reply lands at its op's index in the requester's result.
+//
+// A receive buffer of capacity `cap` is structure-of-arrays, so the owner's
+// batch kernels read its keys and values in place:
+//   keys u32[cap] @ 0 | vals u32[cap] @ 4cap | meta u64[cap] @ 8cap | tags u8[cap] @ 16cap
+// meta = src_index | (uint64)src_rank << 32.
 constexpr uint32_t kMaxPeers = 64;
 struct PeerPtrs {
     void* p[kMaxPeers];
 };
+constexpr int kPushItems = 8;                    // ops per thread per tile (tile = 2048 ops)
 
-// Each block bins a tile of kTileItems ops per thread by destination shard in
-// shared memory, reserves its range in every destination's receive buffer with
-// ONE system-scope atomic on that shard's counter (so the atomics crossing
-// NVLink scale with tiles, not ops), then stores one 16-B record per op.
-// Records past `cap` are not stored (the owner sees count > cap and fails).
+// Each block takes a tile of 2048 ops: it hashes them to their shards, ranks
+// them per shard in shared memory and stages them there grouped by shard; it
+// reserves the tile's range in every destination with ONE system-scope atomic
+// on that shard's counter (atomics crossing NVLink scale with tiles, not ops);
+// then the staged tile is copied out so that consecutive threads store to
+// consecutive addresses of one destination's range (coalesced peer stores).
+// Ops past `cap` are not stored (the owner sees count > cap and fails).
 __global__ void __launch_bounds__(kThreads) k_route_push(HashDest dest, const uint32_t* __restrict__ vals,
                                                          const uint8_t* __restrict__ tags, uint64_t n,
                                                          uint32_t world, uint32_t src_rank, PeerPtrs recv,
                                                          PeerPtrs recv_count, uint64_t cap) {
-    extern __shared__ unsigned long long base[];            // per-destination base of this tile
-    unsigned* cnt = (unsigned*)(base + world);
-    const uint64_t tile = (uint64_t)kThreads * kTileItems;
-    for (uint64_t t0 = (uint64_t)blockIdx.x * tile; t0 < n; t0 += (uint64_t)gridDim.x * tile) {
+    constexpr int T = kThreads * kPushItems;
+    __shared__ uint32_t s_key[T], s_val[T], s_idx[T];
+    __shared__ uint8_t s_tag[T], s_dst[T];
+    __shared__ unsigned cnt[kMaxPeers], off[kMaxPeers + 1];
+    __shared__ unsigned long long base[kMaxPeers];
+    for (uint64_t t0 = (uint64_t)blockIdx.x * T; t0 < n; t0 += (uint64_t)gridDim.x * T) {
+        const unsigned nt = (unsigned)((n - t0) < (uint64_t)T ? (n - t0) : (uint64_t)T);
         for (uint32_t w = threadIdx.x; w < world; w += blockDim.x) cnt[w] = 0;
         __syncthreads();
-        uint32_t dd[kTileItems], rk[kTileItems];
+        uint32_t dd[kPushItems], rk[kPushItems];
 #pragma unroll
-        for (int j = 0; j < kTileItems; j++) {
-            const uint64_t i = t0 + (uint64_t)j * kThreads + threadIdx.x;
-            dd[j] = i < n ? dest(i) : 0xFFFFFFFFu;
-            rk[j] = i < n ? atomicAdd(&cnt[dd[j]], 1u) : 0u;
+        for (int j = 0; j < kPushItems; j++) {
+            const unsigned li = j * kThreads + threadIdx.x;
+            dd[j] = li < nt ? dest(t0 + li) : 0xFFFFFFFFu;
+            rk[j] = li < nt ? atomicAdd(&cnt[dd[j]], 1u) : 0u;
         }
         __syncthreads();
+        if (threadIdx.x == 0) {
+            unsigned acc = 0;
+            for (uint32_t w = 0; w < world; w++) { off[w] = acc; acc += cnt[w]; }
+            off[world] = acc;
+        }
         for (uint32_t w = threadIdx.x; w < world; w += blockDim.x)
             base[w] = cnt[w] ? atomicAdd_system((unsigned long long*)recv_count.p[w], (unsigned long long)cnt[w])
                              : 0ull;
         __syncthreads();
 #pragma unroll
-        for (int j = 0; j < kTileItems; j++) {
-            const uint64_t i = t0 + (uint64_t)j * kThreads + threadIdx.x;
-            if (dd[j] != 0xFFFFFFFFu) {
-                const uint64_t pos = base[dd[j]] + rk[j];
-                if (pos < cap) {
-                    const uint4 r = make_uint4(dest.keys[i], vals ? vals[i] : 0u, (uint32_t)i,
-                                               (src_rank << 8) | (tags ? tags[i] : 0u));
-                    reinterpret_cast<uint4*>(recv.p[dd[j]])[pos] = r;
-                }
+        for (int j = 0; j < kPushItems; j++) {
+            const unsigned li = j * kThreads + threadIdx.x;
+            if (li < nt) {
+                const unsigned p = off[dd[j]] + rk[j];
+                const uint64_t i = t0 + li;
+                s_key[p] = dest.keys[i];
+                s_val[p] = vals ? vals[i] : 0u;
+                s_idx[p] = (uint32_t)i;
+                s_tag[p] = tags ? tags[i] : 0u;
+                s_dst[p] = (uint8_t)dd[j];
+            }
+        }
+        __syncthreads();
+        for (unsigned p = threadIdx.x; p < nt; p += kThreads) {
+            const uint32_t w = s_dst[p];
+            const uint64_t g = base[w] + (p - off[w]);
+            if (g < cap) {
+                char* b = (char*)recv.p[w];
+                reinterpret_cast<uint32_t*>(b)[g] = s_key[p];
+                if (vals) reinterpret_cast<uint32_t*>(b + 4 * cap)[g] = s_val[p];
+                reinterpret_cast<unsigned long long*>(b + 8 * cap)[g] =
+                    (unsigned long long)s_idx[p] | ((unsigned long long)src_rank << 32);
+                if (tags) reinterpret_cast<uint8_t*>(b + 16 * cap)[g] = s_tag[p];
             }
         }
         __syncthreads();
@@ -1019,33 +1048,21 @@ __global__ void __launch_bounds__(kThreads) k_route_push(HashDest dest, const ui
     __threadfence_system();
 }
 
-// Owner side: records -> the key / value / tag arrays the batch kernels read.
-__global__ void __launch_bounds__(kThreads) k_route_unpack(const uint4* __restrict__ recs, uint64_t n,
-                                                           uint32_t* __restrict__ keys, uint32_t* __restrict__ vals,
-                                                           uint8_t* __restrict__ tags) {
-    for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n; i += (uint64_t)gridDim.x * kThreads) {
-        const uint4 r = recs[i];
-        keys[i] = r.x;
-        if (vals) vals[i] = r.y;
-        if (tags) tags[i] = (uint8_t)(r.w & 0xFFu);
-    }
-}
-
-// Combine: the result of record j goes to index src_index of its requester's
-// result arrays (peer pointers), i.e. straight into request order.
-__global__ void __launch_bounds__(kThreads) k_route_reply(const uint4* __restrict__ recs, uint64_t n,
+// Combine: the result of received op j goes to index src_index of its
+// requester's result arrays (peer pointers), i.e. straight into request order.
+__global__ void __launch_bounds__(kThreads) k_route_reply(const unsigned long long* __restrict__ meta, uint64_t n,
                                                           const uint32_t* __restrict__ rv,
                                                           const uint8_t* __restrict__ rs, PeerPtrs out_vals,
                                                           PeerPtrs out_status) {
     constexpr int IT = 4;
     for (uint64_t b0 = (uint64_t)blockIdx.x * kThreads * IT; b0 < n; b0 += (uint64_t)gridDim.x * kThreads * IT) {
-        uint4 r[IT];
+        unsigned long long m[IT];
         uint32_t v[IT];
         uint8_t s8[IT];
 #pragma unroll
         for (int j = 0; j < IT; j++) {
             const uint64_t i = b0 + (uint64_t)j * kThreads + threadIdx.x;
-            r[j] = i < n ? recs[i] : make_uint4(0, 0, 0, 0);
+            m[j] = i < n ? meta[i] : 0ull;
             v[j] = (i < n && rv) ? rv[i] : 0u;
             s8[j] = (i < n && rs) ? rs[i] : 0u;
         }
@@ -1053,9 +1070,9 @@ __global__ void __launch_bounds__(kThreads) k_route_reply(const uint4* __restric
         for (int j = 0; j < IT; j++) {
             const uint64_t i = b0 + (uint64_t)j * kThreads + threadIdx.x;
             if (i < n) {
-                const uint32_t src = r[j].w >> 8;
-                if (rv) reinterpret_cast<uint32_t*>(out_vals.p[src])[r[j].z] = v[j];
-                if (rs) reinterpret_cast<uint8_t*>(out_status.p[src])[r[j].z] = s8[j];
+                const uint32_t src = (uint32_t)(m[j] >> 32), idx = (uint32_t)m[j];
+                if (rv) reinterpret_cast<uint32_t*>(out_vals.p[src])[idx] = v[j];
+                if (rs) reinterpret_cast<uint8_t*>(out_status.p[src])[idx] = s8[j];
             }
         }
     }

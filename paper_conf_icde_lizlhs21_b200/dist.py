@@ -171,12 +171,12 @@ class DistTable:
 class PeerRouter:
     """Fused dispatch / combine over peer memory (dyc_route_push / dyc_route_reply;
     DESIGN.md §7).  Each rank owns, in plain cudaMalloc buffers shared through
-    CUDA IPC: a receive buffer of world * max_ops 16-B records, its uint64
+    CUDA IPC: a receive buffer of world * max_ops ops (17 B each, SoA), its uint64
     receive counter, and its result arrays (u32 values, u8 status) for up to
     max_ops ops.  A batch is
 
-        push (every rank: hash, reserve, store records into the owners' buffers)
-        -> barrier -> owner: unpack, ONE local batch, reply (results stored at
+        push (every rank: hash, reserve, store ops into the owners' buffers)
+        -> barrier -> owner: ONE local batch on the buffer in place, reply (results at
         the op's index in the requester's result arrays), reset counter
         -> barrier -> results are in request order.
 
@@ -190,7 +190,7 @@ class PeerRouter:
         self.dt, self.max_ops = dt, max_ops
         W, r = dt.world, dt.rank
         self.cap = W * max_ops
-        self.recv = PeerBuffer(16 * self.cap)
+        self.recv = PeerBuffer(17 * self.cap)          # DYC_ROUTE_RECV_BYTES: keys | values | meta | tags
         self.cnt = PeerBuffer(8)
         self.rv = PeerBuffer(4 * max_ops)
         self.rs = PeerBuffer(max_ops)
@@ -200,10 +200,6 @@ class PeerRouter:
         dt.dist.all_gather_object(allh, mine, group=dt.group)
         ptrs = [[b.ptr for b in bufs] if w == r else [b.open(h) for b, h in zip(bufs, allh[w])] for w in range(W)]
         self.recv_p, self.cnt_p, self.rv_p, self.rs_p = ([p[i] for p in ptrs] for i in range(4))
-        dev = torch.device("cuda", torch.cuda.current_device())
-        self.k = torch.empty(self.cap, dtype=torch.int32, device=dev)
-        self.v = torch.empty(self.cap, dtype=torch.int32, device=dev)
-        self.t = torch.empty(self.cap, dtype=torch.uint8, device=dev)
         self.count = self.cnt.tensor(1, torch.int64)
         self.out_v = self.rv.tensor(max_ops, torch.int32)
         self.out_s = self.rs.tensor(max_ops, torch.uint8)
@@ -226,10 +222,9 @@ class PeerRouter:
         if m > self.cap:
             raise RuntimeError(f"receive buffer overflow: {m} records > {self.cap}")
         dt.last_recv = m
-        k = self.k[:m]
-        v = self.v[:m] if values is not None else None
-        t = self.t[:m] if tags is not None else None
-        Table.route_unpack(self.recv.ptr, m, k, v, t)
+        k, v, t = Table.recv_views(self.recv, self.cap, m)       # the owner's batch, in place
+        v = v if values is not None else None
+        t = t if tags is not None else None
         if begin is not None:
             begin(m)
         res = op(k, v) if tags is None else op(k, v, t)
@@ -237,10 +232,10 @@ class PeerRouter:
         if end is not None:
             end()
         if n_out == 1:
-            Table.route_reply(self.recv.ptr, m, dt.world, status=res[0], out_status_ptrs=self.rs_p)
+            Table.route_reply(self.recv.ptr, self.cap, m, dt.world, status=res[0], out_status_ptrs=self.rs_p)
         else:
-            Table.route_reply(self.recv.ptr, m, dt.world, vals=res[0], status=res[1], out_val_ptrs=self.rv_p,
-                              out_status_ptrs=self.rs_p)
+            Table.route_reply(self.recv.ptr, self.cap, m, dt.world, vals=res[0], status=res[1],
+                              out_val_ptrs=self.rv_p, out_status_ptrs=self.rs_p)
         self.count.zero_()
         self._barrier()
         out_s = self.out_s[:n].clone()

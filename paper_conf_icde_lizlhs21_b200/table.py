@@ -65,16 +65,19 @@ class PeerBuffer:
         self._opened.append(int(p.value))
         return int(p.value)
 
-    def tensor(self, n: int, dtype):
-        """Zero-copy torch view of the first n elements (__cuda_array_interface__)."""
+    def tensor(self, n: int, dtype, offset: int = 0):
+        """Zero-copy torch view of n elements at byte `offset` (__cuda_array_interface__)."""
         torch = _torch()
         typestr = {torch.int32: "<i4", torch.uint8: "|u1", torch.int64: "<i8"}[dtype]
         size = n * torch.tensor([], dtype=dtype).element_size()
-        if size > self.nbytes:
-            raise ValueError("view larger than the buffer")
+        if offset + size > self.nbytes:
+            raise ValueError("view outside the buffer")
+        if n == 0:
+            return torch.empty(0, dtype=dtype, device="cuda")
+        ptr = self.ptr + offset
 
         class _View:
-            __cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (self.ptr, False), "version": 3,
+            __cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False), "version": 3,
                                         "strides": None, "stream": None}
         return torch.as_tensor(_View(), device="cuda")
 
@@ -420,9 +423,9 @@ class Table:
     # ------------------------------------------- fused routing over peer memory
     def route_push(self, keys, values, world: int, src_rank: int, recv_ptrs, count_ptrs, recv_cap: int,
                    tags=None, stream=None):
-        """Dispatch (dyc_route_push): every op is stored as a 16-B record in its
-        shard's receive buffer.  recv_ptrs / count_ptrs: `world` device
-        addresses (ints; peer pointers from PeerBuffer.open or local ones)."""
+        """Dispatch (dyc_route_push): every op goes to its shard's receive buffer
+        (structure-of-arrays, see recv_views).  recv_ptrs / count_ptrs: `world`
+        device addresses (ints; peer pointers from PeerBuffer.open or local ones)."""
         _check_u32(keys, "keys")
         L.check(self._lib.dyc_route_push(self._h, keys.data_ptr(), values.data_ptr() if values is not None else None,
                                          tags.data_ptr() if tags is not None else None, keys.numel(), world,
@@ -430,20 +433,20 @@ class Table:
                                          recv_cap, _stream_ptr(stream)), "dyc_route_push")
 
     @staticmethod
-    def route_unpack(recs_ptr: int, n: int, keys, values=None, tags=None, stream=None):
-        """Records at device address recs_ptr -> keys[:n] (and values / tags)."""
-        L.check(L.load_library().dyc_route_unpack(recs_ptr, n, keys.data_ptr(),
-                                                  values.data_ptr() if values is not None else None,
-                                                  tags.data_ptr() if tags is not None else None,
-                                                  _stream_ptr(stream)), "dyc_route_unpack")
+    def recv_views(buf: "PeerBuffer", cap: int, m: int):
+        """(keys, values, tags) views of the first m received ops of a receive
+        buffer of capacity cap (keys @0, values @4cap, meta @8cap, tags @16cap)."""
+        torch = _torch()
+        return (buf.tensor(m, torch.int32, 0), buf.tensor(m, torch.int32, 4 * cap),
+                buf.tensor(m, torch.uint8, 16 * cap))
 
     @staticmethod
-    def route_reply(recs_ptr: int, n: int, world: int, vals=None, status=None, out_val_ptrs=None,
+    def route_reply(recv_ptr: int, recv_cap: int, n: int, world: int, vals=None, status=None, out_val_ptrs=None,
                     out_status_ptrs=None, stream=None):
-        """Combine (dyc_route_reply): result j goes to its requester's result
-        arrays (device addresses per rank) at the op's index."""
+        """Combine (dyc_route_reply): result j of the receive buffer at recv_ptr
+        goes to its requester's result arrays (device addresses per rank)."""
         L.check(L.load_library().dyc_route_reply(
-            recs_ptr, n, vals.data_ptr() if vals is not None else None,
+            recv_ptr, recv_cap, n, vals.data_ptr() if vals is not None else None,
             status.data_ptr() if status is not None else None, world,
             _ptr_array(out_val_ptrs, world) if vals is not None else None,
             _ptr_array(out_status_ptrs, world) if status is not None else None,

@@ -1,10 +1,10 @@
 """Fused routing over peer memory (S11): dyc_route_push (hash,
-reserve, store records into the owners' receive buffers) and dyc_route_reply
+reserve, store ops into the owners' receive buffers) and dyc_route_reply
 (results stored at the op's index in the requester's arrays).
 
 1. G virtual shards on one GPU: every "rank" pushes its slice of a batch into
-   all G receive buffers (local pointers), every owner runs its records as one
-   batch and replies; per-op results and the union of the shards' contents
+   all G receive buffers (local pointers), every owner runs its received ops as
+   one batch in place and replies; per-op results and the union of the shards' contents
    must equal the single-table oracle (ops on different keys never interact).
 2. Two processes on cuda:0 (gloo process group): DistTable(p2p=True) with the
    receive/result buffers mapped through real CUDA IPC handles.
@@ -34,7 +34,7 @@ def virtual_batch(shards, op, keys, vals=None, tags=None, n_out=2):
     n = keys.numel()
     cuts = [n * r // G for r in range(G + 1)]
     cap = n + 1
-    recv = [PeerBuffer(16 * cap) for _ in range(G)]
+    recv = [PeerBuffer(17 * cap) for _ in range(G)]
     cnt = [PeerBuffer(8) for _ in range(G)]
     out_v = torch.full((n,), 7, dtype=torch.int32, device="cuda")
     out_s = torch.full((n,), 9, dtype=torch.uint8, device="cuda")
@@ -52,10 +52,9 @@ def virtual_batch(shards, op, keys, vals=None, tags=None, n_out=2):
         sp = [out_s.data_ptr() + cuts[r] for r in range(G)]
         for s in range(G):
             m = counts[s]
-            k = torch.empty(m, dtype=torch.int32, device="cuda")
-            v = torch.empty(m, dtype=torch.int32, device="cuda") if vals is not None else None
-            t = torch.empty(m, dtype=torch.uint8, device="cuda") if tags is not None else None
-            Table.route_unpack(recv[s].ptr, m, k, v, t)
+            k, v, t = Table.recv_views(recv[s], cap, m)
+            v = v if vals is not None else None
+            t = t if tags is not None else None
             # every record routed here hashes to this shard
             if m:
                 dest = shards[s].route_count(k, G).cpu().numpy()
@@ -63,9 +62,10 @@ def virtual_batch(shards, op, keys, vals=None, tags=None, n_out=2):
             res = op(shards[s], k, v, t)
             res = res if isinstance(res, tuple) else (res,)
             if n_out == 1:
-                Table.route_reply(recv[s].ptr, m, G, status=res[0], out_status_ptrs=sp)
+                Table.route_reply(recv[s].ptr, cap, m, G, status=res[0], out_status_ptrs=sp)
             else:
-                Table.route_reply(recv[s].ptr, m, G, vals=res[0], status=res[1], out_val_ptrs=vp, out_status_ptrs=sp)
+                Table.route_reply(recv[s].ptr, cap, m, G, vals=res[0], status=res[1], out_val_ptrs=vp,
+                                  out_status_ptrs=sp)
         torch.cuda.synchronize()
     finally:
         for b in recv + cnt:
@@ -122,7 +122,7 @@ def test_p2p_push_overflow_is_detected():
     """Records past recv_cap are dropped and the counter still counts them."""
     sh = Table(d=4, init_capacity=1024, seed=SEED)
     keys = dev(W.key_range(0, 5000, 3))
-    recv, cnt = PeerBuffer(16 * 100), PeerBuffer(8)
+    recv, cnt = PeerBuffer(17 * 100), PeerBuffer(8)
     try:
         sh.route_push(keys, None, 1, 0, [recv.ptr], [cnt.ptr], 100)
         torch.cuda.synchronize()
