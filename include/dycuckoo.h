@@ -111,6 +111,8 @@ typedef struct {
     uint64_t bytes_cached;            /* released buffers kept for reuse (dyc_trim frees them) */
     uint64_t n_live_resize;           /* resizes committed through dyc_resize_begin/commit */
     uint64_t n_deferred;              /* ops deferred because their subtable was being resized */
+    uint64_t n_device_alloc;          /* cudaMalloc calls (buffers not served by the cache) */
+    double   alloc_ms;                /* host milliseconds spent inside those cudaMalloc calls */
 } dyc_stats_t;
 
 /* Fills *cfg with the defaults: d=4, B=8, alpha=0.3, beta=0.85 (Table

@@ -10,6 +10,7 @@
 //           whose residuals needed a failure upsize ends the loop, Q17b).
 // All comparisons are `(double)m <op> bound*(double)N` on the host (Q29).
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -121,6 +122,8 @@ struct dyc_table {
         cudaEvent_t start = nullptr, done = nullptr;
     } rz;
     uint64_t n_live_resize = 0, n_deferred = 0;
+    uint64_t n_device_alloc = 0;
+    double alloc_ms = 0.0;
     // region-binned execution of large batches (dyc_binned.cuh, dyc_set_binning)
     int bin_mode = 0;                      // 0 off (direct kernels), 1 binned whenever eligible
     int bin_rlog2 = 0;                     // log2 buckets per region (0: ~32 MB regions)
@@ -241,12 +244,15 @@ dyc_status dev_alloc(dyc_table* t, void** p, uint64_t bytes, cudaStream_t st) {
             return DYC_OK;
         }
     }
+    const auto t0 = std::chrono::steady_clock::now();
     cudaError_t e = cudaMalloc(p, bytes);
     if (e == cudaErrorMemoryAllocation && !t->cache.empty()) {
         cudaGetLastError();
         trim_cache(t);
         e = cudaMalloc(p, bytes);
     }
+    t->n_device_alloc++;
+    t->alloc_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     if (e != cudaSuccess) {
         cudaGetLastError();
         *p = nullptr;
@@ -403,7 +409,7 @@ dyc_status downsize_launch(dyc_table* t, uint32_t ti, cudaStream_t st) {
     TRY(zero_one(t, C_RESIDUAL, st));
     {
         ProfScope ps(t, DYC_PROF_DOWNSIZE, st);
-        k_downsize<B><<<grid_for(h * B, kThreads * kResU), kThreads, 0, st>>>(t->sub[ti], (unsigned long long*)p,
+        k_downsize<B><<<grid_for(h * B, kThreads * kResUD), kThreads, 0, st>>>(t->sub[ti], (unsigned long long*)p,
                                                                        (uint32_t)h, t->list[0], t->d_ctr);
     }
     CU(cudaGetLastError());
@@ -563,7 +569,7 @@ dyc_status live_begin(dyc_table* t, int direction, int subtable, cudaStream_t st
         r.res[1] = (unsigned long long*)r1;
         CU(cudaMemsetAsync(r.ctr, 0, C_N * 8, rs));
         ProfScope ps(t, DYC_PROF_DOWNSIZE, rs);
-        k_downsize<B><<<grid_for(nn * B, kThreads * kResU), kThreads, 0, rs>>>(t->sub[ti], (unsigned long long*)p,
+        k_downsize<B><<<grid_for(nn * B, kThreads * kResUD), kThreads, 0, rs>>>(t->sub[ti], (unsigned long long*)p,
                                                                        (uint32_t)nn, r.res[0], r.ctr);
     }
     CU(cudaGetLastError());
@@ -1201,6 +1207,8 @@ dyc_status stats_impl(dyc_table* t, dyc_stats_t* out, cudaStream_t st) {
     out->last_insert_evictions = t->last_evict;
     out->n_live_resize = t->n_live_resize;
     out->n_deferred = t->n_deferred;
+    out->n_device_alloc = t->n_device_alloc;
+    out->alloc_ms = t->alloc_ms;
     return DYC_OK;
 }
 

@@ -681,7 +681,14 @@ __global__ void __launch_bounds__(kThreads) k_apply(TableView tv, const unsigned
 // HBM), the two new buckets are assembled in a per-warp shared-memory tile, and
 // lane s then writes slot s of both, so every store instruction of a warp covers
 // 256 contiguous bytes.
-constexpr int kResU = 4;
+#ifndef DYC_RES_U_UP
+#define DYC_RES_U_UP 4
+#endif
+#ifndef DYC_RES_U_DOWN
+#define DYC_RES_U_DOWN 4
+#endif
+constexpr int kResU = DYC_RES_U_UP;      // slots per thread per pass, upsize
+constexpr int kResUD = DYC_RES_U_DOWN;   // new slots per thread per pass, downsize
 
 template <int B>
 __global__ void __launch_bounds__(kThreads) k_upsize(const unsigned long long* __restrict__ old_s,
@@ -740,23 +747,30 @@ __global__ void __launch_bounds__(kThreads) k_downsize(const unsigned long long*
                                                        unsigned long long* __restrict__ ctr) {
     static_assert(B <= 32 && (32 % B) == 0, "bucket must divide a warp");
     __shared__ unsigned long long tile[kThreads / 32][32];
+    // residuals of one pass are gathered per block and appended with ONE
+    // global atomic (a per-warp append put ~0.4M atomics on one counter)
+    __shared__ unsigned long long s_res[kThreads * kResUD];
+    __shared__ unsigned s_nres;
+    __shared__ unsigned long long s_gbase;
+    if (threadIdx.x == 0) s_nres = 0;
+    __syncthreads();
     const uint64_t total = (uint64_t)h * B;
     const unsigned lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const unsigned gbase = lane & ~(unsigned)(B - 1);
     const unsigned gmask = (B == 32) ? kFull : (((1u << B) - 1u) << gbase);
     const unsigned lt = lanemask_lt() & gmask;
     unsigned long long nres = 0;
-    for (uint64_t base = (uint64_t)blockIdx.x * kThreads * kResU; base < total;
-         base += (uint64_t)gridDim.x * kThreads * kResU) {
-        unsigned long long e1[kResU], e2[kResU];
+    for (uint64_t base = (uint64_t)blockIdx.x * kThreads * kResUD; base < total;
+         base += (uint64_t)gridDim.x * kThreads * kResUD) {
+        unsigned long long e1[kResUD], e2[kResUD];
 #pragma unroll
-        for (int u = 0; u < kResU; u++) {
+        for (int u = 0; u < kResUD; u++) {
             const uint64_t g = base + (uint64_t)u * kThreads + threadIdx.x;
             e1[u] = g < total ? __ldcs(old_s + g) : kEmptySlot;
             e2[u] = g < total ? __ldcs(old_s + g + total) : kEmptySlot;
         }
 #pragma unroll
-        for (int u = 0; u < kResU; u++) {
+        for (int u = 0; u < kResUD; u++) {
             const uint64_t g = base + (uint64_t)u * kThreads + threadIdx.x;
             const bool o1 = key_of(e1[u]) != kEmptyKey, o2 = key_of(e2[u]) != kEmptyKey;
             const unsigned m1 = __ballot_sync(kFull, o1) & gmask;
@@ -773,8 +787,22 @@ __global__ void __launch_bounds__(kThreads) k_downsize(const unsigned long long*
             __syncwarp();
             if (g < total) __stcs(new_s + g, v);
             nres += res;
-            warp_append(res, e2[u], residual, ctr + C_RESIDUAL);
+            const unsigned rb = __ballot_sync(kFull, res);
+            unsigned wb = 0;
+            if (rb && lane == 0) wb = atomicAdd(&s_nres, (unsigned)__popc(rb));
+            wb = __shfl_sync(kFull, wb, 0);
+            if (res) s_res[wb + __popc(rb & lanemask_lt())] = e2[u];
         }
+        __syncthreads();
+        const unsigned nb = s_nres;
+        if (nb) {
+            if (threadIdx.x == 0) s_gbase = atomicAdd(ctr + C_RESIDUAL, (unsigned long long)nb);
+            __syncthreads();
+            for (unsigned i = threadIdx.x; i < nb; i += kThreads) residual[s_gbase + i] = s_res[i];
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) s_nres = 0;
+        __syncthreads();
     }
     block_add<kThreads>(ctr + C_RES_TOTAL, nres);
 }

@@ -463,7 +463,7 @@ def bench_c5(args, rank, world, local, metric, ClockSampler):
                   "found_in_mixed": int(checks[1]), "expected_found": len(mixed) * (batch // 4),
                   "inserted_in_mixed": int(checks[2]), "expected_inserted_in_mixed": int(exp_mixed[0]),
                   "deleted_in_mixed": int(checks[3]), "expected_deleted_in_mixed": int(exp_mixed[1])},
-        "shard0": {"fill": st["fill"], "buckets": st["buckets"], "m": st["m"], "n_upsize": st["n_upsize"],
+        "shard0": {"fill": st["fill"], "buckets": st["buckets"], "m": st["m"], "n_upsize": st["n_upsize"], "n_device_alloc": st["n_device_alloc"], "alloc_ms": st["alloc_ms"],
                    "n_downsize": st["n_downsize"], "bytes": st["bytes_allocated"]},
         "kernel_ms_rank0": {k: round(v[0], 2) for k, v in prof.items() if v[1]},
         "kernel_calls_rank0": {k: v[1] for k, v in prof.items() if v[1]},

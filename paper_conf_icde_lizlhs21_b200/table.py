@@ -312,7 +312,8 @@ class Table:
                     bytes_allocated=s.bytes_allocated, last_insert_new=s.last_insert_new,
                     last_insert_pending=s.last_insert_pending,
                     last_insert_evictions=s.last_insert_evictions, bytes_cached=s.bytes_cached,
-                    n_live_resize=s.n_live_resize, n_deferred=s.n_deferred)
+                    n_live_resize=s.n_live_resize, n_deferred=s.n_deferred,
+                    n_device_alloc=s.n_device_alloc, alloc_ms=s.alloc_ms)
 
     def dump(self, stream=None):
         """(kv uint64, table uint32, bucket uint64) host arrays, unspecified order."""
