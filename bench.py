@@ -240,8 +240,9 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
         "k_delete": n_del * (reads_delete * bkt + sec + 9),
         # upsize: stream the subtable in (8 B/slot) and twice its size out (16 B/slot)
         "k_upsize": slots_sub * 24,
-        # downsize: stream twice the new size in, the new size out
-        "k_downsize": slots_sub * 12,
+        # downsize of the subtable the step doubled: 2*slots_sub slots in (16 B
+        # per new slot), slots_sub out (8 B)
+        "k_downsize": slots_sub * 24,
     }
     kern = {k: prof[k][0] / args.steps for k in bytes_alg if prof[k][1]}
     dom = max(kern, key=kern.get)
