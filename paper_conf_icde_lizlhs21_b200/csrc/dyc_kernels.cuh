@@ -691,7 +691,7 @@ constexpr int kResU = DYC_RES_U_UP;      // slots per thread per pass, upsize
 constexpr int kResUD = DYC_RES_U_DOWN;   // new slots per thread per pass, downsize
 
 template <int B>
-__global__ void __launch_bounds__(kThreads) k_upsize(const unsigned long long* __restrict__ old_s,
+__global__ void __launch_bounds__(kThreads, 8) k_upsize(const unsigned long long* __restrict__ old_s,
                                                      unsigned long long* __restrict__ new_s, uint32_t n_old,
                                                      uint32_t a, uint32_t b, uint64_t magic2, uint32_t n2) {
     static_assert(B <= 32 && (32 % B) == 0, "bucket must divide a warp");

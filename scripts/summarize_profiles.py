@@ -126,7 +126,7 @@ def main(tag):
     md += ["", "## Roofline of the bench line", "",
            f"- Dominant kernel: `{r['kernel']}`, {r['launch_ms']:.3f} ms per launch.",
            f"- Achieved: {r['achieved']:.0f} GB/s of algorithmic bytes.",
-           f"  - That is {r['frac']:.3f} of the measured 6454 GB/s copy peak.",
+           f"  - That is {r['frac']:.3f} of the measured {r['peak']:.0f} GB/s copy peak.",
            f"  - It is {r['frac_of_random_ceiling']:.3f} of the live random-bucket ceiling "
            f"({r['random_bucket_ceiling']['gbs']:.0f} GB/s = {r['random_bucket_ceiling']['gprobes_per_s']:.1f} G bucket reads/s).",
            f"- Traffic (ncu `dram__bytes_read.sum + dram__bytes_write.sum` per launch): "
