@@ -817,8 +817,9 @@ def bench_stream(args, local):
         run()
     torch.cuda.synchronize()
     rec = []
-    g.profile(True)
     g.launch_count(reset=True)
+    # the timed pass runs without the library's per-kernel event scopes; the
+    # kernel times come from a separate profiled replay below
     with ClockSampler(local) as clk:
         a = torch.cuda.Event(enable_timing=True)
         b = torch.cuda.Event(enable_timing=True)
@@ -842,6 +843,23 @@ def bench_stream(args, local):
         torch.cuda.synchronize()
     total_ms = a.elapsed_time(b)
     launches = g.launch_count()
+    g.clear()
+    g.profile(True)
+    run_profiled_ms = None
+    pa, pb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    pa.record(stream)
+    for op, ops, k, v in staged:
+        if op == "insert":
+            g.insert(k, v)
+        elif op == "find":
+            g.find(k)
+        elif op == "delete":
+            g.delete(k)
+        else:
+            g.mixed(ops, k, v)
+    pb.record(stream)
+    torch.cuda.synchronize()
+    run_profiled_ms = pa.elapsed_time(pb)
     prof = g.profile_read()
     g.profile(False)
     per = {"insert": [0, 0.0], "find": [0, 0.0], "delete": [0, 0.0], "mixed": [0, 0.0]}
@@ -878,6 +896,8 @@ def bench_stream(args, local):
         "table_bytes": {"max": max(mem), "final": mem[-1]},
         "resizes": {k: st[k] for k in ("n_upsize", "n_downsize", "n_fail_upsize", "n_residual")},
         "kernel_ms": {k: round(v[0], 3) for k, v in prof.items() if v[1]},
+        "kernel_ms_source": "separate replay with the library's per-kernel event scopes on "
+                            f"(that pass: {run_profiled_ms:.2f} ms; the timed pass runs without them)",
         "kernel_calls": {k: v[1] for k, v in prof.items() if v[1]},
         "gpu_launches": launches, "clocks": clk.summary(), "generator_seconds": gen_s,
         "roofline": None, "cpu_baseline": None, "e2e": None,
