@@ -34,7 +34,7 @@ class DistTable:
     `chunks` (collectives are issued in the same order everywhere)."""
 
     def __init__(self, shard, group=None, force_route: bool = False, chunks: int = 4, p2p: bool = False,
-                 max_ops: Optional[int] = None):
+                 max_ops: Optional[int] = None, p2p_buffers=None, p2p_sync=None):
         import torch.distributed as dist
         self.force_route = force_route
         self.dist = dist
@@ -48,7 +48,7 @@ class DistTable:
         if p2p:
             if not max_ops:
                 raise ValueError("p2p routing needs max_ops (the largest batch any rank issues)")
-            self.p2p = PeerRouter(self, int(max_ops))
+            self.p2p = PeerRouter(self, int(max_ops), buffer_factory=p2p_buffers, sync=p2p_sync)
 
     # ------------------------------------------------------------ exchange
     def _a2a(self, x, send_splits, recv_splits, async_op=False):
@@ -184,16 +184,21 @@ class PeerRouter:
     used; the barriers are host barriers of the process group after a stream
     sync (they order the peer stores, which complete with their kernels)."""
 
-    def __init__(self, dt, max_ops: int):
+    def __init__(self, dt, max_ops: int, buffer_factory=None, sync=None):
+        """buffer_factory(nbytes) -> a PeerBuffer-like object and sync() (the
+        stream sync before each barrier) default to table.PeerBuffer and a CUDA
+        stream sync; the CPU tests inject shared-memory stand-ins."""
         import torch
-        from .table import PeerBuffer
+        if buffer_factory is None:
+            from .table import PeerBuffer as buffer_factory
+        self._sync = sync if sync is not None else (lambda: torch.cuda.current_stream().synchronize())
         self.dt, self.max_ops = dt, max_ops
         W, r = dt.world, dt.rank
         self.cap = W * max_ops
-        self.recv = PeerBuffer(17 * self.cap)          # DYC_ROUTE_RECV_BYTES: keys | values | meta | tags
-        self.cnt = PeerBuffer(8)
-        self.rv = PeerBuffer(4 * max_ops)
-        self.rs = PeerBuffer(max_ops)
+        self.recv = buffer_factory(17 * self.cap)      # DYC_ROUTE_RECV_BYTES: keys | values | meta | tags
+        self.cnt = buffer_factory(8)
+        self.rv = buffer_factory(4 * max_ops)
+        self.rs = buffer_factory(max_ops)
         bufs = (self.recv, self.cnt, self.rv, self.rs)
         mine = [b.handle() for b in bufs]
         allh = [None] * W
@@ -206,12 +211,10 @@ class PeerRouter:
         self._barrier()
 
     def _barrier(self):
-        import torch
-        torch.cuda.current_stream().synchronize()
+        self._sync()
         self.dt.dist.barrier(group=self.dt.group)
 
     def run(self, op, keys, values, n_out, begin, end, tags):
-        from .table import Table
         dt = self.dt
         n = keys.numel()
         if n > self.max_ops:
@@ -222,7 +225,7 @@ class PeerRouter:
         if m > self.cap:
             raise RuntimeError(f"receive buffer overflow: {m} records > {self.cap}")
         dt.last_recv = m
-        k, v, t = Table.recv_views(self.recv, self.cap, m)       # the owner's batch, in place
+        k, v, t = dt.shard.recv_views(self.recv, self.cap, m)    # the owner's batch, in place
         v = v if values is not None else None
         t = t if tags is not None else None
         if begin is not None:
@@ -232,16 +235,17 @@ class PeerRouter:
         if end is not None:
             end()
         if n_out == 1:
-            Table.route_reply(self.recv.ptr, self.cap, m, dt.world, status=res[0], out_status_ptrs=self.rs_p)
+            dt.shard.route_reply(self.recv.ptr, self.cap, m, dt.world, status=res[0], out_status_ptrs=self.rs_p)
         else:
-            Table.route_reply(self.recv.ptr, self.cap, m, dt.world, vals=res[0], status=res[1],
-                              out_val_ptrs=self.rv_p, out_status_ptrs=self.rs_p)
+            dt.shard.route_reply(self.recv.ptr, self.cap, m, dt.world, vals=res[0], status=res[1],
+                                 out_val_ptrs=self.rv_p, out_status_ptrs=self.rs_p)
         self.count.zero_()
         self._barrier()
         out_s = self.out_s[:n].clone()
         return out_s if n_out == 1 else (self.out_v[:n].clone(), out_s)
 
     def close(self):
+        self.count = self.out_v = self.out_s = None       # views into the buffers go first
         for b in (self.recv, self.cnt, self.rv, self.rs):
             b.close()
 
