@@ -286,11 +286,16 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
     placed = (n_ins - pend) / max(1, n_ins)
     acc_model = {"k_find": (probes_find, 0.0, n_find), "k_upsert": (reads_upsert, placed, n_ins),
                  "k_delete": (reads_delete, 1.0, n_del)}
-    acc_frac = {}
+    acc_frac, acc_frac_io = {}, {}
+    io_bytes = 9.0            # streamed per op: key 4 in + value 4 in/out + status/flag 1 out
     for k, (r_, w_, units) in acc_model.items():
         if k in kern and kern[k] > 0:
             ceiling = 1.0 / (r_ / R + w_ * cw)
             acc_frac[k] = round(units / (kern[k] * 1e-3) / ceiling, 4)
+            # SURVEY §8(d)'s ceiling: the same random accesses plus the same
+            # streaming IO, the latter at the measured copy bandwidth
+            ceiling_io = 1.0 / (r_ / R + w_ * cw + io_bytes / (peak * 1e9))
+            acc_frac_io[k] = round(units / (kern[k] * 1e-3) / ceiling_io, 4)
     traffic, traffic_src = None, None
     pdir = os.path.join(ROOT, "profiles")
     tr_files = sorted(f for f in os.listdir(pdir) if f.endswith("_traffic.json")) if os.path.isdir(pdir) else []
@@ -316,6 +321,7 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
                            "what": "dyc_bench_gather(_ex): random bucket reads, and reads each followed by a store "
                                    "into the bucket; ceiling(kernel) = 1/(reads/R + writes*(1/M - 1/R))"},
         "frac_of_access_ceiling": acc_frac,
+        "frac_of_access_ceiling_with_io": acc_frac_io,
         "kernel_ms_per_step": {k: round(v, 4) for k, v in kern.items()},
         "other_kernels_ms_per_step": round(prof["other"][0] / args.steps, 4),
         "model": {"phi": phi, "hit_rate": hit_rate, "evictions_per_insert": E, "probes_per_find": probes_find,
