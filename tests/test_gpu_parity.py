@@ -98,18 +98,22 @@ def test_hash_params_match_oracle(oracle_mod):
 
 
 # ------------------------------------------------------------------ configs
-def test_c1_parity_every_batch(oracle_mod):
-    """Config C1 (BASELINE.json configs[0]) end to end; 17 upsizes, 49 downsizes."""
-    g, o = run_parity(oracle_mod, W.c1_rand_small())
+@pytest.mark.parametrize("seed", [None, 0xD7C10001, 0xD7C10002])
+def test_c1_parity_every_batch(oracle_mod, seed):
+    """Config C1 (BASELINE.json configs[0]) end to end, three seeds (SURVEY
+    §8(d): correctness runs use three); 17 upsizes, 49 downsizes (the schedule
+    depends on m only, so on no seed)."""
+    g, o = run_parity(oracle_mod, W.c1_rand_small(seed_cfg=seed))
     s = g.stats()
     assert (s["n_upsize"], s["n_downsize"], s["n_fail_upsize"]) == (17, 49, 0)
     assert s["buckets"] == [1, 1, 1, 1] and s["m"] == 0
 
 
-@pytest.mark.parametrize("log2_n,extra", [(16, 0), (20, 12345)])
-def test_c2_shape_parity(oracle_mod, log2_n, extra):
-    """Config C2's shape at oracle-friendly sizes, with a ragged tail."""
-    wl = W.c2_rand_static(log2_n=log2_n)
+@pytest.mark.parametrize("log2_n,extra,seed", [(16, 0, None), (16, 777, 0xD7C20001), (16, 31, 0xD7C20002),
+                                               (20, 12345, None)])
+def test_c2_shape_parity(oracle_mod, log2_n, extra, seed):
+    """Config C2's shape at oracle-friendly sizes, with a ragged tail; three seeds at 2^16."""
+    wl = W.c2_rand_static(log2_n=log2_n, seed_cfg=seed)
     if extra:
         more = W.key_range(1 << 30, extra, 99)
         b0 = wl.batches[0]
@@ -329,21 +333,23 @@ def test_c2_full_size_sampled(mode):
 
 
 # ------------------------------------------------------------------ dynamic configs
-@pytest.mark.parametrize("shape", ["TW", "RE"])
-def test_c3_dynamic_parity(oracle_mod, shape):
+@pytest.mark.parametrize("shape,seed", [("TW", None), ("RE", None), ("TW", 0xD7C30001), ("RE", 0xD7C30002)])
+def test_c3_dynamic_parity(oracle_mod, shape, seed):
     """Config C3's shape (sliding window, swap pass, two cycles) at small scale:
     up- and downsizes repeat; contents and the resize schedule match every batch."""
-    wl = W.c3_dynamic(scale=0.001, shape=shape, batch=5000, cycles=2, init_capacity=1024)
+    wl = W.c3_dynamic(scale=0.001, shape=shape, batch=5000, cycles=2, init_capacity=1024, seed_cfg=seed)
     g, o = run_parity(oracle_mod, wl, B=8, layout_every=False)
     check_layout(g, o)
     s = g.stats()
     assert s["n_upsize"] > 0 and s["n_downsize"] > 0
 
 
-def test_c4_zipf_mixed_parity(oracle_mod):
+@pytest.mark.parametrize("seed", [None, 0xD7C40001, 0xD7C40002])
+def test_c4_zipf_mixed_parity(oracle_mod, seed):
     """Config C4's shape: Zipf(0.99) mixed 50/30/20 batches through dyc_mixed_batch
-    (reading Q10: find -> insert -> delete), grow then drain, two cycles."""
-    meta, batches = W.c4_zipf_mixed(U=60000, distinct=6000, grow_batches=6, cycles=2, init_capacity=1024)
+    (reading Q10: find -> insert -> delete), grow then drain, two cycles; three seeds."""
+    meta, batches = W.c4_zipf_mixed(U=60000, distinct=6000, grow_batches=6, cycles=2, init_capacity=1024,
+                                    seed_cfg=seed)
     g = Table(d=4, init_capacity=meta.init_capacity, alpha=meta.alpha, beta=meta.beta, bucket_slots=8)
     o = oracle_mod.OracleTable(d=4, init_capacity=meta.init_capacity, alpha=meta.alpha, beta=meta.beta,
                                bucket_slots=8)
