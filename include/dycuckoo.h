@@ -113,6 +113,8 @@ typedef struct {
     uint64_t n_deferred;              /* ops deferred because their subtable was being resized */
     uint64_t n_device_alloc;          /* cudaMalloc calls (buffers not served by the cache) */
     double   alloc_ms;                /* host milliseconds spent inside those cudaMalloc calls */
+    uint64_t n_sync;                  /* counter read-backs: the host waited on the stream (S6) */
+    double   sync_ms;                 /* host milliseconds spent in those waits                */
 } dyc_stats_t;
 
 /* Fills *cfg with the defaults: d=4, B=8, alpha=0.3, beta=0.85 (Table

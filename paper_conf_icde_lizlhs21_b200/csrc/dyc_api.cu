@@ -124,6 +124,8 @@ struct dyc_table {
     uint64_t n_live_resize = 0, n_deferred = 0;
     uint64_t n_device_alloc = 0;
     double alloc_ms = 0.0;
+    uint64_t n_sync = 0;          // counter read-backs (host waits on the stream)
+    double sync_ms = 0.0;
     // region-binned execution of large batches (dyc_binned.cuh, dyc_set_binning)
     int bin_mode = 0;                      // 0 off (direct kernels), 1 binned whenever eligible
     int bin_rlog2 = 0;                     // log2 buckets per region (0: ~32 MB regions)
@@ -287,7 +289,10 @@ void dev_free(dyc_table* t, void* p, cudaStream_t st) {
 
 dyc_status read_ctr(dyc_table* t, cudaStream_t st) {
     CU(cudaMemcpyAsync(t->h_ctr, t->d_ctr, C_N * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+    const auto t0 = std::chrono::steady_clock::now();
     CU(cudaStreamSynchronize(st));
+    t->sync_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    t->n_sync++;
     return DYC_OK;
 }
 
@@ -1209,6 +1214,8 @@ dyc_status stats_impl(dyc_table* t, dyc_stats_t* out, cudaStream_t st) {
     out->n_deferred = t->n_deferred;
     out->n_device_alloc = t->n_device_alloc;
     out->alloc_ms = t->alloc_ms;
+    out->n_sync = t->n_sync;
+    out->sync_ms = t->sync_ms;
     return DYC_OK;
 }
 
