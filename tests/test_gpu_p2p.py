@@ -181,3 +181,36 @@ def test_p2p_two_processes_ipc(tmp_path, oracle_mod):
     s.close()
     mp.spawn(_worker, args=(2, port, 14, str(tmp_path)), nprocs=2, join=True)
     assert (tmp_path / "ok").exists()
+
+
+def test_p2p_entry_points_reject_bad_arguments():
+    """Argument checks of the peer-routing C ABI (include/dycuckoo.h)."""
+    import ctypes as C
+    from paper_conf_icde_lizlhs21_b200 import _lib as L
+    sh = Table(d=4, init_capacity=1024, seed=SEED)
+    keys = dev(W.key_range(0, 100, 5))
+    recv, cnt = PeerBuffer(17 * 128), PeerBuffer(8)
+    lib = L.load_library()
+    try:
+        with pytest.raises(ValueError):                       # pointer list shorter than world
+            sh.route_push(keys, None, 2, 0, [recv.ptr], [cnt.ptr], 128)
+        arr = lambda ps: C.cast((C.c_void_p * len(ps))(*ps), C.c_void_p)  # noqa: E731
+        s = torch.cuda.current_stream().cuda_stream
+        for world in (0, 65):
+            assert lib.dyc_route_push(sh.handle, keys.data_ptr(), None, None, 100, world, 0,
+                                      arr([recv.ptr] * 65), arr([cnt.ptr] * 65), 128, s) == L.DYC_ERR_INVALID_ARG
+        assert lib.dyc_route_push(sh.handle, keys.data_ptr(), None, None, 100, 1, 0, arr([0]), arr([cnt.ptr]),
+                                  128, s) == L.DYC_ERR_INVALID_ARG          # null peer pointer
+        st = torch.zeros(100, dtype=torch.uint8, device="cuda")
+        # a result array without destinations, and n > recv_cap
+        assert lib.dyc_route_reply(recv.ptr, 128, 100, None, st.data_ptr(), 1, None, None, s) == L.DYC_ERR_INVALID_ARG
+        assert lib.dyc_route_reply(recv.ptr, 128, 129, None, st.data_ptr(), 1, None, arr([st.data_ptr()]),
+                                   s) == L.DYC_ERR_INVALID_ARG
+        assert lib.dyc_ipc_alloc(0, C.byref(C.c_void_p())) == L.DYC_ERR_INVALID_ARG
+        assert lib.dyc_ipc_get_handle(None, None) == L.DYC_ERR_INVALID_ARG
+        # n == 0 is a no-op
+        assert lib.dyc_route_push(sh.handle, keys.data_ptr(), None, None, 0, 1, 0, arr([recv.ptr]), arr([cnt.ptr]),
+                                  128, s) == L.DYC_OK
+    finally:
+        recv.close()
+        cnt.close()
