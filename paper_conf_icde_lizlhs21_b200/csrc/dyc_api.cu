@@ -1836,7 +1836,7 @@ dyc_status dyc_route_push(dyc_table* t, const uint32_t* d_keys, const uint32_t* 
     {
         ProfScope ps(t, DYC_PROF_OTHER, S(stream));
         const HashDest hd{t->a[sh], t->b[sh], world, fastmod_magic(world), d_keys};
-        k_route_push<<<std::min<unsigned>(grid_for(n, (uint64_t)kThreads * kPushItems), t->num_sms * 4), kThreads,
+        k_route_push<<<std::min<unsigned>(grid_for(n, (uint64_t)kThreads * kPushItems), t->num_sms * DYC_PUSH_BPS), kThreads,
                        0, S(stream)>>>(hd, d_vals, d_tags, n, world, src_rank, rp, cp, recv_cap);
     }
     CU(cudaGetLastError());

@@ -868,11 +868,29 @@ __global__ void k_hash_probe(TableView tv, const uint32_t* __restrict__ keys, ui
 // the batch even when G is 1.
 constexpr int kTileItems = 8;
 
+// Warp-aggregated shared-memory counter increment: the lanes of a warp that
+// share a destination are grouped with __match_any_sync and their leader adds
+// the group's size with ONE atomic; each lane gets its rank inside the
+// destination.  (One atomic per lane on a shared counter serialises 32-way
+// when every op has the same destination: G = 1, or an op-code split.)
+// Every lane of the warp must call it; lanes with valid == false take no slot.
+__device__ __forceinline__ unsigned warp_rank_add(unsigned* counters, uint32_t d, bool valid) {
+    const uint32_t key = valid ? d : 0xFFFFFFFFu;
+    const unsigned peers = __match_any_sync(kFull, key);
+    const unsigned leader = __ffs(peers) - 1;
+    const unsigned lane = threadIdx.x & 31;
+    unsigned b = 0;
+    if (valid && lane == leader) b = atomicAdd(&counters[d], (unsigned)__popc(peers));
+    b = __shfl_sync(kFull, b, leader);
+    return b + __popc(peers & ((1u << lane) - 1u));
+}
+
 struct HashDest {
     uint32_t a, b, world;
     uint64_t magic;
     const uint32_t* keys;
     __device__ __forceinline__ uint32_t operator()(uint64_t i) const { return fastmod(hx(a, b, keys[i]), magic, world); }
+    __device__ __forceinline__ uint32_t of_key(uint32_t k) const { return fastmod(hx(a, b, k), magic, world); }
 };
 struct OpDest {
     const uint8_t* ops;
@@ -893,7 +911,7 @@ __global__ void __launch_bounds__(kThreads) k_group_count(Dest dest, uint64_t n,
 #pragma unroll
         for (int j = 0; j < IT; j++) {
             const uint64_t i = b0 + (uint64_t)j * kThreads + threadIdx.x;
-            if (i < n) atomicAdd(&mine[dest(i)], 1u);
+            warp_rank_add(mine, i < n ? dest(i) : 0u, i < n);
         }
     }
     __syncthreads();
@@ -927,7 +945,7 @@ __global__ void __launch_bounds__(kThreads) k_group_scatter(Dest dest, const uin
         for (int j = 0; j < kTileItems; j++) {
             const uint64_t i = t0 + (uint64_t)j * kThreads + threadIdx.x;
             dd[j] = i < n ? dest(i) : 0xFFFFFFFFu;
-            rk[j] = i < n ? atomicAdd(&cnt[dd[j]], 1u) : 0u;  // rank within (tile, dest)
+            rk[j] = warp_rank_add(cnt, dd[j], i < n);           // rank within (tile, dest)
         }
         __syncthreads();
         for (uint32_t w = threadIdx.x; w < world; w += blockDim.x)
@@ -1007,6 +1025,12 @@ struct PeerPtrs {
     void* p[kMaxPeers];
 };
 constexpr int kPushItems = 8;                    // ops per thread per tile (tile = 2048 ops)
+#ifndef DYC_PUSH_ATOMIC
+#define DYC_PUSH_ATOMIC atomicAdd_system
+#endif
+#ifndef DYC_PUSH_BPS
+#define DYC_PUSH_BPS 4                           // resident push blocks per SM (persistent grid)
+#endif
 
 // Each block takes a tile of 2048 ops: it hashes them to their shards, ranks
 // them per shard in shared memory and stages them there grouped by shard; it
@@ -1024,7 +1048,26 @@ __global__ void __launch_bounds__(kThreads) k_route_push(HashDest dest, const ui
     __shared__ uint8_t s_tag[T], s_dst[T];
     __shared__ unsigned cnt[kMaxPeers], off[kMaxPeers + 1];
     __shared__ unsigned long long base[kMaxPeers];
-    for (uint64_t t0 = (uint64_t)blockIdx.x * T; t0 < n; t0 += (uint64_t)gridDim.x * T) {
+    // the tile's keys, values and op codes are loaded into registers in one go,
+    // and the next tile's loads are issued before the current tile is copied
+    // out, so each tile exposes at most one memory latency
+    uint32_t kk[kPushItems], vv[kPushItems];
+    uint8_t tg[kPushItems];
+    auto load_tile = [&](uint64_t t0) {
+        const unsigned nt = t0 < n ? (unsigned)((n - t0) < (uint64_t)T ? (n - t0) : (uint64_t)T) : 0u;
+#pragma unroll
+        for (int j = 0; j < kPushItems; j++) {
+            const unsigned li = j * kThreads + threadIdx.x;
+            const bool ok = li < nt;
+            kk[j] = ok ? __ldcs(dest.keys + t0 + li) : 0u;
+            vv[j] = (ok && vals) ? __ldcs(vals + t0 + li) : 0u;
+            tg[j] = (ok && tags) ? tags[t0 + li] : (uint8_t)0;
+        }
+    };
+    const uint64_t stride = (uint64_t)gridDim.x * T;
+    uint64_t t0 = (uint64_t)blockIdx.x * T;
+    if (t0 < n) load_tile(t0);
+    for (; t0 < n; t0 += stride) {
         const unsigned nt = (unsigned)((n - t0) < (uint64_t)T ? (n - t0) : (uint64_t)T);
         for (uint32_t w = threadIdx.x; w < world; w += blockDim.x) cnt[w] = 0;
         __syncthreads();
@@ -1032,8 +1075,8 @@ __global__ void __launch_bounds__(kThreads) k_route_push(HashDest dest, const ui
 #pragma unroll
         for (int j = 0; j < kPushItems; j++) {
             const unsigned li = j * kThreads + threadIdx.x;
-            dd[j] = li < nt ? dest(t0 + li) : 0xFFFFFFFFu;
-            rk[j] = li < nt ? atomicAdd(&cnt[dd[j]], 1u) : 0u;
+            dd[j] = li < nt ? dest.of_key(kk[j]) : 0xFFFFFFFFu;
+            rk[j] = warp_rank_add(cnt, dd[j], li < nt);
         }
         __syncthreads();
         if (threadIdx.x == 0) {
@@ -1042,7 +1085,7 @@ __global__ void __launch_bounds__(kThreads) k_route_push(HashDest dest, const ui
             off[world] = acc;
         }
         for (uint32_t w = threadIdx.x; w < world; w += blockDim.x)
-            base[w] = cnt[w] ? atomicAdd_system((unsigned long long*)recv_count.p[w], (unsigned long long)cnt[w])
+            base[w] = cnt[w] ? DYC_PUSH_ATOMIC((unsigned long long*)recv_count.p[w], (unsigned long long)cnt[w])
                              : 0ull;
         __syncthreads();
 #pragma unroll
@@ -1050,15 +1093,15 @@ __global__ void __launch_bounds__(kThreads) k_route_push(HashDest dest, const ui
             const unsigned li = j * kThreads + threadIdx.x;
             if (li < nt) {
                 const unsigned p = off[dd[j]] + rk[j];
-                const uint64_t i = t0 + li;
-                s_key[p] = dest.keys[i];
-                s_val[p] = vals ? vals[i] : 0u;
-                s_idx[p] = (uint32_t)i;
-                s_tag[p] = tags ? tags[i] : 0u;
+                s_key[p] = kk[j];
+                s_val[p] = vv[j];
+                s_idx[p] = (uint32_t)(t0 + li);
+                s_tag[p] = tg[j];
                 s_dst[p] = (uint8_t)dd[j];
             }
         }
         __syncthreads();
+        if (t0 + stride < n) load_tile(t0 + stride);          // in flight during the copy-out
         for (unsigned p = threadIdx.x; p < nt; p += kThreads) {
             const uint32_t w = s_dst[p];
             const uint64_t g = base[w] + (p - off[w]);
