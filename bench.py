@@ -824,6 +824,7 @@ def bench_stream(args, local):
     torch.cuda.synchronize()
     rec = []
     g.launch_count(reset=True)
+    st_before = g.stats()
     # the timed pass runs without the library's per-kernel event scopes; the
     # kernel times come from a separate profiled replay below
     with ClockSampler(local) as clk:
@@ -849,6 +850,12 @@ def bench_stream(args, local):
         torch.cuda.synchronize()
     total_ms = a.elapsed_time(b)
     launches = g.launch_count()
+    st_timed = g.stats()
+    resizes = {k: st_timed[k] - st_before[k] for k in ("n_upsize", "n_downsize", "n_fail_upsize", "n_residual")}
+    host_waits = {"n_sync": st_timed["n_sync"] - st_before["n_sync"],
+                  "sync_ms": round(st_timed["sync_ms"] - st_before["sync_ms"], 3),
+                  "n_device_alloc": st_timed["n_device_alloc"] - st_before["n_device_alloc"],
+                  "alloc_ms": round(st_timed["alloc_ms"] - st_before["alloc_ms"], 3)}
     g.clear()
     g.profile(True)
     run_profiled_ms = None
@@ -900,7 +907,8 @@ def bench_stream(args, local):
         "fill_track": {"min_after_mutation": min(x for x, (op, *_r) in zip(track, staged) if op != "find"),
                        "max": max(track), "final": track[-1], "every_batch": track if len(track) <= 400 else None},
         "table_bytes": {"max": max(mem), "final": mem[-1]},
-        "resizes": {k: st[k] for k in ("n_upsize", "n_downsize", "n_fail_upsize", "n_residual")},
+        "resizes": resizes,
+        "host_waits_timed_pass": host_waits,
         "kernel_ms": {k: round(v[0], 3) for k, v in prof.items() if v[1]},
         "kernel_ms_source": "separate replay with the library's per-kernel event scopes on "
                             f"(that pass: {run_profiled_ms:.2f} ms; the timed pass runs without them)",

@@ -1328,8 +1328,15 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
     t->cfg = *cfg;
     cudaGetDevice(&t->device);
     cudaDeviceGetAttribute(&t->num_sms, cudaDevAttrMultiProcessorCount, t->device);
+    // persistent k_place grid: exactly one wave of the instance this table
+    // launches (the register count, hence the residency, depends on B)
     int occ = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_place<4>, kThreads, 0);
+    switch (cfg->bucket_slots) {
+        case 4: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_place<4>, kThreads, 0); break;
+        case 8: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_place<8>, kThreads, 0); break;
+        case 16: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_place<16>, kThreads, 0); break;
+        default: cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_place<32>, kThreads, 0); break;
+    }
     t->place_blocks = t->num_sms * std::max(1, occ);
     uint64_t st = cfg->seed;
     for (uint32_t s = 0; s < d + 2; s++) {

@@ -117,17 +117,30 @@ dyc_status w_ensure_lists(dyw_table* t, uint64_t n, cudaStream_t st) {
     return DYC_OK;
 }
 
+// Persistent grid of exactly one wave for kernel `k` (its residency depends on
+// its register count; a grid past one wave leaves a partial second wave).
+template <class K>
+unsigned w_one_wave(K k, int sms) {
+    int occ = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k, dyw::kThreads, 0);
+    return (unsigned)(sms * std::max(1, occ));
+}
+
 template <int L, int W>
 dyc_status w_launch_place(dyw_table* t, const dyw::KVList& src, const u64* d_count, uint64_t h_count,
                           const dyw::KVList& fail, cudaStream_t st) {
     t->launches++;
-    const unsigned grid = (unsigned)(t->num_sms * 8);
     if (L == dyw::PACK) {
-        if (W == 1) dyw::k_wplace_lockfree<<<grid, dyw::kThreads, 0, st>>>(t->view(), src, d_count, h_count, fail, t->d_ctr);
+        if (W == 1) {
+            static const unsigned g = w_one_wave(dyw::k_wplace_lockfree, t->num_sms);
+            dyw::k_wplace_lockfree<<<g, dyw::kThreads, 0, st>>>(t->view(), src, d_count, h_count, fail, t->d_ctr);
+        }
     } else if (t->cfg.mode == DYW_MODE_VOTER) {
-        dyw::k_wplace_voter<W><<<grid, dyw::kThreads, 0, st>>>(t->view(), src, d_count, h_count, fail, t->d_ctr);
+        static const unsigned g = w_one_wave(dyw::k_wplace_voter<W>, t->num_sms);
+        dyw::k_wplace_voter<W><<<g, dyw::kThreads, 0, st>>>(t->view(), src, d_count, h_count, fail, t->d_ctr);
     } else {
-        dyw::k_wplace_grouped<W><<<grid, dyw::kThreads, 0, st>>>(t->view(), src, d_count, h_count, fail, t->d_ctr);
+        static const unsigned g = w_one_wave(dyw::k_wplace_grouped<W>, t->num_sms);
+        dyw::k_wplace_grouped<W><<<g, dyw::kThreads, 0, st>>>(t->view(), src, d_count, h_count, fail, t->d_ctr);
     }
     CU(cudaGetLastError());
     return DYC_OK;
