@@ -228,7 +228,9 @@ dyc_status dyc_resize_query(const dyc_table* t, int* in_flight, int* kernel_done
 
 /* Returns the buffers the table keeps for reuse (released subtables after a
  * resize, old scratch) to the device.  Resizing frees a subtable's old buffer
- * into this cache, so up/down cycles do not pay cudaMalloc each time. */
+ * into this cache, so up/down cycles do not pay cudaMalloc each time.  The
+ * cache holds at most the table's high-water size + 256 MB (oldest buffers are
+ * freed first beyond that). */
 dyc_status dyc_trim(dyc_table* t);
 
 /* Empties the table without resizing (all slots EMPTY, m = 0). */

@@ -124,6 +124,7 @@ struct dyc_table {
     uint64_t n_live_resize = 0, n_deferred = 0;
     uint64_t n_device_alloc = 0;
     double alloc_ms = 0.0;
+    uint64_t peak_table_bytes = 0;   // high-water mark of the subtables' bytes (cache cap)
     uint64_t n_sync = 0;          // counter read-backs (host waits on the stream)
     double sync_ms = 0.0;
     // region-binned execution of large batches (dyc_binned.cuh, dyc_set_binning)
@@ -276,8 +277,15 @@ void dev_free(dyc_table* t, void* p, cudaStream_t st) {
     cudaEventRecord(ev, st);
     t->cache.push_back({p, bytes, ev});
     t->cache_bytes += bytes;
-    uint64_t cap = 256ull << 20;
-    for (uint32_t i = 0; i < t->cfg.d; i++) cap += t->nb[i] * t->cfg.bucket_slots * 8;
+    // keep up to the table's high-water size (+256 MB) cached, not just its
+    // current size: a shrink phase would otherwise free (cudaFree syncs the
+    // device) exactly the buffers the next growth phase allocates again, and
+    // fresh cudaMalloc calls are where the stream configs' run-to-run variance
+    // came from (profiles/r1t_c5_variance.md).  dyc_trim releases the cache.
+    uint64_t cur = 0;
+    for (uint32_t i = 0; i < t->cfg.d; i++) cur += t->nb[i] * t->cfg.bucket_slots * 8;
+    t->peak_table_bytes = std::max(t->peak_table_bytes, cur);
+    const uint64_t cap = (256ull << 20) + t->peak_table_bytes;
     while (t->cache_bytes > cap && !t->cache.empty()) {      // oldest first
         cudaEventSynchronize(t->cache.front().ev);
         cudaFree(t->cache.front().p);
