@@ -299,6 +299,9 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
     traffic, traffic_src = None, None
     pdir = os.path.join(ROOT, "profiles")
     tr_files = sorted(f for f in os.listdir(pdir) if f.endswith("_traffic.json")) if os.path.isdir(pdir) else []
+    latest = os.path.join(pdir, "traffic_latest.json")
+    if os.path.exists(latest):
+        tr_files = [json.load(open(latest))["file"]]
     # the captured traffic is per launch of the unchunked C2 kernel: only comparable
     # when the timed path launches the dominant kernel once per step (not routed)
     if tr_files and args.log2n == 27 and args.bucket_slots == 8 and n_ins == (1 << 27) and calls == 1:

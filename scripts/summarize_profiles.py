@@ -137,6 +137,8 @@ def main(tag):
            ""]
     open(os.path.join(PROF, f"{tag}_summary.md"), "w").write("\n".join(md) + "\n")
     json.dump({k: v for k, v in traffic.items()}, open(os.path.join(PROF, f"{tag}_traffic.json"), "w"), indent=1)
+    # the pass bench.py reads its roofline traffic from (tag names do not sort by date)
+    json.dump({"tag": tag, "file": f"{tag}_traffic.json"}, open(os.path.join(PROF, "traffic_latest.json"), "w"), indent=1)
     print("\n".join(md))
 
 
