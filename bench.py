@@ -57,7 +57,7 @@ def parse():
     ap.add_argument("--impl", default="dycuckoo", choices=["dycuckoo", "reference"])
     ap.add_argument("--log2n", type=int, default=27, help="C2 batch size 2^log2n (27 = BASELINE configs[1])")
     ap.add_argument("--bucket-slots", type=int, default=8)
-    ap.add_argument("--cpu-log2n", type=int, default=23, help="oracle sample size for cpu_baseline")
+    ap.add_argument("--cpu-log2n", type=int, default=25, help="oracle sample size for cpu_baseline")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-rehash", action="store_true")
