@@ -89,6 +89,11 @@ struct dyc_table {
     // baseline clears all.  Downsizes and placements (first-fit, evictions)
     // preserve it.
     uint32_t clean = 0;
+    // m is exact unless a delete batch skipped its counter read-back (m_lazy):
+    // then the removals wait in d_ctr[C_REMOVED] and m is an upper bound until
+    // the next read_ctr applies them (flush_m before any decision that needs m).
+    bool m_lazy = false;
+    uint64_t del_n = 0;                    // ops of the delete batch in flight
     bool count_probes = false;             // dyc_probe_count_enable (measurement)
     unsigned long long* d_probe = nullptr; // {ops, second probes} x {find, upsert, delete}
     unsigned long long* list[2] = {nullptr, nullptr};
@@ -301,11 +306,27 @@ dyc_status read_ctr(dyc_table* t, cudaStream_t st) {
     CU(cudaStreamSynchronize(st));
     t->sync_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     t->n_sync++;
+    // every read-back applies the removals counted since the last one (the
+    // delete batches whose own read-back was skipped included)
+    const unsigned long long removed = t->h_ctr[C_REMOVED];
+    if (removed) {
+        t->m -= removed;
+        t->clean = 0;   // emptied slots break the first-choice-full invariant
+        CU(cudaMemsetAsync(t->d_ctr + C_REMOVED, 0, sizeof(unsigned long long), st));
+    }
+    t->m_lazy = false;
     return DYC_OK;
 }
 
+dyc_status flush_m(dyc_table* t, cudaStream_t st) {
+    return t->m_lazy ? read_ctr(t, st) : DYC_OK;
+}
+
+// zeroes every counter but C_REMOVED (owned by read_ctr: removals not yet
+// applied to m)
 dyc_status zero_ctr(dyc_table* t, cudaStream_t st) {
-    CU(cudaMemsetAsync(t->d_ctr, 0, C_N * sizeof(unsigned long long), st));
+    CU(cudaMemsetAsync(t->d_ctr, 0, C_REMOVED * sizeof(unsigned long long), st));
+    CU(cudaMemsetAsync(t->d_ctr + C_REMOVED + 1, 0, (C_N - C_REMOVED - 1) * sizeof(unsigned long long), st));
     return DYC_OK;
 }
 
@@ -452,6 +473,7 @@ dyc_status downsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
 // settled once at the end (Q17: retry, then failure-triggered upsizes).
 template <int B>
 dyc_status enforce_lower(dyc_table* t, cudaStream_t st) {
+    TRY(flush_m(t, st));
     uint64_t nb[DYC_MAX_D];
     for (uint32_t i = 0; i < t->cfg.d; i++) nb[i] = t->nb[i];
     std::vector<uint32_t> plan;
@@ -552,6 +574,7 @@ dyc_status live_begin(dyc_table* t, int direction, int subtable, cudaStream_t st
     auto& r = t->rz;
     if (r.active) return set_err(DYC_ERR_INVALID_ARG, "a resize is already in flight (dyc_resize_commit first)");
     if (t->part_op) return set_err(DYC_ERR_INVALID_ARG, "a batch is open (dyc_*_end first)");
+    TRY(flush_m(t, st));
     int ti = -1;
     TRY(pick_resize(t, direction, subtable, ti));
     if (!r.start) CU(cudaEventCreateWithFlags(&r.start, cudaEventDisableTiming));
@@ -601,6 +624,7 @@ dyc_status live_begin(dyc_table* t, int direction, int subtable, cudaStream_t st
 // it has to act.
 template <int B>
 dyc_status policy_lower(dyc_table* t, cudaStream_t st) {
+    TRY(flush_m(t, st));
     if (t->rz.active) {
         if (!((double)t->m < t->cfg.alpha * (double)t->N_after())) return DYC_OK;
         TRY(live_commit<B>(t, st));
@@ -840,6 +864,8 @@ dyc_status binned_ins(dyc_table* t, const BinCtx& bc, const uint32_t* keys, cons
 // need that subtable (deferred updates, keys with no free non-locked slot).
 template <int B>
 dyc_status insert_begin(dyc_table* t, uint64_t n, cudaStream_t st, bool& fuse) {
+    // m may be an upper bound (m_lazy): below beta with it, below beta for sure
+    if (t->m_lazy && (t->rz.active || (double)(t->m + n) > t->cfg.beta * (double)t->N())) TRY(flush_m(t, st));
     if (t->rz.active && (double)(t->m + n) > t->cfg.beta * (double)t->N_after()) TRY(live_commit<B>(t, st));
     TRY(ensure_lists(t, n, st));
     TRY(zero_ctr(t, st));
@@ -936,7 +962,8 @@ dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t
 // one k_delete per chunk + end (m, deferred removals, alpha loop).
 template <int B>
 dyc_status delete_prep(dyc_table* t, uint64_t n, cudaStream_t st) {
-    TRY(zero_one(t, C_REMOVED, st));
+    if (t->rz.active) TRY(flush_m(t, st));
+    t->del_n = n;
     if (t->rz.active) {
         TRY(ensure_lists(t, n, st));
         TRY(zero_one(t, C_DEFER, st));
@@ -963,9 +990,15 @@ dyc_status delete_chunk(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint
 
 template <int B>
 dyc_status delete_end(dyc_table* t, cudaStream_t st) {
-    TRY(read_ctr(t, st));
-    t->m -= t->h_ctr[C_REMOVED];
-    if (t->h_ctr[C_REMOVED]) t->clean = 0;   // emptied slots break the invariant
+    // no resize in flight and m - n >= alpha*N: the alpha loop cannot fire, so
+    // the removals stay on the device until the next read-back (m_lazy)
+    if (!t->rz.active && t->m >= t->del_n &&
+        (double)(t->m - t->del_n) >= t->cfg.alpha * (double)t->N()) {
+        if (t->del_n) t->clean = 0;
+        t->m_lazy = true;
+        return DYC_OK;
+    }
+    TRY(read_ctr(t, st));   // applies the removals to m
     if (t->rz.active && t->h_ctr[C_DEFER]) {
         const uint64_t dfr = t->h_ctr[C_DEFER];
         t->n_deferred += dfr;
@@ -1160,6 +1193,7 @@ dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaSt
 template <int B>
 dyc_status resize_impl(dyc_table* t, int direction, int subtable, int method, cudaStream_t st) {
     TRY(live_commit<B>(t, st));
+    TRY(flush_m(t, st));
     if (direction == 0) {
         while ((double)t->m > t->cfg.beta * (double)t->N()) {
             TRY(upsize_table<B>(t, (uint32_t)t->smallest(), st));
@@ -1231,6 +1265,7 @@ template <int B>
 dyc_status dump_impl(dyc_table* t, uint64_t* h_kv, uint32_t* h_tab, uint64_t* h_bkt, uint64_t cap, uint64_t* n_out,
                      cudaStream_t st) {
     TRY(live_commit<B>(t, st));
+    TRY(flush_m(t, st));
     const uint64_t m = t->m;
     void *kv = nullptr, *tb = nullptr, *bk = nullptr;
     TRY(dev_alloc(t, &kv, m * 8, st));
@@ -1368,6 +1403,8 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
         }
     }
     if (s == DYC_OK && cudaMalloc(&t->d_ctr, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMalloc");
+    // C_REMOVED is only ever zeroed by read_ctr after it applies the count
+    if (s == DYC_OK && cudaMemset(t->d_ctr, 0, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMemset");
     if (s == DYC_OK && cudaMalloc(&t->d_probe, 6 * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMalloc");
     if (s == DYC_OK && cudaMemset(t->d_probe, 0, 6 * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMemset");
     t->clean = (1u << d) - 1u;      // an empty table satisfies the invariant
@@ -1591,6 +1628,7 @@ dyc_status dyc_clear(dyc_table* t, dyc_stream_t stream) {
     if (t->rz.active) TRY(live_commit_any(t, S(stream)));
     for (uint32_t i = 0; i < t->cfg.d; i++)
         CU(cudaMemsetAsync(t->sub[i], 0xFF, t->nb[i] * t->cfg.bucket_slots * 8, S(stream)));
+    TRY(flush_m(t, S(stream)));   // settles the removals counted on the device
     t->m = 0;
     t->clean = (1u << t->cfg.d) - 1u;
     return DYC_OK;
