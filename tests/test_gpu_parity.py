@@ -394,3 +394,40 @@ def test_batch_in_parts_equals_one_batch(oracle_mod):
             np.testing.assert_array_equal(f.cpu().numpy(), of)
         np.testing.assert_array_equal(g.sorted_kv(), o.sorted_kv())
         assert g.stats()["buckets"] == o.stats()["buckets"], f"schedule diverged at batch {i}"
+
+
+def test_lazy_delete_readback_keeps_policy_exact(oracle_mod):
+    """Delete batches that cannot trigger the alpha loop (m - n >= alpha*N,
+    P:L305) leave their removal count on the device; the next insert whose
+    upper bound m + n crosses beta*N must apply it first, so the resize
+    schedule stays the oracle's (no spurious upsize)."""
+    rng = np.random.default_rng(0x1A2B)
+    keys = rng.choice(np.arange(1, 1 << 30, dtype=np.uint32), size=70000, replace=False)
+    vals = rng.integers(0, 1 << 31, size=keys.size, dtype=np.uint32)
+    g = Table(d=4, init_capacity=1 << 16, alpha=0.3, beta=0.85, bucket_slots=8, seed=7)
+    o = oracle_mod.OracleTable(d=4, init_capacity=1 << 16, alpha=0.3, beta=0.85, bucket_slots=8, seed=7)
+    g.insert(dev(keys[:50000]), dev(vals[:50000]))
+    o.insert(keys[:50000], vals[:50000])
+    s0 = g.stats()
+    for j in range(5):
+        dk = keys[j * 2000:(j + 1) * 2000]
+        _, st = g.delete(dev(dk))
+        _, ost = o.delete(dk)
+        np.testing.assert_array_equal(st.cpu().numpy(), ost)
+    s1 = g.stats()
+    assert s1["n_sync"] - s0["n_sync"] < 5, "delete batches still read their counters back"
+    assert s1["m"] == o.stats()["m"] == 40000
+    g.insert(dev(keys[50000:60000]), dev(vals[50000:60000]))
+    o.insert(keys[50000:60000], vals[50000:60000])
+    for j in range(5, 8):                      # lazy again, then an insert crossing beta*N
+        dk = keys[j * 2000:(j + 1) * 2000]
+        g.delete(dev(dk))
+        o.delete(dk)
+    g.insert(dev(keys[60000:70000]), dev(vals[60000:70000]))
+    o.insert(keys[60000:70000], vals[60000:70000])
+    gs, os_ = g.stats(), o.stats()
+    assert gs["m"] == os_["m"]
+    assert gs["buckets"] == os_["buckets"]
+    assert gs["n_upsize"] == os_["n_upsize"]
+    np.testing.assert_array_equal(g.sorted_kv(), o.sorted_kv())
+    check_layout(g, o)
