@@ -678,3 +678,12 @@ int dyo_place_one(dyo_table *T, uint32_t key, uint32_t val)
     if (r != DYO_OK) settle_homeless(T, &hl, 1);
     return r;
 }
+
+/* Test-only hook for the negative pins of dyo_check_invariants (I4): shift the
+ * per-subtable counter m_t by delta without touching the slots. */
+int dyo_debug_adjust_count(dyo_table *T, uint32_t t, int64_t delta)
+{
+    if (t >= T->d) return -1;
+    T->m_t[t] = (uint64_t)((int64_t)T->m_t[t] + delta);
+    return 0;
+}

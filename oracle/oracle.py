@@ -74,6 +74,8 @@ def oracle_lib():
         lib.dyo_poke.restype = I32
         lib.dyo_peek.argtypes = [P, U32, U64, U32]
         lib.dyo_peek.restype = U64
+        lib.dyo_debug_adjust_count.argtypes = [P, U32, C.c_int64]
+        lib.dyo_debug_adjust_count.restype = I32
         lib.dyo_place_one.argtypes = [P, U32, U32]
         lib.dyo_place_one.restype = I32
         _lib = lib
@@ -206,6 +208,11 @@ class OracleTable:
     def peek(self, t: int, b: int, s: int) -> Tuple[int, int]:
         x = int(self._lib.dyo_peek(self._t, t, b, s))
         return x & 0xFFFFFFFF, x >> 32
+
+    def debug_adjust_count(self, t: int, delta: int) -> None:
+        """Corrupts the counter m_t (negative pins of check_invariants, I4)."""
+        if self._lib.dyo_debug_adjust_count(self._t, t, delta) != 0:
+            raise IndexError("subtable out of range")
 
     def place_one(self, key: int, val: int) -> int:
         return int(self._lib.dyo_place_one(self._t, key, val))

@@ -92,7 +92,12 @@ struct dyc_table {
     // m is exact unless a delete batch skipped its counter read-back (m_lazy):
     // then the removals wait in d_ctr[C_REMOVED] and m is an upper bound until
     // the next read_ctr applies them (flush_m before any decision that needs m).
+    // lazy_n bounds the removals still pending (the summed sizes of the delete
+    // batches that skipped their read-back), so m - lazy_n is a lower bound of
+    // the live count; lazy_ev marks the last such batch on its stream.
     bool m_lazy = false;
+    uint64_t lazy_n = 0;
+    cudaEvent_t lazy_ev = nullptr;
     uint64_t del_n = 0;                    // ops of the delete batch in flight
     bool count_probes = false;             // dyc_probe_count_enable (measurement)
     unsigned long long* d_probe = nullptr; // {ops, second probes} x {find, upsert, delete}
@@ -301,6 +306,9 @@ void dev_free(dyc_table* t, void* p, cudaStream_t st) {
 }
 
 dyc_status read_ctr(dyc_table* t, cudaStream_t st) {
+    // a lazy delete may have run on another stream: its removals must have
+    // landed in C_REMOVED before the copy and the reset below
+    if (t->m_lazy && t->lazy_ev) CU(cudaStreamWaitEvent(st, t->lazy_ev, 0));
     CU(cudaMemcpyAsync(t->h_ctr, t->d_ctr, C_N * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
     const auto t0 = std::chrono::steady_clock::now();
     CU(cudaStreamSynchronize(st));
@@ -315,6 +323,7 @@ dyc_status read_ctr(dyc_table* t, cudaStream_t st) {
         CU(cudaMemsetAsync(t->d_ctr + C_REMOVED, 0, sizeof(unsigned long long), st));
     }
     t->m_lazy = false;
+    t->lazy_n = 0;
     return DYC_OK;
 }
 
@@ -990,11 +999,17 @@ dyc_status delete_chunk(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint
 
 template <int B>
 dyc_status delete_end(dyc_table* t, cudaStream_t st) {
-    // no resize in flight and m - n >= alpha*N: the alpha loop cannot fire, so
-    // the removals stay on the device until the next read-back (m_lazy)
-    if (!t->rz.active && t->m >= t->del_n &&
-        (double)(t->m - t->del_n) >= t->cfg.alpha * (double)t->N()) {
+    // no resize in flight and a LOWER bound of m after this batch (m minus
+    // every removal that may still be pending, this batch's included) is
+    // >= alpha*N: the alpha loop cannot fire, so the removals stay on
+    // the device until the next read-back (m_lazy).  m itself is then an upper
+    // bound, which is what the beta test of the next insert needs.
+    const uint64_t pend = t->lazy_n + t->del_n;
+    if (!t->rz.active && t->m >= pend && (double)(t->m - pend) >= t->cfg.alpha * (double)t->N()) {
         if (t->del_n) t->clean = 0;
+        if (!t->lazy_ev) CU(cudaEventCreateWithFlags(&t->lazy_ev, cudaEventDisableTiming));
+        CU(cudaEventRecord(t->lazy_ev, st));
+        t->lazy_n = pend;
         t->m_lazy = true;
         return DYC_OK;
     }
@@ -1440,6 +1455,7 @@ dyc_status dyc_destroy(dyc_table* t) {
     if (t->rz.ctr) cudaFree(t->rz.ctr);
     if (t->rz.start) cudaEventDestroy(t->rz.start);
     if (t->rz.done) cudaEventDestroy(t->rz.done);
+    if (t->lazy_ev) cudaEventDestroy(t->lazy_ev);
     if (t->h_ctr) cudaFreeHost(t->h_ctr);
     if (t->cp_in) cudaStreamDestroy(t->cp_in);
     if (t->cp_out) cudaStreamDestroy(t->cp_out);
@@ -1645,6 +1661,15 @@ dyc_status dyc_stats(dyc_table* t, dyc_stats_t* out, dyc_stream_t stream) {
     TRY(enter(t, stream));
     if (!out) return set_err(DYC_ERR_INVALID_ARG, "null out");
     DISPATCH_B(t, stats_impl<B_>(t, out, S(stream)));
+}
+
+dyc_status dyc_shape(const dyc_table* t, uint64_t* buckets, uint64_t* m, uint64_t* m_pending) {
+    TRY(check_table(t));
+    if (buckets)
+        for (uint32_t i = 0; i < t->cfg.d; i++) buckets[i] = t->nb[i];
+    if (m) *m = t->m;
+    if (m_pending) *m_pending = t->m_lazy ? t->lazy_n : 0;
+    return DYC_OK;
 }
 
 dyc_status dyc_dump(dyc_table* t, uint64_t* h_kv, uint32_t* h_table, uint64_t* h_bucket, uint64_t cap,

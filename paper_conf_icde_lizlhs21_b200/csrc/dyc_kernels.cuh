@@ -1191,7 +1191,7 @@ __global__ void __launch_bounds__(kThreads) k_gather(unsigned long long* __restr
         if (WRITE) {
 #pragma unroll
             for (int j = 0; j < ILP; j++)
-                if (g.sub == 0 && wp[j]) st_u64_cg(wp[j] + (acc & 3), s[j][0] + 1);
+                if (g.sub == 0 && wp[j]) st_u64_cg(wp[j], s[j][0] + 1);   // address: own probe only
         }
     }
     if (acc == 0x0123456789ABCDEFull) *sink = acc;   // keeps the loads alive

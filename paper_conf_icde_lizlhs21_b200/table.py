@@ -301,6 +301,18 @@ class Table:
     def clear(self, stream=None):
         L.check(self._lib.dyc_clear(self._h, _stream_ptr(stream)), "dyc_clear")
 
+    def shape(self) -> Tuple[list, int, int]:
+        """(buckets per subtable, m, removals possibly pending) from the host's
+        view, without touching the device (dyc_shape: never synchronizes)."""
+        nb = np.zeros(self.d, dtype=np.uint64)
+        m, pend = C.c_uint64(), C.c_uint64()
+        L.check(self._lib.dyc_shape(self._h, nb.ctypes.data_as(C.c_void_p), C.byref(m), C.byref(pend)),
+                "dyc_shape")
+        return [int(x) for x in nb], int(m.value), int(pend.value)
+
+    def _buckets_host(self):
+        return self.shape()[0]
+
     def stats(self, stream=None) -> Dict:
         s = L.dyc_stats_t()
         L.check(self._lib.dyc_stats(self._h, C.byref(s), _stream_ptr(stream)), "dyc_stats")

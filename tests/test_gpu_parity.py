@@ -431,3 +431,56 @@ def test_lazy_delete_readback_keeps_policy_exact(oracle_mod):
     assert gs["n_upsize"] == os_["n_upsize"]
     np.testing.assert_array_equal(g.sorted_kv(), o.sorted_kv())
     check_layout(g, o)
+
+
+def test_lazy_deletes_crossing_alpha_downsize_like_oracle(oracle_mod):
+    """Consecutive delete batches that together cross alpha*N, with no stats()
+    or dump() in between (either would make m exact again): the skip test must
+    use a lower bound of m (every pending removal subtracted), so the alpha
+    loop fires in the same batch as in the oracle.  C1's eight
+    delete batches back to back, then C1-like batches at a larger scale."""
+    for n_keys, batch in ((65536, 8192), (200000, 10000)):
+        wl = W.c1_rand_small(n_keys=n_keys, batch=batch)
+        g, o = make_pair(oracle_mod, wl, B=8)
+        sizes_g, sizes_o = [], []
+        dels = [b for b in wl.batches if b.op == "delete"]
+        ins = [b for b in wl.batches if b.op == "insert"]
+        for b in ins:
+            g.insert(dev(b.keys), dev(b.values))
+            o.insert(b.keys, b.values)
+        s0 = g.stats()
+        assert s0["buckets"] == o.stats()["buckets"]
+        outs = []
+        for b in dels:                       # no stats/dump between the batches
+            outs.append(g.delete(dev(b.keys)))
+            o.delete(b.keys)
+            sizes_o.append(o.stats()["buckets"])
+            sizes_g.append(list(g._buckets_host()))
+        for b, (v, st) in zip(dels, outs):
+            assert (st.cpu().numpy() == 1).all()
+            np.testing.assert_array_equal(host_u32(v), W.val_of(b.keys, 0))
+        assert sizes_g == sizes_o, "downsize schedule diverged from the oracle's"
+        gs, os_ = g.stats(), o.stats()
+        assert gs["n_downsize"] == os_["n_downsize"] and gs["m"] == os_["m"] == 0
+        assert gs["buckets"] == os_["buckets"]
+
+
+def test_lazy_delete_on_other_stream_then_stats(oracle_mod):
+    """A delete that skips its read-back on stream A, then stats() on stream B
+    without any host wait: the read-back must wait for A's removals (event)
+    before reading and resetting the device count."""
+    n = 1 << 21
+    keys = W.key_range(0, n, 4242)
+    vals = W.val_of(keys, 0)
+    g = Table(d=4, init_capacity=int(n / 0.8), alpha=0.1, beta=0.85, bucket_slots=8)
+    g.insert(dev(keys), dev(vals))
+    torch.cuda.synchronize()
+    sa = torch.cuda.Stream()
+    kd = dev(keys[: n // 4])
+    torch.cuda.synchronize()
+    s0 = g.stats()["n_sync"]
+    with torch.cuda.stream(sa):
+        g.delete(kd, stream=sa)
+    s = g.stats(stream=torch.cuda.current_stream())
+    assert s["n_sync"] - s0 <= 2, "the delete was expected to skip its read-back"
+    assert s["m"] == n - n // 4 and sum(s["count"]) == s["m"]
