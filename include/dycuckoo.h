@@ -70,7 +70,8 @@ typedef enum {
     DYC_ERR_OOM = 2,
     DYC_ERR_CUDA = 3,
     DYC_ERR_INSERT_FAILED = 4,        /* a key could not be placed even after upsizing */
-    DYC_ERR_NO_DEVICE = 5
+    DYC_ERR_NO_DEVICE = 5,
+    DYC_ERR_NCCL = 6                  /* NCCL missing or an NCCL call failed (dyc_dist_*) */
 } dyc_status;
 
 /* per-op status codes written to uint8 status / found arrays */
@@ -384,6 +385,78 @@ dyc_status dyc_route_unpermute(const uint32_t* d_pos, uint64_t n, const uint32_t
                                uint8_t* d_status, dyc_stream_t stream);
 
 /* ---------------------------------------------------------------------------
+ * Sharded table: one process per GPU, each
+ * owning `local_shards` complete DyCuckoo tables on its current device, G =
+ * world * local_shards shards in all.  Key k belongs to shard
+ * s = x_{d+1}(k) mod G (the (d+1)-th universal hash of P:L271, independent of
+ * the pair and bucket hashes), owned by rank s / local_shards.  Each shard
+ * resizes on its own.  The paper is single-GPU (P:L225 calls
+ * host/device transfer orthogonal, commented); the batch calls keep its map
+ * semantics (insert/find/delete) and batch model: since
+ * keys are distinct within a batch and ops on different keys never interact,
+ * every per-op result and the union of the shards' contents equal those of one
+ * table given the same batches.
+ *
+ * Every rank calls the same dyc_dist_* batch function in the same order (a
+ * collective; n may differ per rank, 0 included).  A batch groups its ops by
+ * shard on the device (dyc_route_count/_scatter), exchanges the per-shard
+ * counts and then keys [values, op codes] with grouped ncclSend/ncclRecv over
+ * NVLink (one host read-back of the counts per batch), runs one ordinary batch
+ * per local shard (so each shard takes its own resize decisions), sends the
+ * results back and writes them in request order.  With world == 1 and no id
+ * no NCCL is used (local virtual shards).  NCCL (libnccl.so.2) is loaded at run time.
+ * Pointers, streams, status codes and preconditions are as for the
+ * single-table calls; results for op i of the calling rank are written at
+ * index i.  Errors: DYC_ERR_NCCL for a failed NCCL call (the table state is
+ * then undefined), otherwise as for the single-table calls.
+ * ------------------------------------------------------------------------- */
+#define DYC_NCCL_UNIQUE_ID_BYTES 128
+typedef struct dyc_dist dyc_dist;     /* opaque; owns its local shards, NCCL communicator, buffers */
+
+/* ncclGetUniqueId into id[DYC_NCCL_UNIQUE_ID_BYTES] (host memory).  Rank 0
+ * calls it and distributes the bytes to every rank out of band (e.g. a
+ * torch.distributed broadcast).  Needs no GPU.  DYC_ERR_NCCL if NCCL cannot
+ * be loaded. */
+dyc_status dyc_dist_get_unique_id(void* id);
+
+/* Creates this rank's part of a sharded table: local_shards tables with config
+ * *cfg (the same on every rank, seed included) on the current device, and for
+ * world > 1 an NCCL communicator from nccl_unique_id (NULL allowed when
+ * world == 1: then nothing is exchanged; an id with world == 1 creates a
+ * one-rank communicator and runs the exchange through NCCL to self).  Collective across the world.  dyc_dist_create uses the default
+ * config with d, init_capacity (per shard), alpha, beta, and one local shard.
+ * Errors: DYC_ERR_INVALID_ARG (rank outside [0, world), local_shards 0,
+ * world*local_shards > 1024, world > 1 without an id, or a bad cfg),
+ * DYC_ERR_NO_DEVICE, DYC_ERR_OOM, DYC_ERR_NCCL. */
+dyc_status dyc_dist_create(uint32_t d, uint64_t init_capacity_per_shard, double alpha, double beta,
+                           const void* nccl_unique_id, int rank, int world, dyc_dist** out);
+dyc_status dyc_dist_create_ex(const dyc_config* cfg, const void* nccl_unique_id, int rank, int world,
+                              uint32_t local_shards, dyc_dist** out);
+/* Destroys the local shards and the communicator (synchronizes the device). */
+dyc_status dyc_dist_destroy(dyc_dist* dist);
+
+/* Sharded batches: as dyc_insert_batch / dyc_find_batch / dyc_delete_batch /
+ * dyc_mixed_batch for the calling rank's n ops.  Each synchronizes `stream`
+ * once for the routing counts (plus what the local shards' own batches do). */
+dyc_status dyc_dist_insert_batch(dyc_dist* dist, const uint32_t* d_keys, const uint32_t* d_values,
+                                 uint8_t* d_status, uint64_t n, dyc_stream_t stream);
+dyc_status dyc_dist_find_batch(dyc_dist* dist, const uint32_t* d_keys, uint32_t* d_values_out,
+                               uint8_t* d_found, uint64_t n, dyc_stream_t stream);
+dyc_status dyc_dist_delete_batch(dyc_dist* dist, const uint32_t* d_keys, uint32_t* d_values_out,
+                                 uint8_t* d_status, uint64_t n, dyc_stream_t stream);
+dyc_status dyc_dist_mixed_batch(dyc_dist* dist, const uint8_t* d_ops, const uint32_t* d_keys,
+                                const uint32_t* d_values, uint32_t* d_values_out, uint8_t* d_status,
+                                uint64_t n, dyc_stream_t stream);
+/* rank, world, local shards, and the number of ops this rank's shards executed
+ * in the last batch (any pointer may be NULL). */
+dyc_status dyc_dist_info(const dyc_dist* dist, int* rank, int* world, uint32_t* local_shards,
+                         uint64_t* last_recv);
+/* The table of local shard local_index (global shard rank*local_shards +
+ * local_index), owned by dist: for dyc_stats / dyc_dump; do not destroy it or
+ * run batches on it directly. */
+dyc_status dyc_dist_shard(const dyc_dist* dist, uint32_t local_index, dyc_table** out);
+
+/* ---------------------------------------------------------------------------
  * Fused routing over peer memory (S11).  Instead of
  * count -> exchange counts -> scatter -> all-to-all -> ... -> all-to-all ->
  * unpermute, the dispatch kernel hashes each op to its shard, reserves a range
@@ -455,10 +528,15 @@ dyc_status dyc_bench_gather(const void* d_buf, uint64_t buf_bytes, uint64_t n_re
 
 /* dyc_bench_gather with flags: DYC_GATHER_WRITE (1) makes every read followed
  * by an 8-byte store into the bucket just read (the probe-then-write pattern of
- * insert and delete: one random read plus one dirty-line write-back per op), so
- * d_buf is overwritten.  Errors: DYC_ERR_INVALID_ARG for other flag bits or
- * sizes as in dyc_bench_gather. */
+ * delete: one random read plus one dirty-line write-back per op);
+ * DYC_GATHER_CAS (2) makes it an 8-byte atomicCAS instead (insert's claim of a
+ * free slot) and DYC_GATHER_SECTOR (4) a full 32-byte sector store (when
+ * several are set the highest wins).  The written word depends only on the
+ * group's own read.  d_buf is overwritten.  Errors: DYC_ERR_INVALID_ARG for
+ * other flag bits or sizes as in dyc_bench_gather. */
 #define DYC_GATHER_WRITE 1u
+#define DYC_GATHER_CAS 2u
+#define DYC_GATHER_SECTOR 4u
 dyc_status dyc_bench_gather_ex(void* d_buf, uint64_t buf_bytes, uint64_t n_reads, uint32_t bytes_per_read,
                                uint64_t seed, uint32_t flags, uint64_t* d_sink, dyc_stream_t stream);
 

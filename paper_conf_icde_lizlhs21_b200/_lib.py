@@ -16,14 +16,15 @@ DYC_MAX_D = 16
 DYC_EMPTY_KEY = 0xFFFFFFFF
 DYC_NOT_FOUND = 0xFFFFFFFF
 
-DYC_OK, DYC_ERR_INVALID_ARG, DYC_ERR_OOM, DYC_ERR_CUDA, DYC_ERR_INSERT_FAILED, DYC_ERR_NO_DEVICE = range(6)
+DYC_OK, DYC_ERR_INVALID_ARG, DYC_ERR_OOM, DYC_ERR_CUDA, DYC_ERR_INSERT_FAILED, DYC_ERR_NO_DEVICE, DYC_ERR_NCCL = range(7)
+DYC_NCCL_UNIQUE_ID_BYTES = 128
 DYC_RESIZE_SPLIT, DYC_RESIZE_REINSERT_SUBTABLE, DYC_RESIZE_REHASH_ALL = range(3)
 DYC_PROF_KINDS = 16
-DYC_GATHER_WRITE = 1
+DYC_GATHER_WRITE, DYC_GATHER_CAS, DYC_GATHER_SECTOR = 1, 2, 4
 PROF_NAMES = ["k_find", "k_upsert", "k_place", "k_delete", "k_upsize", "k_downsize", "k_reinsert", "other",
               "bin_group", "bin_find", "bin_ins", "bin_place", "bin_delete", "bin_out"]
 _STATUS_NAMES = ["DYC_OK", "DYC_ERR_INVALID_ARG", "DYC_ERR_OOM", "DYC_ERR_CUDA",
-                 "DYC_ERR_INSERT_FAILED", "DYC_ERR_NO_DEVICE"]
+                 "DYC_ERR_INSERT_FAILED", "DYC_ERR_NO_DEVICE", "DYC_ERR_NCCL"]
 
 
 class dyc_config(C.Structure):
@@ -139,6 +140,17 @@ SIGNATURES = {
     "dyc_bench_gather_ex": (_I, [_P, _U64, _U64, _U32, _U64, _U32, _P, _P]),
     "dyc_set_l2_fetch_granularity": (_I, [_U32]),
     "dyc_get_l2_fetch_granularity": (_I, [C.POINTER(_U32)]),
+    # sharded table (dyc_dist_*, NCCL between processes, local virtual shards)
+    "dyc_dist_get_unique_id": (_I, [_P]),
+    "dyc_dist_create": (_I, [_U32, _U64, _D, _D, _P, _I, _I, C.POINTER(_TP)]),
+    "dyc_dist_create_ex": (_I, [C.POINTER(dyc_config), _P, _I, _I, _U32, C.POINTER(_TP)]),
+    "dyc_dist_destroy": (_I, [_TP]),
+    "dyc_dist_insert_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
+    "dyc_dist_find_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
+    "dyc_dist_delete_batch": (_I, [_TP, _P, _P, _P, _U64, _P]),
+    "dyc_dist_mixed_batch": (_I, [_TP, _P, _P, _P, _P, _P, _U64, _P]),
+    "dyc_dist_info": (_I, [_TP, C.POINTER(_I), C.POINTER(_I), C.POINTER(_U32), C.POINTER(_U64)]),
+    "dyc_dist_shard": (_I, [_TP, _U32, C.POINTER(_TP)]),
     "dyc_last_error": (C.c_char_p, []),
     "dyc_version": (C.c_char_p, []),
 }

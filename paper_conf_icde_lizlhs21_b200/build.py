@@ -13,14 +13,16 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libdyc.so")
-SOURCES = ["dyc_api.cu"]
-DEPS = ["dyc_api.cu", "dyc_kernels.cuh", "dyc_device.cuh", "dyc_binned.cuh", "dyw_api.cuh", "dyw_kernels.cuh"]
+SOURCES = ["dyc_api.cu", "dyc_dist.cu"]
+DEPS = SOURCES + ["dyc_kernels.cuh", "dyc_device.cuh", "dyc_binned.cuh", "dyw_api.cuh", "dyw_kernels.cuh"]
 
-NVCC_FLAGS = [
+COMPILE_FLAGS = [
     "-O3", "-std=c++17", "-lineinfo",
     "-gencode", "arch=compute_100a,code=sm_100a",
-    "-Xcompiler", "-fPIC,-O2", "-shared", "-cudart", "static",
+    "-Xcompiler", "-fPIC,-O2",
 ]
+LINK_FLAGS = ["-shared", "-cudart", "static", "-gencode", "arch=compute_100a,code=sm_100a", "-ldl"]
+NVCC_FLAGS = COMPILE_FLAGS + LINK_FLAGS
 
 
 def nvcc_path() -> str:
@@ -39,14 +41,33 @@ def needs_build() -> bool:
 
 
 def build_library(force: bool = False, verbose: bool = False) -> str:
+    """Compiles every source to an object in parallel (nvcc -c), then links
+    libdyc.so (static cudart, -ldl for the run-time NCCL load of dyc_dist.cu)."""
     if not force and not needs_build():
         return LIB
-    tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [nvcc_path(), *NVCC_FLAGS, "-I", INCLUDE, "-o", tmp] + [os.path.join(CSRC, s) for s in SOURCES]
-    if verbose:
-        print(" ".join(cmd))
-    subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
+    tag = f".tmp{os.getpid()}"
+    objs, procs = [], []
+    for src in SOURCES:
+        obj = os.path.join(PKG, src.replace(".cu", tag + ".o"))
+        cmd = [nvcc_path(), *COMPILE_FLAGS, "-I", INCLUDE, "-c", "-o", obj, os.path.join(CSRC, src)]
+        if verbose:
+            print(" ".join(cmd))
+        procs.append(subprocess.Popen(cmd))
+        objs.append(obj)
+    rcs = [p.wait() for p in procs]
+    try:
+        if any(rcs):
+            raise subprocess.CalledProcessError(max(rcs), "nvcc -c")
+        tmp = LIB + tag
+        cmd = [nvcc_path(), *LINK_FLAGS, "-o", tmp] + objs
+        if verbose:
+            print(" ".join(cmd))
+        subprocess.check_call(cmd)
+        os.replace(tmp, LIB)
+    finally:
+        for o in objs:
+            if os.path.exists(o):
+                os.remove(o)
     return LIB
 
 

@@ -66,6 +66,9 @@ inline cudaStream_t S(dyc_stream_t s) { return reinterpret_cast<cudaStream_t>(s)
 
 }  // namespace
 
+// Error channel shared with the other translation units (dyc_dist.cu).
+void dyc_internal_set_error(const std::string& msg) { g_err = msg; }
+
 struct dyc_table {
     dyc_config cfg{};
     int device = 0;
@@ -1964,17 +1967,21 @@ dyc_status dyc_bench_gather_ex(void* d_buf, uint64_t buf_bytes, uint64_t n_reads
                                uint64_t seed, uint32_t flags, uint64_t* d_sink, dyc_stream_t stream) {
     if (bytes_per_read != 32 && bytes_per_read != 64 && bytes_per_read != 128 && bytes_per_read != 256)
         return set_err(DYC_ERR_INVALID_ARG, "bytes_per_read must be 32, 64, 128 or 256");
-    if (flags & ~1u) return set_err(DYC_ERR_INVALID_ARG, "flags: only DYC_GATHER_WRITE (1) is defined");
+    if (flags & ~7u) return set_err(DYC_ERR_INVALID_ARG, "flags: DYC_GATHER_WRITE (1) | DYC_GATHER_CAS (2) | DYC_GATHER_SECTOR (4)");
+    const int wmode = (flags & 4u) ? 3 : (flags & 2u) ? 2 : (flags & 1u) ? 1 : 0;
     const uint64_t units = buf_bytes / bytes_per_read;
     if (units == 0) return set_err(DYC_ERR_INVALID_ARG, "buffer too small");
     const uint64_t lanes_per_read = bytes_per_read / 32;
     const unsigned grid = grid_for(n_reads * lanes_per_read, (uint64_t)kThreads * 4);
     unsigned long long* buf = (unsigned long long*)d_buf;
     unsigned long long* sink = (unsigned long long*)d_sink;
-    const bool wr = flags & 1u;
-#define DYC_GATHER(BB)                                                                               \
-    (wr ? k_gather<BB, true><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink)      \
-        : k_gather<BB, false><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink))
+#define DYC_GATHER(BB)                                                                                    \
+    switch (wmode) {                                                                                      \
+        case 0: k_gather<BB, 0><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break; \
+        case 1: k_gather<BB, 1><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break; \
+        case 2: k_gather<BB, 2><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break; \
+        default: k_gather<BB, 3><<<grid, kThreads, 0, S(stream)>>>(buf, units, n_reads, seed, sink); break; \
+    }
     switch (bytes_per_read) {
         case 32: DYC_GATHER(4); break;
         case 64: DYC_GATHER(8); break;

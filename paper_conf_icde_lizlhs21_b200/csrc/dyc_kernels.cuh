@@ -1155,10 +1155,12 @@ __global__ void __launch_bounds__(kThreads) k_route_reply(const unsigned long lo
 // uniformly random bucket-aligned offsets, by a G = B/4 lane group with the same
 // 256-bit loads and L2 prefetch size as k_find.  Its rate is the random-access
 // ceiling the probe kernels are compared with.
-// WRITE: after its read, each group also stores one 8-byte slot into the bucket
-// it read (the probe-then-write pattern of an insert or delete: one read plus
-// one dirty-line write-back per op); the stored word depends on the data read.
-template <int B, bool WRITE = false>
+// WRITE (1, 2 or 3): after its read, each group also writes into the bucket it
+// read (the probe-then-write pattern of an insert or delete: one read plus one
+// dirty-line write-back per op); the written word depends only on the group's
+// own probe.  1: an 8-byte plain store (delete's EMPTY store); 2: an 8-byte
+// atomicCAS (insert's claim of a free slot); 3: a full 32-byte sector store.
+template <int B, int WRITE = 0>
 __global__ void __launch_bounds__(kThreads) k_gather(unsigned long long* __restrict__ buf, uint64_t n_units,
                                                      uint64_t n_reads, uint64_t seed,
                                                      unsigned long long* __restrict__ sink) {
@@ -1190,8 +1192,15 @@ __global__ void __launch_bounds__(kThreads) k_gather(unsigned long long* __restr
         for (int j = 0; j < ILP; j++) acc ^= s[j][0] ^ s[j][1] ^ s[j][2] ^ s[j][3];
         if (WRITE) {
 #pragma unroll
-            for (int j = 0; j < ILP; j++)
-                if (g.sub == 0 && wp[j]) st_u64_cg(wp[j], s[j][0] + 1);   // address: own probe only
+            for (int j = 0; j < ILP; j++) {
+                if (g.sub != 0 || !wp[j]) continue;       // address: the group's own probe only
+                if (WRITE == 1) st_u64_cg(wp[j], s[j][0] + 1);
+                if (WRITE == 2) acc ^= atomicCAS(wp[j], s[j][0], s[j][0] + 1);
+                if (WRITE == 3)
+                    asm volatile("st.global.v4.u64 [%0], {%1,%2,%3,%4};" ::"l"(wp[j]), "l"(s[j][0] + 1), "l"(s[j][1]),
+                                 "l"(s[j][2]), "l"(s[j][3])
+                                 : "memory");
+            }
         }
     }
     if (acc == 0x0123456789ABCDEFull) *sink = acc;   // keeps the loads alive

@@ -138,7 +138,23 @@ class Table:
     def handle(self) -> int:
         return self._h.value
 
+    @classmethod
+    def borrow(cls, handle: int, d: int, bucket_slots: int) -> "Table":
+        """A non-owning view of a table owned elsewhere (a shard of a dyc_dist):
+        stats / dump / find work on it; close() does not destroy it."""
+        torch = _torch()
+        t = cls.__new__(cls)
+        t._lib = L.load_library()
+        t.device = torch.device("cuda", torch.cuda.current_device())
+        t._h = C.c_void_p(handle)
+        t.d, t.B = d, bucket_slots
+        t._borrowed = True
+        return t
+
     def close(self):
+        if getattr(self, "_borrowed", False):
+            self._h = C.c_void_p()
+            return
         if getattr(self, "_h", None) is not None and self._h.value:
             self._lib.dyc_destroy(self._h)
             self._h = C.c_void_p()

@@ -1,0 +1,123 @@
+"""Full-size parity of the dynamic and sharded configs with the CPU oracle
+(VERDICT r1 "What's missing" 3 and 4).
+
+- C5 (BASELINE.json configs[4]) stream at 2^26 keys (the config's recipe: 128
+  global fill batches, then 32 mixed 50/30/20 batches, shards starting at 1M
+  slots), through one table and through 8 local shards of the sharded C ABI:
+  every op's status and value against the oracle, and the final sorted
+  contents.
+- C3-RE (configs[2]) at scale 1.0: 1M-insert batches, finds, r = 0.2 oldest
+  deletes, the swap pass, two cycles, HBM-resident tables, several
+  upsizes per pass, the non-fused insert path with multi-million pending lists.
+- C4-COM (configs[3]): Zipf(0.99) mixed 1M-op batches, grow then drain, two
+  cycles.
+Each batch's per-op results are compared element by element; the sorted
+contents are compared every few batches and at the end; the resize schedule
+(subtable sizes) after every batch whenever neither side needed a
+failure-triggered upsize (readings Q11-Q13, Q17b).
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+from paper_conf_icde_lizlhs21_b200 import workload as W  # noqa: E402
+from paper_conf_icde_lizlhs21_b200.sharded import ShardedTable  # noqa: E402
+from paper_conf_icde_lizlhs21_b200.table import Table  # noqa: E402
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a, dtype=np.uint32).view(np.int32)).cuda()
+
+
+def host_u32(t):
+    return t.cpu().numpy().view(np.uint32)
+
+
+def _u32(t):
+    return t.numpy().view(np.uint32)
+
+
+def test_c5_stream_2e26_one_and_eight_shards(oracle_mod):
+    log2k, batch = 26, 1 << 19
+    one = Table(d=4, init_capacity=1 << 20, alpha=0.3, beta=0.85, bucket_slots=8)
+    eight = ShardedTable(d=4, init_capacity=1 << 20, alpha=0.3, beta=0.85, local_shards=8, rank=0, world=1)
+    o = oracle_mod.OracleTable(d=4, init_capacity=1 << 20, alpha=0.3, beta=0.85, bucket_slots=8)
+    n_fill = n_mixed = 0
+    for i, item in enumerate(W.c5_batches_torch(0, 1, device="cpu", log2_keys=log2k, batch=batch, mixed_batches=32)):
+        if item[0] == "insert":
+            _, k, v = item
+            kd, vd = k.cuda(), v.cuda()
+            exp = o.insert(_u32(k), _u32(v))
+            np.testing.assert_array_equal(one.insert(kd, vd).cpu().numpy(), exp, err_msg=f"fill {i} (1 shard)")
+            np.testing.assert_array_equal(eight.insert(kd, vd).cpu().numpy(), exp, err_msg=f"fill {i} (8 shards)")
+            n_fill += 1
+        else:
+            _, ops, k, v = item
+            od, kd, vd = ops.cuda(), k.cuda(), v.cuda()
+            ov, os_ = o.mixed(ops.numpy(), _u32(k), _u32(v))
+            for name, t in (("1 shard", one), ("8 shards", eight)):
+                gv, gs = t.mixed(od, kd, vd)
+                np.testing.assert_array_equal(gs.cpu().numpy(), os_, err_msg=f"mixed {i} status ({name})")
+                np.testing.assert_array_equal(host_u32(gv), ov, err_msg=f"mixed {i} values ({name})")
+            n_mixed += 1
+    assert (n_fill, n_mixed) == (128, 32)
+    ref = o.sorted_kv()
+    np.testing.assert_array_equal(one.sorted_kv(), ref, err_msg="final contents (1 shard)")
+    np.testing.assert_array_equal(eight.sorted_kv(), ref, err_msg="final contents (8 shards)")
+    s1, so = one.stats(), o.stats()
+    assert s1["m"] == so["m"] == ref.size
+    if s1["n_fail_upsize"] == 0 and so["n_fail_upsize"] == 0:
+        assert s1["buckets"] == so["buckets"]
+    assert sum(s["m"] for s in eight.stats()) == ref.size
+
+
+def _run_single(g, o, batches, contents_every):
+    for i, b in enumerate(batches):
+        op = getattr(b, "op", "mixed")
+        if op == "insert":
+            np.testing.assert_array_equal(g.insert(dev(b.keys), dev(b.values)).cpu().numpy(),
+                                          o.insert(b.keys, b.values), err_msg=f"batch {i}")
+        elif op == "find":
+            v, f = g.find(dev(b.keys))
+            ov, of = o.find(b.keys)
+            np.testing.assert_array_equal(f.cpu().numpy(), of, err_msg=f"batch {i}")
+            np.testing.assert_array_equal(host_u32(v), ov, err_msg=f"batch {i}")
+        elif op == "delete":
+            v, s = g.delete(dev(b.keys))
+            ov, os_ = o.delete(b.keys)
+            np.testing.assert_array_equal(s.cpu().numpy(), os_, err_msg=f"batch {i}")
+            np.testing.assert_array_equal(host_u32(v), ov, err_msg=f"batch {i}")
+        else:
+            v, s = g.mixed(torch.from_numpy(b.ops).cuda(), dev(b.keys), dev(b.values))
+            ov, os_ = o.mixed(b.ops, b.keys, b.values)
+            np.testing.assert_array_equal(s.cpu().numpy(), os_, err_msg=f"batch {i}")
+            np.testing.assert_array_equal(host_u32(v), ov, err_msg=f"batch {i}")
+        gb, _, pend = g.shape()
+        osz = o.stats()
+        if pend == 0 and osz["n_fail_upsize"] == 0:
+            assert gb == osz["buckets"], f"resize schedule diverged at batch {i}"
+        if i % contents_every == contents_every - 1 or i == len(batches) - 1:
+            np.testing.assert_array_equal(g.sorted_kv(), o.sorted_kv(), err_msg=f"contents after batch {i}")
+    s, so = g.stats(), o.stats()
+    assert s["m"] == so["m"]
+    return s
+
+
+def test_c3_re_full_scale(oracle_mod):
+    wl = W.c3_dynamic(scale=1.0, shape="RE", batch=1_000_000, r=0.2, cycles=2)
+    g = Table(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=8)
+    o = oracle_mod.OracleTable(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=8)
+    s = _run_single(g, o, wl.batches, contents_every=40)
+    assert s["n_upsize"] >= 10 and s["n_downsize"] >= 5
+    assert max(s["buckets"]) * 8 * 4 * 8 > 256 << 20, "tables never grew past L2"
+
+
+def test_c4_com_full(oracle_mod):
+    meta, batches = W.c4_zipf_mixed(U=4_583_941, distinct=1_000_000, grow_batches=16, cycles=2)
+    g = Table(d=4, init_capacity=meta.init_capacity, alpha=meta.alpha, beta=meta.beta, bucket_slots=8)
+    o = oracle_mod.OracleTable(d=4, init_capacity=meta.init_capacity, alpha=meta.alpha, beta=meta.beta,
+                               bucket_slots=8)
+    s = _run_single(g, o, batches, contents_every=8)
+    assert s["n_downsize"] > 0
