@@ -97,8 +97,19 @@ typedef struct {
     uint64_t init_capacity;  /* slots; n0 = max(1, ceil(init_capacity/(d*B))) buckets per subtable (Q13) */
     uint64_t seed;           /* SplitMix64 seed of the hash constants a_s, b_s (Q1)  */
     uint32_t max_hops;       /* L_max: eviction hops per attempt before the failure list (Q6) */
-    uint32_t flags;          /* reserved, 0                                          */
+    uint32_t flags;          /* placement policy: 0 = two-choice first-fit (reading Q3,
+                                default); DYC_PLACE_PAPER_WEIGHTED = the paper's rule     */
 } dyc_config;
+
+/* dyc_config.flags: the paper's balancing rule (SURVEY §8(f)
+ * NEXT-4): a new pair goes to table i of its pair with probability
+ * proportional to n_i / C(m_i, 2) (a snapshot of the per-subtable counts taken
+ * at the start of each insert batch and after each resize of it, one streaming
+ * count pass over the table), and evictions start in that table.  Results are
+ * identical to first-fit (placement only changes where keys live); find and
+ * the insert existence check always probe both buckets in this mode, since the
+ * first-choice-full invariant does not hold under it. */
+#define DYC_PLACE_PAPER_WEIGHTED 1u
 
 typedef struct {
     uint64_t m;                       /* live keys Σ m_t                          */
@@ -284,28 +295,6 @@ dyc_status dyc_find_batch_host(dyc_table* t, const uint32_t* h_keys, uint32_t* h
 dyc_status dyc_delete_batch_host(dyc_table* t, const uint32_t* h_keys, uint32_t* h_values_out,
                                  uint8_t* h_status, uint64_t n, dyc_stream_t stream);
 
-/* Region-binned execution of large batches (SURVEY §8(a) S3-S5, S7 on B200's L2).
- * A batch of n ops over a table of NB buckets probes every bucket about n/NB
- * times per pass; when the table is much larger than L2 those probes are random
- * HBM accesses ("random accesses ... are expensive").  Binned mode
- * groups the ops by the region (2^region_log2 consecutive buckets) of the bucket
- * each pass probes, so the blocks in flight probe one L2-sized region at a time,
- * and writes the per-op results back in request order through L2-sized windows
- * of 2^out_log2 ops.  Results, statuses and the resize policy are identical to
- * the direct kernels (same passes: probe h^{t1}, then h^{t2}, P:L485-486,
- * P:L591-592; existence over both buckets before first-fit placement, Q3/Q7).
- * mode: 0 = off (default: the direct kernels), 1 = binned whenever eligible.
- * Eligible: n < 2^30, no resize in flight, and for inserts no upsize needed
- * before placement ((m + n) <= beta*N).  Measured on B200 (DESIGN.md §5,
- * profiles/r1g_binned.md) it is slower than the direct kernels at config C2, so
- * it is opt-in.  region_log2 = 0 picks ~32 MB regions; out_log2 = 0 picks 2^20
- * ops; both are raised as needed to keep at most 1024 bins.  Scratch: up to 32
- * bytes per op, owned by the table.  Errors: DYC_ERR_INVALID_ARG for mode
- * outside 0..1, region_log2 > 31 or out_log2 > 29. */
-dyc_status dyc_set_binning(dyc_table* t, int mode, int region_log2, int out_log2);
-/* Batches executed in binned mode so far, and the region count of the last one. */
-dyc_status dyc_get_binning(const dyc_table* t, uint64_t* n_binned_batches, uint32_t* last_regions);
-
 /* Kernel launch counter (for the bench's gpu_launches claim): number of kernels
  * this table has launched since creation or the last reset. */
 uint64_t dyc_launch_count(const dyc_table* t, int reset);
@@ -318,12 +307,7 @@ uint64_t dyc_launch_count(const dyc_table* t, int reset);
 #define DYC_PROF_KINDS 16
 enum {
     DYC_PROF_FIND = 0, DYC_PROF_UPSERT = 1, DYC_PROF_PLACE = 2, DYC_PROF_DELETE = 3,
-    DYC_PROF_UPSIZE = 4, DYC_PROF_DOWNSIZE = 5, DYC_PROF_REINSERT = 6, DYC_PROF_OTHER = 7,
-    /* region-binned execution (dyc_set_binning): grouping (k_bin_hist, k_bin_offsets,
-     * k_bin_scatter), find passes F1+F2, insert existence passes I1+I2, insert
-     * placement passes I3+I4, delete passes D1+D2, results in request order */
-    DYC_PROF_BIN_GROUP = 8, DYC_PROF_BIN_FIND = 9, DYC_PROF_BIN_INS = 10, DYC_PROF_BIN_PLACE = 11,
-    DYC_PROF_BIN_DELETE = 12, DYC_PROF_BIN_OUT = 13
+    DYC_PROF_UPSIZE = 4, DYC_PROF_DOWNSIZE = 5, DYC_PROF_REINSERT = 6, DYC_PROF_OTHER = 7
 };
 dyc_status dyc_profile_enable(dyc_table* t, int enable);
 dyc_status dyc_profile_read(dyc_table* t, double* ms, uint64_t* calls);
@@ -345,7 +329,7 @@ dyc_status dyc_probe_count_read(dyc_table* t, uint64_t* out6);
  * table, so find and the existence check of insert skip the second probe
  * (still <= 2 probes).  Set for every t by dyc_create / dyc_clear;
  * cleared for t by an upsize or a live resize of t, and for all t by a batch
- * that removed keys, a binned insert or a reinsert baseline (dyc_resize_ex
+ * that removed keys or a reinsert baseline (dyc_resize_ex
  * methods 1, 2).  Downsizes and placements preserve it.  Results never depend
  * on it, only the probe count does.  Batches on one table must not overlap in
  * time (one stream, or ordered by events): a delete running concurrently with

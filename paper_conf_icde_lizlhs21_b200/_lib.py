@@ -18,11 +18,11 @@ DYC_NOT_FOUND = 0xFFFFFFFF
 
 DYC_OK, DYC_ERR_INVALID_ARG, DYC_ERR_OOM, DYC_ERR_CUDA, DYC_ERR_INSERT_FAILED, DYC_ERR_NO_DEVICE, DYC_ERR_NCCL = range(7)
 DYC_NCCL_UNIQUE_ID_BYTES = 128
+DYC_PLACE_PAPER_WEIGHTED = 1
 DYC_RESIZE_SPLIT, DYC_RESIZE_REINSERT_SUBTABLE, DYC_RESIZE_REHASH_ALL = range(3)
 DYC_PROF_KINDS = 16
 DYC_GATHER_WRITE, DYC_GATHER_CAS, DYC_GATHER_SECTOR = 1, 2, 4
-PROF_NAMES = ["k_find", "k_upsert", "k_place", "k_delete", "k_upsize", "k_downsize", "k_reinsert", "other",
-              "bin_group", "bin_find", "bin_ins", "bin_place", "bin_delete", "bin_out"]
+PROF_NAMES = ["k_find", "k_upsert", "k_place", "k_delete", "k_upsize", "k_downsize", "k_reinsert", "other"]
 _STATUS_NAMES = ["DYC_OK", "DYC_ERR_INVALID_ARG", "DYC_ERR_OOM", "DYC_ERR_CUDA",
                  "DYC_ERR_INSERT_FAILED", "DYC_ERR_NO_DEVICE", "DYC_ERR_NCCL"]
 
@@ -119,8 +119,6 @@ SIGNATURES = {
     "dyc_find_batch_host": (_I, [_TP, _P, _P, _P, _U64, _P]),
     "dyc_delete_batch_host": (_I, [_TP, _P, _P, _P, _U64, _P]),
     "dyc_launch_count": (_U64, [_TP, _I]),
-    "dyc_set_binning": (_I, [_TP, _I, _I, _I]),
-    "dyc_get_binning": (_I, [_TP, C.POINTER(_U64), C.POINTER(_U32)]),
     "dyc_profile_enable": (_I, [_TP, _I]),
     "dyc_profile_read": (_I, [_TP, _P, _P]),
     "dyc_probe_count_enable": (_I, [_TP, _I]),

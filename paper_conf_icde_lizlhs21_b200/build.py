@@ -14,7 +14,7 @@ CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libdyc.so")
 SOURCES = ["dyc_api.cu", "dyc_dist.cu"]
-DEPS = SOURCES + ["dyc_kernels.cuh", "dyc_device.cuh", "dyc_binned.cuh", "dyw_api.cuh", "dyw_kernels.cuh"]
+DEPS = SOURCES + ["dyc_kernels.cuh", "dyc_device.cuh", "dyw_api.cuh", "dyw_kernels.cuh"]
 
 COMPILE_FLAGS = [
     "-O3", "-std=c++17", "-lineinfo",

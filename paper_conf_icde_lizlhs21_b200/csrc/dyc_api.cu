@@ -23,7 +23,6 @@
 #include "dycuckoo.h"
 #include "dyc_device.cuh"
 #include "dyc_kernels.cuh"
-#include "dyc_binned.cuh"
 
 using namespace dyc;
 
@@ -88,7 +87,7 @@ struct dyc_table {
     // first-choice-full invariant per subtable (TableView::clean):
     // set for all on create / clear; an upsize of t (split buckets are no longer
     // full) or a live resize of t clears bit t; a batch that removed keys, a
-    // binned insert (its cleanup pass removes tentative copies) or a reinsert
+    // reinsert
     // baseline clears all.  Downsizes and placements (first-fit, evictions)
     // preserve it.
     uint32_t clean = 0;
@@ -102,6 +101,11 @@ struct dyc_table {
     uint64_t lazy_n = 0;
     cudaEvent_t lazy_ev = nullptr;
     uint64_t del_n = 0;                    // ops of the delete batch in flight
+    // placement policy (dyc_config.flags): first-fit (reading Q3) or the
+    // paper's weighted rule; the latter keeps d_w, a per-batch
+    // snapshot of n_t / C(m_t, 2), and gives up the first-choice-full invariant
+    bool weighted = false;
+    float* d_w = nullptr;
     bool count_probes = false;             // dyc_probe_count_enable (measurement)
     unsigned long long* d_probe = nullptr; // {ops, second probes} x {find, upsert, delete}
     unsigned long long* list[2] = {nullptr, nullptr};
@@ -140,14 +144,6 @@ struct dyc_table {
     uint64_t peak_table_bytes = 0;   // high-water mark of the subtables' bytes (cache cap)
     uint64_t n_sync = 0;          // counter read-backs (host waits on the stream)
     double sync_ms = 0.0;
-    // region-binned execution of large batches (dyc_binned.cuh, dyc_set_binning)
-    int bin_mode = 0;                      // 0 off (direct kernels), 1 binned whenever eligible
-    int bin_rlog2 = 0;                     // log2 buckets per region (0: ~32 MB regions)
-    int bin_olog2 = 20;                    // log2 ops per result group
-    uint32_t* bin_buf = nullptr;           // per-op record streams (u32 words)
-    uint64_t bin_cap = 0;                  // words
-    uint64_t n_binned = 0;                 // batches run binned
-    uint32_t last_regions = 0;
     // per-kernel event profiling (dyc_profile_*)
     bool prof = false;
     struct Rec { int kind; cudaEvent_t a, b; };
@@ -199,8 +195,9 @@ struct dyc_table {
         v.dm1 = cfg.d - 1;
         v.recip_dm1 = (65536u + v.dm1 - 1) / v.dm1;
         v.max_hops = cfg.max_hops;
-        v.clean = rz.active ? (clean & ~(1u << rz.ti)) : clean;
+        v.clean = weighted ? 0u : (rz.active ? (clean & ~(1u << rz.ti)) : clean);
         v.probe = count_probes ? d_probe : nullptr;
+        v.wsel = weighted ? d_w : nullptr;
         return v;
     }
 };
@@ -366,6 +363,26 @@ dyc_status ensure_lists(dyc_table* t, uint64_t n, cudaStream_t st) {
     return DYC_OK;
 }
 
+// Paper-weighted mode: snapshot w[t] = n_t / C(m_t, 2) from a count
+// of every subtable (one streaming pass over the table, in stream order, so it
+// sees the state the next placement kernel starts from).
+template <int B>
+dyc_status refresh_weights(dyc_table* t, cudaStream_t st) {
+    if (!t->weighted) return DYC_OK;
+    CU(cudaMemsetAsync(t->d_ctr + C_COUNT0, 0, t->cfg.d * sizeof(unsigned long long), st));
+    const TableView tv = t->view();
+    for (uint32_t i = 0; i < t->cfg.d; i++) {
+        ProfScope ps(t, DYC_PROF_OTHER, st);
+        k_count<B><<<grid_for(t->nb[i] * B, kThreads * 8), kThreads, 0, st>>>(tv, i, t->d_ctr);
+    }
+    {
+        ProfScope ps(t, DYC_PROF_OTHER, st);
+        k_weights<<<1, 32, 0, st>>>(tv, B, t->d_ctr, t->d_w);
+    }
+    CU(cudaGetLastError());
+    return DYC_OK;
+}
+
 template <int B>
 dyc_status upsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
     const uint64_t n_old = t->nb[ti], n_new = 2 * n_old;
@@ -462,6 +479,7 @@ dyc_status downsize_launch(dyc_table* t, uint32_t ti, cudaStream_t st) {
     dev_free(t, t->sub[ti], st);
     t->sub[ti] = (unsigned long long*)p;
     t->nb[ti] = h;
+    TRY(refresh_weights<B>(t, st));
     return launch_place<B>(t, 0, t->d_ctr + C_RESIDUAL, 0, true, st);
 }
 
@@ -652,218 +670,6 @@ dyc_status launch_apply(dyc_table* t, const unsigned long long* list, bool del, 
     return DYC_OK;
 }
 
-// ------------------------------------------------------------------ binned path
-// Region-binned execution (dyc_binned.cuh) of batches much larger than L2:
-// opt-in (dyc_set_binning mode 1); see profiles/r1g_binned.md for its
-// measurements against the direct kernels.  Eligible: no resize in flight,
-// n < 2^30 ops.
-bool bin_plan(dyc_table* t, uint64_t n, BinCtx& bc) {
-    if (t->bin_mode != 1 || t->rz.active || n == 0 || n >= (1ull << 30)) return false;
-    const uint64_t bucket_bytes = (uint64_t)t->cfg.bucket_slots * 8;
-    uint32_t rl = (uint32_t)t->bin_rlog2;
-    if (rl == 0)
-        while ((bucket_bytes << (rl + 1)) <= (32ull << 20)) rl++;     // 32 MB regions (measured best)
-    auto regions = [&](uint32_t r) {
-        uint64_t R = 0;
-        for (uint32_t i = 0; i < t->cfg.d; i++) R += (t->nb[i] + (1ull << r) - 1) >> r;
-        return R;
-    };
-    while (regions(rl) > kMaxBins) rl++;
-    uint32_t ol = std::max<uint32_t>(kChunkShift, (uint32_t)t->bin_olog2);
-    while (((n + (1ull << ol) - 1) >> ol) > kMaxBins) ol++;
-    memset(&bc, 0, sizeof(bc));
-    uint64_t acc = 0;
-    for (uint32_t i = 0; i < t->cfg.d; i++) {       // subtables start on region boundaries
-        bc.gbase[i] = acc;
-        acc += ((t->nb[i] + (1ull << rl) - 1) >> rl) << rl;
-    }
-    if (acc > 0xFFFFFFFFull) return false;          // global bucket indices are 32-bit
-    bc.rshift = rl;
-    bc.R = (uint32_t)(acc >> rl);
-    bc.ishift = ol;
-    bc.Rout = (uint32_t)((n + (1ull << ol) - 1) >> ol);
-    bc.P = (uint32_t)(t->num_sms * kBinBPS);
-    return true;
-}
-
-// Scratch of one binned batch.  Region streams A (t1 regions) and Bq (t2
-// regions) of uint4 records, the result stream (uint2 find/delete, uint32
-// insert); each with per-chunk fills, bin bases and cursors (dyc_binned.cuh).
-struct BinPlan {
-    uint32_t chA, chR;                   // chunks allocated per region stream / result stream
-    uint32_t *baseA, *ctrA, *baseB, *ctrB, *baseR, *ctrR, *tiles;
-    uint32_t *fillA, *fillB, *fillR;
-    uint4 *A, *Bq;
-    void* Res;
-};
-
-// Chunks of a region stream: the bins' expected capacities (the same integer
-// formula as k_bin_init_regions), rounded to kPoolAlign, plus a worst-case pool.
-uint32_t region_stream_chunks(const dyc_table* t, const BinCtx& bc, uint64_t n, uint32_t passes) {
-    uint64_t area = 0;
-    for (uint32_t r = 0; r < bc.R; r++) {
-        const uint64_t g0 = (uint64_t)r << bc.rshift;
-        uint32_t ti = 0;
-        for (uint32_t u = 1; u < t->cfg.d; u++)
-            if (bc.gbase[u] <= g0) ti = u;
-        const uint64_t lo = g0 - bc.gbase[ti];
-        const uint64_t hi = std::min<uint64_t>(t->nb[ti], lo + (1ull << bc.rshift));
-        area += bin_cap_chunks(region_expect(n, t->cfg.d, t->nb[ti], hi > lo ? hi - lo : 0), bc.P, passes);
-    }
-    area = (area + kPoolAlign - 1) / kPoolAlign * kPoolAlign;
-    const uint64_t pool = (n + kChunk - 1) / kChunk + (uint64_t)passes * bc.P * bc.R + kPoolAlign;
-    return (uint32_t)(area + pool);
-}
-
-dyc_status bin_alloc(dyc_table* t, const BinCtx& bc, uint64_t n, BinPlan& pl, cudaStream_t st) {
-    pl.chA = region_stream_chunks(t, bc, n, 1);
-    pl.chR = bc.Rout * (((1u << bc.ishift) >> kChunkShift) + 2 * (bc.P + 1));
-    const uint64_t small = 6ull * (kMaxBins + 1) + kTileCtrs;
-    const uint64_t words = small + 2ull * pl.chA + pl.chR + 8          // counters, fills (+ align)
-                           + 2ull * pl.chA * kChunk * 4                // A, Bq records (4 words each)
-                           + (uint64_t)pl.chR * kChunk * 2;            // results (<= 2 words each)
-    if (words > t->bin_cap) {
-        if (t->bin_buf) dev_free(t, t->bin_buf, st);
-        t->bin_buf = nullptr;
-        t->bin_cap = 0;
-        TRY(dev_alloc(t, (void**)&t->bin_buf, words * 4, st));
-        t->bin_cap = words;
-    }
-    uint32_t* w = t->bin_buf;
-    pl.baseA = w; w += kMaxBins + 1;
-    pl.ctrA = w;  w += kMaxBins + 1;
-    pl.baseB = w; w += kMaxBins + 1;
-    pl.ctrB = w;  w += kMaxBins + 1;
-    pl.baseR = w; w += kMaxBins + 1;
-    pl.ctrR = w;  w += kMaxBins + 1;
-    pl.tiles = w; w += kTileCtrs;
-    pl.fillA = w; w += pl.chA;
-    pl.fillB = w; w += pl.chA;
-    pl.fillR = w; w += pl.chR;
-    w = (uint32_t*)(((uintptr_t)w + 15) & ~(uintptr_t)15);
-    pl.A = (uint4*)w;  w += (uint64_t)pl.chA * kChunk * 4;
-    pl.Bq = (uint4*)w; w += (uint64_t)pl.chA * kChunk * 4;
-    pl.Res = w;
-    return DYC_OK;
-}
-
-template <class Rec>
-Stream<Rec> stream_of(Rec* rec, uint32_t* fill, uint32_t* ctr, const uint32_t* base, uint32_t nbins, uint32_t nch) {
-    return Stream<Rec>{rec, fill, ctr, base, nbins, nch};
-}
-
-// Emptying a region stream before a kernel fills it: chunk fills to 0 and the
-// bin ranges / cursors from the expected counts.
-dyc_status region_reset(dyc_table* t, const BinCtx& bc, uint64_t n, uint32_t* fill, uint32_t nch, uint32_t* base,
-                        uint32_t* ctr, cudaStream_t st) {
-    CU(cudaMemsetAsync(fill, 0, (size_t)nch * 4, st));
-    k_bin_init_regions<<<1, 1024, 0, st>>>(t->view(), bc, n, 1, base, ctr);
-    t->launches++;
-    return DYC_OK;
-}
-
-template <class K>
-void allow_smem(K kernel) {
-    cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024);
-}
-
-// Bin ranges of streams A and R, tile counters, then the grouping of the batch
-// by the region of h^{t1} into stream A.
-dyc_status bin_group(dyc_table* t, const BinCtx& bc, const uint32_t* keys, const uint32_t* vals, uint64_t n,
-                     uint32_t* rv_out, uint8_t* rs_out, BinPlan& pl, cudaStream_t st) {
-    const TableView tv = t->view();
-    ProfScope ps(t, DYC_PROF_BIN_GROUP, st);
-    TRY(region_reset(t, bc, n, pl.fillA, pl.chA, pl.baseA, pl.ctrA, st));
-    CU(cudaMemsetAsync(pl.fillR, 0, (size_t)pl.chR * 4, st));
-    k_bin_init_results<<<1, 1024, 0, st>>>(bc, 2, pl.baseR, pl.ctrR, pl.tiles);
-    allow_smem(k_bin_scatter);
-    const Stream<uint4> A = stream_of(pl.A, pl.fillA, pl.ctrA, pl.baseA, bc.R, pl.chA);
-    k_bin_scatter<<<bc.P, kThreads, 6 * bc.R * 4, st>>>(tv, bc, keys, vals, n, A, rv_out, rs_out);
-    t->launches++;
-    CU(cudaGetLastError());
-    return DYC_OK;
-}
-
-template <int B>
-constexpr int bin_U() { return B <= 8 ? DYC_BIN_U : (B == 16 ? 2 : 1); }
-
-// find (DEL = false) / delete (DEL = true): group by t1 region, F1/D1, F2/D2,
-// results back in request order.
-template <int B, bool DEL>
-dyc_status binned_fd(dyc_table* t, const BinCtx& bc, const uint32_t* keys, uint32_t* vals, uint8_t* flag, uint64_t n,
-                     cudaStream_t st) {
-    constexpr int U = bin_U<B>();
-    BinPlan pl{};
-    TRY(bin_alloc(t, bc, n, pl, st));
-    TRY(bin_group(t, bc, keys, nullptr, n, vals, flag, pl, st));
-    TRY(region_reset(t, bc, n, pl.fillB, pl.chA, pl.baseB, pl.ctrB, st));
-    const TableView tv = t->view();
-    const Stream<uint4> A = stream_of(pl.A, pl.fillA, pl.ctrA, pl.baseA, bc.R, pl.chA);
-    const Stream<uint4> Bs = stream_of(pl.Bq, pl.fillB, pl.ctrB, pl.baseB, bc.R, pl.chA);
-    const Stream<uint2> Rs = stream_of((uint2*)pl.Res, pl.fillR, pl.ctrR, pl.baseR, bc.Rout, pl.chR);
-    {
-        ProfScope ps(t, DEL ? DYC_PROF_BIN_DELETE : DYC_PROF_BIN_FIND, st);
-        allow_smem(k_bin_fd<B, U, DEL, false>);
-        allow_smem(k_bin_fd<B, U, DEL, true>);
-        k_bin_fd<B, U, DEL, false><<<bc.P, kThreads, 6 * (bc.R + bc.Rout) * 4, st>>>(tv, bc, A, Bs, Rs, pl.tiles,
-                                                                                     t->d_ctr);
-        k_bin_fd<B, U, DEL, true><<<bc.P, kThreads, 6 * bc.Rout * 4, st>>>(tv, bc, Bs, Bs, Rs, pl.tiles + 1,
-                                                                           t->d_ctr);
-        t->launches++;
-    }
-    CU(cudaGetLastError());
-    if (vals || flag) {
-        ProfScope ps(t, DYC_PROF_BIN_OUT, st);
-        k_bin_out<uint2><<<grid_for((uint64_t)pl.chR * kChunk, (uint64_t)kThreads * 8), kThreads, 0, st>>>(Rs, vals,
-                                                                                                      flag);
-    }
-    CU(cudaGetLastError());
-    t->n_binned++;
-    t->last_regions = bc.R;
-    return DYC_OK;
-}
-
-// insert (FUSE case): group by t1 region, I1 (t1 existence + tentative t1
-// placement), I2 (t2 existence, t2 placement), I3 (cleanup of tentative copies
-// of keys that existed in t2); pending keys are then placed by insert_end.
-template <int B>
-dyc_status binned_ins(dyc_table* t, const BinCtx& bc, const uint32_t* keys, const uint32_t* vals, uint8_t* status,
-                      uint64_t n, cudaStream_t st) {
-    constexpr int U = bin_U<B>();
-    BinPlan pl{};
-    TRY(bin_alloc(t, bc, n, pl, st));
-    TRY(bin_group(t, bc, keys, vals, n, nullptr, status, pl, st));
-    const TableView tv = t->view();
-    const Stream<uint4> A = stream_of(pl.A, pl.fillA, pl.ctrA, pl.baseA, bc.R, pl.chA);
-    const Stream<uint4> Bs = stream_of(pl.Bq, pl.fillB, pl.ctrB, pl.baseB, bc.R, pl.chA);
-    const Stream<uint32_t> Rs = stream_of(status ? (uint32_t*)pl.Res : (uint32_t*)nullptr, pl.fillR, pl.ctrR,
-                                          pl.baseR, bc.Rout, pl.chR);
-    unsigned long long* pend = t->list[0];
-    {
-        ProfScope ps(t, DYC_PROF_BIN_INS, st);
-        allow_smem(k_bin_ins<B, U, false>);
-        allow_smem(k_bin_ins<B, U, true>);
-        TRY(region_reset(t, bc, n, pl.fillB, pl.chA, pl.baseB, pl.ctrB, st));
-        k_bin_ins<B, U, false><<<bc.P, kThreads, 6 * (bc.R + bc.Rout) * 4, st>>>(tv, bc, A, Bs, Rs, pend, pl.tiles,
-                                                                                 t->d_ctr);
-        TRY(region_reset(t, bc, n, pl.fillA, pl.chA, pl.baseA, pl.ctrA, st));
-        k_bin_ins<B, U, true><<<bc.P, kThreads, 6 * (bc.R + bc.Rout) * 4, st>>>(tv, bc, Bs, A, Rs, pend,
-                                                                                pl.tiles + 1, t->d_ctr);
-        k_bin_cleanup<B, U><<<bc.P, kThreads, 0, st>>>(tv, bc, A, pl.tiles + 2, t->d_ctr);
-        t->launches += 2;
-    }
-    CU(cudaGetLastError());
-    if (status) {
-        ProfScope ps(t, DYC_PROF_BIN_OUT, st);
-        k_bin_out<uint32_t><<<grid_for((uint64_t)pl.chR * kChunk, (uint64_t)kThreads * 8), kThreads, 0, st>>>(
-            Rs, nullptr, status);
-    }
-    CU(cudaGetLastError());
-    t->n_binned++;
-    t->last_regions = bc.R;
-    return DYC_OK;
-}
-
 // insert = begin (scratch, counters, FUSE decision) + one k_upsert per chunk of
 // the batch + end (resize decision, placement, failures, alpha loop).  Splitting
 // the upsert into chunks is invisible to the semantics: every chunk only probes,
@@ -881,6 +687,7 @@ dyc_status insert_begin(dyc_table* t, uint64_t n, cudaStream_t st, bool& fuse) {
     if (t->rz.active && (double)(t->m + n) > t->cfg.beta * (double)t->N_after()) TRY(live_commit<B>(t, st));
     TRY(ensure_lists(t, n, st));
     TRY(zero_ctr(t, st));
+    TRY(refresh_weights<B>(t, st));
     fuse = t->rz.active || (double)(t->m + n) <= t->cfg.beta * (double)t->N();
     return DYC_OK;
 }
@@ -930,6 +737,7 @@ dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
             TRY(upsize_table<B>(t, (uint32_t)t->smallest(), st));
             t->n_upsize++;
         }
+        TRY(refresh_weights<B>(t, st));   // after an upsize the bigger table draws more
     }
     const uint64_t ev0 = t->n_evict;
     dyc_status s = place_and_settle<B>(t, 0, t->d_ctr + C_PENDING, 0, !fuse, st);
@@ -946,12 +754,7 @@ dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals,
                        cudaStream_t st) {
     bool fuse = false;
     TRY(insert_begin<B>(t, n, st, fuse));
-    BinCtx bc;
-    if (fuse && bin_plan(t, n, bc)) {
-        t->clean = 0;               // its cleanup pass removes tentative t1 copies
-        TRY(binned_ins<B>(t, bc, keys, vals, status, n, st));
-    }
-    else TRY(insert_chunk<B>(t, keys, vals, status, n, fuse, st));
+    TRY(insert_chunk<B>(t, keys, vals, status, n, fuse, st));
     return insert_end<B>(t, fuse, st);
 }
 
@@ -960,8 +763,6 @@ dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t
                      cudaStream_t st) {
     constexpr int ILP = (B <= 16) ? DYC_FIND_ILP : 2;
     constexpr uint64_t per_block = (uint64_t)(kThreads / (B / 4)) * ILP;   // queries per block per pass
-    BinCtx bc;
-    if (bin_plan(t, n, bc)) return binned_fd<B, false>(t, bc, keys, vals, found, n, st);
     {
         ProfScope ps(t, DYC_PROF_FIND, st);
         k_find<B, ILP><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n);
@@ -1030,9 +831,7 @@ template <int B>
 dyc_status delete_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
                        cudaStream_t st) {
     TRY(delete_prep<B>(t, n, st));
-    BinCtx bc;
-    if (bin_plan(t, n, bc)) TRY((binned_fd<B, true>(t, bc, keys, vals, status, n, st)));
-    else TRY(delete_chunk<B>(t, keys, vals, status, n, st));
+    TRY(delete_chunk<B>(t, keys, vals, status, n, st));
     return delete_end<B>(t, st);
 }
 
@@ -1380,6 +1179,8 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
     if (cfg->alpha > cfg->beta * (double)d / (double)(d + 1))
         return set_err(DYC_ERR_INVALID_ARG, "need alpha <= beta*d/(d+1) (P:L315-318)");
     if (cfg->max_hops < 1) return set_err(DYC_ERR_INVALID_ARG, "max_hops must be >= 1");
+    if (cfg->flags & ~(uint32_t)DYC_PLACE_PAPER_WEIGHTED)
+        return set_err(DYC_ERR_INVALID_ARG, "flags: only DYC_PLACE_PAPER_WEIGHTED is defined");
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
         cudaGetLastError();
@@ -1425,6 +1226,9 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
     if (s == DYC_OK && cudaMemset(t->d_ctr, 0, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMemset");
     if (s == DYC_OK && cudaMalloc(&t->d_probe, 6 * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMalloc");
     if (s == DYC_OK && cudaMemset(t->d_probe, 0, 6 * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMemset");
+    t->weighted = (cfg->flags & DYC_PLACE_PAPER_WEIGHTED) != 0;
+    if (s == DYC_OK && cudaMalloc(&t->d_w, DYC_MAX_D * sizeof(float)) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMalloc");
+    if (s == DYC_OK && cudaMemset(t->d_w, 0, DYC_MAX_D * sizeof(float)) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMemset");
     t->clean = (1u << d) - 1u;      // an empty table satisfies the invariant
     if (s == DYC_OK && cudaMallocHost(&t->h_ctr, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMallocHost");
     if (s == DYC_OK && cudaDeviceSynchronize() != cudaSuccess) s = cuda_err(cudaGetLastError(), "create");
@@ -1455,6 +1259,7 @@ dyc_status dyc_destroy(dyc_table* t) {
     trim_cache(t);
     if (t->d_ctr) cudaFree(t->d_ctr);
     if (t->d_probe) cudaFree(t->d_probe);
+    if (t->d_w) cudaFree(t->d_w);
     if (t->rz.ctr) cudaFree(t->rz.ctr);
     if (t->rz.start) cudaEventDestroy(t->rz.start);
     if (t->rz.done) cudaEventDestroy(t->rz.done);
@@ -1724,23 +1529,6 @@ dyc_status dyc_delete_batch_host(dyc_table* t, const uint32_t* h_keys, uint32_t*
     if (n == 0) return DYC_OK;
     if (!h_keys) return set_err(DYC_ERR_INVALID_ARG, "null keys");
     DISPATCH_B(t, delete_host_impl<B_>(t, h_keys, h_values_out, h_status, n, S(stream)));
-}
-
-dyc_status dyc_set_binning(dyc_table* t, int mode, int region_log2, int out_log2) {
-    TRY(check_table(t));
-    if (mode < 0 || mode > 1 || region_log2 < 0 || region_log2 > 31 || out_log2 < 0 || out_log2 > 29)
-        return set_err(DYC_ERR_INVALID_ARG, "dyc_set_binning: mode 0..1, region_log2 0..31, out_log2 0..29");
-    t->bin_mode = mode;
-    t->bin_rlog2 = region_log2;
-    t->bin_olog2 = out_log2 ? out_log2 : 20;
-    return DYC_OK;
-}
-
-dyc_status dyc_get_binning(const dyc_table* t, uint64_t* n_binned_batches, uint32_t* last_regions) {
-    TRY(check_table(t));
-    if (n_binned_batches) *n_binned_batches = t->n_binned;
-    if (last_regions) *last_regions = t->last_regions;
-    return DYC_OK;
 }
 
 uint64_t dyc_launch_count(const dyc_table* t, int reset) {

@@ -53,6 +53,10 @@ struct TableView {
     // measurement only (dyc_probe_count_enable): {ops, second probes} per kernel
     // kind (find, upsert, delete); nullptr in normal operation
     unsigned long long* probe;
+    // the paper's balancing rule (DYC_PLACE_PAPER_WEIGHTED):
+    // w[t] = n_t / max(C(m_t, 2), 1) per subtable, a snapshot taken at
+    // the start of the batch; nullptr = two-choice first-fit (reading Q3)
+    const float* wsel;
 };
 
 // Shared-memory copy of the per-subtable fields, indexed by a lane-varying t.
@@ -60,12 +64,18 @@ struct SmemView {
     SubView sub[kMaxD];
     uint32_t a[kMaxD + 2];
     uint32_t b[kMaxD + 2];
+    float w[kMaxD];              // TableView::wsel copied (0 when first-fit)
+    uint32_t weighted;
 };
 
 __device__ __forceinline__ void load_view(const TableView& tv, SmemView& s) {
     const uint32_t i = threadIdx.x;
-    if (i < tv.d) s.sub[i] = tv.sub[i];
+    if (i < tv.d) {
+        s.sub[i] = tv.sub[i];
+        s.w[i] = tv.wsel ? tv.wsel[i] : 0.f;
+    }
     if (i < tv.d + 2) { s.a[i] = tv.a[i]; s.b[i] = tv.b[i]; }
+    if (i == 0) s.weighted = tv.wsel != nullptr;
     __syncthreads();
 }
 
@@ -97,6 +107,18 @@ __device__ __forceinline__ Pair pair_of(const TableView& tv, uint32_t k) {
     uint32_t f = (q * tv.recip_dm1) >> 16;
     uint32_t r = q - f * tv.dm1;
     return Pair{f, r + (r >= f ? 1u : 0u)};
+}
+
+// The paper's initial table choice (also after an upsize P:L384): a new
+// pair goes to table i of its pair with probability proportional to
+// n_i / C(m_i, 2).  The uniform draw is a hash of the key (counter-based, so a
+// key's choice is fixed within a batch).  Returns true for the second table.
+__device__ __forceinline__ bool weighted_second(const SmemView& s, uint32_t t1, uint32_t t2, uint32_t k) {
+    const float w1 = s.w[t1], w2 = s.w[t2];
+    uint32_t x = k ^ 0x2545F491u;
+    x ^= x >> 16; x *= 0x7FEB352Du; x ^= x >> 15; x *= 0x846CA68Bu; x ^= x >> 16;
+    const float u = (float)(x >> 8) * (1.0f / 16777216.0f);
+    return u * (w1 + w2) >= w1;
 }
 
 __device__ __forceinline__ uint32_t bucket_of(const SmemView& s, uint32_t t, uint32_t k) {

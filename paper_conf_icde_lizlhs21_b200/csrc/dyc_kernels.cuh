@@ -57,7 +57,6 @@ enum CounterIdx : int {
     C_SECOND = 8,     // keys in their second-choice subtable (stats)
     C_RES_TOTAL = 9,  // residuals over several downsizes of one alpha loop
     C_DEFER = 10,     // ops on a subtable locked by a resize in flight (NEXT-1)
-    C_CLEANUP = 11,   // binned insert: keys placed in t1 by I1 that turned out to live in t2
     C_COUNT0 = 16,    // per-subtable live counts [16, 32)
     C_N = 32
 };
@@ -331,6 +330,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
         bool need2[U], isnew[U], placed[U];
         int j1[U], j2[U];
         bool lk1[U], lk2[U];
+        bool ch2[U];                     // paper-weighted mode: the new key's table is t2
 #if DYC_UPSERT_SPEC
         // speculative: both candidate buckets are read together (one round trip);
         // the t2 read is wasted only for keys found in t1 (updates)
@@ -345,6 +345,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                 const Pair p = pair_of(tv, k[u]);
                 lk1[u] = LK && p.t1 == locked;
                 lk2[u] = LK && p.t2 == locked;
+                ch2[u] = sv.weighted && weighted_second(sv, p.t1, p.t2, k[u]);
                 b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
                 b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
                 probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
@@ -376,6 +377,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                 const Pair p = pair_of(tv, k[u]);
                 lk1[u] = LK && p.t1 == locked;
                 lk2[u] = LK && p.t2 == locked;
+                ch2[u] = sv.weighted && weighted_second(sv, p.t1, p.t2, k[u]);
                 c1[u] = ((tv.clean >> p.t1) & 1u) && !lk1[u];
                 b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
                 b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
@@ -422,6 +424,15 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
             placed[u] = false;
         }
         if (FUSE) {
+            // paper-weighted mode: only the chosen table's bucket is a candidate
+            // (P:L361); a full one sends the key to k_place, which evicts there
+            if (sv.weighted) {
+#pragma unroll
+                for (int u = 0; u < U; u++) {
+                    if (ch2[u]) em1[u] = 0;
+                    else em2[u] = 0;
+                }
+            }
             coop_cas_multi<G, U>(g, b1, em1, isnew, kv, placed);
             coop_cas_multi<G, U>(g, b2, em2, isnew, kv, placed);
         }
@@ -487,8 +498,9 @@ __global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv
             // without first-fit, hop 0 evicts from t1 without a probe: k_upsert
             // saw that bucket full; its t2 bucket may be unread (first-choice-full
             // shortcut) and evicting from a non-full bucket would break the
-            // invariant for the victim
-            t = p.t1;
+            // invariant for the victim.  Paper-weighted mode: the chosen table
+            // plays t1's part (probed once, then evicted from).
+            t = (sv.weighted && weighted_second(sv, p.t1, p.t2, k)) ? p.t2 : p.t1;
             hop = 0;
         }
         if (!__any_sync(kFull, phase >= 0)) break;
@@ -514,7 +526,8 @@ __global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv
             phase = -1;
         } else if (act && phase < 2) {
             const Pair p = pair_of(tv, k);
-            if (phase == 0) { phase = 1; t = p.t2; }
+            if (sv.weighted) { phase = 2; hop = 0; }        // evict from the chosen table
+            else if (phase == 0) { phase = 1; t = p.t2; }
             else { phase = 2; hop = 0; t = (mix32(k) & 1u) ? p.t2 : p.t1; }
         } else if (evict) {
             ev += (g.sub == 0);
@@ -808,6 +821,18 @@ __global__ void __launch_bounds__(kThreads) k_downsize(const unsigned long long*
 }
 
 // ---------------------------------------------------------- stats / dump (S10)
+// Paper-weighted placement snapshot: w[t] = n_t / max(C(m_t, 2), 1)
+// from the live counts k_count left in ctr[C_COUNT0 + t] (n_t in slots; the
+// common factor B cancels in the ratio).
+__global__ void k_weights(TableView tv, uint32_t B, const unsigned long long* __restrict__ ctr, float* __restrict__ w) {
+    const uint32_t t = threadIdx.x;
+    if (t >= tv.d) return;
+    const double m = (double)ctr[C_COUNT0 + t];
+    double c = m * (m - 1.0) / 2.0;
+    if (c < 1.0) c = 1.0;
+    w[t] = (float)((double)tv.sub[t].n * (double)B / c);
+}
+
 template <int B>
 __global__ void __launch_bounds__(kThreads) k_count(TableView tv, uint32_t t, unsigned long long* __restrict__ ctr) {
     const unsigned long long* slots = tv.sub[t].slots;

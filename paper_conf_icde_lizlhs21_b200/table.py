@@ -102,7 +102,7 @@ class Table:
 
     def __init__(self, d: int = 4, init_capacity: int = 4096, alpha: float = 0.3, beta: float = 0.85,
                  bucket_slots: int = 8, seed: int = 0x5EED0001, max_hops: int = 64, device=None,
-                 binning: Optional[Tuple[int, int, int]] = None):
+                 placement: str = "first_fit"):
         torch = _torch()
         self._lib = L.load_library()
         if not torch.cuda.is_available():
@@ -113,26 +113,16 @@ class Table:
         L.check(self._lib.dyc_config_default(C.byref(cfg)), "dyc_config_default")
         cfg.d, cfg.bucket_slots, cfg.alpha, cfg.beta = d, bucket_slots, alpha, beta
         cfg.init_capacity, cfg.seed, cfg.max_hops = init_capacity, seed, max_hops
+        if placement not in ("first_fit", "paper_weighted"):
+            raise ValueError("placement must be 'first_fit' (reading Q3) or 'paper_weighted' (P:L361)")
+        cfg.flags = L.DYC_PLACE_PAPER_WEIGHTED if placement == "paper_weighted" else 0
+        self.placement = placement
         self.cfg = cfg
         h = C.c_void_p()
         with torch.cuda.device(self.device):
             L.check(self._lib.dyc_create_ex(C.byref(cfg), C.byref(h)), "dyc_create_ex")
         self._h = h
         self.d, self.B = d, bucket_slots
-        if binning is not None:
-            self.set_binning(*binning)
-
-    def set_binning(self, mode: int = 0, region_log2: int = 0, out_log2: int = 0) -> None:
-        """Region-binned execution of large batches (dyc_set_binning): mode 0 off
-        (direct kernels, default), 1 binned whenever eligible; region_log2 /
-        out_log2 = 0 pick the defaults."""
-        L.check(self._lib.dyc_set_binning(self._h, mode, region_log2, out_log2), "dyc_set_binning")
-
-    def binning_info(self) -> Tuple[int, int]:
-        """(batches executed binned so far, regions of the last one)."""
-        n, r = C.c_uint64(), C.c_uint32()
-        L.check(self._lib.dyc_get_binning(self._h, C.byref(n), C.byref(r)), "dyc_get_binning")
-        return int(n.value), int(r.value)
 
     @property
     def handle(self) -> int:

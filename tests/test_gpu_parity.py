@@ -28,9 +28,9 @@ def host_u32(t):
     return t.cpu().numpy().view(np.uint32)
 
 
-def make_pair(oracle_mod, wl, B=4, max_hops=64, seed=0x5EED0001, binning=None):
+def make_pair(oracle_mod, wl, B=4, max_hops=64, seed=0x5EED0001):
     g = Table(d=wl.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta,
-              bucket_slots=B, max_hops=max_hops, seed=seed, binning=binning)
+              bucket_slots=B, max_hops=max_hops, seed=seed)
     o = oracle_mod.OracleTable(d=wl.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta,
                                bucket_slots=B, max_hops=max_hops, seed=seed)
     return g, o
@@ -44,8 +44,8 @@ def check_layout(g, o):
     assert sum(st["count"]) == st["m"] == kv.size, "I4: device counts != m"
 
 
-def run_parity(oracle_mod, wl, B=4, max_hops=64, layout_every=True, compare_sizes=True, binning=None):
-    g, o = make_pair(oracle_mod, wl, B=B, max_hops=max_hops, binning=binning)
+def run_parity(oracle_mod, wl, B=4, max_hops=64, layout_every=True, compare_sizes=True):
+    g, o = make_pair(oracle_mod, wl, B=B, max_hops=max_hops)
     for i, b in enumerate(wl.batches):
         kd = dev(b.keys)
         if b.op == "insert":
@@ -295,8 +295,7 @@ def test_host_entry_points_chunked(oracle_mod):
 
 # ------------------------------------------------------------------ full size (C2)
 @pytest.mark.slow
-@pytest.mark.parametrize("mode", [0, 1])
-def test_c2_full_size_sampled(mode):
+def test_c2_full_size_sampled():
     """BASELINE.json configs[1] at full size (2^27 keys, fill 0.85), in the
     launch configuration bench.py times.  Expected results follow from the
     generator: hits return val(k,0), misses NOT_FOUND; every delete hits; the
@@ -304,8 +303,7 @@ def test_c2_full_size_sampled(mode):
     (checked on a sample of 2^20 keys one by one)."""
     wl = W.c2_rand_static(log2_n=27)
     ins, fnd, dele = wl.batches
-    g = Table(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=8,
-              binning=(mode, 0, 0))    # 0: direct kernels (bench.py's configuration), 1: region-binned
+    g = Table(d=4, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=8)
     st = g.insert(dev(ins.keys), dev(ins.values))
     assert int((st == 1).sum()) == ins.keys.size
     s = g.stats()
@@ -323,7 +321,6 @@ def test_c2_full_size_sampled(mode):
     np.testing.assert_array_equal(host_u32(vd), W.val_of(dele.keys, 0))
     s = g.stats()
     assert s["m"] == ins.keys.size - dele.keys.size and s["n_downsize"] == 0
-    assert g.binning_info()[0] == (3 if mode == 1 else 0)
     rng = np.random.Generator(np.random.PCG64(5))
     sample = ins.keys[rng.choice(ins.keys.size, size=1 << 20, replace=False)]
     v, f = g.find(dev(sample))
