@@ -135,6 +135,7 @@ typedef struct {
     double   alloc_ms;                /* host milliseconds spent inside those cudaMalloc calls */
     uint64_t n_sync;                  /* counter read-backs: the host waited on the stream (S6) */
     double   sync_ms;                 /* host milliseconds spent in those waits                */
+    uint64_t n_pending;               /* new keys handed to the eviction kernel by all insert batches */
 } dyc_stats_t;
 
 /* Fills *cfg with the defaults: d=4, B=8, alpha=0.3, beta=0.85 (Table

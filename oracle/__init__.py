@@ -8,3 +8,4 @@ outputs are pinned ("parity unpinned": placement positions, φ, eviction counts)
 """
 from .oracle import OracleTable, build_oracle, oracle_lib  # noqa: F401
 from .oracle_wide import OracleWideTable, build_oracle_wide, oracle_wide_lib  # noqa: F401,E402
+from .brute import BruteMapCpp, build_brute  # noqa: F401,E402

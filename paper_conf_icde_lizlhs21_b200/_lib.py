@@ -43,7 +43,7 @@ class dyc_stats_t(C.Structure):
                 ("last_insert_pending", C.c_uint64), ("last_insert_evictions", C.c_uint64),
                 ("bytes_cached", C.c_uint64), ("n_live_resize", C.c_uint64), ("n_deferred", C.c_uint64),
                 ("n_device_alloc", C.c_uint64), ("alloc_ms", C.c_double),
-                ("n_sync", C.c_uint64), ("sync_ms", C.c_double)]
+                ("n_sync", C.c_uint64), ("sync_ms", C.c_double), ("n_pending", C.c_uint64)]
 
 
 class dyw_config(C.Structure):

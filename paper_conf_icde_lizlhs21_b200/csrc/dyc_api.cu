@@ -121,6 +121,7 @@ struct dyc_table {
     void* mix = nullptr;                   // scratch of dyc_mixed_batch
     uint64_t mix_cap = 0;
     uint64_t n_upsize = 0, n_downsize = 0, n_fail_upsize = 0, n_residual = 0, n_evict = 0, n_place_retry = 0;
+    uint64_t n_pending_total = 0;          // new keys handed to k_place by all insert batches
     uint64_t launches = 0;
     uint64_t last_new = 0, last_pending = 0, last_evict = 0;
     cudaStream_t last = nullptr;
@@ -726,6 +727,7 @@ dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
         t->m += ins;
         t->last_new = ins;
         t->last_pending = pend;
+        t->n_pending_total += pend;
         t->last_evict = t->n_evict - ev0;
         return policy_lower<B>(t, st);
     }
@@ -744,6 +746,7 @@ dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
     t->m += t->h_ctr[C_INSERTED];   // counters were read by place_and_settle
     t->last_new = t->h_ctr[C_INSERTED];
     t->last_pending = t->h_ctr[C_PENDING];
+    t->n_pending_total += t->h_ctr[C_PENDING];
     t->last_evict = t->n_evict - ev0;
     if (s != DYC_OK) return s;
     return enforce_lower<B>(t, st);
@@ -1075,6 +1078,7 @@ dyc_status stats_impl(dyc_table* t, dyc_stats_t* out, cudaStream_t st) {
     out->alloc_ms = t->alloc_ms;
     out->n_sync = t->n_sync;
     out->sync_ms = t->sync_ms;
+    out->n_pending = t->n_pending_total;
     return DYC_OK;
 }
 

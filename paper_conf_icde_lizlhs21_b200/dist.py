@@ -1,20 +1,27 @@
 """Hash-partitioned DyCuckoo across the ranks of a torch.distributed group
-(DESIGN.md §7).
+(DESIGN.md §7): the Python-orchestrated routers and the
+multi-GPU bench drivers.
+
+The product path for sharding is the C ABI (dyc_dist_*, sharded.py), where
+the routing and the NCCL exchange run inside libdyc.so.  This module keeps:
+
+- DistTable: the same routing orchestrated from Python over
+  torch.distributed all-to-all (the round-1 path, the baseline the C ABI
+  replaced; its CPU orchestration tests run over gloo), and
+- PeerRouter (DistTable(p2p=True)): fused dispatch/combine kernels that store
+  straight into peer memory (CUDA IPC), with host barriers between phases,
+- bench_multi_gpu / bench_c5: the bench's N > 1 and C5 drivers (C ABI by
+  default, the fused peer path with --p2p).
 
 Keys are owned by shard(k) = x_{d+1}(k) mod G (the (d+1)-th universal hash of
 P:L271, independent of the pair and bucket hashes).  Every rank holds one full
 DyCuckoo table (its own d subtables and [alpha, beta] resizing); since ops on
 different keys never interact, the union of the shards has exactly the
-single-table semantics.  A batch issued on any rank is routed:
+single-table semantics.  DistTable routes a batch as
 
     route_count (kernel)  ->  all_to_all(counts)  ->  route_scatter (kernel)
     ->  all_to_all(keys[, values])  ->  local batch on the owner (kernels)
     ->  all_to_all(replies)  ->  route_unpermute (kernel)
-
-torch.distributed (NCCL over NVLink on GPUs, gloo in the CPU tests) is the
-plumbing for the exchanges; every data-parallel step runs in libdyc.so.  The
-per-rank table is any object with the Table interface (insert/find/delete/
-route_*); the CPU tests inject a plain one to exercise this orchestration.
 """
 from __future__ import annotations
 
@@ -264,12 +271,21 @@ def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_pea
     from . import workload as W
     from .table import Table
 
+    from .sharded import ShardedTable, new_unique_id
     n = 1 << args.log2n
     cap, k_ins, v_ins, k_find, k_del = W.c2_rand_static_torch(args.log2n, device="cuda", key_base=rank * n,
                                                               miss_base=rank * n)
-    shard = Table(d=4, init_capacity=cap, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
     p2p = getattr(args, "p2p", False)
-    dt = DistTable(shard, force_route=True, p2p=p2p, max_ops=n if p2p else None)  # router even at N=1
+    if p2p:
+        # fused dispatch/combine over peer memory, orchestrated here
+        shard = Table(d=4, init_capacity=cap, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
+        dt = DistTable(shard, force_route=True, p2p=True, max_ops=n)
+    else:
+        # the sharded C ABI (dyc_dist_*): routing and NCCL exchange inside libdyc.so;
+        # at N = 1 a one-rank communicator keeps the NCCL exchange on the path
+        dt = ShardedTable(d=4, init_capacity=cap, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots,
+                          unique_id=new_unique_id() if world == 1 else None)
+        shard = dt
     stream = torch.cuda.current_stream()
 
     def step(evs=None):
@@ -295,6 +311,7 @@ def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_pea
     shard.clear()
     dt.insert(k_ins, v_ins)
     s_ins = shard.stats()
+    s_ins = s_ins[0] if isinstance(s_ins, list) else s_ins
     phi = s_ins["n_second_table"] / max(1, s_ins["m"])
     for _ in range(args.warmup):
         step()
@@ -360,7 +377,7 @@ def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_pea
         e2e = {"value": n_ops / float(t.item()) / 1e6, "unit": "Mops/s",
                "h2d_bytes_per_step": 4 * n + 4 * n + 4 * n + 4 * (n // 2),
                "d2h_bytes_per_step": n + 5 * n + 5 * (n // 2), "ms_per_step": 1e3 * float(t.item()),
-               "path": "pinned host batch -> DistTable (route, NCCL all-to-all, local kernels) -> host"}
+               "path": "pinned host batch -> sharded table (route, NCCL exchange, local kernels) -> host"}
     if rank != 0:
         return None
     return {
@@ -369,9 +386,10 @@ def bench_multi_gpu(args, rank, world, local, metric, ClockSampler, measured_pea
         "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
         "config": {"workload": f"C2-shaped batch per rank (2^{args.log2n} inserts, 2^{args.log2n} finds 50% hit, "
                                f"2^{args.log2n - 1} deletes), hash-partitioned over {world} shards, "
-                               "NCCL all-to-all routing", "d": 4, "alpha": 0.3, "beta": 0.85,
+                               "routed to the owning shards", "d": 4, "alpha": 0.3, "beta": 0.85,
                    "bucket_slots": args.bucket_slots, "parallelism": f"shard{world}",
-                   "routing": "p2p (fused push/reply over peer memory)" if p2p else "nccl all-to-all",
+                   "routing": "p2p (fused push/reply over peer memory)" if p2p else
+                   "dyc_dist_* C ABI: grouped ncclSend/ncclRecv inside libdyc.so",
                    "l2": "inputs and tables larger than L2; no flush needed"},
         "phase_ms_rank0": phases,
         "check": {"all_inserted_ranks": int(ok[0].item()), "found_total": int(ok[1].item()),
@@ -398,11 +416,17 @@ def bench_c5(args, rank, world, local, metric, ClockSampler):
     log2k = getattr(args, "c5_log2keys", 31)
     # 128 fill batches at every scale (2^31 keys: 16M per batch, the config);
     # keeps the 32 mixed batches' deletes below the live-find range at any scale
+    from .sharded import ShardedTable, new_unique_id
     batch = 1 << min(24, log2k - 7)
-    shard = Table(d=4, init_capacity=1 << 20, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
     p2p = getattr(args, "p2p", False)
-    dt = DistTable(shard, force_route=getattr(args, "routed", False) or p2p, p2p=p2p,
-                   max_ops=(batch + world - 1) // world if p2p else None)
+    if p2p:
+        shard = Table(d=4, init_capacity=1 << 20, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots)
+        dt = DistTable(shard, force_route=True, p2p=True, max_ops=(batch + world - 1) // world)
+    else:
+        routed = getattr(args, "routed", False)
+        dt = ShardedTable(d=4, init_capacity=1 << 20, alpha=0.3, beta=0.85, bucket_slots=args.bucket_slots,
+                          unique_id=new_unique_id() if (world == 1 and routed) else None)
+        shard = dt
     stream = torch.cuda.current_stream()
     gen = W.c5_batches_torch(rank, world, device="cuda", log2_keys=log2k, batch=batch, mixed_batches=32)
     fill, mixed = [], []
@@ -441,6 +465,7 @@ def bench_c5(args, rank, world, local, metric, ClockSampler):
     prof = shard.profile_read()
     shard.profile(False)
     st = shard.stats()
+    st = st[0] if isinstance(st, list) else st
     fill_ms, mixed_ms = float(t[0]), float(t[1])
     r_t = torch.tensor([reserved], dtype=torch.int64, device="cuda")
     if world > 1:
@@ -459,7 +484,8 @@ def bench_c5(args, rank, world, local, metric, ClockSampler):
                    "d": 4, "alpha": 0.3, "beta": 0.85, "bucket_slots": args.bucket_slots,
                    "parallelism": f"shard{world}", "init_capacity_per_shard": 1 << 20,
                    "routing": "p2p (fused push/reply over peer memory)" if p2p else
-                   ("nccl all-to-all" if (world > 1 or getattr(args, "routed", False)) else "local")},
+                   ("dyc_dist_* C ABI: grouped ncclSend/ncclRecv inside libdyc.so"
+                    if (world > 1 or getattr(args, "routed", False)) else "dyc_dist_* C ABI, one shard (no exchange)")},
         "phases": {"fill_ms": fill_ms, "fill_mops": n_fill / fill_ms / 1e3,
                    "mixed_ms": mixed_ms, "mixed_mops": n_mixed / mixed_ms / 1e3},
         "check": {"inserted_fill": int(checks[0]), "expected_fill": n_fill - reserved_all,

@@ -150,6 +150,27 @@ class ShardedTable:
         L.check(self._lib.dyc_dist_shard(self._h, local_index, C.byref(h)), "dyc_dist_shard")
         return Table.borrow(h.value, self.d, self.B)
 
+    def clear(self, stream=None) -> None:
+        for i in range(self.local_shards):
+            self.shard(i).clear(stream)
+
+    def profile(self, enable: bool = True) -> None:
+        for i in range(self.local_shards):
+            self.shard(i).profile(enable)
+
+    def profile_read(self) -> Dict[str, tuple]:
+        """Per-kernel (ms, launches) summed over the local shards."""
+        tot: Dict[str, list] = {}
+        for i in range(self.local_shards):
+            for k, (ms, calls) in self.shard(i).profile_read().items():
+                t = tot.setdefault(k, [0.0, 0])
+                t[0] += ms
+                t[1] += calls
+        return {k: (v[0], v[1]) for k, v in tot.items()}
+
+    def launch_count(self, reset: bool = False) -> int:
+        return sum(self.shard(i).launch_count(reset=reset) for i in range(self.local_shards))
+
     def stats(self) -> List[Dict]:
         return [self.shard(i).stats() for i in range(self.local_shards)]
 

@@ -331,7 +331,8 @@ class Table:
                     last_insert_pending=s.last_insert_pending,
                     last_insert_evictions=s.last_insert_evictions, bytes_cached=s.bytes_cached,
                     n_live_resize=s.n_live_resize, n_deferred=s.n_deferred,
-                    n_device_alloc=s.n_device_alloc, alloc_ms=s.alloc_ms, n_sync=s.n_sync, sync_ms=s.sync_ms)
+                    n_device_alloc=s.n_device_alloc, alloc_ms=s.alloc_ms, n_sync=s.n_sync, sync_ms=s.sync_ms,
+                    n_pending=s.n_pending)
 
     def dump(self, stream=None):
         """(kv uint64, table uint32, bucket uint64) host arrays, unspecified order."""

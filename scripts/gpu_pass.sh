@@ -18,7 +18,7 @@ for step in "$@"; do
     launches) timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_$R.csv python bench.py --steps 2 --warmup 1 --profile-only > /dev/null 2>&1; echo "launches rc=$?" ;;
     ncu) timeout 1500 ncu --set full --clock-control none --import-source on -k regex:"k_upsert|k_find|k_delete|k_place" -c 4 -o gpurun_out/prof_$R python bench.py --steps 1 --warmup 0 --profile-only > gpurun_out/ncu_full_$R.log 2>&1; tail -2 gpurun_out/ncu_full_$R.log ;;
     gather) timeout 600 python scripts/gather_wall.py > gpurun_out/gather_$R.log 2>&1; tail -3 gpurun_out/gather_$R.log
-            GATHER_REPS=1 timeout 1500 ncu --set full --clock-control none -k regex:k_gather -o gpurun_out/gather_ncu_$R python scripts/gather_wall.py > gpurun_out/gather_ncu_$R.log 2>&1; tail -2 gpurun_out/gather_ncu_$R.log ;;
+            ;;
     sanitize)
       for tool in memcheck racecheck synccheck; do
         timeout 1500 compute-sanitizer --tool $tool --error-exitcode 9 python scripts/sanitize_streams.py > gpurun_out/${tool}_$R.txt 2>&1; echo "$tool rc=$?"; tail -2 gpurun_out/${tool}_$R.txt

@@ -118,3 +118,28 @@ def test_create_rejects_infeasible_bounds(oracle_mod):
         oracle_mod.OracleTable(d=2, alpha=0.6, beta=0.85)    # 0.567
     with pytest.raises(ValueError):
         oracle_mod.OracleTable(d=1)
+
+
+def test_cpp_brute_map_equals_python_dict():
+    """The std::unordered_map baseline (oracle/brute_map.cpp, BASELINE.md §3 (ii))
+    gives the dict model's results on a random stream with mixed batches."""
+    import numpy as np
+    from oracle import BruteMapCpp
+    from paper_conf_icde_lizlhs21_b200 import workload as W
+    from tests.bruteforce import BruteMap
+    a, b = BruteMapCpp(), BruteMap()
+    wl = W.random_op_stream(99, n_batches=30, batch=2000, universe=3000)
+    for bt in wl.batches:
+        if bt.op == "insert":
+            np.testing.assert_array_equal(a.insert(bt.keys, bt.values), b.insert(bt.keys, bt.values))
+        elif bt.op == "find":
+            for x, y in zip(a.find(bt.keys), b.find(bt.keys)):
+                np.testing.assert_array_equal(x, y)
+        else:
+            for x, y in zip(a.delete(bt.keys), b.delete(bt.keys)):
+                np.testing.assert_array_equal(x, y)
+    _, mixed = W.c4_zipf_mixed(U=20000, distinct=2000, grow_batches=3, cycles=1)
+    for mb in mixed:
+        for x, y in zip(a.mixed(mb.ops, mb.keys, mb.values), b.mixed(mb.ops, mb.keys, mb.values)):
+            np.testing.assert_array_equal(x, y)
+    assert len(a) == len(b.m)
