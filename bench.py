@@ -68,6 +68,9 @@ def parse():
     ap.add_argument("--scale", type=float, default=1.0, help="c3: stream scale; c4: universe scale")
     ap.add_argument("--c5-log2keys", type=int, default=31, help="c5: log2 of the total key count")
     ap.add_argument("--d", type=int, default=4, help="number of subtables (paper default 4, P:L804)")
+    ap.add_argument("--placement", default="first_fit", choices=["first_fit", "paper_weighted"],
+                    help="initial table choice: two-choice first-fit (reading Q3) or the paper's n_i/C(m_i,2) "
+                         "rule (P:L361; NEXT-4 ablation)")
     ap.add_argument("--alpha", type=float, default=None, help="lower fill bound (c3/c4 sweeps, Table tbl:parameters)")
     ap.add_argument("--beta", type=float, default=None, help="upper fill bound (sweeps; c2 fill target)")
     ap.add_argument("--r", type=float, default=0.2, help="c3: deletes per insert (P:L732-733)")
@@ -473,7 +476,7 @@ def main():
     cap, k_ins, v_ins, k_find, k_del = W.c2_rand_static_torch(args.log2n, device="cuda", beta=beta)
 
     stream = torch.cuda.current_stream()
-    g = Table(d=args.d, init_capacity=cap, alpha=0.3 if args.alpha is None else args.alpha,
+    g = Table(d=args.d, init_capacity=cap, placement=args.placement, alpha=0.3 if args.alpha is None else args.alpha,
               beta=min(0.99, beta + 1e-6) if beta > 0.85 else 0.85, bucket_slots=args.bucket_slots)
     st_ins = torch.empty(n, dtype=torch.uint8, device="cuda")
     v_out = torch.empty(n, dtype=torch.int32, device="cuda")
@@ -750,6 +753,7 @@ def main():
                                f"2^{args.log2n} finds (50% hit), one subtable upsize, 2^{args.log2n - 1} deletes, "
                                "one subtable downsize",
                    "d": args.d, "alpha": 0.3, "beta": beta, "bucket_slots": args.bucket_slots,
+                   "placement": args.placement,
                    "table_bytes": int(s_ins["N"] * 8),
                    "l2": "inputs and table larger than L2 (126 MB); no flush needed"},
         "phase_ms": phase_ms,
@@ -762,6 +766,8 @@ def main():
         "gpu_launches": launches,
         "clocks": clk.summary(),
         "table": {"fill_after_insert": s_ins["fill"], "phi": phi,
+                  "per_table_fill": [round(c / (nb * args.bucket_slots), 4) for c, nb in zip(s_ins["count"], s_ins["buckets"])],
+                  "evictions_per_insert": s_ins["last_insert_evictions"] / max(1, s_ins["last_insert_new"]),
                   "pending_after_upsert": pend, "evictions": s_ins["last_insert_evictions"]},
     }
     emit(line)
@@ -882,7 +888,8 @@ def bench_stream(args, local):
         name = (f"C4 {shape}-shaped Zipf(0.99) mixed 50/30/20 batches of {D} distinct keys over U={U}, "
                 "grow 16 batches then drain, 2 cycles")
     gen_s = time.time() - t0
-    g = Table(d=args.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=args.bucket_slots)
+    g = Table(d=args.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=args.bucket_slots,
+              placement=args.placement)
     dev = lambda a: torch.from_numpy(np.ascontiguousarray(a, dtype=np.uint32).view(np.int32)).cuda()  # noqa: E731
     staged = []
     for b in batches:
@@ -978,6 +985,7 @@ def bench_stream(args, local):
     # fill-factor track: replay untimed with a stats call after every batch
     g.clear()
     track, mem = [], []
+    peak_st = None
     for op, ops, k, v in staged:
         if op == "insert":
             g.insert(k, v)
@@ -990,6 +998,8 @@ def bench_stream(args, local):
         st = g.stats()
         track.append(round(st["fill"], 4))
         mem.append(st["N"] * 8)
+        if peak_st is None or st["m"] > peak_st["m"]:
+            peak_st = st
     st = g.stats()
     n_ops = sum(c for _, c, _, _, _ in rec)
     ops_line = {f"{k}_mops": (v[0] / v[1] / 1e3 if v[1] else None) for k, v in per.items() if v[0]}
@@ -1009,12 +1019,18 @@ def bench_stream(args, local):
         "metric": METRIC, "value": n_ops / total_ms / 1e3, "unit": "Mops/s", "n_gpus": 1, "steps": 1,
         "warmup": args.warmup, "ms_per_step": total_ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": name, "d": args.d, "alpha": wl.alpha, "beta": wl.beta,
+        "config": {"workload": name, "d": args.d, "alpha": wl.alpha, "beta": wl.beta, "placement": args.placement,
                    "bucket_slots": args.bucket_slots, "batches": len(staged), "ops": n_ops},
         "ops": ops_line,
         "fill_track": {"min_after_mutation": min(x for x, (op, *_r) in zip(track, staged) if op != "find"),
                        "max": max(track), "final": track[-1], "every_batch": track if len(track) <= 400 else None},
         "table_bytes": {"max": max(mem), "final": mem[-1]},
+        "at_peak_live": {"m": peak_st["m"], "fill": round(peak_st["fill"], 4),
+                         "phi": round(peak_st["n_second_table"] / max(1, peak_st["m"]), 4),
+                         "per_table_fill": [round(c / (nb * args.bucket_slots), 4)
+                                            for c, nb in zip(peak_st["count"], peak_st["buckets"])],
+                         "evictions_per_new_key_whole_stream": round(st["n_evict"] / max(1, sum(
+                             c for op, c, *_ in rec if op == "insert")), 4)},
         "resizes": resizes,
         "host_waits_timed_pass": host_waits,
         "kernel_ms": {k: round(v[0], 3) for k, v in prof.items() if v[1]},

@@ -27,17 +27,20 @@
  * - Arrays are dense, element i belongs to op i.  No alignment beyond the
  *   element type is required.
  * - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
- *   Work is stream-ordered.  find never blocks the host.  insert synchronizes
- *   `stream` once (twice when a resize decision needs the number of new keys)
- *   to read the batch counters that drive the resize policy (S6).  A delete
- *   synchronizes only when the alpha loop might fire: when a lower bound of m
- *   after it (m minus every removal still pending, its own n included) is
- *   >= alpha*N it returns without waiting, leaves its removal count on the
- *   device and records an event on `stream`; the next call that needs the exact
- *   m (on any stream) waits for that event before reading the count.  So the
- *   lower fill bound still holds after every batch.  Batches
- *   on one table must not overlap in time: issue them on one stream, or order
- *   them across streams with events.
+ *   Work is stream-ordered.  find never blocks the host.  A mutating batch
+ *   waits for `stream` only when a resize decision needs the exact live count
+ *   (S6): an insert whose upper bound m + n may exceed beta*N reads the number
+ *   of new keys back once before placing them (Q11); a delete, or an
+ *   insert, after which a lower bound of m may fall below alpha*N reads the
+ *   counts back for the alpha loop.  Otherwise the batch returns without
+ *   waiting: its counts stay in accumulating device counters and are applied
+ *   at the next read-back (which first waits for an event recorded on the lazy
+ *   batch's stream, so another stream may issue it).  Pairs that an insert
+ *   could not place within max_hops hops wait in a device stash that find,
+ *   insert and delete consult until the next read-back places them, upsizing
+ *   on failure (Q17); results are never affected.  Batches on one
+ *   table must not overlap in time: issue them on one stream, or order them
+ *   across streams with events.
  * - Batches are single-type.  Keys must be distinct within a batch
  *   (precondition, reading Q9); violating it never corrupts the table but the
  *   final value of a duplicated key is unspecified.
@@ -262,11 +265,12 @@ dyc_status dyc_stats(dyc_table* t, dyc_stats_t* out, dyc_stream_t stream);
 
 /* Host view of the table's shape, without touching the device (never
  * synchronizes): buckets[d] (nullable) = |h^t| per subtable as the resize
- * policy has left it, *m (nullable) = the live count the host holds, and
- * *m_pending (nullable) = an upper bound of removals counted on the device but
- * not yet applied (lazy delete read-back): the exact count lies in
- * [m - m_pending, m].  A resize in flight (dyc_resize_begin) is not included. */
-dyc_status dyc_shape(const dyc_table* t, uint64_t* buckets, uint64_t* m, uint64_t* m_pending);
+ * policy has left it; batches that skipped their counter read-back (see the
+ * stream semantics above) leave the live count known only within
+ * [*m_lo, *m_hi] (equal when nothing is pending); *n_fail_upsize = upsizes so
+ * far that placement failures triggered.  Any pointer may be NULL.
+ * A resize in flight (dyc_resize_begin) is not included. */
+dyc_status dyc_shape(const dyc_table* t, uint64_t* buckets, uint64_t* m_lo, uint64_t* m_hi, uint64_t* n_fail_upsize);
 
 /* Copies the live contents to host arrays (tests/diagnostics, not timed).
  * h_kv[i] = key | (uint64)value << 32; h_table[i] / h_bucket[i] (nullable) give

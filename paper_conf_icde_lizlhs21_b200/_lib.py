@@ -112,7 +112,7 @@ SIGNATURES = {
     "dyc_trim": (_I, [_TP]),
     "dyc_stats": (_I, [_TP, C.POINTER(dyc_stats_t), _P]),
     "dyc_dump": (_I, [_TP, _P, _P, _P, _U64, C.POINTER(_U64), _P]),
-    "dyc_shape": (_I, [_TP, _P, C.POINTER(_U64), C.POINTER(_U64)]),
+    "dyc_shape": (_I, [_TP, _P, C.POINTER(_U64), C.POINTER(_U64), C.POINTER(_U64)]),
     "dyc_hash_params": (_I, [_TP, _P, _P]),
     "dyc_hash_probe": (_I, [_TP, _P, _U64, _P, _P, _P]),
     "dyc_insert_batch_host": (_I, [_TP, _P, _P, _P, _U64, _P]),

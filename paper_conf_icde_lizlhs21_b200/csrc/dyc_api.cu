@@ -91,15 +91,23 @@ struct dyc_table {
     // baseline clears all.  Downsizes and placements (first-fit, evictions)
     // preserve it.
     uint32_t clean = 0;
-    // m is exact unless a delete batch skipped its counter read-back (m_lazy):
-    // then the removals wait in d_ctr[C_REMOVED] and m is an upper bound until
-    // the next read_ctr applies them (flush_m before any decision that needs m).
-    // lazy_n bounds the removals still pending (the summed sizes of the delete
-    // batches that skipped their read-back), so m - lazy_n is a lower bound of
-    // the live count; lazy_ev marks the last such batch on its stream.
+    // m is the live count as of the last counter read-back.  A batch that cannot
+    // trigger a resize decision skips its read-back (lazy): its counts wait in
+    // the accumulating device counters (C_ADDED, C_REMOVED, ...) until the next
+    // read_ctr applies them, and the exact count lies in
+    // [m - lazy_del, m + lazy_add] (flush_m before any decision that needs it).
+    // lazy_ev marks the last lazy batch on its stream (ev_pending until read).
     bool m_lazy = false;
-    uint64_t lazy_n = 0;
+    uint64_t lazy_del = 0, lazy_add = 0;
     cudaEvent_t lazy_ev = nullptr;
+    bool ev_pending = false;
+    bool ins_lazy = false;                 // the last insert's per-batch stats are still on the device
+    uint64_t ins_n = 0;                    // ops of the insert batch in flight
+    // stash (dyc_kernels.cuh stash_find): pairs a lazily settled insert could
+    // not place; the next sync_state settles them (retry, failure upsizes)
+    unsigned long long* stash = nullptr;
+    uint64_t stash_cap = 0;
+    uint64_t stash_bound = 0;              // upper bound of its entries since the last settle
     uint64_t del_n = 0;                    // ops of the delete batch in flight
     // placement policy (dyc_config.flags): first-fit (reading Q3) or the
     // paper's weighted rule; the latter keeps d_w, a per-batch
@@ -199,6 +207,8 @@ struct dyc_table {
         v.clean = weighted ? 0u : (rz.active ? (clean & ~(1u << rz.ti)) : clean);
         v.probe = count_probes ? d_probe : nullptr;
         v.wsel = weighted ? d_w : nullptr;
+        v.stash = stash;
+        v.stash_n = d_ctr ? d_ctr + C_STASH : nullptr;
         return v;
     }
 };
@@ -307,36 +317,49 @@ void dev_free(dyc_table* t, void* p, cudaStream_t st) {
 }
 
 dyc_status read_ctr(dyc_table* t, cudaStream_t st) {
-    // a lazy delete may have run on another stream: its removals must have
-    // landed in C_REMOVED before the copy and the reset below
-    if (t->m_lazy && t->lazy_ev) CU(cudaStreamWaitEvent(st, t->lazy_ev, 0));
+    // a lazy batch may have run on another stream: its counts must have landed
+    // in the accumulators before the copy and the reset below
+    if (t->ev_pending && t->lazy_ev) CU(cudaStreamWaitEvent(st, t->lazy_ev, 0));
     CU(cudaMemcpyAsync(t->h_ctr, t->d_ctr, C_N * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
     const auto t0 = std::chrono::steady_clock::now();
     CU(cudaStreamSynchronize(st));
     t->sync_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     t->n_sync++;
-    // every read-back applies the removals counted since the last one (the
-    // delete batches whose own read-back was skipped included)
-    const unsigned long long removed = t->h_ctr[C_REMOVED];
-    if (removed) {
-        t->m -= removed;
-        t->clean = 0;   // emptied slots break the first-choice-full invariant
-        CU(cudaMemsetAsync(t->d_ctr + C_REMOVED, 0, sizeof(unsigned long long), st));
+    // every read-back applies what the batches counted since the last one (the
+    // lazy ones included): live-count changes, evictions, pending keys
+    const unsigned long long* h = t->h_ctr;
+    const unsigned long long added = h[C_ADDED], removed = h[C_REMOVED];
+    t->m = t->m + added - removed;
+    if (removed) t->clean = 0;   // emptied slots break the first-choice-full invariant
+    t->n_evict += h[C_EVICT];
+    t->n_pending_total += h[C_PEND_ACC];
+    if (t->ins_lazy) {
+        t->last_new = h[C_INSERTED];
+        t->last_pending = h[C_PENDING];
+        t->last_evict = h[C_EVICT];
+        t->ins_lazy = false;
     }
+    if (added | removed | h[C_EVICT] | h[C_PEND_ACC])
+        CU(cudaMemsetAsync(t->d_ctr + C_REMOVED, 0, (C_COUNT0 - C_REMOVED) * sizeof(unsigned long long), st));
     t->m_lazy = false;
-    t->lazy_n = 0;
+    t->ev_pending = false;
+    t->lazy_del = t->lazy_add = 0;
     return DYC_OK;
 }
 
-dyc_status flush_m(dyc_table* t, cudaStream_t st) {
-    return t->m_lazy ? read_ctr(t, st) : DYC_OK;
+// zeroes the per-batch counters ([0, C_ACC0) and the per-subtable counts); the
+// accumulators and the stash count belong to read_ctr / the stash settling
+dyc_status zero_ctr(dyc_table* t, cudaStream_t st) {
+    CU(cudaMemsetAsync(t->d_ctr, 0, C_ACC0 * sizeof(unsigned long long), st));
+    CU(cudaMemsetAsync(t->d_ctr + C_COUNT0, 0, (C_N - C_COUNT0) * sizeof(unsigned long long), st));
+    return DYC_OK;
 }
 
-// zeroes every counter but C_REMOVED (owned by read_ctr: removals not yet
-// applied to m)
-dyc_status zero_ctr(dyc_table* t, cudaStream_t st) {
-    CU(cudaMemsetAsync(t->d_ctr, 0, C_REMOVED * sizeof(unsigned long long), st));
-    CU(cudaMemsetAsync(t->d_ctr + C_REMOVED + 1, 0, (C_N - C_REMOVED - 1) * sizeof(unsigned long long), st));
+// A lazy batch returns without a host wait: remember its stream position.
+dyc_status mark_lazy(dyc_table* t, cudaStream_t st) {
+    if (!t->lazy_ev) CU(cudaEventCreateWithFlags(&t->lazy_ev, cudaEventDisableTiming));
+    CU(cudaEventRecord(t->lazy_ev, st));
+    t->ev_pending = true;
     return DYC_OK;
 }
 
@@ -367,6 +390,20 @@ dyc_status ensure_lists(dyc_table* t, uint64_t n, cudaStream_t st) {
 // Paper-weighted mode: snapshot w[t] = n_t / C(m_t, 2) from a count
 // of every subtable (one streaming pass over the table, in stream order, so it
 // sees the state the next placement kernel starts from).
+// Stash capacity for `need` entries; live entries are carried over (in stream order).
+dyc_status ensure_stash(dyc_table* t, uint64_t need, cudaStream_t st) {
+    if (need <= t->stash_cap) return DYC_OK;
+    const uint64_t cap = std::max<uint64_t>(need, 2 * t->stash_cap);
+    void* p = nullptr;
+    TRY(dev_alloc(t, &p, cap * 8, st));
+    if (t->stash && t->stash_bound)
+        CU(cudaMemcpyAsync(p, t->stash, t->stash_cap * 8, cudaMemcpyDeviceToDevice, st));
+    dev_free(t, t->stash, st);
+    t->stash = (unsigned long long*)p;
+    t->stash_cap = cap;
+    return DYC_OK;
+}
+
 template <int B>
 dyc_status refresh_weights(dyc_table* t, cudaStream_t st) {
     if (!t->weighted) return DYC_OK;
@@ -419,7 +456,6 @@ dyc_status settle(dyc_table* t, int cur, uint64_t nfail, cudaStream_t st, unsign
         round++;
         t->n_place_retry++;
         TRY(zero_one(t, C_FAIL, st));
-        TRY(zero_one(t, C_EVICT, st));
         {
             ProfScope ps(t, DYC_PROF_PLACE, st);
             k_place<B><<<grid_for(nfail, kThreads / (B / 4)), kThreads, 0, st>>>(t->view(), L[cur], nullptr, nfail,
@@ -427,7 +463,6 @@ dyc_status settle(dyc_table* t, int cur, uint64_t nfail, cudaStream_t st, unsign
         }
         CU(cudaGetLastError());
         TRY(read_ctr(t, st));
-        t->n_evict += t->h_ctr[C_EVICT];
         nfail = t->h_ctr[C_FAIL];
         cur = 1 - cur;
         if (round > 64) return set_err(DYC_ERR_INSERT_FAILED, "placement kept failing after 64 upsizes");
@@ -452,11 +487,41 @@ template <int B>
 dyc_status place_and_settle(dyc_table* t, int src, const unsigned long long* d_count, uint64_t h_count,
                             bool first_fit, cudaStream_t st) {
     TRY(zero_one(t, C_FAIL, st));
-    TRY(zero_one(t, C_EVICT, st));
     TRY(launch_place<B>(t, src, d_count, h_count, first_fit, st));
     TRY(read_ctr(t, st));
-    t->n_evict += t->h_ctr[C_EVICT];
     return settle<B>(t, 1 - src, t->h_ctr[C_FAIL], st);
+}
+
+// Settles the stash (pairs the lazily settled inserts could not place):
+// one placement pass over it, then the usual retry / failure-upsize loop (Q17).
+template <int B>
+dyc_status settle_stash(dyc_table* t, cudaStream_t st) {
+    const uint64_t S = t->h_ctr[C_STASH];
+    TRY(ensure_lists(t, S, st));
+    TRY(zero_one(t, C_FAIL, st));
+    {
+        ProfScope ps(t, DYC_PROF_PLACE, st);
+        k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->stash, nullptr, S, t->list[1], t->d_ctr, true);
+    }
+    CU(cudaGetLastError());
+    TRY(zero_one(t, C_STASH, st));
+    t->stash_bound = 0;
+    TRY(read_ctr(t, st));
+    return settle<B>(t, 1, t->h_ctr[C_FAIL], st);
+}
+
+// Exact state: apply every count still on the device and settle the stash.
+template <int B>
+dyc_status sync_state(dyc_table* t, cudaStream_t st) {
+    TRY(read_ctr(t, st));
+    if (t->h_ctr[C_STASH]) return settle_stash<B>(t, st);
+    t->stash_bound = 0;
+    return DYC_OK;
+}
+
+template <int B>
+dyc_status flush_m(dyc_table* t, cudaStream_t st) {
+    return (t->m_lazy || t->ev_pending || t->stash_bound) ? sync_state<B>(t, st) : DYC_OK;
 }
 
 // Halves subtable ti: merge kernel, then residual placement into
@@ -488,11 +553,9 @@ template <int B>
 dyc_status downsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
     TRY(ensure_lists(t, (t->nb[ti] / 2) * B, st));
     TRY(zero_one(t, C_FAIL, st));
-    TRY(zero_one(t, C_EVICT, st));
     TRY(zero_one(t, C_RES_TOTAL, st));
     TRY(downsize_launch<B>(t, ti, st));
     TRY(read_ctr(t, st));
-    t->n_evict += t->h_ctr[C_EVICT];
     t->n_residual += t->h_ctr[C_RES_TOTAL];
     return settle<B>(t, 1, t->h_ctr[C_FAIL], st);
 }
@@ -504,7 +567,7 @@ dyc_status downsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
 // settled once at the end (Q17: retry, then failure-triggered upsizes).
 template <int B>
 dyc_status enforce_lower(dyc_table* t, cudaStream_t st) {
-    TRY(flush_m(t, st));
+    TRY(flush_m<B>(t, st));
     uint64_t nb[DYC_MAX_D];
     for (uint32_t i = 0; i < t->cfg.d; i++) nb[i] = t->nb[i];
     std::vector<uint32_t> plan;
@@ -526,14 +589,12 @@ dyc_status enforce_lower(dyc_table* t, cudaStream_t st) {
     if (plan.empty()) return DYC_OK;
     TRY(ensure_lists(t, std::min<uint64_t>(res_bound, t->m + 1) + 1, st));
     TRY(zero_one(t, C_FAIL, st));
-    TRY(zero_one(t, C_EVICT, st));
     TRY(zero_one(t, C_RES_TOTAL, st));
     for (uint32_t ti : plan) {
         TRY(downsize_launch<B>(t, ti, st));
         t->n_downsize++;
     }
     TRY(read_ctr(t, st));
-    t->n_evict += t->h_ctr[C_EVICT];
     t->n_residual += t->h_ctr[C_RES_TOTAL];
     TRY(settle<B>(t, 1, t->h_ctr[C_FAIL], st));
     return DYC_OK;
@@ -562,7 +623,6 @@ dyc_status live_commit(dyc_table* t, cudaStream_t st) {
     }
     t->n_downsize++;
     TRY(zero_one(t, C_FAIL, st));
-    TRY(zero_one(t, C_EVICT, st));
     {
         ProfScope ps(t, DYC_PROF_PLACE, st);
         k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), r.res[0], r.ctr + C_RESIDUAL, 0, r.res[1],
@@ -571,7 +631,6 @@ dyc_status live_commit(dyc_table* t, cudaStream_t st) {
     CU(cudaGetLastError());
     CU(cudaMemcpyAsync(t->d_ctr + C_RES_TOTAL, r.ctr + C_RES_TOTAL, 8, cudaMemcpyDeviceToDevice, st));
     TRY(read_ctr(t, st));
-    t->n_evict += t->h_ctr[C_EVICT];
     t->n_residual += t->h_ctr[C_RES_TOTAL];
     TRY(settle<B>(t, 1, t->h_ctr[C_FAIL], st, r.res));
     dev_free(t, r.res[0], st);
@@ -605,7 +664,7 @@ dyc_status live_begin(dyc_table* t, int direction, int subtable, cudaStream_t st
     auto& r = t->rz;
     if (r.active) return set_err(DYC_ERR_INVALID_ARG, "a resize is already in flight (dyc_resize_commit first)");
     if (t->part_op) return set_err(DYC_ERR_INVALID_ARG, "a batch is open (dyc_*_end first)");
-    TRY(flush_m(t, st));
+    TRY(flush_m<B>(t, st));
     int ti = -1;
     TRY(pick_resize(t, direction, subtable, ti));
     if (!r.start) CU(cudaEventCreateWithFlags(&r.start, cudaEventDisableTiming));
@@ -655,7 +714,7 @@ dyc_status live_begin(dyc_table* t, int direction, int subtable, cudaStream_t st
 // it has to act.
 template <int B>
 dyc_status policy_lower(dyc_table* t, cudaStream_t st) {
-    TRY(flush_m(t, st));
+    TRY(flush_m<B>(t, st));
     if (t->rz.active) {
         if (!((double)t->m < t->cfg.alpha * (double)t->N_after())) return DYC_OK;
         TRY(live_commit<B>(t, st));
@@ -683,13 +742,18 @@ dyc_status launch_apply(dyc_table* t, const unsigned long long* list, bool del, 
 // need that subtable (deferred updates, keys with no free non-locked slot).
 template <int B>
 dyc_status insert_begin(dyc_table* t, uint64_t n, cudaStream_t st, bool& fuse) {
-    // m may be an upper bound (m_lazy): below beta with it, below beta for sure
-    if (t->m_lazy && (t->rz.active || (double)(t->m + n) > t->cfg.beta * (double)t->N())) TRY(flush_m(t, st));
+    // with lazy counts the live count is at most m + lazy_add: below beta with
+    // that bound, below beta for sure; otherwise the decision needs the exact m
+    const bool lazy = t->m_lazy || t->ev_pending || t->stash_bound;
+    if (lazy && (t->rz.active || (double)(t->m + t->lazy_add + n) > t->cfg.beta * (double)t->N()))
+        TRY(flush_m<B>(t, st));
     if (t->rz.active && (double)(t->m + n) > t->cfg.beta * (double)t->N_after()) TRY(live_commit<B>(t, st));
     TRY(ensure_lists(t, n, st));
+    TRY(ensure_stash(t, t->stash_bound + n, st));
     TRY(zero_ctr(t, st));
     TRY(refresh_weights<B>(t, st));
-    fuse = t->rz.active || (double)(t->m + n) <= t->cfg.beta * (double)t->N();
+    t->ins_n = n;
+    fuse = t->rz.active || (double)(t->m + t->lazy_add + n) <= t->cfg.beta * (double)t->N();
     return DYC_OK;
 }
 
@@ -724,7 +788,6 @@ dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
             if (dfr) TRY(launch_apply<B>(t, t->list[1], false, dfr, st));
             if (pend) TRY(place_and_settle<B>(t, 0, t->d_ctr + C_PENDING, 0, true, st));
         }
-        t->m += ins;
         t->last_new = ins;
         t->last_pending = pend;
         t->n_pending_total += pend;
@@ -732,23 +795,35 @@ dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
         return policy_lower<B>(t, st);
     }
     if (!fuse) {
-        // the resize decision needs n_new before any placement (Q11)
+        // the resize decision needs n_new before any placement (Q11):
+        // after the read-back m includes this batch's new keys
         TRY(read_ctr(t, st));
-        const uint64_t n_new = t->h_ctr[C_INSERTED];
-        while ((double)(t->m + n_new) > t->cfg.beta * (double)t->N()) {
+        while ((double)t->m > t->cfg.beta * (double)t->N()) {
             TRY(upsize_table<B>(t, (uint32_t)t->smallest(), st));
             t->n_upsize++;
         }
         TRY(refresh_weights<B>(t, st));   // after an upsize the bigger table draws more
     }
-    const uint64_t ev0 = t->n_evict;
-    dyc_status s = place_and_settle<B>(t, 0, t->d_ctr + C_PENDING, 0, !fuse, st);
-    t->m += t->h_ctr[C_INSERTED];   // counters were read by place_and_settle
-    t->last_new = t->h_ctr[C_INSERTED];
-    t->last_pending = t->h_ctr[C_PENDING];
-    t->n_pending_total += t->h_ctr[C_PENDING];
-    t->last_evict = t->n_evict - ev0;
-    if (s != DYC_OK) return s;
+    // placement of the keys whose candidate buckets were full; pairs still
+    // homeless after L_max hops go to the stash, which every later batch
+    // consults and the next exact read-back settles (Q17), so the
+    // batch ends without a host wait
+    {
+        ProfScope ps(t, DYC_PROF_PLACE, st);
+        k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->list[0], t->d_ctr + C_PENDING, 0, t->stash,
+                                                         t->d_ctr, !fuse, t->d_ctr + C_STASH,
+                                                         t->d_ctr + C_PEND_ACC);
+    }
+    CU(cudaGetLastError());
+    t->stash_bound += t->ins_n;
+    t->ins_lazy = true;
+    if (fuse) {
+        t->lazy_add += t->ins_n;
+        t->m_lazy = true;
+    }
+    TRY(mark_lazy(t, st));
+    // the alpha loop cannot fire while a lower bound of m is >= alpha*N
+    if (t->m >= t->lazy_del && (double)(t->m - t->lazy_del) >= t->cfg.alpha * (double)t->N()) return DYC_OK;
     return enforce_lower<B>(t, st);
 }
 
@@ -778,7 +853,7 @@ dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t
 // one k_delete per chunk + end (m, deferred removals, alpha loop).
 template <int B>
 dyc_status delete_prep(dyc_table* t, uint64_t n, cudaStream_t st) {
-    if (t->rz.active) TRY(flush_m(t, st));
+    if (t->rz.active) TRY(flush_m<B>(t, st));
     t->del_n = n;
     if (t->rz.active) {
         TRY(ensure_lists(t, n, st));
@@ -811,12 +886,11 @@ dyc_status delete_end(dyc_table* t, cudaStream_t st) {
     // >= alpha*N: the alpha loop cannot fire, so the removals stay on
     // the device until the next read-back (m_lazy).  m itself is then an upper
     // bound, which is what the beta test of the next insert needs.
-    const uint64_t pend = t->lazy_n + t->del_n;
+    const uint64_t pend = t->lazy_del + t->del_n;
     if (!t->rz.active && t->m >= pend && (double)(t->m - pend) >= t->cfg.alpha * (double)t->N()) {
         if (t->del_n) t->clean = 0;
-        if (!t->lazy_ev) CU(cudaEventCreateWithFlags(&t->lazy_ev, cudaEventDisableTiming));
-        CU(cudaEventRecord(t->lazy_ev, st));
-        t->lazy_n = pend;
+        TRY(mark_lazy(t, st));
+        t->lazy_del = pend;
         t->m_lazy = true;
         return DYC_OK;
     }
@@ -1001,7 +1075,6 @@ dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaSt
         CU(cudaGetLastError());
     }
     TRY(read_ctr(t, st));
-    t->n_evict += t->h_ctr[C_EVICT];
     const uint64_t nfail = t->h_ctr[C_FAIL];
     for (uint32_t i = 0; i < d; i++)
         if (touched[i]) dev_free(t, old[i], st);
@@ -1013,7 +1086,7 @@ dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaSt
 template <int B>
 dyc_status resize_impl(dyc_table* t, int direction, int subtable, int method, cudaStream_t st) {
     TRY(live_commit<B>(t, st));
-    TRY(flush_m(t, st));
+    TRY(flush_m<B>(t, st));
     if (direction == 0) {
         while ((double)t->m > t->cfg.beta * (double)t->N()) {
             TRY(upsize_table<B>(t, (uint32_t)t->smallest(), st));
@@ -1042,6 +1115,7 @@ dyc_status resize_impl(dyc_table* t, int direction, int subtable, int method, cu
 template <int B>
 dyc_status stats_impl(dyc_table* t, dyc_stats_t* out, cudaStream_t st) {
     TRY(live_commit<B>(t, st));
+    TRY(flush_m<B>(t, st));        // exact counts, empty stash
     TRY(zero_ctr(t, st));
     const TableView tv = t->view();
     for (uint32_t i = 0; i < t->cfg.d; i++) {
@@ -1086,7 +1160,7 @@ template <int B>
 dyc_status dump_impl(dyc_table* t, uint64_t* h_kv, uint32_t* h_tab, uint64_t* h_bkt, uint64_t cap, uint64_t* n_out,
                      cudaStream_t st) {
     TRY(live_commit<B>(t, st));
-    TRY(flush_m(t, st));
+    TRY(flush_m<B>(t, st));
     const uint64_t m = t->m;
     void *kv = nullptr, *tb = nullptr, *bk = nullptr;
     TRY(dev_alloc(t, &kv, m * 8, st));
@@ -1456,7 +1530,11 @@ dyc_status dyc_clear(dyc_table* t, dyc_stream_t stream) {
     if (t->rz.active) TRY(live_commit_any(t, S(stream)));
     for (uint32_t i = 0; i < t->cfg.d; i++)
         CU(cudaMemsetAsync(t->sub[i], 0xFF, t->nb[i] * t->cfg.bucket_slots * 8, S(stream)));
-    TRY(flush_m(t, S(stream)));   // settles the removals counted on the device
+    // the counts still on the device are read (statistics) and the stash is
+    // discarded with the rest of the contents
+    if (t->m_lazy || t->ev_pending) TRY(read_ctr(t, S(stream)));
+    CU(cudaMemsetAsync(t->d_ctr + C_STASH, 0, sizeof(unsigned long long), S(stream)));
+    t->stash_bound = 0;
     t->m = 0;
     t->clean = (1u << t->cfg.d) - 1u;
     return DYC_OK;
@@ -1475,12 +1553,13 @@ dyc_status dyc_stats(dyc_table* t, dyc_stats_t* out, dyc_stream_t stream) {
     DISPATCH_B(t, stats_impl<B_>(t, out, S(stream)));
 }
 
-dyc_status dyc_shape(const dyc_table* t, uint64_t* buckets, uint64_t* m, uint64_t* m_pending) {
+dyc_status dyc_shape(const dyc_table* t, uint64_t* buckets, uint64_t* m_lo, uint64_t* m_hi, uint64_t* n_fail_upsize) {
     TRY(check_table(t));
     if (buckets)
         for (uint32_t i = 0; i < t->cfg.d; i++) buckets[i] = t->nb[i];
-    if (m) *m = t->m;
-    if (m_pending) *m_pending = t->m_lazy ? t->lazy_n : 0;
+    if (m_lo) *m_lo = t->m >= t->lazy_del ? t->m - t->lazy_del : 0;
+    if (m_hi) *m_hi = t->m + t->lazy_add;
+    if (n_fail_upsize) *n_fail_upsize = t->n_fail_upsize;
     return DYC_OK;
 }
 

@@ -57,6 +57,10 @@ struct TableView {
     // w[t] = n_t / max(C(m_t, 2), 1) per subtable, a snapshot taken at
     // the start of the batch; nullptr = two-choice first-fit (reading Q3)
     const float* wsel;
+    // homeless pairs of lazily settled insert batches (dyc_kernels.cuh
+    // stash_find) and their count (a device counter)
+    unsigned long long* stash;
+    const unsigned long long* stash_n;
 };
 
 // Shared-memory copy of the per-subtable fields, indexed by a lane-varying t.

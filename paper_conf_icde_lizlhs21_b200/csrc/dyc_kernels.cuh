@@ -45,18 +45,26 @@ constexpr int kThreads = 256;
 #define DYC_FIND_ILP 4
 #endif
 
+// Device counters.  [0, C_ACC0) are per batch (zeroed when a batch starts);
+// [C_ACC0, C_COUNT0) accumulate across batches until the host reads them back
+// (read_ctr applies them to its live count and statistics, then zeroes them),
+// so a batch that does not need an exact count can return without a host wait.
 enum CounterIdx : int {
     C_PENDING = 0,    // new keys handed to k_place
     C_INSERTED = 1,   // ops with status INSERTED
     C_UPDATED = 2,    // ops with status UPDATED
-    C_FAIL = 3,       // homeless pairs appended by k_place
-    C_EVICT = 4,      // eviction hops
-    C_REMOVED = 5,    // delete hits
-    C_RESIDUAL = 6,   // downsize residuals
-    C_DUMP = 7,       // dump cursor
-    C_SECOND = 8,     // keys in their second-choice subtable (stats)
-    C_RES_TOTAL = 9,  // residuals over several downsizes of one alpha loop
-    C_DEFER = 10,     // ops on a subtable locked by a resize in flight (NEXT-1)
+    C_FAIL = 3,       // homeless pairs appended by k_place (synchronous settling)
+    C_RESIDUAL = 4,   // downsize residuals
+    C_DUMP = 5,       // dump cursor
+    C_SECOND = 6,     // keys in their second-choice subtable (stats)
+    C_RES_TOTAL = 7,  // residuals over several downsizes of one alpha loop
+    C_DEFER = 8,      // ops on a subtable locked by a resize in flight (NEXT-1)
+    C_ACC0 = 11,
+    C_STASH = 11,     // pairs in the stash (homeless after a lazily settled batch)
+    C_REMOVED = 12,   // delete hits
+    C_EVICT = 13,     // eviction hops
+    C_ADDED = 14,     // INSERTED statuses (live-count increments)
+    C_PEND_ACC = 15,  // new keys handed to k_place (statistics)
     C_COUNT0 = 16,    // per-subtable live counts [16, 32)
     C_N = 32
 };
@@ -132,6 +140,27 @@ __device__ __forceinline__ unsigned empty_mask(const unsigned long long (&s)[4])
     return m;
 }
 
+// ------------------------------------------------------------------- stash
+// Pairs that an insert batch could not place within L_max hops wait in
+// the stash until the host's next read-back settles them (retry, then
+// failure-triggered upsizes, Q17); until then they are live keys of the map, so
+// find, the existence check of insert and delete look there after both
+// candidate buckets missed (the stash is empty in normal operation: one load of
+// its count per thread).  Returns the stash index of k, or -1.  The group's
+// lead lane scans; the result is broadcast.
+template <int G>
+__device__ __forceinline__ int64_t stash_find(const Grp<G>& g, const TableView& tv, uint64_t sn, uint32_t k, bool want) {
+    int64_t at = -1;
+    if (g.sub == 0 && want && k != kEmptyKey)
+        for (uint64_t j = 0; j < sn; j++)
+            if (key_of(*(volatile unsigned long long*)(tv.stash + j)) == k) { at = (int64_t)j; break; }
+    return (int64_t)__shfl_sync(kFull, (unsigned long long)at, g.base);
+}
+
+__device__ __forceinline__ uint64_t stash_count(const TableView& tv) {
+    return tv.stash_n ? *(volatile const unsigned long long*)tv.stash_n : 0ull;
+}
+
 // ----------------------------------------------------------------- find (S3)
 // ILP queries per group; all first probes are issued back to back, then the
 // second probes (predicated, only after a first-probe miss: <= 2 lookups).
@@ -149,6 +178,7 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
     const uint64_t wtile = (uint64_t)QPW * ILP;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
+    const uint64_t sn = stash_count(tv);
     unsigned long long n_ops = 0, n_p2 = 0;
     for (uint64_t base = w * wtile; base < n; base += nwarps * wtile) {
         uint32_t k[ILP], v[ILP];
@@ -189,6 +219,10 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
             const unsigned hb = g.ballot(lh);
             const uint32_t v2 = g.bcast32(lv, first_lane(hb));
             if (hb) { f[j] = true; v[j] = v2; }
+            if (sn) {
+                const int64_t at = stash_find(g, tv, sn, k[j], !f[j]);
+                if (at >= 0) { f[j] = true; v[j] = val_of(tv.stash[at]); }
+            }
             const uint64_t i = base + (uint64_t)j * QPW + grp;
             if (g.sub == 0 && i < n) {
                 vals[i] = f[j] ? v[j] : kEmptyKey;
@@ -317,6 +351,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
     const unsigned grp = g.lane / G;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
+    const uint64_t sn = stash_count(tv);
     unsigned long long n_ins = 0, n_upd = 0, n_ops = 0, n_p2 = 0;
     for (uint64_t base = w * (QPW * U); base < n; base += nwarps * (QPW * U)) {
         // per op only the match position and the free-slot mask of each bucket
@@ -422,6 +457,14 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
             if (LK) warp_append(g.sub == 0 && ((h1[u] && lk1[u]) || (h2[u] && lk2[u])), kv[u], defer, ctr + C_DEFER);
             isnew[u] = k[u] != kEmptyKey && h1[u] == 0 && h2[u] == 0;
             placed[u] = false;
+            if (sn) {                       // a stashed pair is present: update it in place
+                const int64_t at = stash_find(g, tv, sn, k[u], isnew[u]);
+                if (at >= 0) {
+                    if (g.sub == 0) st_u64_cg(tv.stash + at, kv[u]);
+                    isnew[u] = false;
+                    h1[u] |= 1u;            // status UPDATED below
+                }
+            }
         }
         if (FUSE) {
             // paper-weighted mode: only the chosen table's bucket is a candidate
@@ -447,6 +490,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
         }
     }
     block_add<kThreads>(ctr + C_INSERTED, n_ins);
+    block_add<kThreads>(ctr + C_ADDED, n_ins);
     block_add<kThreads>(ctr + C_UPDATED, n_upd);
     if (tv.probe) {
         block_add<kThreads>(tv.probe + 2, n_ops);
@@ -470,12 +514,16 @@ template <int B>
 __global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv, const unsigned long long* __restrict__ list,
                                                     const unsigned long long* count_ptr, uint64_t count_host,
                                                     unsigned long long* __restrict__ fail_list,
-                                                    unsigned long long* __restrict__ ctr, bool first_fit) {
+                                                    unsigned long long* __restrict__ ctr, bool first_fit,
+                                                    unsigned long long* __restrict__ fail_cursor = nullptr,
+                                                    unsigned long long* __restrict__ pend_acc = nullptr) {
     constexpr int G = B / 4;
     __shared__ SmemView sv;
     load_view(tv, sv);
     const Grp<G> g;
     const uint64_t cnt = count_ptr ? *(volatile const unsigned long long*)count_ptr : count_host;
+    if (pend_acc && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(pend_acc, (unsigned long long)cnt);
+    unsigned long long* const fcur = fail_cursor ? fail_cursor : ctr + C_FAIL;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
     const uint64_t per = (cnt + nwarps - 1) / nwarps;
@@ -490,7 +538,7 @@ __global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv
         const unsigned want = __ballot_sync(kFull, idle && g.sub == 0);   // one bit per idle group leader
         const uint64_t mine = next + __popc(want & ((1u << g.base) - 1u)); // idle leaders before this group
         next += __popc(want);
-        if (idle && mine < end) {
+        if (idle && mine < end && key_of(list[mine]) != kEmptyKey) {   // (a stash tombstone is skipped)
             kv = list[mine];
             k = key_of(kv);
             const Pair p = pair_of(tv, k);
@@ -542,7 +590,7 @@ __global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv
                 if (hop >= tv.max_hops) { fail = true; phase = -1; }
             }
         }
-        warp_append(g.sub == 0 && fail, kv, fail_list, ctr + C_FAIL);
+        warp_append(g.sub == 0 && fail, kv, fail_list, fcur);
     }
     block_add<kThreads>(ctr + C_EVICT, ev);
 }
@@ -590,6 +638,7 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
     const unsigned grp = g.lane / G;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
+    const uint64_t sn = stash_count(tv);
     unsigned long long removed = 0, n_ops = 0, n_p2 = 0;
     for (uint64_t base = w * (QPW * U); base < n; base += nwarps * (QPW * U)) {
         uint64_t i[U];
@@ -637,9 +686,18 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
             if (LK) warp_append(g.sub == 0 && ((h1[u] && lk1[u]) || (h2 && lk2[u])), make_kv(k[u], 0u), defer, ctr + C_DEFER);
             const uint32_t o1 = g.bcast32(lv1, first_lane(h1[u]));
             const uint32_t o2 = g.bcast32(lv2, first_lane(h2));
-            const bool hit = (h1[u] | h2) != 0;
+            bool hit = (h1[u] | h2) != 0;
+            uint32_t ov = h1[u] ? o1 : (h2 ? o2 : kEmptyKey);
+            if (sn) {                       // a stashed pair: remove it from the stash
+                const int64_t at = stash_find(g, tv, sn, k[u], !hit && k[u] != kEmptyKey);
+                if (at >= 0) {
+                    ov = val_of(tv.stash[at]);
+                    if (g.sub == 0) st_u64_cg(tv.stash + at, kEmptySlot);
+                    hit = true;
+                }
+            }
             if (g.sub == 0 && i[u] < n) {
-                if (old_vals) old_vals[i[u]] = h1[u] ? o1 : (h2 ? o2 : kEmptyKey);
+                if (old_vals) old_vals[i[u]] = ov;
                 if (status) status[i[u]] = hit ? 1 : 0;
             }
             removed += (g.sub == 0 && hit);

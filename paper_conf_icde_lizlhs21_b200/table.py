@@ -307,17 +307,19 @@ class Table:
     def clear(self, stream=None):
         L.check(self._lib.dyc_clear(self._h, _stream_ptr(stream)), "dyc_clear")
 
-    def shape(self) -> Tuple[list, int, int]:
-        """(buckets per subtable, m, removals possibly pending) from the host's
-        view, without touching the device (dyc_shape: never synchronizes)."""
+    def shape(self) -> Dict:
+        """Host view without touching the device (dyc_shape: never synchronizes):
+        buckets per subtable, the live-count bounds m_lo <= m <= m_hi left by
+        batches that skipped their read-back, failure-triggered upsizes so far."""
         nb = np.zeros(self.d, dtype=np.uint64)
-        m, pend = C.c_uint64(), C.c_uint64()
-        L.check(self._lib.dyc_shape(self._h, nb.ctypes.data_as(C.c_void_p), C.byref(m), C.byref(pend)),
+        lo, hi, nf = C.c_uint64(), C.c_uint64(), C.c_uint64()
+        L.check(self._lib.dyc_shape(self._h, nb.ctypes.data_as(C.c_void_p), C.byref(lo), C.byref(hi), C.byref(nf)),
                 "dyc_shape")
-        return [int(x) for x in nb], int(m.value), int(pend.value)
+        return {"buckets": [int(x) for x in nb], "m_lo": int(lo.value), "m_hi": int(hi.value),
+                "n_fail_upsize": int(nf.value)}
 
     def _buckets_host(self):
-        return self.shape()[0]
+        return self.shape()["buckets"]
 
     def stats(self, stream=None) -> Dict:
         s = L.dyc_stats_t()

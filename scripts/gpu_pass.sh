@@ -25,6 +25,15 @@ for step in "$@"; do
       done ;;
     configs) for c in c1 "c3 --shape RE" "c3 --shape TW" "c4 --shape LINE" "c4 --shape COM"; do
                n=$(echo "$c" | tr -c 'a-zA-Z0-9' '_'); timeout 1200 python bench.py --config $c > gpurun_out/cfg_${R}_$n.json 2> gpurun_out/cfg_${R}_$n.err; head -c 250 gpurun_out/cfg_${R}_$n.json; echo; done ;;
+    ablation)   # NEXT-4: placement rule x d x bucket width at C2, placement rule at C3-RE (x0.25)
+      for pl in first_fit paper_weighted; do
+        for d in 2 3 4 6 8; do
+          timeout 900 python bench.py --placement $pl --d $d --steps 3 --warmup 3 --no-e2e --no-cpu-baseline --no-rehash > gpurun_out/abl_${R}_${pl}_d$d.json 2> gpurun_out/abl_${R}_${pl}_d$d.err; head -c 200 gpurun_out/abl_${R}_${pl}_d$d.json; echo
+        done
+        timeout 900 python bench.py --placement $pl --bucket-slots 16 --steps 3 --warmup 3 --no-e2e --no-cpu-baseline --no-rehash > gpurun_out/abl_${R}_${pl}_B16.json 2>&1; head -c 200 gpurun_out/abl_${R}_${pl}_B16.json; echo
+        timeout 900 python bench.py --placement $pl --bucket-slots 4 --steps 3 --warmup 3 --no-e2e --no-cpu-baseline --no-rehash > gpurun_out/abl_${R}_${pl}_B4.json 2>&1; head -c 200 gpurun_out/abl_${R}_${pl}_B4.json; echo
+        timeout 900 python bench.py --config c3 --shape RE --scale 0.25 --placement $pl --no-cpu-baseline > gpurun_out/abl_${R}_${pl}_c3.json 2>&1; head -c 200 gpurun_out/abl_${R}_${pl}_c3.json; echo
+      done ;;
     *) echo "unknown step $step" ;;
   esac
 done

@@ -35,5 +35,5 @@ def test_gather_rejects_bad_arguments():
     sink = torch.zeros(1, dtype=torch.int64, device="cuda")
     s = torch.cuda.current_stream().cuda_stream
     assert L.dyc_bench_gather(buf.data_ptr(), buf.numel(), 16, 48, 1, sink.data_ptr(), s) == L.DYC_ERR_INVALID_ARG
-    assert L.dyc_bench_gather_ex(buf.data_ptr(), buf.numel(), 16, 64, 1, 2, sink.data_ptr(), s) == L.DYC_ERR_INVALID_ARG
+    assert L.dyc_bench_gather_ex(buf.data_ptr(), buf.numel(), 16, 64, 1, 8, sink.data_ptr(), s) == L.DYC_ERR_INVALID_ARG
     assert L.dyc_bench_gather(buf.data_ptr(), 16, 16, 64, 1, sink.data_ptr(), s) == L.DYC_ERR_INVALID_ARG
