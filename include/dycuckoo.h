@@ -198,10 +198,14 @@ dyc_status dyc_delete_batch(dyc_table* t, const uint32_t* d_keys, uint32_t* d_va
  * mixed batches ambiguous (commented); reading Q10: keys are distinct
  * across the whole batch and the phases run find -> insert -> delete, so finds
  * observe the table before the batch.  The ops are grouped by type on the
- * device, run as three single-type batches, and the results returned in request
- * order: d_values_out[i] (nullable) = found / removed value, DYC_NOT_FOUND on a
- * miss and for inserts; d_status[i] (nullable) = the op's status code.
- * Synchronizes `stream` (the phase sizes are needed on the host). */
+ * device into fixed regions of a scratch buffer and run as three single-type
+ * batches whose op counts stay on the device (the kernels read them), so the
+ * grouping adds no host wait; the results return in request order:
+ * d_values_out[i] (nullable) = found / removed value, DYC_NOT_FOUND on a miss
+ * and for inserts; d_status[i] (nullable) = the op's status code; d_values
+ * may be NULL (inserts then store 0).  An op code outside 0..2 gets status
+ * DYC_OP_NONE and has no effect.  n < 2^30.  Scratch: about 56 bytes per op,
+ * owned by the table. */
 enum { DYC_MIX_FIND = 0, DYC_MIX_INSERT = 1, DYC_MIX_DELETE = 2 };
 dyc_status dyc_mixed_batch(dyc_table* t, const uint8_t* d_ops, const uint32_t* d_keys,
                            const uint32_t* d_values, uint32_t* d_values_out, uint8_t* d_status,

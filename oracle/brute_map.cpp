@@ -59,6 +59,8 @@ void bm_delete_batch(void* h, const uint32_t* keys, uint32_t* vals, uint8_t* sta
 void bm_mixed_batch(void* h, const uint8_t* ops, const uint32_t* keys, const uint32_t* vals, uint32_t* vals_out,
                     uint8_t* status, uint64_t n) {
     auto& m = static_cast<Map*>(h)->m;
+    for (uint64_t i = 0; i < n; i++)
+        if (ops[i] > 2) { vals_out[i] = kEmpty; status[i] = 0; }   // no operation (reading Q10)
     for (int phase = 0; phase < 3; phase++)
         for (uint64_t i = 0; i < n; i++) {
             if (ops[i] != phase) continue;

@@ -508,6 +508,13 @@ void dyo_mixed_batch(dyo_table *T, const uint8_t *ops, const uint32_t *keys, con
     uint32_t *v = (uint32_t *)malloc((n + 1) * sizeof(uint32_t));
     uint32_t *ov = (uint32_t *)malloc((n + 1) * sizeof(uint32_t));
     uint8_t *st = (uint8_t *)malloc(n + 1);
+    /* an op code outside 0..2 is no operation: status NONE, value NOT_FOUND
+       (reading Q10) */
+    for (uint64_t i = 0; i < n; i++)
+        if (ops[i] > 2) {
+            if (vals_out) vals_out[i] = DYO_EMPTY;
+            if (status) status[i] = 0;
+        }
     for (uint8_t op = 0; op < 3; op++) {
         uint64_t c = 0;
         for (uint64_t i = 0; i < n; i++)

@@ -759,18 +759,20 @@ dyc_status insert_begin(dyc_table* t, uint64_t n, cudaStream_t st, bool& fuse) {
 
 template <int B>
 dyc_status insert_chunk(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* status, uint64_t n,
-                        bool fuse, cudaStream_t st) {
+                        bool fuse, cudaStream_t st, const unsigned long long* n_dev = nullptr) {
     constexpr int U = DYC_UPSERT_U;
     const unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
     {
         ProfScope ps(t, DYC_PROF_UPSERT, st);
         if (t->rz.active)
             k_upsert<B, true, U, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0],
-                                                                  t->d_ctr, t->rz.ti, t->list[1]);
+                                                                  t->d_ctr, t->rz.ti, t->list[1], n_dev);
         else if (fuse)
-            k_upsert<B, true, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
+            k_upsert<B, true, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr,
+                                                            0xFFFFFFFFu, nullptr, n_dev);
         else
-            k_upsert<B, false, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr);
+            k_upsert<B, false, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr,
+                                                             0xFFFFFFFFu, nullptr, n_dev);
     }
     CU(cudaGetLastError());
     return DYC_OK;
@@ -838,12 +840,12 @@ dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals,
 
 template <int B>
 dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* found, uint64_t n,
-                     cudaStream_t st) {
+                     cudaStream_t st, const unsigned long long* n_dev = nullptr) {
     constexpr int ILP = (B <= 16) ? DYC_FIND_ILP : 2;
     constexpr uint64_t per_block = (uint64_t)(kThreads / (B / 4)) * ILP;   // queries per block per pass
     {
         ProfScope ps(t, DYC_PROF_FIND, st);
-        k_find<B, ILP><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n);
+        k_find<B, ILP><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
     }
     CU(cudaGetLastError());
     return DYC_OK;
@@ -864,16 +866,17 @@ dyc_status delete_prep(dyc_table* t, uint64_t n, cudaStream_t st) {
 
 template <int B>
 dyc_status delete_chunk(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
-                        cudaStream_t st) {
+                        cudaStream_t st, const unsigned long long* n_dev = nullptr) {
     {
         ProfScope ps(t, DYC_PROF_DELETE, st);
         constexpr int U = DYC_DELETE_U;
         const unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
         if (t->rz.active)
             k_delete<B, U, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, t->rz.ti,
-                                                            t->list[0]);
+                                                            t->list[0], n_dev);
         else
-            k_delete<B, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr);
+            k_delete<B, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, 0xFFFFFFFFu,
+                                                      nullptr, n_dev);
     }
     CU(cudaGetLastError());
     return DYC_OK;
@@ -1192,6 +1195,59 @@ dyc_status dump_impl(dyc_table* t, uint64_t* h_kv, uint32_t* h_tab, uint64_t* h_
     return DYC_OK;
 }
 
+// Mixed batch (reading Q10: finds, then inserts, then deletes).  The ops are
+// grouped by op code on the device into fixed regions [c*n, (c+1)*n) of the
+// scratch; each phase runs on its region with its count read by the kernels on
+// the device, so the grouping costs no host wait and each phase waits only
+// when its own resize decision needs the exact live count.  Op codes outside
+// 0..2 land in region 3 and get status DYC_OP_NONE.
+template <int B>
+dyc_status mixed_impl(dyc_table* t, const uint8_t* d_ops, const uint32_t* d_keys, const uint32_t* d_values,
+                      uint32_t* d_values_out, uint8_t* d_status, uint64_t n, cudaStream_t st) {
+    const uint64_t need = n * (4 * 4 + 4 * 4 + 4 * 4 + 4 + 4) + 256;   // k, v, out v (4n each), status (4n), pos
+    if (need > t->mix_cap) {
+        if (t->mix) dev_free(t, t->mix, st);
+        t->mix = nullptr;
+        t->mix_cap = 0;
+        TRY(dev_alloc(t, &t->mix, need, st));
+        t->mix_cap = need;
+    }
+    unsigned long long* cnt = (unsigned long long*)t->mix;      // [0..4) counts, [4..8) cursors
+    uint32_t* k = (uint32_t*)(cnt + 8);
+    uint32_t* v = k + 4 * n;
+    uint32_t* ov = v + 4 * n;
+    uint32_t* pos = ov + 4 * n;
+    uint8_t* sts = (uint8_t*)(pos + n);
+    CU(cudaMemsetAsync(cnt, 0, 8 * 8, st));
+    {
+        ProfScope ps(t, DYC_PROF_OTHER, st);
+        const OpDest od{d_ops};
+        k_group_count<OpDest><<<std::min<unsigned>(grid_for(n, kThreads * 4), t->num_sms * 8), kThreads,
+                                (kThreads / 32) * 4 * 4, st>>>(od, n, 4, cnt);
+        k_fixed_bases<<<1, 32, 0, st>>>(cnt + 4, 4, n);
+        k_group_scatter<OpDest><<<grid_for(n, (uint64_t)kThreads * kTileItems), kThreads, 4 * 12, st>>>(
+            od, d_keys, d_values, n, 4, cnt + 4, k, v, pos);
+    }
+    CU(cudaGetLastError());
+    // phase 1: finds observe the table before the batch
+    TRY(find_impl<B>(t, k, ov, sts, n, st, cnt + 0));
+    // phase 2: inserts (one batch of at most n new keys)
+    bool fuse = false;
+    TRY(insert_begin<B>(t, n, st, fuse));
+    TRY(insert_chunk<B>(t, k + n, v + n, sts + n, n, fuse, st, cnt + 1));
+    TRY(insert_end<B>(t, fuse, st));
+    CU(cudaMemsetAsync(ov + n, 0xFF, n * 4, st));
+    // phase 3: deletes
+    TRY(delete_prep<B>(t, n, st));
+    TRY(delete_chunk<B>(t, k + 2 * n, ov + 2 * n, sts + 2 * n, n, st, cnt + 2));
+    TRY(delete_end<B>(t, st));
+    // region 3: invalid op codes
+    CU(cudaMemsetAsync(ov + 3 * n, 0xFF, n * 4, st));
+    CU(cudaMemsetAsync(sts + 3 * n, 0, n, st));
+    return dyc_route_unpermute(pos, n, d_values_out ? ov : nullptr, d_status ? sts : nullptr, d_values_out, d_status,
+                               st);
+}
+
 #define DISPATCH_B(t, CALL)                                                        \
     switch ((t)->cfg.bucket_slots) {                                               \
         case 4: { constexpr int B_ = 4; return CALL; }                             \
@@ -1441,50 +1497,8 @@ dyc_status dyc_mixed_batch(dyc_table* t, const uint8_t* d_ops, const uint32_t* d
     TRY(enter(t, stream));
     if (n == 0) return DYC_OK;
     if (!d_ops || !d_keys) return set_err(DYC_ERR_INVALID_ARG, "null ops/keys");
-    if (n > 0xFFFFFFFFull) return set_err(DYC_ERR_INVALID_ARG, "mixed batch must be < 2^32 ops");
-    cudaStream_t st = S(stream);
-    // scratch: keys, values, out values (u32 x n each), pos (u32 x n), status (u8 x n), 8 counters
-    const uint64_t need = n * 17 + 128;
-    if (need > t->mix_cap) {
-        if (t->mix) dev_free(t, t->mix, st);
-        t->mix = nullptr;
-        t->mix_cap = 0;
-        TRY(dev_alloc(t, &t->mix, need, st));
-        t->mix_cap = need;
-    }
-    unsigned long long* cnt = (unsigned long long*)t->mix;      // [0..4) counts, [4..8) cursors
-    uint32_t* k = (uint32_t*)(cnt + 8);
-    uint32_t* v = k + n;
-    uint32_t* ov = v + n;
-    uint32_t* pos = ov + n;
-    uint8_t* sts = (uint8_t*)(pos + n);
-    CU(cudaMemsetAsync(cnt, 0, 8 * 8, st));
-    {
-        ProfScope ps(t, DYC_PROF_OTHER, st);
-        const OpDest od{d_ops};
-        k_group_count<OpDest><<<std::min<unsigned>(grid_for(n, kThreads * 4), t->num_sms * 8), kThreads,
-                                (kThreads / 32) * 4 * 4, st>>>(
-            od, n, 4, cnt);
-        k_route_offsets<<<1, 32, 0, st>>>(cnt, 4, cnt + 4);
-        k_group_scatter<OpDest><<<grid_for(n, (uint64_t)kThreads * kTileItems), kThreads, 4 * 12, st>>>(
-            od, d_keys, d_values, n, 4, cnt + 4, k, v, pos);
-    }
-    CU(cudaGetLastError());
-    unsigned long long h[4];
-    CU(cudaMemcpyAsync(h, cnt, sizeof(h), cudaMemcpyDeviceToHost, st));
-    CU(cudaStreamSynchronize(st));
-    if (h[3]) return set_err(DYC_ERR_INVALID_ARG, "op codes must be 0 (find), 1 (insert) or 2 (delete)");
-    const uint64_t nf = h[0], ni = h[1], nd = h[2];
-    // phases: find -> insert -> delete (Q10)
-    if (nf) TRY(dyc_find_batch(t, k, ov, sts, nf, stream));
-    if (ni) {
-        TRY(dyc_insert_batch(t, k + nf, v + nf, sts + nf, ni, stream));
-        CU(cudaMemsetAsync(ov + nf, 0xFF, ni * 4, st));
-    }
-    if (nd) TRY(dyc_delete_batch(t, k + nf + ni, ov + nf + ni, sts + nf + ni, nd, stream));
-    TRY(dyc_route_unpermute(pos, n, d_values_out ? ov : nullptr, d_status ? sts : nullptr, d_values_out, d_status,
-                            stream));
-    return DYC_OK;
+    if (n > 0xFFFFFFFFull / 4) return set_err(DYC_ERR_INVALID_ARG, "mixed batch must be < 2^30 ops");
+    DISPATCH_B(t, mixed_impl<B_>(t, d_ops, d_keys, d_values, d_values_out, d_status, n, S(stream)));
 }
 
 dyc_status dyc_resize_ex(dyc_table* t, int direction, int subtable, int method, dyc_stream_t stream) {

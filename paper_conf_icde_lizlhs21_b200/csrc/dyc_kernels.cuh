@@ -169,10 +169,11 @@ __device__ __forceinline__ uint64_t stash_count(const TableView& tv) {
 template <int B, int ILP>
 __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, const uint32_t* __restrict__ keys,
                                                    uint32_t* __restrict__ vals, uint8_t* __restrict__ found,
-                                                   uint64_t n) {
+                                                   uint64_t n, const unsigned long long* __restrict__ n_dev = nullptr) {
     constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
+    if (n_dev) n = min(n, (uint64_t)*n_dev);     // op count known on the device only (mixed batches)
     const Grp<G> g;
     const unsigned grp = g.lane / G;
     const uint64_t wtile = (uint64_t)QPW * ILP;
@@ -343,10 +344,12 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                                                      unsigned long long* __restrict__ pending,
                                                      unsigned long long* __restrict__ ctr,
                                                      uint32_t locked = 0xFFFFFFFFu,
-                                                     unsigned long long* __restrict__ defer = nullptr) {
+                                                     unsigned long long* __restrict__ defer = nullptr,
+                                                     const unsigned long long* __restrict__ n_dev = nullptr) {
     constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
+    if (n_dev) n = min(n, (uint64_t)*n_dev);     // op count known on the device only (mixed batches)
     const Grp<G> g;
     const unsigned grp = g.lane / G;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
@@ -630,10 +633,12 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
                                                      uint8_t* __restrict__ status, uint64_t n,
                                                      unsigned long long* __restrict__ ctr,
                                                      uint32_t locked = 0xFFFFFFFFu,
-                                                     unsigned long long* __restrict__ defer = nullptr) {
+                                                     unsigned long long* __restrict__ defer = nullptr,
+                                                     const unsigned long long* __restrict__ n_dev = nullptr) {
     constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
+    if (n_dev) n = min(n, (uint64_t)*n_dev);     // op count known on the device only (mixed batches)
     const Grp<G> g;
     const unsigned grp = g.lane / G;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
@@ -1047,6 +1052,13 @@ __global__ void __launch_bounds__(kThreads) k_group_scatter(Dest dest, const uin
         }
         __syncthreads();
     }
+}
+
+// Fixed region bases for the phases of a mixed batch: op code c's ops go to
+// [c*n, (c+1)*n) of the scratch, so every phase's keys start at an address the
+// host knows while its count stays on the device (no host wait).
+__global__ void k_fixed_bases(unsigned long long* __restrict__ cursor, uint32_t regions, uint64_t n) {
+    if (threadIdx.x < regions) cursor[threadIdx.x] = (unsigned long long)threadIdx.x * n;
 }
 
 // Exclusive prefix sum of the per-destination counts into the scatter cursors (one block).
