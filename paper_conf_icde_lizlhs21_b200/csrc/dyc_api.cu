@@ -208,7 +208,7 @@ struct dyc_table {
         v.probe = count_probes ? d_probe : nullptr;
         v.wsel = weighted ? d_w : nullptr;
         v.stash = stash;
-        v.stash_n = d_ctr ? d_ctr + C_STASH : nullptr;
+        v.stash_n = (d_ctr && stash_bound) ? d_ctr + C_STASH : nullptr;   // known empty: no load at all
         return v;
     }
 };
@@ -790,21 +790,24 @@ dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
             if (dfr) TRY(launch_apply<B>(t, t->list[1], false, dfr, st));
             if (pend) TRY(place_and_settle<B>(t, 0, t->d_ctr + C_PENDING, 0, true, st));
         }
+        t->m += ins;
         t->last_new = ins;
         t->last_pending = pend;
         t->n_pending_total += pend;
         t->last_evict = t->n_evict - ev0;
         return policy_lower<B>(t, st);
     }
+    uint64_t add_bound = t->ins_n;
     if (!fuse) {
-        // the resize decision needs n_new before any placement (Q11):
-        // after the read-back m includes this batch's new keys
+        // the resize decision needs n_new before any placement (Q11)
         TRY(read_ctr(t, st));
-        while ((double)t->m > t->cfg.beta * (double)t->N()) {
+        const uint64_t n_new = t->h_ctr[C_INSERTED];
+        while ((double)(t->m + n_new) > t->cfg.beta * (double)t->N()) {
             TRY(upsize_table<B>(t, (uint32_t)t->smallest(), st));
             t->n_upsize++;
         }
         TRY(refresh_weights<B>(t, st));   // after an upsize the bigger table draws more
+        add_bound = n_new;
     }
     // placement of the keys whose candidate buckets were full; pairs still
     // homeless after L_max hops go to the stash, which every later batch
@@ -813,16 +816,13 @@ dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
     {
         ProfScope ps(t, DYC_PROF_PLACE, st);
         k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->list[0], t->d_ctr + C_PENDING, 0, t->stash,
-                                                         t->d_ctr, !fuse, t->d_ctr + C_STASH,
-                                                         t->d_ctr + C_PEND_ACC);
+                                                         t->d_ctr, !fuse, t->d_ctr + C_STASH, true);
     }
     CU(cudaGetLastError());
-    t->stash_bound += t->ins_n;
+    t->stash_bound += add_bound;
     t->ins_lazy = true;
-    if (fuse) {
-        t->lazy_add += t->ins_n;
-        t->m_lazy = true;
-    }
+    t->lazy_add += add_bound;     // the batch's INSERTED count reaches m at the next read-back
+    t->m_lazy = true;
     TRY(mark_lazy(t, st));
     // the alpha loop cannot fire while a lower bound of m is >= alpha*N
     if (t->m >= t->lazy_del && (double)(t->m - t->lazy_del) >= t->cfg.alpha * (double)t->N()) return DYC_OK;

@@ -493,7 +493,6 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
         }
     }
     block_add<kThreads>(ctr + C_INSERTED, n_ins);
-    block_add<kThreads>(ctr + C_ADDED, n_ins);
     block_add<kThreads>(ctr + C_UPDATED, n_upd);
     if (tv.probe) {
         block_add<kThreads>(tv.probe + 2, n_ops);
@@ -519,13 +518,18 @@ __global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv
                                                     unsigned long long* __restrict__ fail_list,
                                                     unsigned long long* __restrict__ ctr, bool first_fit,
                                                     unsigned long long* __restrict__ fail_cursor = nullptr,
-                                                    unsigned long long* __restrict__ pend_acc = nullptr) {
+                                                    bool lazy_counts = false) {
     constexpr int G = B / 4;
     __shared__ SmemView sv;
     load_view(tv, sv);
     const Grp<G> g;
     const uint64_t cnt = count_ptr ? *(volatile const unsigned long long*)count_ptr : count_host;
-    if (pend_acc && blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(pend_acc, (unsigned long long)cnt);
+    // the placement of a lazily settled insert batch also moves the batch's
+    // counts into the accumulators (k_upsert has finished: stream order)
+    if (lazy_counts && blockIdx.x == 0 && threadIdx.x == 0) {
+        atomicAdd(ctr + C_PEND_ACC, (unsigned long long)cnt);
+        atomicAdd(ctr + C_ADDED, *(volatile const unsigned long long*)(ctr + C_INSERTED));
+    }
     unsigned long long* const fcur = fail_cursor ? fail_cursor : ctr + C_FAIL;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);

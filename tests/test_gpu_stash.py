@@ -22,11 +22,16 @@ from tests.test_gpu_parity import dev, host_u32  # noqa: E402
 def test_stash_is_consulted_until_settled(oracle_mod, B):
     d, n0 = 4, 64
     init = d * B * n0
-    g = Table(d=d, init_capacity=init, alpha=0.02, beta=0.85, bucket_slots=B, max_hops=1, seed=0xC0FFEE)
-    o = oracle_mod.OracleTable(d=d, init_capacity=init, alpha=0.02, beta=0.85, bucket_slots=B, max_hops=1,
+    g = Table(d=d, init_capacity=init, alpha=0.05, beta=0.85, bucket_slots=B, max_hops=1, seed=0xC0FFEE)
+    o = oracle_mod.OracleTable(d=d, init_capacity=init, alpha=0.05, beta=0.85, bucket_slots=B, max_hops=1,
                                seed=0xC0FFEE)
-    hot = hot_keys(o, n0, (0, 1), 5, 9, want=600)
-    a, b = hot[:300], hot[300:400]
+    hot = hot_keys(o, n0, (0, 1), 5, 9, want=260)
+    a, b = hot[:200], hot[200:250]
+    # background keys first, read back exactly: from here on a lower bound of
+    # m stays above alpha*N, so no batch below needs a read-back
+    bg = np.setdiff1d(W.key_range(1 << 29, int(0.4 * init), 3), hot)
+    g.insert(dev(bg), dev(W.val_of(bg, 0)))
+    o.insert(bg, W.val_of(bg, 0))
     s0 = g.stats()
 
     def ins(k, ver):
@@ -45,7 +50,7 @@ def test_stash_is_consulted_until_settled(oracle_mod, B):
         np.testing.assert_array_equal(st.cpu().numpy(), ost)
         np.testing.assert_array_equal(host_u32(v), ov)
 
-    ins(a, 0)                                   # 300 keys, 2B slots: most fail -> stash (no read-back)
+    ins(a, 0)                                   # 200 keys, 2B slots: most fail -> stash (no read-back)
     sh = g.shape()
     assert sh["m_hi"] > sh["m_lo"], "the insert was expected to skip its read-back"
     fnd(np.concatenate([a, b, W.key_range(1 << 31, 50, 1)]))     # stash hits, misses
