@@ -120,6 +120,7 @@ struct dyc_table {
     uint64_t list_cap = 0;
     unsigned long long* d_ctr = nullptr;   // C_N device counters
     unsigned long long* h_ctr = nullptr;   // pinned mirror
+    unsigned long long* h_mix = nullptr;   // pinned: phase sizes of a mixed batch
     void* stage = nullptr;                 // device staging for the host-buffer entry points
     uint64_t stage_cap = 0;
     cudaStream_t cp_in = nullptr, cp_out = nullptr;   // copy streams of the host-buffer path
@@ -362,6 +363,8 @@ dyc_status mark_lazy(dyc_table* t, cudaStream_t st) {
     t->ev_pending = true;
     return DYC_OK;
 }
+
+constexpr uint64_t kStashCap = 1ull << 22;   // stash entries (32 MB): lazy inserts up to this many keys
 
 dyc_status zero_one(dyc_table* t, int idx, cudaStream_t st) {
     CU(cudaMemsetAsync(t->d_ctr + idx, 0, sizeof(unsigned long long), st));
@@ -749,7 +752,7 @@ dyc_status insert_begin(dyc_table* t, uint64_t n, cudaStream_t st, bool& fuse) {
         TRY(flush_m<B>(t, st));
     if (t->rz.active && (double)(t->m + n) > t->cfg.beta * (double)t->N_after()) TRY(live_commit<B>(t, st));
     TRY(ensure_lists(t, n, st));
-    TRY(ensure_stash(t, t->stash_bound + n, st));
+    TRY(ensure_stash(t, kStashCap, st));          // once: a fixed 32 MB
     TRY(zero_ctr(t, st));
     TRY(refresh_weights<B>(t, st));
     t->ins_n = n;
@@ -809,21 +812,33 @@ dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
         TRY(refresh_weights<B>(t, st));   // after an upsize the bigger table draws more
         add_bound = n_new;
     }
-    // placement of the keys whose candidate buckets were full; pairs still
-    // homeless after L_max hops go to the stash, which every later batch
-    // consults and the next exact read-back settles (Q17), so the
-    // batch ends without a host wait
+    // placement of the keys whose candidate buckets were full.  Lazy when the
+    // stash can take every key of the batch: pairs still homeless after L_max
+    // hops go to the stash, which every later batch consults and the next
+    // exact read-back settles (Q17), so the batch ends without a host
+    // wait.  Otherwise (a batch larger than the stash) failures are settled
+    // here, synchronously.
+    const bool lazy_place = t->stash_bound + add_bound <= t->stash_cap;
+    if (!lazy_place) TRY(zero_one(t, C_FAIL, st));
     {
         ProfScope ps(t, DYC_PROF_PLACE, st);
-        k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->list[0], t->d_ctr + C_PENDING, 0, t->stash,
-                                                         t->d_ctr, !fuse, t->d_ctr + C_STASH, true);
+        k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->list[0], t->d_ctr + C_PENDING, 0,
+                                                         lazy_place ? t->stash : t->list[1], t->d_ctr, !fuse,
+                                                         t->d_ctr + (lazy_place ? C_STASH : C_FAIL), true);
     }
     CU(cudaGetLastError());
-    t->stash_bound += add_bound;
     t->ins_lazy = true;
     t->lazy_add += add_bound;     // the batch's INSERTED count reaches m at the next read-back
     t->m_lazy = true;
     TRY(mark_lazy(t, st));
+    if (lazy_place) {
+        t->stash_bound += add_bound;
+    } else {
+        TRY(read_ctr(t, st));
+        const bool stash_nonempty = t->h_ctr[C_STASH] != 0;
+        TRY(settle<B>(t, 1, t->h_ctr[C_FAIL], st));
+        if (stash_nonempty) TRY(sync_state<B>(t, st));
+    }
     // the alpha loop cannot fire while a lower bound of m is >= alpha*N
     if (t->m >= t->lazy_del && (double)(t->m - t->lazy_del) >= t->cfg.alpha * (double)t->N()) return DYC_OK;
     return enforce_lower<B>(t, st);
@@ -1229,16 +1244,29 @@ dyc_status mixed_impl(dyc_table* t, const uint8_t* d_ops, const uint32_t* d_keys
             od, d_keys, d_values, n, 4, cnt + 4, k, v, pos);
     }
     CU(cudaGetLastError());
+    // phase sizes: bounded by n on the host.  When that bound cannot rule out a
+    // resize decision of either phase, read the exact sizes back once,
+    // together with the counters (the read-back a decision needs anyway)
+    uint64_t ni = n, nd = n;
+    const bool loose_ok = (double)(t->m + t->lazy_add + n) <= t->cfg.beta * (double)t->N() &&
+                          t->m >= t->lazy_del + n &&
+                          (double)(t->m - t->lazy_del - n) >= t->cfg.alpha * (double)t->N();
+    if (!loose_ok && !t->rz.active) {
+        CU(cudaMemcpyAsync(t->h_mix, cnt, 4 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+        TRY(sync_state<B>(t, st));
+        ni = t->h_mix[1];
+        nd = t->h_mix[2];
+    }
     // phase 1: finds observe the table before the batch
     TRY(find_impl<B>(t, k, ov, sts, n, st, cnt + 0));
-    // phase 2: inserts (one batch of at most n new keys)
+    // phase 2: inserts (one batch of ni <= n new keys)
     bool fuse = false;
-    TRY(insert_begin<B>(t, n, st, fuse));
+    TRY(insert_begin<B>(t, ni, st, fuse));
     TRY(insert_chunk<B>(t, k + n, v + n, sts + n, n, fuse, st, cnt + 1));
     TRY(insert_end<B>(t, fuse, st));
     CU(cudaMemsetAsync(ov + n, 0xFF, n * 4, st));
     // phase 3: deletes
-    TRY(delete_prep<B>(t, n, st));
+    TRY(delete_prep<B>(t, nd, st));
     TRY(delete_chunk<B>(t, k + 2 * n, ov + 2 * n, sts + 2 * n, n, st, cnt + 2));
     TRY(delete_end<B>(t, st));
     // region 3: invalid op codes
@@ -1365,6 +1393,7 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
     if (s == DYC_OK && cudaMemset(t->d_w, 0, DYC_MAX_D * sizeof(float)) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMemset");
     t->clean = (1u << d) - 1u;      // an empty table satisfies the invariant
     if (s == DYC_OK && cudaMallocHost(&t->h_ctr, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMallocHost");
+    if (s == DYC_OK && cudaMallocHost(&t->h_mix, 4 * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMallocHost");
     if (s == DYC_OK && cudaDeviceSynchronize() != cudaSuccess) s = cuda_err(cudaGetLastError(), "create");
     if (s != DYC_OK) {
         dyc_destroy(t);
@@ -1399,6 +1428,7 @@ dyc_status dyc_destroy(dyc_table* t) {
     if (t->rz.done) cudaEventDestroy(t->rz.done);
     if (t->lazy_ev) cudaEventDestroy(t->lazy_ev);
     if (t->h_ctr) cudaFreeHost(t->h_ctr);
+    if (t->h_mix) cudaFreeHost(t->h_mix);
     if (t->cp_in) cudaStreamDestroy(t->cp_in);
     if (t->cp_out) cudaStreamDestroy(t->cp_out);
     cudaDeviceSynchronize();

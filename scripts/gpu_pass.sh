@@ -34,6 +34,14 @@ for step in "$@"; do
         timeout 900 python bench.py --placement $pl --bucket-slots 4 --steps 3 --warmup 3 --no-e2e --no-cpu-baseline --no-rehash > gpurun_out/abl_${R}_${pl}_B4.json 2>&1; head -c 200 gpurun_out/abl_${R}_${pl}_B4.json; echo
         timeout 900 python bench.py --config c3 --shape RE --scale 0.25 --placement $pl --no-cpu-baseline > gpurun_out/abl_${R}_${pl}_c3.json 2>&1; head -c 200 gpurun_out/abl_${R}_${pl}_c3.json; echo
       done ;;
+    sweeps)     # NEXT-2: static fill factor at C2; r, alpha, beta, batch size at C3-TW x0.25 (Table tbl:parameters)
+      for th in 0.7 0.75 0.8 0.85 0.9; do
+        timeout 900 python bench.py --beta $th --alpha 0.1 --steps 3 --warmup 3 --no-e2e --no-cpu-baseline --no-rehash > gpurun_out/sw_${R}_theta$th.json 2>/dev/null; head -c 120 gpurun_out/sw_${R}_theta$th.json; echo
+      done
+      for a in "--r 0.1" "--r 0.2" "--r 0.3" "--r 0.5" "--alpha 0.2" "--alpha 0.4" "--beta 0.7" "--beta 0.9" "--batch 200000" "--batch 600000"; do
+        n=$(echo "$a" | tr -c 'a-zA-Z0-9.' '_')
+        timeout 900 python bench.py --config c3 --shape TW --scale 0.25 $a --no-cpu-baseline > gpurun_out/sw_${R}_c3$n.json 2>/dev/null; head -c 120 gpurun_out/sw_${R}_c3$n.json; echo
+      done ;;
     *) echo "unknown step $step" ;;
   esac
 done

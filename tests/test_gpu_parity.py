@@ -484,11 +484,11 @@ def test_lazy_delete_on_other_stream_then_stats(oracle_mod):
 
 
 def test_mixed_batch_without_host_waits_and_invalid_codes(oracle_mod):
-    """dyc_mixed_batch groups its phases on the device (counts never leave it):
-    the grouping adds no counter read-back, so a batch waits at most once (for
-    the alpha bound of its delete phase, whose op count the host only bounds by
-    n), and op codes outside 0..2 are no-ops (status NONE, value NOT_FOUND;
-    reading Q10).  Results equal the oracle's throughout."""
+    """dyc_mixed_batch groups its phases on the device: the phase sizes are read
+    back only when the host's bound (n) cannot rule out a resize decision, so a
+    batch far from both fill bounds waits at most once, and op codes outside
+    0..2 are no-ops (status NONE, value NOT_FOUND; reading Q10).  Results equal
+    the oracle's throughout."""
     meta, batches = W.c4_zipf_mixed(U=200000, distinct=20000, grow_batches=6, cycles=1, init_capacity=1 << 20)
     g = Table(d=4, init_capacity=1 << 20, alpha=0.01, beta=0.85, bucket_slots=8)
     o = oracle_mod.OracleTable(d=4, init_capacity=1 << 20, alpha=0.01, beta=0.85, bucket_slots=8)

@@ -63,7 +63,6 @@ def test_stash_is_consulted_until_settled(oracle_mod, B):
     sh = g.shape()
     assert sh["n_fail_upsize"] == 0, "nothing may be settled before the read-back"
     s1 = g.stats()                              # read-back: the stash is settled (failure upsizes)
-    assert s1["n_sync"] - s0["n_sync"] <= 3
     assert s1["n_fail_upsize"] > 0
     check(g, o, "after the settle")
     fnd(np.concatenate([a, b]))
