@@ -65,6 +65,9 @@ inline cudaStream_t S(dyc_stream_t s) { return reinterpret_cast<cudaStream_t>(s)
 
 }  // namespace
 
+// The placement kernel of the table's mode (first-fit or paper-weighted).
+#define DYC_PLACE_K(BB) (t->weighted ? k_place<BB, true> : k_place<BB, false>)
+
 // Error channel shared with the other translation units (dyc_dist.cu).
 void dyc_internal_set_error(const std::string& msg) { g_err = msg; }
 
@@ -461,8 +464,8 @@ dyc_status settle(dyc_table* t, int cur, uint64_t nfail, cudaStream_t st, unsign
         TRY(zero_one(t, C_FAIL, st));
         {
             ProfScope ps(t, DYC_PROF_PLACE, st);
-            k_place<B><<<grid_for(nfail, kThreads / (B / 4)), kThreads, 0, st>>>(t->view(), L[cur], nullptr, nfail,
-                                                                              L[1 - cur], t->d_ctr, true);
+            DYC_PLACE_K(B)<<<grid_for(nfail, kThreads / (B / 4)), kThreads, 0, st>>>(t->view(), L[cur], nullptr, nfail,
+                                                                              L[1 - cur], t->d_ctr, true, nullptr, false);
         }
         CU(cudaGetLastError());
         TRY(read_ctr(t, st));
@@ -479,8 +482,8 @@ template <int B>
 dyc_status launch_place(dyc_table* t, int src, const unsigned long long* d_count, uint64_t h_count, bool first_fit,
                         cudaStream_t st) {
     ProfScope ps(t, DYC_PROF_PLACE, st);
-    k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->list[src], d_count, h_count, t->list[1 - src],
-                                                     t->d_ctr, first_fit);
+    DYC_PLACE_K(B)<<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->list[src], d_count, h_count, t->list[1 - src],
+                                                     t->d_ctr, first_fit, nullptr, false);
     CU(cudaGetLastError());
     return DYC_OK;
 }
@@ -504,7 +507,7 @@ dyc_status settle_stash(dyc_table* t, cudaStream_t st) {
     TRY(zero_one(t, C_FAIL, st));
     {
         ProfScope ps(t, DYC_PROF_PLACE, st);
-        k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->stash, nullptr, S, t->list[1], t->d_ctr, true);
+        DYC_PLACE_K(B)<<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->stash, nullptr, S, t->list[1], t->d_ctr, true, nullptr, false);
     }
     CU(cudaGetLastError());
     TRY(zero_one(t, C_STASH, st));
@@ -628,8 +631,8 @@ dyc_status live_commit(dyc_table* t, cudaStream_t st) {
     TRY(zero_one(t, C_FAIL, st));
     {
         ProfScope ps(t, DYC_PROF_PLACE, st);
-        k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), r.res[0], r.ctr + C_RESIDUAL, 0, r.res[1],
-                                                         t->d_ctr, true);
+        DYC_PLACE_K(B)<<<t->place_blocks, kThreads, 0, st>>>(t->view(), r.res[0], r.ctr + C_RESIDUAL, 0, r.res[1],
+                                                         t->d_ctr, true, nullptr, false);
     }
     CU(cudaGetLastError());
     CU(cudaMemcpyAsync(t->d_ctr + C_RES_TOTAL, r.ctr + C_RES_TOTAL, 8, cudaMemcpyDeviceToDevice, st));
@@ -767,15 +770,24 @@ dyc_status insert_chunk(dyc_table* t, const uint32_t* keys, const uint32_t* vals
     const unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
     {
         ProfScope ps(t, DYC_PROF_UPSERT, st);
-        if (t->rz.active)
-            k_upsert<B, true, U, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0],
-                                                                  t->d_ctr, t->rz.ti, t->list[1], n_dev);
-        else if (fuse)
-            k_upsert<B, true, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr,
-                                                            0xFFFFFFFFu, nullptr, n_dev);
-        else
-            k_upsert<B, false, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->list[0], t->d_ctr,
-                                                             0xFFFFFFFFu, nullptr, n_dev);
+        const bool sp = t->stash_bound != 0;
+        const unsigned long long* nd = n_dev;
+        unsigned long long* pl = t->list[0];
+#define DYC_UPSERT_LAUNCH(FU, LKV, DEFER)                                                                      \
+    do {                                                                                                      \
+        const uint32_t lk = LKV ? t->rz.ti : 0xFFFFFFFFu;                                                     \
+        if (t->weighted) {                                                                                    \
+            if (sp) k_upsert<B, FU, U, LKV, true, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, pl, t->d_ctr, lk, DEFER, nd); \
+            else k_upsert<B, FU, U, LKV, true, false><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, pl, t->d_ctr, lk, DEFER, nd); \
+        } else {                                                                                              \
+            if (sp) k_upsert<B, FU, U, LKV, false, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, pl, t->d_ctr, lk, DEFER, nd); \
+            else k_upsert<B, FU, U, LKV, false, false><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, pl, t->d_ctr, lk, DEFER, nd); \
+        }                                                                                                     \
+    } while (0)
+        if (t->rz.active) DYC_UPSERT_LAUNCH(true, true, t->list[1]);
+        else if (fuse) DYC_UPSERT_LAUNCH(true, false, nullptr);
+        else DYC_UPSERT_LAUNCH(false, false, nullptr);
+#undef DYC_UPSERT_LAUNCH
     }
     CU(cudaGetLastError());
     return DYC_OK;
@@ -822,7 +834,7 @@ dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
     if (!lazy_place) TRY(zero_one(t, C_FAIL, st));
     {
         ProfScope ps(t, DYC_PROF_PLACE, st);
-        k_place<B><<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->list[0], t->d_ctr + C_PENDING, 0,
+        DYC_PLACE_K(B)<<<t->place_blocks, kThreads, 0, st>>>(t->view(), t->list[0], t->d_ctr + C_PENDING, 0,
                                                          lazy_place ? t->stash : t->list[1], t->d_ctr, !fuse,
                                                          t->d_ctr + (lazy_place ? C_STASH : C_FAIL), true);
     }
@@ -860,7 +872,10 @@ dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t
     constexpr uint64_t per_block = (uint64_t)(kThreads / (B / 4)) * ILP;   // queries per block per pass
     {
         ProfScope ps(t, DYC_PROF_FIND, st);
-        k_find<B, ILP><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
+        if (t->stash_bound)
+            k_find<B, ILP, true><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
+        else
+            k_find<B, ILP, false><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
     }
     CU(cudaGetLastError());
     return DYC_OK;
@@ -886,12 +901,14 @@ dyc_status delete_chunk(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint
         ProfScope ps(t, DYC_PROF_DELETE, st);
         constexpr int U = DYC_DELETE_U;
         const unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
-        if (t->rz.active)
-            k_delete<B, U, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, t->rz.ti,
-                                                            t->list[0], n_dev);
-        else
-            k_delete<B, U><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, 0xFFFFFFFFu,
-                                                      nullptr, n_dev);
+        const bool sp = t->stash_bound != 0;
+        if (t->rz.active) {
+            if (sp) k_delete<B, U, true, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, t->rz.ti, t->list[0], n_dev);
+            else k_delete<B, U, true, false><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, t->rz.ti, t->list[0], n_dev);
+        } else {
+            if (sp) k_delete<B, U, false, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, 0xFFFFFFFFu, nullptr, n_dev);
+            else k_delete<B, U, false, false><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, 0xFFFFFFFFu, nullptr, n_dev);
+        }
     }
     CU(cudaGetLastError());
     return DYC_OK;

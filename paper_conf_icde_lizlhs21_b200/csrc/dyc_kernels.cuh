@@ -166,7 +166,9 @@ __device__ __forceinline__ uint64_t stash_count(const TableView& tv) {
 // second probes (predicated, only after a first-probe miss: <= 2 lookups).
 // A miss in a non-full first-choice bucket of a subtable that holds the
 // first-choice-full invariant (TableView::clean) is final: no second probe.
-template <int B, int ILP>
+// STASH (compile time): the host launches this variant only while the stash
+// may hold pairs (dyc_kernels.cuh stash_find); otherwise no stash code runs.
+template <int B, int ILP, bool STASH = false>
 __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, const uint32_t* __restrict__ keys,
                                                    uint32_t* __restrict__ vals, uint8_t* __restrict__ found,
                                                    uint64_t n, const unsigned long long* __restrict__ n_dev = nullptr) {
@@ -179,7 +181,7 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
     const uint64_t wtile = (uint64_t)QPW * ILP;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
-    const uint64_t sn = stash_count(tv);
+    const uint64_t sn = STASH ? stash_count(tv) : 0ull;
     unsigned long long n_ops = 0, n_p2 = 0;
     for (uint64_t base = w * wtile; base < n; base += nwarps * wtile) {
         uint32_t k[ILP], v[ILP];
@@ -337,7 +339,8 @@ __device__ __forceinline__ void coop_cas_multi(const Grp<G>& g, unsigned long lo
 // its new value is appended to `defer` (applied by k_apply after the resize is
 // committed); a new key may only take a free slot of its OTHER candidate bucket,
 // else it is pending (placed after the commit).
-template <int B, bool FUSE, int U, bool LK = false>
+// W: the paper-weighted placement mode (compile time); STASH as in k_find.
+template <int B, bool FUSE, int U, bool LK = false, bool W = false, bool STASH = false>
 __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView tv, const uint32_t* __restrict__ keys,
                                                      const uint32_t* __restrict__ vals,
                                                      uint8_t* __restrict__ status, uint64_t n,
@@ -354,7 +357,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
     const unsigned grp = g.lane / G;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
-    const uint64_t sn = stash_count(tv);
+    const uint64_t sn = STASH ? stash_count(tv) : 0ull;
     unsigned long long n_ins = 0, n_upd = 0, n_ops = 0, n_p2 = 0;
     for (uint64_t base = w * (QPW * U); base < n; base += nwarps * (QPW * U)) {
         // per op only the match position and the free-slot mask of each bucket
@@ -383,7 +386,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                 const Pair p = pair_of(tv, k[u]);
                 lk1[u] = LK && p.t1 == locked;
                 lk2[u] = LK && p.t2 == locked;
-                ch2[u] = sv.weighted && weighted_second(sv, p.t1, p.t2, k[u]);
+                ch2[u] = W && weighted_second(sv, p.t1, p.t2, k[u]);
                 b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
                 b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
                 probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
@@ -415,7 +418,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                 const Pair p = pair_of(tv, k[u]);
                 lk1[u] = LK && p.t1 == locked;
                 lk2[u] = LK && p.t2 == locked;
-                ch2[u] = sv.weighted && weighted_second(sv, p.t1, p.t2, k[u]);
+                ch2[u] = W && weighted_second(sv, p.t1, p.t2, k[u]);
                 c1[u] = ((tv.clean >> p.t1) & 1u) && !lk1[u];
                 b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
                 b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
@@ -472,7 +475,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
         if (FUSE) {
             // paper-weighted mode: only the chosen table's bucket is a candidate
             // (P:L361); a full one sends the key to k_place, which evicts there
-            if (sv.weighted) {
+            if (W) {
 #pragma unroll
                 for (int u = 0; u < U; u++) {
                     if (ch2[u]) em1[u] = 0;
@@ -512,7 +515,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
 //               exchange a pseudo-random victim (Q5) and carry it to the other
 //               table of ITS pair; after max_hops (Q6) the
 //               carried pair goes to the failure list.
-template <int B>
+template <int B, bool W = false>
 __global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv, const unsigned long long* __restrict__ list,
                                                     const unsigned long long* count_ptr, uint64_t count_host,
                                                     unsigned long long* __restrict__ fail_list,
@@ -555,7 +558,7 @@ __global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv
             // shortcut) and evicting from a non-full bucket would break the
             // invariant for the victim.  Paper-weighted mode: the chosen table
             // plays t1's part (probed once, then evicted from).
-            t = (sv.weighted && weighted_second(sv, p.t1, p.t2, k)) ? p.t2 : p.t1;
+            t = (W && weighted_second(sv, p.t1, p.t2, k)) ? p.t2 : p.t1;
             hop = 0;
         }
         if (!__any_sync(kFull, phase >= 0)) break;
@@ -581,7 +584,7 @@ __global__ void __launch_bounds__(kThreads, DYC_PLACE_MINB) k_place(TableView tv
             phase = -1;
         } else if (act && phase < 2) {
             const Pair p = pair_of(tv, k);
-            if (sv.weighted) { phase = 2; hop = 0; }        // evict from the chosen table
+            if (W) { phase = 2; hop = 0; }                   // evict from the chosen table
             else if (phase == 0) { phase = 1; t = p.t2; }
             else { phase = 2; hop = 0; t = (mix32(k) & 1u) ? p.t2 : p.t1; }
         } else if (evict) {
@@ -631,7 +634,7 @@ __global__ void __launch_bounds__(kThreads) k_reinsert(TableView tv, const unsig
 // LK: a key found in the `locked` subtable (being resized concurrently) is
 // reported DELETED with its old value, and its removal is appended to `defer`
 // (applied by k_apply after the resize is committed).
-template <int B, int U, bool LK = false>
+template <int B, int U, bool LK = false, bool STASH = false>
 __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView tv, const uint32_t* __restrict__ keys,
                                                      uint32_t* __restrict__ old_vals,
                                                      uint8_t* __restrict__ status, uint64_t n,
@@ -647,7 +650,7 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
     const unsigned grp = g.lane / G;
     const uint64_t nwarps = (uint64_t)gridDim.x * (kThreads / 32);
     const uint64_t w = (uint64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
-    const uint64_t sn = stash_count(tv);
+    const uint64_t sn = STASH ? stash_count(tv) : 0ull;
     unsigned long long removed = 0, n_ops = 0, n_p2 = 0;
     for (uint64_t base = w * (QPW * U); base < n; base += nwarps * (QPW * U)) {
         uint64_t i[U];
