@@ -367,7 +367,7 @@ dyc_status mark_lazy(dyc_table* t, cudaStream_t st) {
     return DYC_OK;
 }
 
-constexpr uint64_t kStashCap = 1ull << 22;   // stash entries (32 MB): lazy inserts up to this many keys
+constexpr uint64_t kStashMin = 1ull << 20, kStashMax = 1ull << 26;   // stash entries
 
 dyc_status zero_one(dyc_table* t, int idx, cudaStream_t st) {
     CU(cudaMemsetAsync(t->d_ctr + idx, 0, sizeof(unsigned long long), st));
@@ -755,7 +755,9 @@ dyc_status insert_begin(dyc_table* t, uint64_t n, cudaStream_t st, bool& fuse) {
         TRY(flush_m<B>(t, st));
     if (t->rz.active && (double)(t->m + n) > t->cfg.beta * (double)t->N_after()) TRY(live_commit<B>(t, st));
     TRY(ensure_lists(t, n, st));
-    TRY(ensure_stash(t, kStashCap, st));          // once: a fixed 32 MB
+    // stash capacity: a quarter of the table's slots, 1M..64M pairs (lazy
+    // inserts run until their summed sizes would exceed it)
+    TRY(ensure_stash(t, std::min<uint64_t>(kStashMax, std::max<uint64_t>(kStashMin, t->N() / 4)), st));
     TRY(zero_ctr(t, st));
     TRY(refresh_weights<B>(t, st));
     t->ins_n = n;

@@ -485,19 +485,19 @@ def test_lazy_delete_on_other_stream_then_stats(oracle_mod):
 
 def test_mixed_batch_without_host_waits_and_invalid_codes(oracle_mod):
     """dyc_mixed_batch groups its phases on the device: the phase sizes are read
-    back only when the host's bound (n) cannot rule out a resize decision, so a
-    batch far from both fill bounds waits at most once, and op codes outside
-    0..2 are no-ops (status NONE, value NOT_FOUND; reading Q10).  Results equal
-    the oracle's throughout."""
+    back only when the host's bound (n) cannot rule out a resize decision, so
+    batches far from both fill bounds run without any host wait, and op codes
+    outside 0..2 are no-ops (status NONE, value NOT_FOUND; reading Q10).
+    Results equal the oracle's throughout."""
     meta, batches = W.c4_zipf_mixed(U=200000, distinct=20000, grow_batches=6, cycles=1, init_capacity=1 << 20)
     g = Table(d=4, init_capacity=1 << 20, alpha=0.01, beta=0.85, bucket_slots=8)
     o = oracle_mod.OracleTable(d=4, init_capacity=1 << 20, alpha=0.01, beta=0.85, bucket_slots=8)
-    first = batches[0]
-    g.insert(dev(first.keys), dev(first.values))          # one exact read-back: above alpha from here on
-    o.insert(first.keys, first.values)
+    bg = W.key_range(1 << 30, 200000, 11)                 # background: far above alpha*N from here on
+    g.insert(dev(bg), dev(W.val_of(bg, 0)))
+    o.insert(bg, W.val_of(bg, 0))
     s0 = g.stats()
     rng = np.random.default_rng(3)
-    for i, b in enumerate(batches[1:]):
+    for i, b in enumerate(batches[:8]):
         ops = b.ops.copy()
         ops[rng.choice(ops.size, size=50, replace=False)] = 7          # invalid codes
         v, st = g.mixed(torch.from_numpy(ops).cuda(), dev(b.keys), dev(b.values))
@@ -505,5 +505,5 @@ def test_mixed_batch_without_host_waits_and_invalid_codes(oracle_mod):
         np.testing.assert_array_equal(st.cpu().numpy(), os_, err_msg=f"batch {i} status")
         np.testing.assert_array_equal(host_u32(v), ov, err_msg=f"batch {i} values")
     s1 = g.stats()
-    assert s1["n_sync"] - s0["n_sync"] <= len(batches), s1["n_sync"] - s0["n_sync"]
+    assert s1["n_sync"] - s0["n_sync"] <= 2, s1["n_sync"] - s0["n_sync"]
     np.testing.assert_array_equal(g.sorted_kv(), o.sorted_kv())
