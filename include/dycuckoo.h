@@ -100,9 +100,23 @@ typedef struct {
     uint64_t init_capacity;  /* slots; n0 = max(1, ceil(init_capacity/(d*B))) buckets per subtable (Q13) */
     uint64_t seed;           /* SplitMix64 seed of the hash constants a_s, b_s (Q1)  */
     uint32_t max_hops;       /* L_max: eviction hops per attempt before the failure list (Q6) */
-    uint32_t flags;          /* placement policy: 0 = two-choice first-fit (reading Q3,
-                                default); DYC_PLACE_PAPER_WEIGHTED = the paper's rule     */
+    uint32_t flags;          /* DYC_PLACE_PAPER_WEIGHTED: the paper's placement rule instead
+                                of two-choice first-fit (reading Q3);
+                                DYC_RESIZE_IN_PLACE (set by dyc_config_default): subtables
+                                resize in place in reserved address ranges          */
 } dyc_config;
+
+/* dyc_config.flags: in-place resizing.  Each subtable lives in its own reserved
+ * virtual address range (256 GB of address space) whose physical backing
+ * (cuMemCreate/cuMemMap, 2 MB granules) grows and shrinks with it: an upsize
+ * maps only the new half behind the old buckets and splits bucket b into b and
+ * b + n there; a downsize merges b' and b' + h into b'
+ * and the upper half is unmapped at the next host read-back.  No buffer is
+ * copied or held twice.  Falls back to cudaMalloc buffers when the driver's
+ * virtual-memory API is unavailable; a resize under live traffic
+ * (dyc_resize_begin) or a reinsert baseline (dyc_resize_ex methods 1, 2) moves
+ * that subtable to a cudaMalloc buffer. */
+#define DYC_RESIZE_IN_PLACE 2u
 
 /* dyc_config.flags: the paper's balancing rule (SURVEY §8(f)
  * NEXT-4): a new pair goes to table i of its pair with probability
@@ -139,10 +153,14 @@ typedef struct {
     uint64_t n_sync;                  /* counter read-backs: the host waited on the stream (S6) */
     double   sync_ms;                 /* host milliseconds spent in those waits                */
     uint64_t n_pending;               /* new keys handed to the eviction kernel by all insert batches */
+    uint64_t vm_subtables;            /* subtables resized in place (DYC_RESIZE_IN_PLACE)          */
+    uint64_t vm_mapped_bytes;         /* physical bytes mapped under their address ranges          */
+    uint64_t n_vm_map, n_vm_unmap;    /* physical chunks mapped / unmapped so far                  */
 } dyc_stats_t;
 
 /* Fills *cfg with the defaults: d=4, B=8, alpha=0.3, beta=0.85 (Table
- * `tbl:parameters`), init_capacity=4096, seed=0x5EED0001, max_hops=64. */
+ * `tbl:parameters`), init_capacity=4096, seed=0x5EED0001, max_hops=64,
+ * flags = DYC_RESIZE_IN_PLACE. */
 dyc_status dyc_config_default(dyc_config* cfg);
 
 /* Creates a table on the current CUDA device with the default config except

@@ -19,6 +19,7 @@ DYC_NOT_FOUND = 0xFFFFFFFF
 DYC_OK, DYC_ERR_INVALID_ARG, DYC_ERR_OOM, DYC_ERR_CUDA, DYC_ERR_INSERT_FAILED, DYC_ERR_NO_DEVICE, DYC_ERR_NCCL = range(7)
 DYC_NCCL_UNIQUE_ID_BYTES = 128
 DYC_PLACE_PAPER_WEIGHTED = 1
+DYC_RESIZE_IN_PLACE = 2
 DYC_RESIZE_SPLIT, DYC_RESIZE_REINSERT_SUBTABLE, DYC_RESIZE_REHASH_ALL = range(3)
 DYC_PROF_KINDS = 16
 DYC_GATHER_WRITE, DYC_GATHER_CAS, DYC_GATHER_SECTOR = 1, 2, 4
@@ -43,7 +44,9 @@ class dyc_stats_t(C.Structure):
                 ("last_insert_pending", C.c_uint64), ("last_insert_evictions", C.c_uint64),
                 ("bytes_cached", C.c_uint64), ("n_live_resize", C.c_uint64), ("n_deferred", C.c_uint64),
                 ("n_device_alloc", C.c_uint64), ("alloc_ms", C.c_double),
-                ("n_sync", C.c_uint64), ("sync_ms", C.c_double), ("n_pending", C.c_uint64)]
+                ("n_sync", C.c_uint64), ("sync_ms", C.c_double), ("n_pending", C.c_uint64),
+                ("vm_subtables", C.c_uint64), ("vm_mapped_bytes", C.c_uint64), ("n_vm_map", C.c_uint64),
+                ("n_vm_unmap", C.c_uint64)]
 
 
 class dyw_config(C.Structure):

@@ -18,6 +18,7 @@
 #include <unordered_map>
 #include <vector>
 
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include "dycuckoo.h"
@@ -63,6 +64,45 @@ uint64_t fastmod_magic(uint64_t n) { return n <= 1 ? 0ull : (~0ull / n) + 1ull; 
 
 inline cudaStream_t S(dyc_stream_t s) { return reinterpret_cast<cudaStream_t>(s); }
 
+// ------------------------------------------------------------ virtual memory
+// Subtables can live in a reserved virtual address range whose physical
+// backing grows and shrinks in place (DYC_RESIZE_IN_PLACE): an upsize maps only
+// the new half behind the old buckets and splits there, a
+// downsize merges into the lower half and unmaps the upper one.
+// The driver entry points are fetched through the runtime, so libdyc.so has no
+// link-time libcuda dependency; if any is missing the tables use cudaMalloc.
+struct VmmApi {
+    bool ok = false;
+    CUresult (*reserve)(CUdeviceptr*, size_t, size_t, CUdeviceptr, unsigned long long) = nullptr;
+    CUresult (*addr_free)(CUdeviceptr, size_t) = nullptr;
+    CUresult (*create)(CUmemGenericAllocationHandle*, size_t, const CUmemAllocationProp*, unsigned long long) = nullptr;
+    CUresult (*release)(CUmemGenericAllocationHandle) = nullptr;
+    CUresult (*map)(CUdeviceptr, size_t, size_t, CUmemGenericAllocationHandle, unsigned long long) = nullptr;
+    CUresult (*unmap)(CUdeviceptr, size_t) = nullptr;
+    CUresult (*set_access)(CUdeviceptr, size_t, const CUmemAccessDesc*, size_t) = nullptr;
+    CUresult (*granularity)(size_t*, const CUmemAllocationProp*, CUmemAllocationGranularity_flags) = nullptr;
+};
+
+VmmApi& vmm_api() {
+    static VmmApi v;
+    static bool tried = false;
+    if (tried) return v;
+    tried = true;
+    auto get = [](const char* name, void** fn) {
+        cudaDriverEntryPointQueryResult q;
+        return cudaGetDriverEntryPoint(name, fn, cudaEnableDefault, &q) == cudaSuccess &&
+               q == cudaDriverEntryPointSuccess && *fn;
+    };
+    bool ok = get("cuMemAddressReserve", (void**)&v.reserve) && get("cuMemAddressFree", (void**)&v.addr_free) &&
+              get("cuMemCreate", (void**)&v.create) && get("cuMemRelease", (void**)&v.release) &&
+              get("cuMemMap", (void**)&v.map) && get("cuMemUnmap", (void**)&v.unmap) &&
+              get("cuMemSetAccess", (void**)&v.set_access) &&
+              get("cuMemGetAllocationGranularity", (void**)&v.granularity);
+    cudaGetLastError();
+    v.ok = ok;
+    return v;
+}
+
 }  // namespace
 
 // The placement kernel of the table's mode (first-fit or paper-weighted).
@@ -85,6 +125,18 @@ struct dyc_table {
     std::unordered_map<void*, uint64_t> live;   // pointer -> bytes of live allocations
     unsigned long long* sub[DYC_MAX_D] = {};
     uint64_t nb[DYC_MAX_D] = {};
+    // in-place resizing (DYC_RESIZE_IN_PLACE): subtable t lives in a reserved
+    // virtual range when vm[t].base != 0; chunks are the physical pieces mapped
+    // at its end, in mapping order
+    struct Vm {
+        CUdeviceptr base = 0;
+        size_t reserved = 0, mapped = 0;
+        std::vector<std::pair<CUmemGenericAllocationHandle, size_t>> chunks;
+    } vm[DYC_MAX_D];
+    bool in_place = false;
+    size_t vm_gran = 0;
+    uint32_t vm_shrink_pending = 0;        // subtables halved in place, upper half still mapped
+    uint64_t n_vm_map = 0, n_vm_unmap = 0;
     uint32_t a[DYC_MAX_D + 2] = {}, b[DYC_MAX_D + 2] = {};
     uint64_t m = 0;
     // first-choice-full invariant per subtable (TableView::clean):
@@ -244,6 +296,103 @@ unsigned grid_for(uint64_t work, uint64_t per_block) {
     return (unsigned)g;
 }
 
+// Physical backing of subtable t's virtual range grown to at least `bytes`.
+dyc_status vm_grow(dyc_table* t, uint32_t ti, uint64_t bytes) {
+    VmmApi& A = vmm_api();
+    auto& v = t->vm[ti];
+    while (v.mapped < bytes) {
+        const size_t sz = (bytes - v.mapped + t->vm_gran - 1) / t->vm_gran * t->vm_gran;
+        if (v.mapped + sz > v.reserved) return set_err(DYC_ERR_OOM, "subtable outgrew its reserved address range");
+        CUmemAllocationProp prop{};
+        prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+        prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+        prop.location.id = t->device;
+        CUmemGenericAllocationHandle h;
+        const auto t0 = std::chrono::steady_clock::now();
+        if (A.create(&h, sz, &prop, 0) != CUDA_SUCCESS) return set_err(DYC_ERR_OOM, "cuMemCreate failed");
+        if (A.map(v.base + v.mapped, sz, 0, h, 0) != CUDA_SUCCESS) {
+            A.release(h);
+            return set_err(DYC_ERR_CUDA, "cuMemMap failed");
+        }
+        CUmemAccessDesc acc{};
+        acc.location = prop.location;
+        acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+        if (A.set_access(v.base + v.mapped, sz, &acc, 1) != CUDA_SUCCESS) {
+            A.unmap(v.base + v.mapped, sz);
+            A.release(h);
+            return set_err(DYC_ERR_CUDA, "cuMemSetAccess failed");
+        }
+        t->alloc_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+        v.chunks.push_back({h, sz});
+        v.mapped += sz;
+        t->n_vm_map++;
+    }
+    return DYC_OK;
+}
+
+// Unmaps the chunks of subtable t's range that lie wholly at or beyond `keep`
+// bytes.  The caller guarantees no enqueued work still touches them.
+void vm_shrink(dyc_table* t, uint32_t ti, uint64_t keep) {
+    VmmApi& A = vmm_api();
+    auto& v = t->vm[ti];
+    while (!v.chunks.empty() && v.mapped - v.chunks.back().second >= keep) {
+        const auto c = v.chunks.back();
+        A.unmap(v.base + v.mapped - c.second, c.second);
+        A.release(c.first);
+        v.mapped -= c.second;
+        v.chunks.pop_back();
+        t->n_vm_unmap++;
+    }
+}
+
+// A fresh virtual range for subtable t with `bytes` mapped (false if virtual
+// memory is not available: the caller falls back to cudaMalloc).
+bool vm_create(dyc_table* t, uint32_t ti, uint64_t bytes) {
+    VmmApi& A = vmm_api();
+    if (!t->in_place || !A.ok || t->vm_gran == 0) return false;
+    auto& v = t->vm[ti];
+    const size_t reserve = (size_t)1 << 38;            // 256 GB of address space: any subtable fits
+    if (A.reserve(&v.base, reserve, t->vm_gran, 0, 0) != CUDA_SUCCESS) {
+        v.base = 0;
+        return false;
+    }
+    v.reserved = reserve;
+    v.mapped = 0;
+    if (vm_grow(t, ti, bytes) != DYC_OK) {
+        vm_shrink(t, ti, 0);
+        A.addr_free(v.base, v.reserved);
+        v = dyc_table::Vm();
+        cudaGetLastError();
+        return false;
+    }
+    return true;
+}
+
+// Releases a virtual range (after the work that used it: synchronizes `st`).
+void vm_release_range(dyc_table* t, dyc_table::Vm& v, cudaStream_t st) {
+    if (!v.base) return;
+    cudaStreamSynchronize(st);
+    VmmApi& A = vmm_api();
+    for (auto it = v.chunks.rbegin(); it != v.chunks.rend(); ++it) {
+        v.mapped -= it->second;
+        A.unmap(v.base + v.mapped, it->second);
+        A.release(it->first);
+        t->n_vm_unmap++;
+    }
+    A.addr_free(v.base, v.reserved);
+    v = dyc_table::Vm();
+}
+
+void vm_release(dyc_table* t, uint32_t ti, cudaStream_t st) { vm_release_range(t, t->vm[ti], st); }
+
+// Releases the buffer of subtable ti (virtual range or cached cudaMalloc).
+void dev_free(dyc_table* t, void* p, cudaStream_t st);
+void free_sub(dyc_table* t, uint32_t ti, cudaStream_t st) {
+    if (t->vm[ti].base) vm_release(t, ti, st);
+    else dev_free(t, t->sub[ti], st);
+    t->sub[ti] = nullptr;
+}
+
 void trim_cache(dyc_table* t) {
     for (auto& c : t->cache) {
         cudaFree(c.p);                       // synchronizes the device
@@ -329,6 +478,12 @@ dyc_status read_ctr(dyc_table* t, cudaStream_t st) {
     CU(cudaStreamSynchronize(st));
     t->sync_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     t->n_sync++;
+    // the stream is idle: the upper halves of subtables merged in place can go
+    for (uint32_t i = 0; t->vm_shrink_pending && i < t->cfg.d; i++)
+        if (t->vm_shrink_pending & (1u << i)) {
+            vm_shrink(t, i, t->nb[i] * t->cfg.bucket_slots * 8);
+            t->vm_shrink_pending &= ~(1u << i);
+        }
     // every read-back applies what the batches counted since the last one (the
     // lazy ones included): live-count changes, evictions, pending keys
     const unsigned long long* h = t->h_ctr;
@@ -431,18 +586,31 @@ template <int B>
 dyc_status upsize_table(dyc_table* t, uint32_t ti, cudaStream_t st) {
     const uint64_t n_old = t->nb[ti], n_new = 2 * n_old;
     if (n_new > 0xFFFFFFFFull) return set_err(DYC_ERR_OOM, "subtable would exceed 2^32 buckets");
-    void* p = nullptr;
-    TRY(dev_alloc(t, &p, n_new * B * 8, st));
     const uint64_t slots = n_old * B;
-    {
-        ProfScope ps(t, DYC_PROF_UPSIZE, st);
-        k_upsize<B><<<grid_for(slots, kThreads * kResU), kThreads, 0, st>>>(
-            t->sub[ti], (unsigned long long*)p, (uint32_t)n_old, t->a[ti + 1], t->b[ti + 1], fastmod_magic(n_new),
-            (uint32_t)n_new);
+    if (t->vm[ti].base) {
+        // in place: map the new half behind the old buckets, split there
+        t->vm_shrink_pending &= ~(1u << ti);
+        TRY(vm_grow(t, ti, n_new * B * 8));
+        {
+            ProfScope ps(t, DYC_PROF_UPSIZE, st);
+            k_upsize<B><<<grid_for(slots, kThreads * kResU), kThreads, 0, st>>>(
+                t->sub[ti], t->sub[ti], (uint32_t)n_old, t->a[ti + 1], t->b[ti + 1], fastmod_magic(n_new),
+                (uint32_t)n_new);
+        }
+        CU(cudaGetLastError());
+    } else {
+        void* p = nullptr;
+        TRY(dev_alloc(t, &p, n_new * B * 8, st));
+        {
+            ProfScope ps(t, DYC_PROF_UPSIZE, st);
+            k_upsize<B><<<grid_for(slots, kThreads * kResU), kThreads, 0, st>>>(
+                t->sub[ti], (unsigned long long*)p, (uint32_t)n_old, t->a[ti + 1], t->b[ti + 1], fastmod_magic(n_new),
+                (uint32_t)n_new);
+        }
+        CU(cudaGetLastError());
+        free_sub(t, ti, st);
+        t->sub[ti] = (unsigned long long*)p;
     }
-    CU(cudaGetLastError());
-    dev_free(t, t->sub[ti], st);
-    t->sub[ti] = (unsigned long long*)p;
     t->nb[ti] = n_new;
     t->clean &= ~(1u << ti);        // split buckets are no longer full
     return DYC_OK;
@@ -539,17 +707,29 @@ template <int B>
 dyc_status downsize_launch(dyc_table* t, uint32_t ti, cudaStream_t st) {
     const uint64_t n_old = t->nb[ti], h = n_old / 2;
     if (n_old < 2 || (n_old & 1)) return set_err(DYC_ERR_INVALID_ARG, "subtable cannot be halved");
-    void* p = nullptr;
-    TRY(dev_alloc(t, &p, h * B * 8, st));
     TRY(zero_one(t, C_RESIDUAL, st));
-    {
-        ProfScope ps(t, DYC_PROF_DOWNSIZE, st);
-        k_downsize<B><<<grid_for(h * B, kThreads * kResUD), kThreads, 0, st>>>(t->sub[ti], (unsigned long long*)p,
-                                                                       (uint32_t)h, t->list[0], t->d_ctr);
+    if (t->vm[ti].base) {
+        // in place: merge into the lower half; the upper half is unmapped at the
+        // next host read-back (nothing enqueued after it touches it)
+        {
+            ProfScope ps(t, DYC_PROF_DOWNSIZE, st);
+            k_downsize<B><<<grid_for(h * B, kThreads * kResUD), kThreads, 0, st>>>(t->sub[ti], t->sub[ti], (uint32_t)h,
+                                                                           t->list[0], t->d_ctr);
+        }
+        CU(cudaGetLastError());
+        t->vm_shrink_pending |= 1u << ti;
+    } else {
+        void* p = nullptr;
+        TRY(dev_alloc(t, &p, h * B * 8, st));
+        {
+            ProfScope ps(t, DYC_PROF_DOWNSIZE, st);
+            k_downsize<B><<<grid_for(h * B, kThreads * kResUD), kThreads, 0, st>>>(t->sub[ti], (unsigned long long*)p,
+                                                                           (uint32_t)h, t->list[0], t->d_ctr);
+        }
+        CU(cudaGetLastError());
+        free_sub(t, ti, st);
+        t->sub[ti] = (unsigned long long*)p;
     }
-    CU(cudaGetLastError());
-    dev_free(t, t->sub[ti], st);
-    t->sub[ti] = (unsigned long long*)p;
     t->nb[ti] = h;
     TRY(refresh_weights<B>(t, st));
     return launch_place<B>(t, 0, t->d_ctr + C_RESIDUAL, 0, true, st);
@@ -617,7 +797,8 @@ dyc_status live_commit(dyc_table* t, cudaStream_t st) {
     if (!r.active) return DYC_OK;
     CU(cudaStreamWaitEvent(st, r.done, 0));
     const uint32_t ti = r.ti;
-    dev_free(t, t->sub[ti], st);
+    t->vm_shrink_pending &= ~(1u << ti);
+    free_sub(t, ti, st);
     t->sub[ti] = r.nbuf;
     t->nb[ti] = r.nnb;
     r.active = false;
@@ -1084,6 +1265,7 @@ template <int B>
 dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaStream_t st) {
     const uint32_t d = t->cfg.d;
     unsigned long long* old[DYC_MAX_D] = {};
+    dyc_table::Vm old_vm[DYC_MAX_D];
     uint64_t old_nb[DYC_MAX_D] = {};
     bool touched[DYC_MAX_D] = {};
     for (uint32_t i = 0; i < d; i++) touched[i] = all || (int)i == ti;
@@ -1096,6 +1278,9 @@ dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaSt
         TRY(dev_alloc(t, &p, nn * B * 8, st));
         CU(cudaMemsetAsync(p, 0xFF, nn * B * 8, st));
         old[i] = t->sub[i];
+        old_vm[i] = t->vm[i];
+        t->vm[i] = dyc_table::Vm();
+        t->vm_shrink_pending &= ~(1u << i);
         old_nb[i] = t->nb[i];
         t->sub[i] = (unsigned long long*)p;
         t->nb[i] = nn;
@@ -1114,7 +1299,10 @@ dyc_status reinsert_resize(dyc_table* t, int direction, int ti, bool all, cudaSt
     TRY(read_ctr(t, st));
     const uint64_t nfail = t->h_ctr[C_FAIL];
     for (uint32_t i = 0; i < d; i++)
-        if (touched[i]) dev_free(t, old[i], st);
+        if (touched[i]) {
+            if (old_vm[i].base) vm_release_range(t, old_vm[i], st);
+            else dev_free(t, old[i], st);
+        }
     if (nfail) TRY(place_and_settle<B>(t, 1, nullptr, nfail, true, st));
     t->clean = 0;
     return DYC_OK;
@@ -1190,6 +1378,12 @@ dyc_status stats_impl(dyc_table* t, dyc_stats_t* out, cudaStream_t st) {
     out->n_sync = t->n_sync;
     out->sync_ms = t->sync_ms;
     out->n_pending = t->n_pending_total;
+    for (uint32_t i = 0; i < t->cfg.d; i++) {
+        if (t->vm[i].base) out->vm_subtables++;
+        out->vm_mapped_bytes += t->vm[i].mapped;
+    }
+    out->n_vm_map = t->n_vm_map;
+    out->n_vm_unmap = t->n_vm_unmap;
     return DYC_OK;
 }
 
@@ -1346,6 +1540,7 @@ dyc_status dyc_config_default(dyc_config* cfg) {
     cfg->init_capacity = 4096;
     cfg->seed = 0x5EED0001ull;
     cfg->max_hops = 64;
+    cfg->flags = DYC_RESIZE_IN_PLACE;
     return DYC_OK;
 }
 
@@ -1360,8 +1555,8 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
     if (cfg->alpha > cfg->beta * (double)d / (double)(d + 1))
         return set_err(DYC_ERR_INVALID_ARG, "need alpha <= beta*d/(d+1) (P:L315-318)");
     if (cfg->max_hops < 1) return set_err(DYC_ERR_INVALID_ARG, "max_hops must be >= 1");
-    if (cfg->flags & ~(uint32_t)DYC_PLACE_PAPER_WEIGHTED)
-        return set_err(DYC_ERR_INVALID_ARG, "flags: only DYC_PLACE_PAPER_WEIGHTED is defined");
+    if (cfg->flags & ~(uint32_t)(DYC_PLACE_PAPER_WEIGHTED | DYC_RESIZE_IN_PLACE))
+        return set_err(DYC_ERR_INVALID_ARG, "flags: only DYC_PLACE_PAPER_WEIGHTED | DYC_RESIZE_IN_PLACE are defined");
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
         cudaGetLastError();
@@ -1393,9 +1588,21 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
         return set_err(DYC_ERR_INVALID_ARG, "init_capacity too large");
     }
     dyc_status s = DYC_OK;
+    t->in_place = (cfg->flags & DYC_RESIZE_IN_PLACE) != 0 && vmm_api().ok;
+    if (t->in_place) {
+        CUmemAllocationProp prop{};
+        prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+        prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+        prop.location.id = t->device;
+        size_t g = 0;
+        if (vmm_api().granularity(&g, &prop, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED) != CUDA_SUCCESS || g == 0)
+            t->in_place = false;
+        t->vm_gran = g;
+    }
     for (uint32_t i = 0; i < d && s == DYC_OK; i++) {
         void* p = nullptr;
-        s = dev_alloc(t, &p, per * B * 8, nullptr);
+        if (vm_create(t, i, per * B * 8)) p = (void*)t->vm[i].base;
+        else s = dev_alloc(t, &p, per * B * 8, nullptr);
         if (s == DYC_OK) {
             t->sub[i] = (unsigned long long*)p;
             t->nb[i] = per;
@@ -1436,6 +1643,7 @@ dyc_status dyc_destroy(dyc_table* t) {
     if (!t) return DYC_OK;
     cudaSetDevice(t->device);
     cudaDeviceSynchronize();
+    for (uint32_t i = 0; i < DYC_MAX_D; i++) vm_release(t, i, nullptr);
     for (auto& kv : t->live) cudaFree(kv.first);   // subtables, lists, staging, scratch
     t->live.clear();
     trim_cache(t);

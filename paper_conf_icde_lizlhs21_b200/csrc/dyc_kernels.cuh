@@ -774,8 +774,11 @@ constexpr int kResU = DYC_RES_U_UP;      // slots per thread per pass, upsize
 constexpr int kResUD = DYC_RES_U_DOWN;   // new slots per thread per pass, downsize
 
 template <int B>
-__global__ void __launch_bounds__(kThreads, 8) k_upsize(const unsigned long long* __restrict__ old_s,
-                                                     unsigned long long* __restrict__ new_s, uint32_t n_old,
+// In place (DYC_RESIZE_IN_PLACE) old_s == new_s: bucket b is read and written
+// by the same B lanes (the ballots order every read of b before its writes),
+// and b + n_old is fresh memory no lane reads, so no pointer is __restrict__.
+__global__ void __launch_bounds__(kThreads, 8) k_upsize(const unsigned long long* old_s,
+                                                     unsigned long long* new_s, uint32_t n_old,
                                                      uint32_t a, uint32_t b, uint64_t magic2, uint32_t n2) {
     static_assert(B <= 32 && (32 % B) == 0, "bucket must divide a warp");
     __shared__ unsigned long long tile[kThreads / 32][2][32];
@@ -824,8 +827,10 @@ __global__ void __launch_bounds__(kThreads, 8) k_upsize(const unsigned long long
 // (P:L392-393).  Streams: read 16 B, write 8 B per new slot.  Same streaming
 // layout as k_upsize (kResU slots per thread, per-warp tile, coalesced stores).
 template <int B>
-__global__ void __launch_bounds__(kThreads) k_downsize(const unsigned long long* __restrict__ old_s,
-                                                       unsigned long long* __restrict__ new_s, uint32_t h,
+// In place old_s == new_s: new bucket b' is written only by the lanes that read
+// old b' and b'+h (after the ballots on them); the upper half is unmapped later.
+__global__ void __launch_bounds__(kThreads) k_downsize(const unsigned long long* old_s,
+                                                       unsigned long long* new_s, uint32_t h,
                                                        unsigned long long* __restrict__ residual,
                                                        unsigned long long* __restrict__ ctr) {
     static_assert(B <= 32 && (32 % B) == 0, "bucket must divide a warp");
