@@ -102,8 +102,8 @@ typedef struct {
     uint32_t max_hops;       /* L_max: eviction hops per attempt before the failure list (Q6) */
     uint32_t flags;          /* DYC_PLACE_PAPER_WEIGHTED: the paper's placement rule instead
                                 of two-choice first-fit (reading Q3);
-                                DYC_RESIZE_IN_PLACE (set by dyc_config_default): subtables
-                                resize in place in reserved address ranges          */
+                                DYC_RESIZE_IN_PLACE: subtables resize in place in
+                                reserved address ranges (opt-in)                     */
 } dyc_config;
 
 /* dyc_config.flags: in-place resizing.  Each subtable lives in its own reserved
@@ -115,7 +115,9 @@ typedef struct {
  * copied or held twice.  Falls back to cudaMalloc buffers when the driver's
  * virtual-memory API is unavailable; a resize under live traffic
  * (dyc_resize_begin) or a reinsert baseline (dyc_resize_ex methods 1, 2) moves
- * that subtable to a cudaMalloc buffer. */
+ * that subtable to a cudaMalloc buffer.  Opt-in: on the measured B200 driver,
+ * mapping and unmapping physical memory costs ~28 ms per GB, far more than the
+ * cached cudaMalloc buffers of the default path. */
 #define DYC_RESIZE_IN_PLACE 2u
 
 /* dyc_config.flags: the paper's balancing rule (SURVEY §8(f)
@@ -160,7 +162,7 @@ typedef struct {
 
 /* Fills *cfg with the defaults: d=4, B=8, alpha=0.3, beta=0.85 (Table
  * `tbl:parameters`), init_capacity=4096, seed=0x5EED0001, max_hops=64,
- * flags = DYC_RESIZE_IN_PLACE. */
+ * flags = 0 (first-fit placement, cudaMalloc subtables). */
 dyc_status dyc_config_default(dyc_config* cfg);
 
 /* Creates a table on the current CUDA device with the default config except

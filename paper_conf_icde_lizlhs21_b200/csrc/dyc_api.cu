@@ -1540,7 +1540,7 @@ dyc_status dyc_config_default(dyc_config* cfg) {
     cfg->init_capacity = 4096;
     cfg->seed = 0x5EED0001ull;
     cfg->max_hops = 64;
-    cfg->flags = DYC_RESIZE_IN_PLACE;
+    cfg->flags = 0;          // in-place resizing is opt-in (measured slower here: DESIGN.md §5)
     return DYC_OK;
 }
 

@@ -102,7 +102,7 @@ class Table:
 
     def __init__(self, d: int = 4, init_capacity: int = 4096, alpha: float = 0.3, beta: float = 0.85,
                  bucket_slots: int = 8, seed: int = 0x5EED0001, max_hops: int = 64, device=None,
-                 placement: str = "first_fit", in_place: bool = True):
+                 placement: str = "first_fit", in_place: bool = False):
         torch = _torch()
         self._lib = L.load_library()
         if not torch.cuda.is_available():
@@ -117,8 +117,7 @@ class Table:
             raise ValueError("placement must be 'first_fit' (reading Q3) or 'paper_weighted' (P:L361)")
         cfg.flags = (cfg.flags & ~L.DYC_PLACE_PAPER_WEIGHTED) | (
             L.DYC_PLACE_PAPER_WEIGHTED if placement == "paper_weighted" else 0)
-        if not in_place:
-            cfg.flags &= ~L.DYC_RESIZE_IN_PLACE
+        cfg.flags = (cfg.flags & ~L.DYC_RESIZE_IN_PLACE) | (L.DYC_RESIZE_IN_PLACE if in_place else 0)
         self.placement = placement
         self.cfg = cfg
         h = C.c_void_p()
