@@ -89,7 +89,7 @@ def main(tag):
     K = ncu_raw(tag)
     traffic = {}
     md = [f"# Profile summary `{tag}`", "",
-          "Source: `gpurun` pass `scripts/gpu_full.sh " + tag + "` on one B200 (sm_100a).",
+          "Source: `gpurun` pass `scripts/gpu_pass.sh " + tag + " ... launches ncu` on one B200 (sm_100a).",
           "",
           "- `ncu --metrics gpu__time_duration.sum --clock-control none`: the launch list of",
           "  `bench.py --steps 2 --warmup 1 --profile-only`. These launches are cold-cache and serialised, so",
