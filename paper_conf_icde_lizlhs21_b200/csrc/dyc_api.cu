@@ -1055,10 +1055,7 @@ dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t
     constexpr uint64_t per_block = (uint64_t)(kThreads / (B / 4)) * ILP;   // queries per block per pass
     {
         ProfScope ps(t, DYC_PROF_FIND, st);
-        if (t->stash_bound)
-            k_find<B, ILP, true><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
-        else
-            k_find<B, ILP, false><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
+        k_find<B, ILP><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
     }
     CU(cudaGetLastError());
     return DYC_OK;
