@@ -899,8 +899,21 @@ def bench_stream(args, local):
             staged.append((b.op, None, dev(b.keys), dev(b.values) if b.values is not None else None))
     stream = torch.cuda.current_stream()
 
-    def run():
+    n0 = max(1, -(-wl.init_capacity // (args.d * args.bucket_slots)))   # reading Q13
+
+    def reset():
+        """Every pass starts from the config's empty table of init_capacity
+        slots (the previous pass may have left it larger or smaller); the
+        resizes come from the table's buffer cache and run untimed."""
         g.clear()
+        while min(g.shape()["buckets"]) < n0:
+            g.resize(+1)
+        while max(g.shape()["buckets"]) > n0:
+            g.resize(-1)
+        torch.cuda.synchronize()
+
+    def run():
+        reset()
         for op, ops, k, v in staged:
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
@@ -926,7 +939,7 @@ def bench_stream(args, local):
     with ClockSampler(local) as clk:
         a = torch.cuda.Event(enable_timing=True)
         b = torch.cuda.Event(enable_timing=True)
-        g.clear()
+        reset()
         a.record(stream)
         for op, ops, k, v in staged:
             if op == "insert":
@@ -947,7 +960,7 @@ def bench_stream(args, local):
                   "sync_ms": round(st_timed["sync_ms"] - st_before["sync_ms"], 3),
                   "n_device_alloc": st_timed["n_device_alloc"] - st_before["n_device_alloc"],
                   "alloc_ms": round(st_timed["alloc_ms"] - st_before["alloc_ms"], 3)}
-    g.clear()
+    reset()
     g.profile(True)
     g.probe_count(True)
     st_prof0 = g.stats()
@@ -975,7 +988,7 @@ def bench_stream(args, local):
                                l2_resident=(args.config == "c1"))
     # per-op-type times: one more replay with an event pair around every batch
     # (kept out of the timed pass: the events cost host time per batch)
-    g.clear()
+    reset()
     for op, ops, k, v in staged:
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
@@ -996,7 +1009,7 @@ def bench_stream(args, local):
         per[op][0] += cnt
         per[op][1] += e0.elapsed_time(e1)
     # fill-factor track: replay untimed with a stats call after every batch
-    g.clear()
+    reset()
     track, mem = [], []
     peak_st = None
     for op, ops, k, v in staged:

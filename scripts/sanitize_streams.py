@@ -68,6 +68,26 @@ def main():
     run(*mk(max_hops=1), rs.batches, "failure path")
     st = ShardedTable(d=4, init_capacity=1024, local_shards=3, rank=0, world=1)
     run(st, oracle.OracleTable(d=4, init_capacity=1024, alpha=0.3, beta=0.85, bucket_slots=8), c4, "sharded x3")
+    # fused peer-memory routing (dyc_route_push / dyc_route_reply) with 3 virtual
+    # shards on one GPU: insert, find and delete batches against the oracle
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
+    from test_gpu_p2p import SEED, union_kv, virtual_batch
+    shards = [Table(d=4, init_capacity=1024, alpha=0.3, beta=0.85, seed=SEED) for _ in range(3)]
+    o = oracle.OracleTable(d=4, init_capacity=1024, alpha=0.3, beta=0.85, bucket_slots=8, seed=SEED)
+    kk = W.key_range(0, 6000, 17)
+    vv = W.val_of(kk, 0)
+    st = virtual_batch(shards, lambda t, k, v, _: t.insert(k, v), dev(kk), dev(vv), n_out=1)
+    if not (st.cpu().numpy() == o.insert(kk, vv)).all():
+        raise SystemExit("p2p insert differs from the oracle")
+    q = np.concatenate([kk[::2], W.key_range(1 << 31, 500, 17)])
+    v, f = virtual_batch(shards, lambda t, k, v_, _: t.find(k), dev(q))
+    ov, of = o.find(q)
+    if not ((f.cpu().numpy() == of).all() and (hu(v) == ov).all()):
+        raise SystemExit("p2p find differs from the oracle")
+    v, st = virtual_batch(shards, lambda t, k, v_, _: t.delete(k), dev(kk[1::3]))
+    if not (st.cpu().numpy() == o.delete(kk[1::3])[1]).all() or not (union_kv(shards) == o.sorted_kv()).all():
+        raise SystemExit("p2p delete differs from the oracle")
+    print("p2p x3 ok", flush=True)
     # live resize window (NEXT-1): finds and writes against a resize in flight
     g = Table(d=4, init_capacity=1 << 14, alpha=0.05, beta=0.9)
     o = oracle.OracleTable(d=4, init_capacity=1 << 14, alpha=0.05, beta=0.9, bucket_slots=8)
