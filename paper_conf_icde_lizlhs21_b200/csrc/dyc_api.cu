@@ -176,6 +176,15 @@ struct dyc_table {
     unsigned long long* d_ctr = nullptr;   // C_N device counters
     unsigned long long* h_ctr = nullptr;   // pinned mirror
     unsigned long long* h_mix = nullptr;   // pinned: phase sizes of a mixed batch
+    // phase sizes of lazily run mixed batches, copied back asynchronously: once
+    // a copy has landed (event query, no wait) the bounds that batch added to
+    // lazy_add / lazy_del (n each) shrink to its exact sizes, provided no
+    // read-back has happened since (sync_epoch)
+    struct MixRec { int slot; cudaEvent_t ev; uint64_t epoch, n, ins_bound, del_bound; };
+    std::vector<MixRec> mix_recs;
+    unsigned long long* h_mix_ring = nullptr;   // pinned [kMixRing][4]
+    uint32_t mix_ring_next = 0;
+    uint64_t sync_epoch = 0;
     void* stage = nullptr;                 // device staging for the host-buffer entry points
     uint64_t stage_cap = 0;
     cudaStream_t cp_in = nullptr, cp_out = nullptr;   // copy streams of the host-buffer path
@@ -503,6 +512,7 @@ dyc_status read_ctr(dyc_table* t, cudaStream_t st) {
     t->m_lazy = false;
     t->ev_pending = false;
     t->lazy_del = t->lazy_add = 0;
+    t->sync_epoch++;
     return DYC_OK;
 }
 
@@ -523,6 +533,7 @@ dyc_status mark_lazy(dyc_table* t, cudaStream_t st) {
 }
 
 constexpr uint64_t kStashMin = 1ull << 20, kStashMax = 1ull << 26;   // stash entries
+constexpr uint32_t kMixRing = 16;                                     // async phase-size copies in flight
 
 dyc_status zero_one(dyc_table* t, int idx, cudaStream_t st) {
     CU(cudaMemsetAsync(t->d_ctr + idx, 0, sizeof(unsigned long long), st));
@@ -1457,6 +1468,22 @@ dyc_status mixed_impl(dyc_table* t, const uint8_t* d_ops, const uint32_t* d_keys
     // phase sizes: bounded by n on the host.  When that bound cannot rule out a
     // resize decision of either phase, read the exact sizes back once,
     // together with the counters (the read-back a decision needs anyway)
+    // tighten the bounds with the phase sizes of earlier lazy mixed batches
+    // whose asynchronous copies have landed (no wait)
+    while (!t->mix_recs.empty()) {
+        const dyc_table::MixRec r = t->mix_recs.front();
+        const cudaError_t q = cudaEventQuery(r.ev);
+        if (q == cudaErrorNotReady) break;
+        if (q != cudaSuccess) return cuda_err(q, "cudaEventQuery");
+        if (r.epoch == t->sync_epoch) {
+            const unsigned long long* h = t->h_mix_ring + 4 * r.slot;
+            const uint64_t ei = std::min<uint64_t>(h[1], r.ins_bound), ed = std::min<uint64_t>(h[2], r.del_bound);
+            t->lazy_add -= std::min(t->lazy_add, r.ins_bound - ei);
+            t->lazy_del -= std::min(t->lazy_del, r.del_bound - ed);
+        }
+        t->ev_pool.push_back(r.ev);
+        t->mix_recs.erase(t->mix_recs.begin());
+    }
     uint64_t ni = n, nd = n;
     const bool loose_ok = (double)(t->m + t->lazy_add + n) <= t->cfg.beta * (double)t->N() &&
                           t->m >= t->lazy_del + n &&
@@ -1466,6 +1493,14 @@ dyc_status mixed_impl(dyc_table* t, const uint8_t* d_ops, const uint32_t* d_keys
         TRY(sync_state<B>(t, st));
         ni = t->h_mix[1];
         nd = t->h_mix[2];
+    } else if (t->mix_recs.size() < kMixRing) {
+        // copy the sizes back in the background; a later batch tightens the
+        // bounds this one adds once the copy has landed
+        const int slot = (int)(t->mix_ring_next++ % kMixRing);
+        CU(cudaMemcpyAsync(t->h_mix_ring + 4 * slot, cnt, 4 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+        cudaEvent_t ev = t->ev();
+        CU(cudaEventRecord(ev, st));
+        t->mix_recs.push_back({slot, ev, t->sync_epoch, n, n, n});
     }
     // phase 1: finds observe the table before the batch
     TRY(find_impl<B>(t, k, ov, sts, n, st, cnt + 0));
@@ -1617,6 +1652,8 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
     t->clean = (1u << d) - 1u;      // an empty table satisfies the invariant
     if (s == DYC_OK && cudaMallocHost(&t->h_ctr, C_N * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMallocHost");
     if (s == DYC_OK && cudaMallocHost(&t->h_mix, 4 * 8) != cudaSuccess) s = cuda_err(cudaGetLastError(), "cudaMallocHost");
+    if (s == DYC_OK && cudaMallocHost(&t->h_mix_ring, kMixRing * 4 * 8) != cudaSuccess)
+        s = cuda_err(cudaGetLastError(), "cudaMallocHost");
     if (s == DYC_OK && cudaDeviceSynchronize() != cudaSuccess) s = cuda_err(cudaGetLastError(), "create");
     if (s != DYC_OK) {
         dyc_destroy(t);
@@ -1653,6 +1690,8 @@ dyc_status dyc_destroy(dyc_table* t) {
     if (t->lazy_ev) cudaEventDestroy(t->lazy_ev);
     if (t->h_ctr) cudaFreeHost(t->h_ctr);
     if (t->h_mix) cudaFreeHost(t->h_mix);
+    if (t->h_mix_ring) cudaFreeHost(t->h_mix_ring);
+    for (auto& r : t->mix_recs) cudaEventDestroy(r.ev);
     if (t->cp_in) cudaStreamDestroy(t->cp_in);
     if (t->cp_out) cudaStreamDestroy(t->cp_out);
     cudaDeviceSynchronize();
