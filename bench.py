@@ -232,6 +232,17 @@ def run_oracle_sample(log2n: int, kinds=("oracle", "brute_force")):
     return r
 
 
+def c2_config(args):
+    """The headline workload (BASELINE.json configs[1]), named the same way by
+    both arms of the bench."""
+    return {"workload": f"C2 RAND static (BASELINE.json configs[1]): 2^{args.log2n} inserts to fill 0.85, "
+                        f"2^{args.log2n} finds (50% hit), one subtable upsize, 2^{args.log2n - 1} deletes, "
+                        "one subtable downsize",
+            "d": args.d, "alpha": 0.3, "beta": args.beta or 0.85, "bucket_slots": args.bucket_slots,
+            "placement": args.placement,
+            "l2": "inputs and table larger than L2 (126 MB); no flush needed"}
+
+
 def reference_arm(args, rank, world):
     """--impl reference: the CPU oracle is this tier's reference arm."""
     if rank != 0:
@@ -251,8 +262,8 @@ def reference_arm(args, rank, world):
         "impl": "reference", "metric": METRIC, "value": value, "unit": "Mops/s", "n_gpus": world,
         "steps": K, "warmup": Wm, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": f"C2 RAND static (BASELINE configs[1]) shape, bounded sample 2^{log2n} keys",
-                   "d": 4, "alpha": 0.3, "beta": 0.85, "bucket_slots": 8},
+        "config": {**c2_config(args), "sample": f"each step: C2's shape scaled to 2^{log2n} keys (inserts to fill "
+                                                 "0.85, finds at 50% hit, deletes of half), oracle/dyc_oracle.c"},
         "cpu_baseline": {"value": value, "unit": "Mops/s", "cores": 1, "kind": "oracle",
                          "sample": f"C2 shape at 2^{log2n} keys per step (insert+find+delete)"},
         "e2e": {"value": value, "unit": "Mops/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -749,13 +760,7 @@ def main():
         "metric": METRIC, "value": value, "unit": "Mops/s", "n_gpus": 1, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": f"C2 RAND static (BASELINE.json configs[1]): 2^{args.log2n} inserts to fill 0.85, "
-                               f"2^{args.log2n} finds (50% hit), one subtable upsize, 2^{args.log2n - 1} deletes, "
-                               "one subtable downsize",
-                   "d": args.d, "alpha": 0.3, "beta": beta, "bucket_slots": args.bucket_slots,
-                   "placement": args.placement,
-                   "table_bytes": int(s_ins["N"] * 8),
-                   "l2": "inputs and table larger than L2 (126 MB); no flush needed"},
+        "config": {**c2_config(args), "table_bytes": int(s_ins["N"] * 8)},
         "phase_ms": phase_ms,
         "ops": {"insert_mops": n / phase_ms["insert"] / 1e3, "find_mops": n / phase_ms["find"] / 1e3,
                 "delete_mops": (n // 2) / phase_ms["delete"] / 1e3},
