@@ -130,6 +130,23 @@ typedef struct {
  * first-choice-full invariant does not hold under it. */
 #define DYC_PLACE_PAPER_WEIGHTED 1u
 
+/* dyc_config.flags: chunk-staged execution of large batches (DESIGN.md §5,
+ * "Staged batches").  A single insert (needing no upsize), find or delete batch
+ * of B = 8 whose op count is at least the table's bucket count (and >= 2^20) is
+ * ordered on the device by the 64 KB table chunk (1024 buckets) of each op's
+ * first-choice bucket; each chunk is then read once with a
+ * TMA bulk copy, its ops are applied in shared memory and it is written back
+ * once; ops the first-choice bucket cannot decide go through the direct kernels.
+ * Results are those of the direct path (each op's result depends only on the
+ * table before the batch and its own key, P:L464 with distinct keys, Q9); only
+ * where new keys land may differ.  Scratch: ~30 bytes per op, kept by the table
+ * until dyc_trim.  Not used with a resize in flight, the paper-weighted
+ * placement, a possibly non-empty stash, or the parts / mixed / host-buffer
+ * entry points.  DYC_STAGED_OFF disables it; DYC_STAGED_FORCE uses it for every
+ * eligible batch whatever its size (tests); neither = automatic. */
+#define DYC_STAGED_OFF 4u
+#define DYC_STAGED_FORCE 8u
+
 typedef struct {
     uint64_t m;                       /* live keys Σ m_t                          */
     uint64_t N;                       /* slots Σ n_t * B                          */
@@ -158,6 +175,7 @@ typedef struct {
     uint64_t vm_subtables;            /* subtables resized in place (DYC_RESIZE_IN_PLACE)          */
     uint64_t vm_mapped_bytes;         /* physical bytes mapped under their address ranges          */
     uint64_t n_vm_map, n_vm_unmap;    /* physical chunks mapped / unmapped so far                  */
+    uint64_t n_staged;                /* batches run chunk-staged (DYC_STAGED_*)                   */
 } dyc_stats_t;
 
 /* Fills *cfg with the defaults: d=4, B=8, alpha=0.3, beta=0.85 (Table
@@ -336,7 +354,11 @@ uint64_t dyc_launch_count(const dyc_table* t, int reset);
 #define DYC_PROF_KINDS 16
 enum {
     DYC_PROF_FIND = 0, DYC_PROF_UPSERT = 1, DYC_PROF_PLACE = 2, DYC_PROF_DELETE = 3,
-    DYC_PROF_UPSIZE = 4, DYC_PROF_DOWNSIZE = 5, DYC_PROF_REINSERT = 6, DYC_PROF_OTHER = 7
+    DYC_PROF_UPSIZE = 4, DYC_PROF_DOWNSIZE = 5, DYC_PROF_REINSERT = 6, DYC_PROF_OTHER = 7,
+    DYC_PROF_ST_HIST = 8,     /* staged batches: first-choice buckets + chunk histogram, scan      */
+    DYC_PROF_ST_SCATTER = 9,  /* staged batches: the two ordering passes (by bin, by chunk)        */
+    DYC_PROF_ST_APPLY = 10,   /* staged batches: the per-chunk apply kernel                        */
+    DYC_PROF_ST_UNPERM = 11   /* staged batches: need-list compaction, results to request order    */
 };
 dyc_status dyc_profile_enable(dyc_table* t, int enable);
 dyc_status dyc_profile_read(dyc_table* t, double* ms, uint64_t* calls);

@@ -20,10 +20,13 @@ DYC_OK, DYC_ERR_INVALID_ARG, DYC_ERR_OOM, DYC_ERR_CUDA, DYC_ERR_INSERT_FAILED, D
 DYC_NCCL_UNIQUE_ID_BYTES = 128
 DYC_PLACE_PAPER_WEIGHTED = 1
 DYC_RESIZE_IN_PLACE = 2
+DYC_STAGED_OFF = 4
+DYC_STAGED_FORCE = 8
 DYC_RESIZE_SPLIT, DYC_RESIZE_REINSERT_SUBTABLE, DYC_RESIZE_REHASH_ALL = range(3)
 DYC_PROF_KINDS = 16
 DYC_GATHER_WRITE, DYC_GATHER_CAS, DYC_GATHER_SECTOR = 1, 2, 4
-PROF_NAMES = ["k_find", "k_upsert", "k_place", "k_delete", "k_upsize", "k_downsize", "k_reinsert", "other"]
+PROF_NAMES = ["k_find", "k_upsert", "k_place", "k_delete", "k_upsize", "k_downsize", "k_reinsert", "other",
+              "st_hist", "st_scatter", "st_apply", "st_unperm"]
 _STATUS_NAMES = ["DYC_OK", "DYC_ERR_INVALID_ARG", "DYC_ERR_OOM", "DYC_ERR_CUDA",
                  "DYC_ERR_INSERT_FAILED", "DYC_ERR_NO_DEVICE", "DYC_ERR_NCCL"]
 
@@ -46,7 +49,7 @@ class dyc_stats_t(C.Structure):
                 ("n_device_alloc", C.c_uint64), ("alloc_ms", C.c_double),
                 ("n_sync", C.c_uint64), ("sync_ms", C.c_double), ("n_pending", C.c_uint64),
                 ("vm_subtables", C.c_uint64), ("vm_mapped_bytes", C.c_uint64), ("n_vm_map", C.c_uint64),
-                ("n_vm_unmap", C.c_uint64)]
+                ("n_vm_unmap", C.c_uint64), ("n_staged", C.c_uint64)]
 
 
 class dyw_config(C.Structure):

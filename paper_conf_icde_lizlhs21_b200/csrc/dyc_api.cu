@@ -24,6 +24,7 @@
 #include "dycuckoo.h"
 #include "dyc_device.cuh"
 #include "dyc_kernels.cuh"
+#include "dyc_staged.cuh"
 
 using namespace dyc;
 
@@ -215,6 +216,11 @@ struct dyc_table {
     uint64_t n_live_resize = 0, n_deferred = 0;
     uint64_t n_device_alloc = 0;
     double alloc_ms = 0.0;
+    // chunk-staged execution of large batches (dyc_staged.cuh): one scratch
+    // buffer, grown on demand; n_staged counts the batches that took the path
+    void* stg = nullptr;
+    uint64_t stg_cap = 0;
+    uint64_t n_staged = 0;
     uint64_t peak_table_bytes = 0;   // high-water mark of the subtables' bytes (cache cap)
     uint64_t n_sync = 0;          // counter read-backs (host waits on the stream)
     double sync_ms = 0.0;
@@ -959,9 +965,11 @@ dyc_status insert_begin(dyc_table* t, uint64_t n, cudaStream_t st, bool& fuse) {
 
 template <int B>
 dyc_status insert_chunk(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* status, uint64_t n,
-                        bool fuse, cudaStream_t st, const unsigned long long* n_dev = nullptr) {
+                        bool fuse, cudaStream_t st, const unsigned long long* n_dev = nullptr, unsigned max_grid = 0,
+                        bool skip1 = false) {
     constexpr int U = DYC_UPSERT_U;
-    const unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
+    unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
+    if (max_grid) grid = std::min(grid, max_grid);
     {
         ProfScope ps(t, DYC_PROF_UPSERT, st);
         const bool sp = t->stash_bound != 0;
@@ -978,7 +986,10 @@ dyc_status insert_chunk(dyc_table* t, const uint32_t* keys, const uint32_t* vals
             else k_upsert<B, FU, U, LKV, false, false><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, pl, t->d_ctr, lk, DEFER, nd); \
         }                                                                                                     \
     } while (0)
-        if (t->rz.active) DYC_UPSERT_LAUNCH(true, true, t->list[1]);
+        if (skip1)   // staged batches: first-choice bucket known full, key known absent from it
+            k_upsert<B, true, U, false, false, false, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, pl,
+                                                                                     t->d_ctr, 0xFFFFFFFFu, nullptr, nd);
+        else if (t->rz.active) DYC_UPSERT_LAUNCH(true, true, t->list[1]);
         else if (fuse) DYC_UPSERT_LAUNCH(true, false, nullptr);
         else DYC_UPSERT_LAUNCH(false, false, nullptr);
 #undef DYC_UPSERT_LAUNCH
@@ -1050,23 +1061,34 @@ dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
     return enforce_lower<B>(t, st);
 }
 
+template <int B, int OP>
+dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* out_st, uint32_t* out_r,
+                      uint64_t n, cudaStream_t st);
+bool staged_ok(const dyc_table* t, uint64_t n);
+
 template <int B>
 dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* status, uint64_t n,
                        cudaStream_t st) {
     bool fuse = false;
     TRY(insert_begin<B>(t, n, st, fuse));
-    TRY(insert_chunk<B>(t, keys, vals, status, n, fuse, st));
+    // a large batch that needs no upsize runs chunk-staged (dyc_staged.cuh)
+    if (fuse && staged_ok(t, n) && B == 8) TRY((staged_run<B, 0>(t, keys, vals, status, nullptr, n, st)));
+    else TRY(insert_chunk<B>(t, keys, vals, status, n, fuse, st));
     return insert_end<B>(t, fuse, st);
 }
 
 template <int B>
 dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* found, uint64_t n,
-                     cudaStream_t st, const unsigned long long* n_dev = nullptr) {
+                     cudaStream_t st, const unsigned long long* n_dev = nullptr, unsigned max_grid = 0,
+                     bool skip1 = false) {
     constexpr int ILP = (B <= 16) ? DYC_FIND_ILP : 2;
     constexpr uint64_t per_block = (uint64_t)(kThreads / (B / 4)) * ILP;   // queries per block per pass
+    unsigned grid = grid_for(n, per_block);
+    if (max_grid) grid = std::min(grid, max_grid);
     {
         ProfScope ps(t, DYC_PROF_FIND, st);
-        k_find<B, ILP><<<grid_for(n, per_block), kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
+        if (skip1) k_find<B, ILP, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
+        else k_find<B, ILP><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
     }
     CU(cudaGetLastError());
     return DYC_OK;
@@ -1087,13 +1109,18 @@ dyc_status delete_prep(dyc_table* t, uint64_t n, cudaStream_t st) {
 
 template <int B>
 dyc_status delete_chunk(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
-                        cudaStream_t st, const unsigned long long* n_dev = nullptr) {
+                        cudaStream_t st, const unsigned long long* n_dev = nullptr, unsigned max_grid = 0,
+                        bool skip1 = false) {
     {
         ProfScope ps(t, DYC_PROF_DELETE, st);
         constexpr int U = DYC_DELETE_U;
-        const unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
+        unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
+        if (max_grid) grid = std::min(grid, max_grid);
         const bool sp = t->stash_bound != 0;
-        if (t->rz.active) {
+        if (skip1) {
+            k_delete<B, U, false, false, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr,
+                                                                         0xFFFFFFFFu, nullptr, n_dev);
+        } else if (t->rz.active) {
             if (sp) k_delete<B, U, true, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, t->rz.ti, t->list[0], n_dev);
             else k_delete<B, U, true, false><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, t->rz.ti, t->list[0], n_dev);
         } else {
@@ -1134,8 +1161,174 @@ template <int B>
 dyc_status delete_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
                        cudaStream_t st) {
     TRY(delete_prep<B>(t, n, st));
-    TRY(delete_chunk<B>(t, keys, vals, status, n, st));
+    if (staged_ok(t, n) && B == 8) TRY((staged_run<B, 2>(t, keys, nullptr, status, vals, n, st)));
+    else TRY(delete_chunk<B>(t, keys, vals, status, n, st));
     return delete_end<B>(t, st);
+}
+
+template <int B>
+dyc_status find_top(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* found, uint64_t n, cudaStream_t st) {
+    if (staged_ok(t, n) && B == 8) return staged_run<B, 1>(t, keys, nullptr, found, vals, n, st);
+    return find_impl<B>(t, keys, vals, found, n, st);
+}
+
+// ------------------------------------------------------------------ staged path
+// Chunk-staged execution of a large batch (dyc_staged.cuh): used
+// for B = 8 when the batch has at least as many ops as the table has buckets
+// (auto), or always (DYC_STAGED_FORCE) / never (DYC_STAGED_OFF); never with a
+// resize in flight, the paper-weighted placement, or a possibly non-empty
+// stash (those keep the direct kernels).
+constexpr uint64_t kStagedMinOps = 1ull << 20;
+
+StagedView staged_view(const dyc_table* t) {
+    StagedView s{};
+    uint32_t c = 0;
+    for (uint32_t i = 0; i < t->cfg.d; i++) {
+        s.cbase[i] = c;
+        c += (uint32_t)((t->nb[i] + kStChunk - 1) / kStChunk);
+    }
+    s.cbase[t->cfg.d] = c;
+    s.nc = c;
+    uint32_t s1 = 0;
+    while (((uint64_t)c + (1ull << s1) - 1) >> s1 > (uint64_t)kStBins1) s1++;
+    s.s1 = s1;
+    s.nbins = (uint32_t)(((uint64_t)c + (1ull << s1) - 1) >> s1);
+    return s;
+}
+
+bool staged_ok(const dyc_table* t, uint64_t n) {
+    if (t->cfg.bucket_slots != 8 || t->weighted || t->rz.active || t->stash_bound || n == 0 || n >= (1ull << 31))
+        return false;
+    if (t->cfg.flags & DYC_STAGED_OFF) return false;
+    const StagedView s = staged_view(t);
+    if (s.s1 > (uint32_t)kStMaxS1 || s.nc > kStMaxChunks) return false;
+    if (t->cfg.flags & DYC_STAGED_FORCE) return true;
+    uint64_t buckets = 0;
+    for (uint32_t i = 0; i < t->cfg.d; i++) buckets += t->nb[i];
+    return n >= kStagedMinOps && n >= buckets;
+}
+
+// Scratch of one staged batch of n ops over nc chunks (u32 arrays of n unless noted):
+//   g (first-choice buckets; later the need list), k1 v1 g1 (level-1 order),
+//   k2 v2 (level-2 = chunk order), lb2 spos1 spos2 [u16 x n], st1 st2 [u8 x n],
+//   run1 / roff1 [tiles1 x 256 u32 / 257 u16], run2 / roff2 [tiles2 x ...],
+//   chunk_cnt chunk_off cur2 [nc + 1], bin_off cur1 tile_first [kStBins1 + 1],
+//   need_cnt [u64].  The need list's keys / values / results reuse k1 / v1
+//   (free after the level-2 scatter), its statuses st1.
+struct StagedBufs {
+    uint32_t *g, *k1, *v1, *g1, *k2, *v2, *run1, *run2;
+    uint16_t *lb2, *spos1, *spos2, *roff1, *roff2;
+    uint8_t *st1, *st2;
+    uint32_t *chunk_cnt, *chunk_off, *cur2, *bin_off, *cur1, *tile_first;
+    unsigned long long* need_cnt;
+};
+
+dyc_status staged_bufs(dyc_table* t, uint64_t n, uint32_t nc, uint64_t tiles1, uint64_t tiles2, cudaStream_t st,
+                       StagedBufs& b) {
+    auto al = [](uint64_t x) { return (x + 255) & ~255ull; };
+    const uint64_t a4 = al(4 * n), a2 = al(2 * n), a1 = al(n);
+    const uint64_t r1 = al(4ull * kStRun * tiles1), o1 = al(2ull * kStRoff * tiles1);
+    const uint64_t r2 = al(4ull * kStRun * tiles2), o2 = al(2ull * kStRoff * tiles2);
+    const uint64_t sc = al(4ull * (nc + 1)), sb = al(4ull * (kStBins1 + 1));
+    const uint64_t bytes = 6 * a4 + 3 * a2 + 2 * a1 + r1 + o1 + r2 + o2 + 3 * sc + 3 * sb + 256;
+    if (bytes > t->stg_cap) {
+        dev_free(t, t->stg, st);
+        t->stg = nullptr;
+        t->stg_cap = 0;
+        const uint64_t cap = bytes + bytes / 4;
+        TRY(dev_alloc(t, &t->stg, cap, st));
+        t->stg_cap = cap;
+    }
+    char* p = (char*)t->stg;
+    auto take = [&](uint64_t sz) { char* q = p; p += sz; return q; };
+    b.g = (uint32_t*)take(a4); b.k1 = (uint32_t*)take(a4); b.v1 = (uint32_t*)take(a4); b.g1 = (uint32_t*)take(a4);
+    b.k2 = (uint32_t*)take(a4); b.v2 = (uint32_t*)take(a4);
+    b.lb2 = (uint16_t*)take(a2); b.spos1 = (uint16_t*)take(a2); b.spos2 = (uint16_t*)take(a2);
+    b.st1 = (uint8_t*)take(a1); b.st2 = (uint8_t*)take(a1);
+    b.run1 = (uint32_t*)take(r1); b.roff1 = (uint16_t*)take(o1); b.run2 = (uint32_t*)take(r2); b.roff2 = (uint16_t*)take(o2);
+    b.chunk_cnt = (uint32_t*)take(sc); b.chunk_off = (uint32_t*)take(sc); b.cur2 = (uint32_t*)take(sc);
+    b.bin_off = (uint32_t*)take(sb); b.cur1 = (uint32_t*)take(sb); b.tile_first = (uint32_t*)take(sb);
+    b.need_cnt = (unsigned long long*)take(256);
+    return DYC_OK;
+}
+
+// OP 0 insert (keys, vals -> out_st), 1 find (keys -> out_r values, out_st found),
+// 2 delete (keys -> out_r old values, out_st status).  Outputs are nullable.
+template <int B, int OP>
+dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* out_st, uint32_t* out_r,
+                      uint64_t n, cudaStream_t st) {
+    constexpr bool VALS = OP == 0;
+    const StagedView sv = staged_view(t);
+    const uint64_t tiles1 = (n + kStTile - 1) / kStTile;
+    const uint64_t tiles2 = tiles1 + sv.nbins;
+    StagedBufs b{};
+    TRY(staged_bufs(t, n, sv.nc, tiles1, tiles2, st, b));
+    const uint32_t sm_scatter = (VALS ? 3 : 2) * kStTile * 4 + kStTile;
+    static bool attr_set = false;
+    if (!attr_set) {
+        CU(cudaFuncSetAttribute(k_st_apply<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kStSlots * 8));
+        CU(cudaFuncSetAttribute(k_st_apply<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, kStSlots * 8));
+        CU(cudaFuncSetAttribute(k_st_apply<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, kStSlots * 8));
+        CU(cudaFuncSetAttribute(k_st_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, kStMaxChunks * 4));
+        CU(cudaFuncSetAttribute(k_st_scatter<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 3 * kStTile * 4 + kStTile));
+        CU(cudaFuncSetAttribute(k_st_scatter<2, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 3 * kStTile * 4 + kStTile));
+        attr_set = true;
+    }
+    t->n_staged++;
+    const TableView tv = t->view();
+    const unsigned gstream = (unsigned)std::min<uint64_t>(grid_for(n, kThreads), (uint64_t)t->num_sms * 8);
+    {
+        ProfScope ps(t, DYC_PROF_ST_HIST, st);
+        CU(cudaMemsetAsync(b.chunk_cnt, 0, 4ull * (sv.nc + 1), st));
+        CU(cudaMemsetAsync(b.need_cnt, 0, 8, st));
+        const unsigned per_sm = sv.nc * 4 <= 100u * 1024 ? 2u : 1u;    // two CTAs per SM when both counter sets fit
+        k_st_hist<<<t->num_sms * per_sm, kStHistT, sv.nc * 4, st>>>(tv, sv, keys, n, b.g, b.chunk_cnt);
+        k_st_scan<<<1, 1024, 0, st>>>(sv, b.chunk_cnt, b.chunk_off, b.cur2, b.bin_off, b.cur1, b.tile_first);
+    }
+    {
+        ProfScope ps(t, DYC_PROF_ST_SCATTER, st);
+        k_st_scatter<1, VALS><<<(unsigned)tiles1, kStT, sm_scatter, st>>>(sv, keys, vals, b.g, n, b.bin_off, b.tile_first,
+                                                                         b.cur1, b.k1, b.v1, b.g1, nullptr, b.spos1,
+                                                                         b.run1, b.roff1);
+        k_st_scatter<2, VALS><<<(unsigned)tiles2, kStT, sm_scatter, st>>>(sv, b.k1, b.v1, b.g1, n, b.bin_off, b.tile_first,
+                                                                         b.cur2, b.k2, b.v2, nullptr, b.lb2, b.spos2,
+                                                                         b.run2, b.roff2);
+    }
+    CU(cudaGetLastError());
+    // r2 (sorted 32-bit results of find / delete) lives in v2, which those ops do not carry;
+    // the need list reuses g (free after the level-1 scatter)
+    uint32_t* r2 = OP == 0 ? nullptr : b.v2;
+    uint32_t* need = b.g;
+    {
+        ProfScope ps(t, DYC_PROF_ST_APPLY, st);
+        k_st_apply<OP><<<sv.nc, kThreads, kStSlots * 8, st>>>(tv, sv, b.k2, b.v2, b.lb2, b.chunk_off, b.st2, r2, need,
+                                                             b.need_cnt, t->d_ctr);
+    }
+    CU(cudaGetLastError());
+    // the ops their first-choice bucket could not decide: compacted into k1 / v1,
+    // run through the direct kernel with the first probe skipped, results scattered back
+    const unsigned gneed = (unsigned)t->num_sms * 8;
+    {
+        ProfScope ps(t, DYC_PROF_ST_UNPERM, st);
+        k_st_need_gather<<<gstream, kThreads, 0, st>>>(need, b.need_cnt, b.k2, VALS ? b.v2 : nullptr, b.k1,
+                                                      VALS ? b.v1 : nullptr);
+    }
+    if (OP == 0) TRY(insert_chunk<B>(t, b.k1, b.v1, b.st1, n, true, st, b.need_cnt, gneed, true));
+    else if (OP == 1) TRY(find_impl<B>(t, b.k1, b.v1, b.st1, n, st, b.need_cnt, gneed, true));
+    else TRY(delete_chunk<B>(t, b.k1, b.v1, b.st1, n, st, b.need_cnt, gneed, true));
+    {
+        ProfScope ps(t, DYC_PROF_ST_UNPERM, st);
+        k_st_need_scatter<<<gstream, kThreads, 0, st>>>(need, b.need_cnt, b.st1, OP == 0 ? nullptr : b.v1, b.st2, r2);
+        // back to request order: chunk order -> level-1 order (into st1 / v1) -> caller
+        uint32_t* r1 = OP == 0 ? nullptr : b.v1;
+        k_st_unperm<2><<<(unsigned)tiles2, kStT, 0, st>>>(sv, n, b.bin_off, b.tile_first, b.run2, b.roff2, b.spos2,
+                                                           b.st2, r2, b.st1, r1);
+        if (out_st || out_r)
+            k_st_unperm<1><<<(unsigned)tiles1, kStT, 0, st>>>(sv, n, b.bin_off, b.tile_first, b.run1, b.roff1, b.spos1,
+                                                               b.st1, r1, out_st, out_r);
+    }
+    CU(cudaGetLastError());
+    return DYC_OK;
 }
 
 // ------------------------------------------------------------------ host-buffer path
@@ -1392,6 +1585,7 @@ dyc_status stats_impl(dyc_table* t, dyc_stats_t* out, cudaStream_t st) {
     }
     out->n_vm_map = t->n_vm_map;
     out->n_vm_unmap = t->n_vm_unmap;
+    out->n_staged = t->n_staged;
     return DYC_OK;
 }
 
@@ -1587,8 +1781,11 @@ dyc_status dyc_create_ex(const dyc_config* cfg, dyc_table** out) {
     if (cfg->alpha > cfg->beta * (double)d / (double)(d + 1))
         return set_err(DYC_ERR_INVALID_ARG, "need alpha <= beta*d/(d+1) (P:L315-318)");
     if (cfg->max_hops < 1) return set_err(DYC_ERR_INVALID_ARG, "max_hops must be >= 1");
-    if (cfg->flags & ~(uint32_t)(DYC_PLACE_PAPER_WEIGHTED | DYC_RESIZE_IN_PLACE))
-        return set_err(DYC_ERR_INVALID_ARG, "flags: only DYC_PLACE_PAPER_WEIGHTED | DYC_RESIZE_IN_PLACE are defined");
+    if (cfg->flags & ~(uint32_t)(DYC_PLACE_PAPER_WEIGHTED | DYC_RESIZE_IN_PLACE | DYC_STAGED_OFF | DYC_STAGED_FORCE))
+        return set_err(DYC_ERR_INVALID_ARG, "flags: only DYC_PLACE_PAPER_WEIGHTED | DYC_RESIZE_IN_PLACE | "
+                                            "DYC_STAGED_OFF | DYC_STAGED_FORCE are defined");
+    if ((cfg->flags & DYC_STAGED_OFF) && (cfg->flags & DYC_STAGED_FORCE))
+        return set_err(DYC_ERR_INVALID_ARG, "flags: DYC_STAGED_OFF and DYC_STAGED_FORCE exclude each other");
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
         cudaGetLastError();
@@ -1774,7 +1971,7 @@ dyc_status dyc_find_batch(dyc_table* t, const uint32_t* d_keys, uint32_t* d_valu
     TRY(enter(t, stream));
     if (n == 0) return DYC_OK;
     if (!d_keys || !d_values_out) return set_err(DYC_ERR_INVALID_ARG, "null keys/values_out");
-    DISPATCH_B(t, find_impl<B_>(t, d_keys, d_values_out, d_found, n, S(stream)));
+    DISPATCH_B(t, find_top<B_>(t, d_keys, d_values_out, d_found, n, S(stream)));
 }
 
 dyc_status dyc_delete_batch(dyc_table* t, const uint32_t* d_keys, uint32_t* d_values_out, uint8_t* d_status,
@@ -1850,6 +2047,11 @@ dyc_status dyc_clear(dyc_table* t, dyc_stream_t stream) {
 dyc_status dyc_trim(dyc_table* t) {
     TRY(check_table(t));
     CU(cudaSetDevice(t->device));
+    if (t->stg) {                     // staged-batch scratch (dyc_staged.cuh)
+        dev_free(t, t->stg, t->last);
+        t->stg = nullptr;
+        t->stg_cap = 0;
+    }
     trim_cache(t);
     return DYC_OK;
 }

@@ -173,7 +173,9 @@ __device__ __forceinline__ uint64_t stash_count(const TableView& tv) {
 // host knows the stash is empty): measured 3.87 vs 4.29 ms at C2 against a
 // compile-time variant without it, from instruction scheduling alone
 // (profiles/r2_variants.md).
-template <int B, int ILP>
+// S1 (staged batches, dyc_staged.cuh): every key is known to be absent from its
+// first-choice bucket (the staged pass read it); only the second one is probed.
+template <int B, int ILP, bool S1 = false>
 __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, const uint32_t* __restrict__ keys,
                                                    uint32_t* __restrict__ vals, uint8_t* __restrict__ found,
                                                    uint64_t n, const unsigned long long* __restrict__ n_dev = nullptr) {
@@ -208,7 +210,12 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
             p2[j] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[j]), B) + 4 * g.sub;
 #else
             p2[j] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[j]), B) + 4 * g.sub;
-            probe_nc<B>(bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[j]), B) + 4 * g.sub, s[j]);
+            if (S1) {
+#pragma unroll
+                for (int q = 0; q < 4; q++) s[j][q] = kEmptySlot;
+            } else {
+                probe_nc<B>(bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[j]), B) + 4 * g.sub, s[j]);
+            }
 #if DYC_FIND_ORDER == 1
             asm volatile("" ::: "memory");   // issue this probe before the next query's view reads
 #endif
@@ -223,7 +230,7 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
             const unsigned eb = g.ballot(empty_mask(s[j]) != 0);
             f[j] = hb != 0;
             v[j] = g.bcast32(lv, first_lane(hb));
-            need2[j] = !f[j] && k[j] != kEmptyKey && !(c1[j] && eb != 0);
+            need2[j] = !f[j] && k[j] != kEmptyKey && (S1 || !(c1[j] && eb != 0));
             n_ops += g.sub == 0 && k[j] != kEmptyKey;
             n_p2 += g.sub == 0 && need2[j];
         }
@@ -354,7 +361,10 @@ __device__ __forceinline__ void coop_cas_multi(const Grp<G>& g, unsigned long lo
 // committed); a new key may only take a free slot of its OTHER candidate bucket,
 // else it is pending (placed after the commit).
 // W: the paper-weighted placement mode (compile time); STASH as in k_find.
-template <int B, bool FUSE, int U, bool LK = false, bool W = false, bool STASH = false>
+// S1 as in k_find: the first-choice bucket is known not to hold the key and
+// not to be a placement candidate (staged batches send a key here when its
+// first-choice bucket was full); only the second bucket is probed.
+template <int B, bool FUSE, int U, bool LK = false, bool W = false, bool STASH = false, bool S1 = false>
 __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView tv, const uint32_t* __restrict__ keys,
                                                      const uint32_t* __restrict__ vals,
                                                      uint8_t* __restrict__ status, uint64_t n,
@@ -436,20 +446,25 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                 c1[u] = ((tv.clean >> p.t1) & 1u) && !lk1[u];
                 b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
                 b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
-                probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
+                if (S1) {
+#pragma unroll
+                    for (int q = 0; q < 4; q++) s1[u][q] = kEmptySlot;
+                } else {
+                    probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
+                }
             }
 #pragma unroll
             for (int u = 0; u < U; u++) {
                 const bool active = k[u] != kEmptyKey;
                 j1[u] = match_slot<4>(s1[u], k[u]);
                 const unsigned e = empty_mask(s1[u]);
-                em1[u] = lk1[u] ? 0u : e;
+                em1[u] = (S1 || lk1[u]) ? 0u : e;
                 h1[u] = g.ballot(active && j1[u] >= 0);
                 // first-choice-full invariant: absent from a non-full first-choice
                 // bucket of a clean subtable => absent from the table (no t2 probe)
                 const unsigned eb = g.ballot(e != 0);   // every lane votes (no short circuit)
                 const bool skip = c1[u] && eb != 0;
-                need2[u] = active && h1[u] == 0 && !skip;
+                need2[u] = active && h1[u] == 0 && (S1 || !skip);
                 n_ops += g.sub == 0 && active;
                 n_p2 += g.sub == 0 && need2[u];
             }
@@ -648,7 +663,8 @@ __global__ void __launch_bounds__(kThreads) k_reinsert(TableView tv, const unsig
 // LK: a key found in the `locked` subtable (being resized concurrently) is
 // reported DELETED with its old value, and its removal is appended to `defer`
 // (applied by k_apply after the resize is committed).
-template <int B, int U, bool LK = false, bool STASH = false>
+// S1 as in k_find (staged batches): the key is known absent from its first-choice bucket.
+template <int B, int U, bool LK = false, bool STASH = false, bool S1 = false>
 __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView tv, const uint32_t* __restrict__ keys,
                                                      uint32_t* __restrict__ old_vals,
                                                      uint8_t* __restrict__ status, uint64_t n,
@@ -684,7 +700,12 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
             lk2[u] = LK && p.t2 == locked;
             b1[u] = bucket_ptr(sv, p.t1, bucket_of(sv, p.t1, k[u]), B);
             b2[u] = bucket_ptr(sv, p.t2, bucket_of(sv, p.t2, k[u]), B);
-            probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
+            if (S1) {
+#pragma unroll
+                for (int q = 0; q < 4; q++) s1[u][q] = kEmptySlot;
+            } else {
+                probe_cg<B>(b1[u] + 4 * g.sub, s1[u]);
+            }
         }
 #pragma unroll
         for (int u = 0; u < U; u++) {

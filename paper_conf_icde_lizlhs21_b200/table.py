@@ -102,7 +102,7 @@ class Table:
 
     def __init__(self, d: int = 4, init_capacity: int = 4096, alpha: float = 0.3, beta: float = 0.85,
                  bucket_slots: int = 8, seed: int = 0x5EED0001, max_hops: int = 64, device=None,
-                 placement: str = "first_fit", in_place: bool = False):
+                 placement: str = "first_fit", in_place: bool = False, staged: str = "auto"):
         torch = _torch()
         self._lib = L.load_library()
         if not torch.cuda.is_available():
@@ -118,6 +118,9 @@ class Table:
         cfg.flags = (cfg.flags & ~L.DYC_PLACE_PAPER_WEIGHTED) | (
             L.DYC_PLACE_PAPER_WEIGHTED if placement == "paper_weighted" else 0)
         cfg.flags = (cfg.flags & ~L.DYC_RESIZE_IN_PLACE) | (L.DYC_RESIZE_IN_PLACE if in_place else 0)
+        if staged not in ("auto", "off", "force"):
+            raise ValueError("staged must be 'auto', 'off' or 'force' (DYC_STAGED_*)")
+        cfg.flags |= {"auto": 0, "off": L.DYC_STAGED_OFF, "force": L.DYC_STAGED_FORCE}[staged]
         self.placement = placement
         self.cfg = cfg
         h = C.c_void_p()
@@ -337,7 +340,7 @@ class Table:
                     n_live_resize=s.n_live_resize, n_deferred=s.n_deferred,
                     n_device_alloc=s.n_device_alloc, alloc_ms=s.alloc_ms, n_sync=s.n_sync, sync_ms=s.sync_ms,
                     n_pending=s.n_pending, vm_subtables=s.vm_subtables, vm_mapped_bytes=s.vm_mapped_bytes,
-                    n_vm_map=s.n_vm_map, n_vm_unmap=s.n_vm_unmap)
+                    n_vm_map=s.n_vm_map, n_vm_unmap=s.n_vm_unmap, n_staged=s.n_staged)
 
     def dump(self, stream=None):
         """(kv uint64, table uint32, bucket uint64) host arrays, unspecified order."""
