@@ -77,6 +77,9 @@ def parse():
     ap.add_argument("--batch", type=int, default=None, help="c3: batch size (Table tbl:parameters: 2e5..1e6)")
     ap.add_argument("--shape", default=None, help="c3: TW|RE, c4: LINE|COM")
     ap.add_argument("--wide-modes", default=None, help="--config wide: comma list of voter_W2,grouped_W2,...")
+    ap.add_argument("--staged", default="auto", choices=["auto", "off", "force"],
+                    help="chunk-staged execution of large batches (DYC_STAGED_*; auto = inserts and deletes "
+                         "with at least as many ops as the table has buckets)")
     ap.add_argument("--routed", action="store_true",
                     help="use the sharded router even at N=1 (exercises the N>1 code path)")
     ap.add_argument("--p2p", action="store_true",
@@ -271,7 +274,8 @@ def reference_arm(args, rank, world):
     emit(line)
 
 
-def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi_del, cap, stream, probes=None):
+def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi_del, cap, stream, probes=None,
+                     staged=None, table_bytes=None):
     """Roofline of the dominant kernel.  Algorithmic bytes: every
     probe reads one whole bucket (8*B bytes, the unit the method compares), every
     slot write costs one 32-byte sector, plus the streamed keys/values/status.
@@ -297,23 +301,58 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
         reads_upsert = 1.0 + probes["upsert"][1] / max(1, probes["upsert"][0])
         reads_delete = 1.0 + probes["delete"][1] / max(1, probes["delete"][0])
     slots_sub = (cap // 4 // args.bucket_slots + 1) * args.bucket_slots     # slots of one subtable
+    # Staged phases (dyc_staged.cuh): the chunk passes decide most ops; the probe
+    # kernels then run only on the need list, first probe skipped (S1): their units
+    # are the counted ops and each reads one bucket per counted second probe.
+    staged = staged or {}
+    s1 = {"find": staged.get("find", False), "upsert": staged.get("insert", False),
+          "delete": staged.get("delete", False)}
+    units = {"find": n_find, "upsert": n_ins, "delete": n_del}
+    if probes:
+        units = {k: probes[k][0] for k in units}
+        probes_find = (0.0 if s1["find"] else 1.0) + probes["find"][1] / max(1, probes["find"][0])
+        reads_upsert = (0.0 if s1["upsert"] else 1.0) + probes["upsert"][1] / max(1, probes["upsert"][0])
+        reads_delete = (0.0 if s1["delete"] else 1.0) + probes["delete"][1] / max(1, probes["delete"][0])
+    u_find, u_ins, u_del = units["find"], units["upsert"], units["delete"]
     bytes_alg = {
         # find: first-choice bucket, then the second one unless hit; + key, value, flag
-        "k_find": n_find * (probes_find * bkt + 9),
+        "k_find": u_find * (probes_find * bkt + 9),
         # upsert of new keys: the first-choice bucket, and the second one unless
         # the invariant rules it out (existence check); one sector written for
         # each key placed here; + key, value, status
-        "k_upsert": n_ins * (reads_upsert * bkt + 9) + (n_ins - pend) * sec,
+        "k_upsert": u_ins * (reads_upsert * bkt + 9) + max(0, u_ins - pend) * sec,
         # eviction kernel: per pending key one write; per hop one bucket read + one exchange
         "k_place": pend * sec + ev * (bkt + sec),
         # delete (all hits): 1+φ bucket reads, one sector written; + key, old value, status
-        "k_delete": n_del * (reads_delete * bkt + sec + 9),
+        "k_delete": u_del * (reads_delete * bkt + sec + 9),
         # upsize: stream the subtable in (8 B/slot) and twice its size out (16 B/slot)
         "k_upsize": slots_sub * 24,
         # downsize of the subtable the step doubled: 2*slots_sub slots in (16 B
         # per new slot), slots_sub out (8 B)
         "k_downsize": slots_sub * 24,
     }
+    if any(staged.values()):
+        # streamed bytes per op of the staged passes (DESIGN.md §5 "Staged batches"):
+        # hist: key in, first-choice bucket out (8); scatter: level 1 k,(v),g in and
+        # out + 16-bit sorted index + 32-bit destination (30 / 22), level 2
+        # k,(v),g in, k,(v) + 16-bit bucket + 16-bit index + 32-bit destination
+        # out (28 / 20); apply: k,(v),bucket in, status (+ 32-bit result) out, plus
+        # every touched 64 KB chunk read once (and written back once by insert /
+        # delete); unperm, per level: index and destination in, the result bytes
+        # in and out (8 / 16).
+        T0 = table_bytes or {}
+        per = {"insert": (n_ins, 58.0, 11, 2, 16.0), "find": (n_find, 42.0, 11, 1, 32.0),
+               "delete": (n_del, 42.0, 11, 2, 32.0)}
+        for k in ("st_hist", "st_scatter", "st_apply", "st_unperm"):
+            bytes_alg[k] = 0.0
+        for ph, on in staged.items():
+            if not on:
+                continue
+            nn, sc, ap_, passes, un = per[ph]
+            bytes_alg["st_hist"] += 8.0 * nn
+            bytes_alg["st_scatter"] += sc * nn
+            bytes_alg["st_apply"] += ap_ * nn + passes * T0.get(ph, 0)
+            bytes_alg["st_unperm"] += un * nn
     kern = {k: prof[k][0] / args.steps for k in bytes_alg if prof[k][1]}
     dom = max(kern, key=kern.get)
     calls = prof[dom][1] / args.steps
@@ -360,9 +399,9 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
     M = M_store
     cw_store = max(0.0, 1.0 / M_store - 1.0 / R)
     cw_cas = max(0.0, 1.0 / M_cas - 1.0 / R)
-    placed = (n_ins - pend) / max(1, n_ins)
-    acc_model = {"k_find": (probes_find, 0.0, n_find, 0.0), "k_upsert": (reads_upsert, placed, n_ins, cw_cas),
-                 "k_delete": (reads_delete, 1.0, n_del, cw_store)}
+    placed = max(0, u_ins - pend) / max(1, u_ins)
+    acc_model = {"k_find": (probes_find, 0.0, u_find, 0.0), "k_upsert": (reads_upsert, placed, u_ins, cw_cas),
+                 "k_delete": (reads_delete, 1.0, u_del, cw_store)}
     acc_frac, acc_frac_io = {}, {}
     io_bytes = 9.0            # streamed per op: key 4 in + value 4 in/out + status/flag 1 out
     for k, (r_, w_, units, cw) in acc_model.items():
@@ -376,13 +415,13 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
     # SURVEY §8(d)'s own accounting: one 32-byte sector per probe the kernel
     # issues (counted), one sector per slot written, plus the streamed IO
     survey_bytes = {
-        "k_find": n_find * (probes_find * sec + 9),
-        "k_upsert": n_ins * (reads_upsert * sec + 9) + (n_ins - pend) * sec,
+        "k_find": u_find * (probes_find * sec + 9),
+        "k_upsert": u_ins * (reads_upsert * sec + 9) + max(0, u_ins - pend) * sec,
         "k_place": pend * sec + ev * (sec + sec),
-        "k_delete": n_del * (reads_delete * sec + sec + 9),
+        "k_delete": u_del * (reads_delete * sec + sec + 9),
     }
-    survey = {k: {"bytes_per_op": round(survey_bytes[k] / max(1, {"k_find": n_find, "k_upsert": n_ins,
-                                                                   "k_place": max(1, pend), "k_delete": n_del}[k]), 2),
+    survey = {k: {"bytes_per_op": round(survey_bytes[k] / max(1, {"k_find": u_find, "k_upsert": u_ins,
+                                                                   "k_place": max(1, pend), "k_delete": u_del}[k]), 2),
                   "achieved_gbs": round(survey_bytes[k] / (kern[k] * 1e-3) / 1e9, 1),
                   "frac": round(survey_bytes[k] / (kern[k] * 1e-3) / 1e9 / peak, 4)}
               for k in survey_bytes if k in kern and kern[k] > 0}
@@ -422,6 +461,7 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
         "frac_of_access_ceiling_with_io": acc_frac_io,
         "kernel_ms_per_step": {k: round(v, 4) for k, v in kern.items()},
         "other_kernels_ms_per_step": round(prof["other"][0] / args.steps, 4),
+        "staged_phases": staged,
         "model": {"phi": phi, "hit_rate": hit_rate, "evictions_per_insert": E, "probes_per_find": probes_find,
                   "reads_per_upsert": reads_upsert, "reads_per_delete": reads_delete,
                   "probe_counts": probes, "probe_source": "measured (dyc_probe_count_read, calibration pass)"
@@ -488,7 +528,8 @@ def main():
 
     stream = torch.cuda.current_stream()
     g = Table(d=args.d, init_capacity=cap, placement=args.placement, alpha=0.3 if args.alpha is None else args.alpha,
-              beta=min(0.99, beta + 1e-6) if beta > 0.85 else 0.85, bucket_slots=args.bucket_slots)
+              beta=min(0.99, beta + 1e-6) if beta > 0.85 else 0.85, bucket_slots=args.bucket_slots,
+              staged=args.staged)
     st_ins = torch.empty(n, dtype=torch.uint8, device="cuda")
     v_out = torch.empty(n, dtype=torch.int32, device="cuda")
     f_out = torch.empty(n, dtype=torch.uint8, device="cuda")
@@ -522,17 +563,22 @@ def main():
     # calibration pass (untimed): correctness spot checks + per-phase statistics
     g.clear()
     g.probe_count(True)
+    nst0 = g.stats()["n_staged"]
     g.insert(k_ins, v_ins, st_ins)
     probes = {"upsert": g.probe_count_read()["upsert"]}
     s_ins = g.stats()
+    staged = {"insert": s_ins["n_staged"] > nst0}
     assert s_ins["m"] == n and s_ins["n_upsize"] == 0, s_ins
     g.find(k_find, v_out, f_out)
     probes["find"] = g.probe_count_read()["find"]
+    staged["find"] = g.stats()["n_staged"] > s_ins["n_staged"]
     hit_rate = float(f_out.float().mean().item())
     phi = s_ins["n_second_table"] / max(1, s_ins["m"])
     g.resize(+1)
+    s_up = g.stats()
     g.delete(k_del, dv_out, ds_out)
     probes["delete"] = g.probe_count_read()["delete"]
+    staged["delete"] = g.stats()["n_staged"] > s_up["n_staged"]
     g.probe_count(False)
     assert int(ds_out.sum().item()) == n // 2
     s_del_before = g.stats()
@@ -573,7 +619,9 @@ def main():
 
     # --------------------------------------------------------- roofline
     roofline = compute_roofline(args, prof, n_ins=n, n_find=n, n_del=n // 2, s_ins=s_ins, hit_rate=hit_rate,
-                                phi=phi, phi_del=phi_after_up, cap=cap, stream=stream, probes=probes)
+                                phi=phi, phi_del=phi_after_up, cap=cap, stream=stream, probes=probes,
+                                staged=staged, table_bytes={"insert": s_ins["N"] * 8, "find": s_ins["N"] * 8,
+                                                            "delete": s_up["N"] * 8})
     pend = s_ins["last_insert_pending"]
 
     # --------------------------------------------------------- resize baselines

@@ -131,8 +131,8 @@ typedef struct {
 #define DYC_PLACE_PAPER_WEIGHTED 1u
 
 /* dyc_config.flags: chunk-staged execution of large batches (DESIGN.md §5,
- * "Staged batches").  A single insert (needing no upsize), find or delete batch
- * of B = 8 whose op count is at least the table's bucket count (and >= 2^20) is
+ * "Staged batches").  A single insert (needing no upsize) or delete batch of
+ * B = 8 whose op count is at least the table's bucket count (and >= 2^20) is
  * ordered on the device by the 64 KB table chunk (1024 buckets) of each op's
  * first-choice bucket; each chunk is then read once with a
  * TMA bulk copy, its ops are applied in shared memory and it is written back
@@ -143,7 +143,8 @@ typedef struct {
  * until dyc_trim.  Not used with a resize in flight, the paper-weighted
  * placement, a possibly non-empty stash, or the parts / mixed / host-buffer
  * entry points.  DYC_STAGED_OFF disables it; DYC_STAGED_FORCE uses it for every
- * eligible batch whatever its size (tests); neither = automatic. */
+ * eligible batch whatever its size, finds included (tests; a staged find is
+ * slower than dyc_find_batch's direct kernel at C2); neither = automatic. */
 #define DYC_STAGED_OFF 4u
 #define DYC_STAGED_FORCE 8u
 

@@ -966,7 +966,7 @@ dyc_status insert_begin(dyc_table* t, uint64_t n, cudaStream_t st, bool& fuse) {
 template <int B>
 dyc_status insert_chunk(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* status, uint64_t n,
                         bool fuse, cudaStream_t st, const unsigned long long* n_dev = nullptr, unsigned max_grid = 0,
-                        bool skip1 = false) {
+                        const uint32_t* skip1_idx = nullptr) {
     constexpr int U = DYC_UPSERT_U;
     unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
     if (max_grid) grid = std::min(grid, max_grid);
@@ -986,9 +986,10 @@ dyc_status insert_chunk(dyc_table* t, const uint32_t* keys, const uint32_t* vals
             else k_upsert<B, FU, U, LKV, false, false><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, pl, t->d_ctr, lk, DEFER, nd); \
         }                                                                                                     \
     } while (0)
-        if (skip1)   // staged batches: first-choice bucket known full, key known absent from it
+        if (skip1_idx)   // staged batches: first-choice bucket known full, key known absent from it
             k_upsert<B, true, U, false, false, false, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, pl,
-                                                                                     t->d_ctr, 0xFFFFFFFFu, nullptr, nd);
+                                                                                     t->d_ctr, 0xFFFFFFFFu, nullptr, nd,
+                                                                                     skip1_idx);
         else if (t->rz.active) DYC_UPSERT_LAUNCH(true, true, t->list[1]);
         else if (fuse) DYC_UPSERT_LAUNCH(true, false, nullptr);
         else DYC_UPSERT_LAUNCH(false, false, nullptr);
@@ -1064,7 +1065,7 @@ dyc_status insert_end(dyc_table* t, bool fuse, cudaStream_t st) {
 template <int B, int OP>
 dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* out_st, uint32_t* out_r,
                       uint64_t n, cudaStream_t st);
-bool staged_ok(const dyc_table* t, uint64_t n);
+bool staged_ok(const dyc_table* t, uint64_t n, int op);
 
 template <int B>
 dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals, uint8_t* status, uint64_t n,
@@ -1072,7 +1073,7 @@ dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals,
     bool fuse = false;
     TRY(insert_begin<B>(t, n, st, fuse));
     // a large batch that needs no upsize runs chunk-staged (dyc_staged.cuh)
-    if (fuse && staged_ok(t, n) && B == 8) TRY((staged_run<B, 0>(t, keys, vals, status, nullptr, n, st)));
+    if (fuse && staged_ok(t, n, 0) && B == 8) TRY((staged_run<B, 0>(t, keys, vals, status, nullptr, n, st)));
     else TRY(insert_chunk<B>(t, keys, vals, status, n, fuse, st));
     return insert_end<B>(t, fuse, st);
 }
@@ -1080,14 +1081,14 @@ dyc_status insert_impl(dyc_table* t, const uint32_t* keys, const uint32_t* vals,
 template <int B>
 dyc_status find_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* found, uint64_t n,
                      cudaStream_t st, const unsigned long long* n_dev = nullptr, unsigned max_grid = 0,
-                     bool skip1 = false) {
+                     const uint32_t* skip1_idx = nullptr) {
     constexpr int ILP = (B <= 16) ? DYC_FIND_ILP : 2;
     constexpr uint64_t per_block = (uint64_t)(kThreads / (B / 4)) * ILP;   // queries per block per pass
     unsigned grid = grid_for(n, per_block);
     if (max_grid) grid = std::min(grid, max_grid);
     {
         ProfScope ps(t, DYC_PROF_FIND, st);
-        if (skip1) k_find<B, ILP, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
+        if (skip1_idx) k_find<B, ILP, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev, skip1_idx);
         else k_find<B, ILP><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, found, n, n_dev);
     }
     CU(cudaGetLastError());
@@ -1110,16 +1111,16 @@ dyc_status delete_prep(dyc_table* t, uint64_t n, cudaStream_t st) {
 template <int B>
 dyc_status delete_chunk(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
                         cudaStream_t st, const unsigned long long* n_dev = nullptr, unsigned max_grid = 0,
-                        bool skip1 = false) {
+                        const uint32_t* skip1_idx = nullptr) {
     {
         ProfScope ps(t, DYC_PROF_DELETE, st);
         constexpr int U = DYC_DELETE_U;
         unsigned grid = grid_for(n, (uint64_t)(kThreads / (B / 4)) * U);
         if (max_grid) grid = std::min(grid, max_grid);
         const bool sp = t->stash_bound != 0;
-        if (skip1) {
+        if (skip1_idx) {
             k_delete<B, U, false, false, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr,
-                                                                         0xFFFFFFFFu, nullptr, n_dev);
+                                                                         0xFFFFFFFFu, nullptr, n_dev, skip1_idx);
         } else if (t->rz.active) {
             if (sp) k_delete<B, U, true, true><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, t->rz.ti, t->list[0], n_dev);
             else k_delete<B, U, true, false><<<grid, kThreads, 0, st>>>(t->view(), keys, vals, status, n, t->d_ctr, t->rz.ti, t->list[0], n_dev);
@@ -1161,14 +1162,14 @@ template <int B>
 dyc_status delete_impl(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* status, uint64_t n,
                        cudaStream_t st) {
     TRY(delete_prep<B>(t, n, st));
-    if (staged_ok(t, n) && B == 8) TRY((staged_run<B, 2>(t, keys, nullptr, status, vals, n, st)));
+    if (staged_ok(t, n, 2) && B == 8) TRY((staged_run<B, 2>(t, keys, nullptr, status, vals, n, st)));
     else TRY(delete_chunk<B>(t, keys, vals, status, n, st));
     return delete_end<B>(t, st);
 }
 
 template <int B>
 dyc_status find_top(dyc_table* t, const uint32_t* keys, uint32_t* vals, uint8_t* found, uint64_t n, cudaStream_t st) {
-    if (staged_ok(t, n) && B == 8) return staged_run<B, 1>(t, keys, nullptr, found, vals, n, st);
+    if (staged_ok(t, n, 1) && B == 8) return staged_run<B, 1>(t, keys, nullptr, found, vals, n, st);
     return find_impl<B>(t, keys, vals, found, n, st);
 }
 
@@ -1196,13 +1197,18 @@ StagedView staged_view(const dyc_table* t) {
     return s;
 }
 
-bool staged_ok(const dyc_table* t, uint64_t n) {
+// op: 0 insert, 1 find, 2 delete.  Automatic choice: inserts and deletes only.
+// A staged find decides ~68% of a C2 batch in the chunk pass but must still
+// probe the second bucket of the rest; measured slower than k_find alone
+// (5.4 vs 3.9 ms at C2, profiles/r2_staged.md), so finds stage only when forced.
+bool staged_ok(const dyc_table* t, uint64_t n, int op) {
     if (t->cfg.bucket_slots != 8 || t->weighted || t->rz.active || t->stash_bound || n == 0 || n >= (1ull << 31))
         return false;
     if (t->cfg.flags & DYC_STAGED_OFF) return false;
     const StagedView s = staged_view(t);
     if (s.s1 > (uint32_t)kStMaxS1 || s.nc > kStMaxChunks) return false;
     if (t->cfg.flags & DYC_STAGED_FORCE) return true;
+    if (op == 1) return false;
     uint64_t buckets = 0;
     for (uint32_t i = 0; i < t->cfg.d; i++) buckets += t->nb[i];
     return n >= kStagedMinOps && n >= buckets;
@@ -1216,10 +1222,10 @@ bool staged_ok(const dyc_table* t, uint64_t n) {
 //   need_cnt [u64].  The need list's keys / values / results reuse k1 / v1
 //   (free after the level-2 scatter), its statuses st1.
 struct StagedBufs {
-    uint32_t *g, *k1, *v1, *g1, *k2, *v2, *run1, *run2;
-    uint16_t *lb2, *spos1, *spos2, *roff1, *roff2;
+    uint32_t *g, *k1, *v1, *g1, *k2, *v2, *dmap1, *dmap2;
+    uint16_t *lb2, *spos1, *spos2;
     uint8_t *st1, *st2;
-    uint32_t *chunk_cnt, *chunk_off, *cur2, *bin_off, *cur1, *tile_first;
+    uint32_t *chunk_cnt, *chunk_off, *cur2, *bin_off, *cur1, *tile_first, *tile_bin, *tile_lo, *tile_hi;
     unsigned long long* need_cnt;
 };
 
@@ -1227,10 +1233,10 @@ dyc_status staged_bufs(dyc_table* t, uint64_t n, uint32_t nc, uint64_t tiles1, u
                        StagedBufs& b) {
     auto al = [](uint64_t x) { return (x + 255) & ~255ull; };
     const uint64_t a4 = al(4 * n), a2 = al(2 * n), a1 = al(n);
-    const uint64_t r1 = al(4ull * kStRun * tiles1), o1 = al(2ull * kStRoff * tiles1);
-    const uint64_t r2 = al(4ull * kStRun * tiles2), o2 = al(2ull * kStRoff * tiles2);
+    const uint64_t tt = al(4ull * (tiles2 + 1));
     const uint64_t sc = al(4ull * (nc + 1)), sb = al(4ull * (kStBins1 + 1));
-    const uint64_t bytes = 6 * a4 + 3 * a2 + 2 * a1 + r1 + o1 + r2 + o2 + 3 * sc + 3 * sb + 256;
+    (void)tiles1;
+    const uint64_t bytes = 8 * a4 + 3 * a2 + 2 * a1 + 3 * tt + 3 * sc + 3 * sb + 256;
     if (bytes > t->stg_cap) {
         dev_free(t, t->stg, st);
         t->stg = nullptr;
@@ -1245,7 +1251,8 @@ dyc_status staged_bufs(dyc_table* t, uint64_t n, uint32_t nc, uint64_t tiles1, u
     b.k2 = (uint32_t*)take(a4); b.v2 = (uint32_t*)take(a4);
     b.lb2 = (uint16_t*)take(a2); b.spos1 = (uint16_t*)take(a2); b.spos2 = (uint16_t*)take(a2);
     b.st1 = (uint8_t*)take(a1); b.st2 = (uint8_t*)take(a1);
-    b.run1 = (uint32_t*)take(r1); b.roff1 = (uint16_t*)take(o1); b.run2 = (uint32_t*)take(r2); b.roff2 = (uint16_t*)take(o2);
+    b.dmap1 = (uint32_t*)take(a4); b.dmap2 = (uint32_t*)take(a4);
+    b.tile_bin = (uint32_t*)take(tt); b.tile_lo = (uint32_t*)take(tt); b.tile_hi = (uint32_t*)take(tt);
     b.chunk_cnt = (uint32_t*)take(sc); b.chunk_off = (uint32_t*)take(sc); b.cur2 = (uint32_t*)take(sc);
     b.bin_off = (uint32_t*)take(sb); b.cur1 = (uint32_t*)take(sb); b.tile_first = (uint32_t*)take(sb);
     b.need_cnt = (unsigned long long*)take(256);
@@ -1283,16 +1290,17 @@ dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, 
         CU(cudaMemsetAsync(b.need_cnt, 0, 8, st));
         const unsigned per_sm = sv.nc * 4 <= 100u * 1024 ? 2u : 1u;    // two CTAs per SM when both counter sets fit
         k_st_hist<<<t->num_sms * per_sm, kStHistT, sv.nc * 4, st>>>(tv, sv, keys, n, b.g, b.chunk_cnt);
-        k_st_scan<<<1, 1024, 0, st>>>(sv, b.chunk_cnt, b.chunk_off, b.cur2, b.bin_off, b.cur1, b.tile_first);
+        k_st_scan<<<1, 1024, 0, st>>>(sv, b.chunk_cnt, b.chunk_off, b.cur2, b.bin_off, b.cur1, b.tile_first,
+                                      b.tile_bin, b.tile_lo, b.tile_hi);
     }
     {
         ProfScope ps(t, DYC_PROF_ST_SCATTER, st);
-        k_st_scatter<1, VALS><<<(unsigned)tiles1, kStT, sm_scatter, st>>>(sv, keys, vals, b.g, n, b.bin_off, b.tile_first,
-                                                                         b.cur1, b.k1, b.v1, b.g1, nullptr, b.spos1,
-                                                                         b.run1, b.roff1);
-        k_st_scatter<2, VALS><<<(unsigned)tiles2, kStT, sm_scatter, st>>>(sv, b.k1, b.v1, b.g1, n, b.bin_off, b.tile_first,
-                                                                         b.cur2, b.k2, b.v2, nullptr, b.lb2, b.spos2,
-                                                                         b.run2, b.roff2);
+        k_st_scatter<1, VALS><<<(unsigned)tiles1, kStT, sm_scatter, st>>>(
+            sv, keys, vals, b.g, n, b.tile_first, b.tile_bin, b.tile_lo, b.tile_hi, b.cur1, b.k1, b.v1, b.g1, nullptr,
+            b.spos1, b.dmap1);
+        k_st_scatter<2, VALS><<<(unsigned)tiles2, kStT, sm_scatter, st>>>(
+            sv, b.k1, b.v1, b.g1, n, b.tile_first, b.tile_bin, b.tile_lo, b.tile_hi, b.cur2, b.k2, b.v2, nullptr, b.lb2,
+            b.spos2, b.dmap2);
     }
     CU(cudaGetLastError());
     // r2 (sorted 32-bit results of find / delete) lives in v2, which those ops do not carry;
@@ -1305,27 +1313,22 @@ dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, 
                                                              b.need_cnt, t->d_ctr);
     }
     CU(cudaGetLastError());
-    // the ops their first-choice bucket could not decide: compacted into k1 / v1,
-    // run through the direct kernel with the first probe skipped, results scattered back
+    // the ops their first-choice bucket could not decide (the need list: positions
+    // in the chunk order) run through the direct kernel with the first probe
+    // skipped, reading their keys and writing their results at those positions
     const unsigned gneed = (unsigned)t->num_sms * 8;
+    if (OP == 0) TRY(insert_chunk<B>(t, b.k2, b.v2, b.st2, n, true, st, b.need_cnt, gneed, need));
+    else if (OP == 1) TRY(find_impl<B>(t, b.k2, r2, b.st2, n, st, b.need_cnt, gneed, need));
+    else TRY(delete_chunk<B>(t, b.k2, r2, b.st2, n, st, b.need_cnt, gneed, need));
     {
         ProfScope ps(t, DYC_PROF_ST_UNPERM, st);
-        k_st_need_gather<<<gstream, kThreads, 0, st>>>(need, b.need_cnt, b.k2, VALS ? b.v2 : nullptr, b.k1,
-                                                      VALS ? b.v1 : nullptr);
-    }
-    if (OP == 0) TRY(insert_chunk<B>(t, b.k1, b.v1, b.st1, n, true, st, b.need_cnt, gneed, true));
-    else if (OP == 1) TRY(find_impl<B>(t, b.k1, b.v1, b.st1, n, st, b.need_cnt, gneed, true));
-    else TRY(delete_chunk<B>(t, b.k1, b.v1, b.st1, n, st, b.need_cnt, gneed, true));
-    {
-        ProfScope ps(t, DYC_PROF_ST_UNPERM, st);
-        k_st_need_scatter<<<gstream, kThreads, 0, st>>>(need, b.need_cnt, b.st1, OP == 0 ? nullptr : b.v1, b.st2, r2);
         // back to request order: chunk order -> level-1 order (into st1 / v1) -> caller
         uint32_t* r1 = OP == 0 ? nullptr : b.v1;
-        k_st_unperm<2><<<(unsigned)tiles2, kStT, 0, st>>>(sv, n, b.bin_off, b.tile_first, b.run2, b.roff2, b.spos2,
-                                                           b.st2, r2, b.st1, r1);
+        k_st_unperm<2><<<(unsigned)tiles2, kStT, 0, st>>>(sv, n, b.tile_first, b.tile_bin, b.tile_lo, b.tile_hi,
+                                                           b.dmap2, b.spos2, b.st2, r2, b.st1, r1);
         if (out_st || out_r)
-            k_st_unperm<1><<<(unsigned)tiles1, kStT, 0, st>>>(sv, n, b.bin_off, b.tile_first, b.run1, b.roff1, b.spos1,
-                                                               b.st1, r1, out_st, out_r);
+            k_st_unperm<1><<<(unsigned)tiles1, kStT, 0, st>>>(sv, n, b.tile_first, b.tile_bin, b.tile_lo, b.tile_hi,
+                                                               b.dmap1, b.spos1, b.st1, r1, out_st, out_r);
     }
     CU(cudaGetLastError());
     return DYC_OK;

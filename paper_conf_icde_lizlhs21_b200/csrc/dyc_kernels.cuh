@@ -178,7 +178,9 @@ __device__ __forceinline__ uint64_t stash_count(const TableView& tv) {
 template <int B, int ILP, bool S1 = false>
 __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, const uint32_t* __restrict__ keys,
                                                    uint32_t* __restrict__ vals, uint8_t* __restrict__ found,
-                                                   uint64_t n, const unsigned long long* __restrict__ n_dev = nullptr) {
+                                                   uint64_t n, const unsigned long long* __restrict__ n_dev = nullptr,
+                                                   const uint32_t* __restrict__ idx = nullptr) {
+    // S1: op i is keys[idx[i]], its results go to [idx[i]] (a staged batch's need list)
     constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
@@ -198,7 +200,7 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
             const uint64_t i = base + (uint64_t)j * QPW + grp;
-            k[j] = i < n ? __ldg(keys + i) : kEmptyKey;
+            k[j] = i < n ? __ldg(keys + (S1 ? (uint64_t)__ldg(idx + i) : i)) : kEmptyKey;
         }
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
@@ -249,8 +251,9 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
             }
             const uint64_t i = base + (uint64_t)j * QPW + grp;
             if (g.sub == 0 && i < n) {
-                vals[i] = f[j] ? v[j] : kEmptyKey;
-                if (found) found[i] = f[j] ? 1 : 0;
+                const uint64_t o = S1 ? (uint64_t)__ldg(idx + i) : i;
+                vals[o] = f[j] ? v[j] : kEmptyKey;
+                if (found) found[o] = f[j] ? 1 : 0;
             }
         }
     }
@@ -372,7 +375,9 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                                                      unsigned long long* __restrict__ ctr,
                                                      uint32_t locked = 0xFFFFFFFFu,
                                                      unsigned long long* __restrict__ defer = nullptr,
-                                                     const unsigned long long* __restrict__ n_dev = nullptr) {
+                                                     const unsigned long long* __restrict__ n_dev = nullptr,
+                                                     const uint32_t* __restrict__ idx = nullptr) {
+    // S1: op i is (keys, vals)[idx[i]], its status goes to status[idx[i]] (a staged batch's need list)
     constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
@@ -405,8 +410,9 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
             for (int u = 0; u < U; u++) {
                 i[u] = base + (uint64_t)u * QPW + grp;
                 const bool valid = i[u] < n;
-                k[u] = valid ? __ldg(keys + i[u]) : kEmptyKey;
-                kv[u] = make_kv(k[u], valid ? __ldg(vals + i[u]) : 0u);
+                const uint64_t src = (S1 && valid) ? (uint64_t)__ldg(idx + i[u]) : i[u];
+                k[u] = valid ? __ldg(keys + src) : kEmptyKey;
+                kv[u] = make_kv(k[u], valid ? __ldg(vals + src) : 0u);
                 const Pair p = pair_of(tv, k[u]);
                 lk1[u] = LK && p.t1 == locked;
                 lk2[u] = LK && p.t2 == locked;
@@ -437,8 +443,9 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
             for (int u = 0; u < U; u++) {
                 i[u] = base + (uint64_t)u * QPW + grp;
                 const bool valid = i[u] < n;
-                k[u] = valid ? __ldg(keys + i[u]) : kEmptyKey;
-                kv[u] = make_kv(k[u], valid ? __ldg(vals + i[u]) : 0u);
+                const uint64_t src = (S1 && valid) ? (uint64_t)__ldg(idx + i[u]) : i[u];
+                k[u] = valid ? __ldg(keys + src) : kEmptyKey;
+                kv[u] = make_kv(k[u], valid ? __ldg(vals + src) : 0u);
                 const Pair p = pair_of(tv, k[u]);
                 lk1[u] = LK && p.t1 == locked;
                 lk2[u] = LK && p.t2 == locked;
@@ -518,7 +525,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
 #pragma unroll
         for (int u = 0; u < U; u++) {
             const uint8_t st = k[u] == kEmptyKey ? 0 : ((h1[u] | h2[u]) ? 2 : 1);
-            if (lead && i[u] < n && status) status[i[u]] = st;
+            if (lead && i[u] < n && status) status[S1 ? (uint64_t)__ldg(idx + i[u]) : i[u]] = st;
             warp_append(lead && isnew[u] && !placed[u], kv[u], pending, ctr + C_PENDING);
             n_ins += lead && st == 1;
             n_upd += lead && st == 2;
@@ -671,7 +678,9 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
                                                      unsigned long long* __restrict__ ctr,
                                                      uint32_t locked = 0xFFFFFFFFu,
                                                      unsigned long long* __restrict__ defer = nullptr,
-                                                     const unsigned long long* __restrict__ n_dev = nullptr) {
+                                                     const unsigned long long* __restrict__ n_dev = nullptr,
+                                                     const uint32_t* __restrict__ idx = nullptr) {
+    // S1: op i is keys[idx[i]], its results go to [idx[i]] (a staged batch's need list)
     constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
@@ -694,7 +703,7 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
 #pragma unroll
         for (int u = 0; u < U; u++) {
             i[u] = base + (uint64_t)u * QPW + grp;
-            k[u] = i[u] < n ? __ldg(keys + i[u]) : kEmptyKey;
+            k[u] = i[u] < n ? __ldg(keys + (S1 ? (uint64_t)__ldg(idx + i[u]) : i[u])) : kEmptyKey;
             const Pair p = pair_of(tv, k[u]);
             lk1[u] = LK && p.t1 == locked;
             lk2[u] = LK && p.t2 == locked;
@@ -744,8 +753,9 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
                 }
             }
             if (g.sub == 0 && i[u] < n) {
-                if (old_vals) old_vals[i[u]] = ov;
-                if (status) status[i[u]] = hit ? 1 : 0;
+                const uint64_t o = S1 ? (uint64_t)__ldg(idx + i[u]) : i[u];
+                if (old_vals) old_vals[o] = ov;
+                if (status) status[o] = hit ? 1 : 0;
             }
             removed += (g.sub == 0 && hit);
         }

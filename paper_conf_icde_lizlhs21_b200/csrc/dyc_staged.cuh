@@ -56,8 +56,7 @@ constexpr int kStHistT = 1024;
 constexpr int kStHistPer = 8;
 constexpr int kStApplyU = 4;                      // ops per lane in flight (apply)
 constexpr int kStNeedBuf = 64;                    // per-warp need-list buffer (apply)
-constexpr int kStRun = 256;                       // run-table stride (bins or chunks per tile)
-constexpr int kStRoff = 257;                      // offset-table stride
+constexpr int kStRun = 256;                       // bins (level 1) or chunks of a bin (level 2), at most
 
 struct StagedView {
     uint32_t cbase[kMaxD + 1];   // first chunk of subtable t (prefix of ceil(n_t / kStChunk))
@@ -161,7 +160,8 @@ __global__ void __launch_bounds__(kStHistT) k_st_hist(TableView tv, StagedView s
 __global__ void __launch_bounds__(1024) k_st_scan(StagedView s, const uint32_t* __restrict__ chunk_cnt,
                                                   uint32_t* __restrict__ chunk_off, uint32_t* __restrict__ cur2,
                                                   uint32_t* __restrict__ bin_off, uint32_t* __restrict__ cur1,
-                                                  uint32_t* __restrict__ tile_first) {
+                                                  uint32_t* __restrict__ tile_first, uint32_t* __restrict__ tile_bin,
+                                                  uint32_t* __restrict__ tile_lo, uint32_t* __restrict__ tile_hi) {
     __shared__ uint32_t part[1024];
     const uint32_t per = (s.nc + 1023) / 1024;
     const uint32_t a = min(s.nc, threadIdx.x * per), z = min(s.nc, a + per);
@@ -195,20 +195,27 @@ __global__ void __launch_bounds__(1024) k_st_scan(StagedView s, const uint32_t* 
         bin_off[s.nbins] = chunk_off[s.nc];
         tile_first[s.nbins] = tf;
     }
+    __syncthreads();
+    // the level-2 tiling written out once: tile T of bin b covers
+    // [bin_off[b] + j*kStTile, min(bin_off[b+1], ... + kStTile)), j = T - tile_first[b]
+    for (uint32_t b = threadIdx.x; b < s.nbins; b += 1024) {
+        const uint32_t lo = bin_off[b], hi = bin_off[b + 1];
+        for (uint32_t T = tile_first[b], j = 0; T < tile_first[b + 1]; T++, j++) {
+            tile_bin[T] = b;
+            tile_lo[T] = lo + j * kStTile;
+            tile_hi[T] = min(hi, lo + (j + 1) * kStTile);
+        }
+    }
 }
 
-// Tile T of the level-1 order: the bin whose tile range holds T, and the op range.
-__device__ __forceinline__ bool st_tile2(const StagedView& s, const uint32_t* bin_off, const uint32_t* tile_first,
-                                         uint32_t T, uint32_t& b, uint32_t& lo, uint32_t& hi) {
+// Tile T of the level-1 order (level-2 tiling): its bin and op range (k_st_scan's tables).
+__device__ __forceinline__ bool st_tile2(const StagedView& s, const uint32_t* tile_first, const uint32_t* tile_bin,
+                                         const uint32_t* tile_lo, const uint32_t* tile_hi, uint32_t T, uint32_t& b,
+                                         uint32_t& lo, uint32_t& hi) {
     if (T >= tile_first[s.nbins]) return false;
-    uint32_t a = 0, z = s.nbins;            // largest b with tile_first[b] <= T
-    while (z - a > 1) {
-        const uint32_t m = (a + z) >> 1;
-        if (tile_first[m] <= T) a = m; else z = m;
-    }
-    b = a;
-    lo = bin_off[b] + (T - tile_first[b]) * kStTile;
-    hi = min(bin_off[b + 1], lo + kStTile);
+    b = tile_bin[T];
+    lo = tile_lo[T];
+    hi = tile_hi[T];
     return true;
 }
 
@@ -217,18 +224,19 @@ __device__ __forceinline__ bool st_tile2(const StagedView& s, const uint32_t* bi
 // shared atomics), one global cursor reservation per (tile, bin), coalesced runs
 // out.  LEVEL 1: bins = level-1 bins over the request order; LEVEL 2: the
 // chunks of one level-1 bin over that bin's ops.  spos[op] = the op's index in
-// the tile's sorted order; run[T][b] / roff[T][b] = the bin's global start and
-// its offset in the sorted tile (what k_st_unperm reads back).
+// the tile's sorted order; dmap[tile start + p] = the global position the
+// tile's p-th sorted op went to (what k_st_unperm reads the results back from).
 // Level 2 writes the chunk-local bucket (gb & 1023) as 16 bits instead of gb.
 template <int LEVEL, bool VALS>
-__global__ void __launch_bounds__(kStT) k_st_scatter(StagedView s, const uint32_t* __restrict__ kin,
+__global__ void __launch_bounds__(kStT, 3) k_st_scatter(StagedView s, const uint32_t* __restrict__ kin,
                                                      const uint32_t* __restrict__ vin, const uint32_t* __restrict__ gin,
-                                                     uint64_t n, const uint32_t* __restrict__ bin_off,
-                                                     const uint32_t* __restrict__ tile_first, uint32_t* __restrict__ cur,
+                                                     uint64_t n, const uint32_t* __restrict__ tile_first,
+                                                     const uint32_t* __restrict__ tile_bin,
+                                                     const uint32_t* __restrict__ tile_lo,
+                                                     const uint32_t* __restrict__ tile_hi, uint32_t* __restrict__ cur,
                                                      uint32_t* __restrict__ kout, uint32_t* __restrict__ vout,
                                                      uint32_t* __restrict__ gout, uint16_t* __restrict__ lbout,
-                                                     uint16_t* __restrict__ spos, uint32_t* __restrict__ run,
-                                                     uint16_t* __restrict__ roff) {
+                                                     uint16_t* __restrict__ spos, uint32_t* __restrict__ dmap) {
     extern __shared__ __align__(16) uint32_t sm[];
     uint32_t* sk = sm;                              // [kStTile]
     uint32_t* sg = sm + kStTile;                    // [kStTile]
@@ -244,7 +252,7 @@ __global__ void __launch_bounds__(kStT) k_st_scatter(StagedView s, const uint32_
     } else {
         if (threadIdx.x == 0) {
             uint32_t b = 0, lo = 0, hi = 0;
-            sok = st_tile2(s, bin_off, tile_first, blockIdx.x, b, lo, hi);
+            sok = st_tile2(s, tile_first, tile_bin, tile_lo, tile_hi, blockIdx.x, b, lo, hi);
             sb = b; slo = lo; shi = hi;
         }
         __syncthreads();
@@ -256,7 +264,9 @@ __global__ void __launch_bounds__(kStT) k_st_scatter(StagedView s, const uint32_
     }
     if (threadIdx.x < kStRun) cnt[threadIdx.x] = 0;
     __syncthreads();
-    uint32_t kk[kStPer], vv[kStPer], gg[kStPer], bb[kStPer], rk[kStPer];
+    // (the bin is recomputed from gg where needed: fewer live registers, three CTAs per SM)
+    uint32_t kk[kStPer], vv[kStPer], gg[kStPer], rk[kStPer];
+    auto bin_of = [&](uint32_t g) { return LEVEL == 1 ? g >> (kStLog + s.s1) : (g >> kStLog) - c0; };
 #pragma unroll
     for (int j = 0; j < kStPer; j++) {
         const uint32_t li = j * kStT + threadIdx.x;
@@ -268,8 +278,7 @@ __global__ void __launch_bounds__(kStT) k_st_scatter(StagedView s, const uint32_
 #pragma unroll
     for (int j = 0; j < kStPer; j++) {
         const uint32_t li = j * kStT + threadIdx.x;
-        bb[j] = LEVEL == 1 ? gg[j] >> (kStLog + s.s1) : (gg[j] >> kStLog) - c0;
-        rk[j] = li < tn ? atomicAdd(&cnt[bb[j]], 1u) : 0u;
+        rk[j] = li < tn ? atomicAdd(&cnt[bin_of(gg[j])], 1u) : 0u;
     }
     __syncthreads();
     const uint32_t c = threadIdx.x < nb ? cnt[threadIdx.x] : 0u;
@@ -278,27 +287,27 @@ __global__ void __launch_bounds__(kStT) k_st_scatter(StagedView s, const uint32_
         const uint32_t g = c ? atomicAdd(cur + c0 + threadIdx.x, c) : 0u;
         off[threadIdx.x] = ex;
         gbase[threadIdx.x] = g;
-        run[(uint64_t)blockIdx.x * kStRun + threadIdx.x] = g;
-        roff[(uint64_t)blockIdx.x * kStRoff + threadIdx.x] = (uint16_t)ex;
     }
-    if (threadIdx.x == 0) roff[(uint64_t)blockIdx.x * kStRoff + nb] = (uint16_t)tn;
     __syncthreads();
 #pragma unroll
     for (int j = 0; j < kStPer; j++) {
         const uint32_t li = j * kStT + threadIdx.x;
         if (li < tn) {
-            const uint32_t p = off[bb[j]] + rk[j];
+            const uint32_t b = bin_of(gg[j]);
+            const uint32_t p = off[b] + rk[j];
             sk[p] = kk[j];
             sg[p] = gg[j];
             if (VALS) svl[p] = vv[j];
-            sbin[p] = (uint8_t)bb[j];
+            sbin[p] = (uint8_t)b;
             spos[t0 + li] = (uint16_t)p;
         }
     }
     __syncthreads();
+#pragma unroll 4
     for (uint32_t p = threadIdx.x; p < tn; p += kStT) {
         const uint32_t b = sbin[p];
         const uint32_t d = gbase[b] + (p - off[b]);
+        dmap[t0 + p] = d;
         kout[d] = sk[p];
         if (VALS) vout[d] = svl[p];
         if (LEVEL == 1) gout[d] = sg[p];
@@ -396,16 +405,23 @@ __global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView 
             int hit = -1;
             uint32_t hv = 0;
             unsigned emask = 0;
-            // A 64-byte bucket spans 16 banks starting at bank 0 or 16, so 32
-            // lanes reading slot j of random buckets would meet in 2 bank pairs;
-            // each lane starts at its own rotation instead (16 pairs in use).
-            const uint32_t rot = lb >> 1;
+            // The bucket is read as four 16-byte quads.  A 64-byte bucket starts
+            // at quad group 0 or 4 of the 8 in a 128-byte bank row, so lanes
+            // reading quad q of random buckets would meet in 2 groups; each lane
+            // starts at its own rotation instead (all 8 groups in use).
+            const uint32_t rot = (lb >> 1) & 3u;
 #pragma unroll
-            for (int j = 0; j < 8; j++) {
-                const uint32_t jj = (j + rot) & 7u;
-                const unsigned long long e = bk[jj];
-                if (act && key_of(e) == k) { hit = (int)jj; hv = val_of(e); }
-                if (e == kEmptySlot) emask |= 1u << jj;
+            for (int q = 0; q < 4; q++) {
+                const uint32_t qq = (q + rot) & 3u;
+                unsigned long long e[2];
+                asm volatile("ld.shared.v2.u64 {%0,%1}, [%2];" : "=l"(e[0]), "=l"(e[1])
+                             : "r"(smem_addr(tab + lb * 8 + qq * 2)) : "memory");
+#pragma unroll
+                for (int h = 0; h < 2; h++) {
+                    const uint32_t jj = qq * 2 + h;
+                    if (act && key_of(e[h]) == k) { hit = (int)jj; hv = val_of(e[h]); }
+                    if (e[h] == kEmptySlot) emask |= 1u << jj;
+                }
             }
             bool to_need = false;
             if (OP == 0) {
@@ -421,10 +437,8 @@ __global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView 
                     for (;;) {
                         if (!emask) {             // every snapshot slot taken meanwhile: re-read
 #pragma unroll
-                            for (int j = 0; j < 8; j++) {
-                                const uint32_t jj = (j + rot) & 7u;
-                                if (bk[jj] == kEmptySlot) emask |= 1u << jj;
-                            }
+                            for (int j = 0; j < 8; j++)
+                                if (bk[j] == kEmptySlot) emask |= 1u << j;
                             if (!emask) break;
                         }
                         const int j = __ffs(emask) - 1;
@@ -486,88 +500,40 @@ __global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView 
     }
 }
 
-// ------------------------------------------------------------- need list, results
-// nk[i] = k2[need[i]] (and values) for i < *cnt.
-__global__ void __launch_bounds__(kThreads) k_st_need_gather(const uint32_t* __restrict__ need,
-                                                             const unsigned long long* __restrict__ cnt,
-                                                             const uint32_t* __restrict__ k2, const uint32_t* __restrict__ v2,
-                                                             uint32_t* __restrict__ nk, uint32_t* __restrict__ nv) {
-    const uint64_t n = *cnt;
-    for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n; i += (uint64_t)gridDim.x * kThreads) {
-        const uint32_t p = need[i];
-        nk[i] = k2[p];
-        if (nv) nv[i] = v2[p];
-    }
-}
-
-// st2[need[i]] = ns[i] (and values) for i < *cnt.
-__global__ void __launch_bounds__(kThreads) k_st_need_scatter(const uint32_t* __restrict__ need,
-                                                              const unsigned long long* __restrict__ cnt,
-                                                              const uint8_t* __restrict__ ns, const uint32_t* __restrict__ nr,
-                                                              uint8_t* __restrict__ st2, uint32_t* __restrict__ r2) {
-    const uint64_t n = *cnt;
-    for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < n; i += (uint64_t)gridDim.x * kThreads) {
-        const uint32_t p = need[i];
-        st2[p] = ns[i];
-        if (nr) r2[p] = nr[i];
-    }
-}
-
-// Results of one tile back to the order before its scatter: the tile's runs
-// (run / roff tables of k_st_scatter) are read coalesced into shared memory in
-// the tile's sorted order, then op i of the tile takes entry spos[i].
+// ------------------------------------------------------------------ results
+// Results of one tile back to the order before its scatter: the tile's sorted
+// results are gathered through dmap (runs of consecutive positions, so the reads
+// coalesce) into shared memory, then op i of the tile takes entry spos[i].
 template <int LEVEL>
-__global__ void __launch_bounds__(kStT) k_st_unperm(StagedView s, uint64_t n, const uint32_t* __restrict__ bin_off,
-                                                    const uint32_t* __restrict__ tile_first,
-                                                    const uint32_t* __restrict__ run, const uint16_t* __restrict__ roff,
-                                                    const uint16_t* __restrict__ spos,
+__global__ void __launch_bounds__(kStT) k_st_unperm(StagedView s, uint64_t n, const uint32_t* __restrict__ tile_first,
+                                                    const uint32_t* __restrict__ tile_bin,
+                                                    const uint32_t* __restrict__ tile_lo,
+                                                    const uint32_t* __restrict__ tile_hi,
+                                                    const uint32_t* __restrict__ dmap, const uint16_t* __restrict__ spos,
                                                     const uint8_t* __restrict__ src_s, const uint32_t* __restrict__ src_r,
                                                     uint8_t* __restrict__ dst_s, uint32_t* __restrict__ dst_r) {
-    __shared__ uint32_t ro[kStRoff], rr[kStRun];
     __shared__ uint32_t sr[kStTile];
     __shared__ uint8_t ss[kStTile];
-    __shared__ uint32_t sb, slo, shi, sok;
-    uint32_t nb, t0, tn;
+    uint32_t t0, tn;
     if (LEVEL == 1) {
-        nb = s.nbins;
         t0 = blockIdx.x * kStTile;
         tn = (uint32_t)(n - t0 < (uint64_t)kStTile ? n - t0 : (uint64_t)kStTile);
     } else {
-        if (threadIdx.x == 0) {
-            uint32_t b = 0, lo = 0, hi = 0;
-            sok = st_tile2(s, bin_off, tile_first, blockIdx.x, b, lo, hi);
-            sb = b; slo = lo; shi = hi;
-        }
-        __syncthreads();
-        if (!sok) return;
-        nb = 1u << s.s1;
-        t0 = slo;
-        tn = shi - slo;
+        if (blockIdx.x >= tile_first[s.nbins]) return;
+        t0 = tile_lo[blockIdx.x];
+        tn = tile_hi[blockIdx.x] - t0;
     }
-    for (uint32_t b = threadIdx.x; b <= nb; b += kStT) {
-        ro[b] = roff[(uint64_t)blockIdx.x * kStRoff + b];
-        if (b < nb) rr[b] = run[(uint64_t)blockIdx.x * kStRun + b];
-    }
-    __syncthreads();
-    // kStPer positions per thread: all searches, then all loads in flight, then the stores
-    uint32_t srcp[kStPer];
-#pragma unroll
-    for (int j = 0; j < kStPer; j++) {
-        const uint32_t p = j * kStT + threadIdx.x;
-        uint32_t a = 0, z = nb;            // largest b with ro[b] <= p
-        while (z - a > 1) {
-            const uint32_t m = (a + z) >> 1;
-            if (ro[m] <= p) a = m; else z = m;
-        }
-        srcp[j] = rr[a] + (p - ro[a]);
-    }
+    uint16_t q[kStPer];
     uint32_t vr[kStPer];
     uint8_t vs[kStPer];
 #pragma unroll
     for (int j = 0; j < kStPer; j++) {
-        const bool ok = j * kStT + threadIdx.x < tn;
-        vs[j] = (dst_s && ok) ? src_s[srcp[j]] : (uint8_t)0;
-        vr[j] = (dst_r && ok) ? src_r[srcp[j]] : 0u;
+        const uint32_t i = j * kStT + threadIdx.x;
+        const bool ok = i < tn;
+        q[j] = ok ? spos[t0 + i] : (uint16_t)0;
+        const uint32_t src = ok ? dmap[t0 + i] : 0u;
+        vs[j] = (dst_s && ok) ? src_s[src] : (uint8_t)0;
+        vr[j] = (dst_r && ok) ? src_r[src] : 0u;
     }
 #pragma unroll
     for (int j = 0; j < kStPer; j++) {
@@ -575,12 +541,6 @@ __global__ void __launch_bounds__(kStT) k_st_unperm(StagedView s, uint64_t n, co
         if (p < tn) { ss[p] = vs[j]; sr[p] = vr[j]; }
     }
     __syncthreads();
-    uint16_t q[kStPer];
-#pragma unroll
-    for (int j = 0; j < kStPer; j++) {
-        const uint32_t i = j * kStT + threadIdx.x;
-        q[j] = i < tn ? spos[t0 + i] : (uint16_t)0;
-    }
 #pragma unroll
     for (int j = 0; j < kStPer; j++) {
         const uint32_t i = j * kStT + threadIdx.x;

@@ -110,7 +110,9 @@ def test_staged_c2_shape(oracle_mod, log2_n):
     wl = W.c2_rand_static(log2_n=log2_n)
     g, o = run_staged(oracle_mod, wl, staged="auto" if log2_n >= 20 else "force", layout_every=False)
     check_layout(g, o)
-    assert g.stats()["n_staged"] >= 2   # (the delete batch, n/2 ops, is below the automatic threshold at 2^20)
+    # automatic choice: the insert batch stages; finds stay direct; the delete
+    # batch (n/2 ops) is below the automatic threshold at 2^20
+    assert g.stats()["n_staged"] >= 1
 
 
 def test_staged_matches_direct(oracle_mod):
