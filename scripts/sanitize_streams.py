@@ -1,7 +1,8 @@
 """Small end-to-end workloads for compute-sanitizer (memcheck, racecheck,
 synccheck; scripts/gpu_pass.sh sanitize): C1, C3 and C4 streams at small
 scale, the paper-weighted placement mode, a live resize window, the sharded C
-ABI with local virtual shards, and the failure path (max_hops = 1).  Every
+ABI with local virtual shards, the chunk-staged path (forced), and the failure
+path (max_hops = 1).  Every
 batch is checked against the oracle so a sanitizer-clean run is also a correct
 one.  Exits non-zero on a mismatch."""
 import os
@@ -55,6 +56,7 @@ def main():
                        oracle.OracleTable(d=wl.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta,
                                           bucket_slots=8, **{k: v for k, v in kw.items() if k == "max_hops"}))
     run(*mk(), wl.batches, "C1")
+    run(*mk(staged="force"), wl.batches, "C1-staged")     # chunk-staged path (TMA bulk copies, smem atomics)
     c3 = W.c3_dynamic(scale=0.0005, shape="RE", batch=4000, cycles=1, init_capacity=1024)
     g = Table(d=4, init_capacity=1024, alpha=0.3, beta=0.85)
     run(g, oracle.OracleTable(d=4, init_capacity=1024, alpha=0.3, beta=0.85, bucket_slots=8), c3.batches, "C3-RE")

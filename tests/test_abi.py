@@ -67,6 +67,22 @@ def test_host_only_calls_without_gpu(lib):
     assert lib.dyc_launch_count(None, 0) == 0
 
 
+def test_staged_flags_checked_without_gpu(lib):
+    """DYC_STAGED_OFF and DYC_STAGED_FORCE exclude each other; undefined flag bits
+    are rejected; both are checked before any device is touched."""
+    cfg = L.dyc_config()
+    assert lib.dyc_config_default(C.byref(cfg)) == L.DYC_OK
+    h = C.c_void_p()
+    cfg.flags = L.DYC_STAGED_OFF | L.DYC_STAGED_FORCE
+    assert lib.dyc_create_ex(C.byref(cfg), C.byref(h)) == L.DYC_ERR_INVALID_ARG
+    assert "exclude" in L.last_error()
+    cfg.flags = 16
+    assert lib.dyc_create_ex(C.byref(cfg), C.byref(h)) == L.DYC_ERR_INVALID_ARG
+    for ok in (L.DYC_STAGED_OFF, L.DYC_STAGED_FORCE, 0):
+        cfg.flags = ok            # valid: fails only for want of a device here
+        assert lib.dyc_create_ex(C.byref(cfg), C.byref(h)) in (L.DYC_ERR_NO_DEVICE, L.DYC_OK)
+
+
 def test_library_is_sm100a(lib):
     """The fatbin carries sm_100a SASS (cuobjdump), with 256-bit probe loads."""
     import shutil
