@@ -466,15 +466,19 @@ void dev_free(dyc_table* t, void* p, cudaStream_t st) {
     cudaEventRecord(ev, st);
     t->cache.push_back({p, bytes, ev});
     t->cache_bytes += bytes;
-    // keep up to the table's high-water size (+256 MB) cached, not just its
-    // current size: a shrink phase would otherwise free (cudaFree syncs the
+    // keep up to twice the table's high-water size (+256 MB) cached, not just
+    // its current size: a shrink phase would otherwise free (cudaFree syncs the
     // device) exactly the buffers the next growth phase allocates again, and
     // fresh cudaMalloc calls are where the stream configs' run-to-run variance
-    // came from (profiles/r1t_c5_variance.md).  dyc_trim releases the cache.
+    // came from (profiles/r1t_c5_variance.md; C3-RE's 9 cudaMalloc calls per
+    // pass took 12 ms in r2m and 84 ms in r2n with a cap of one high-water size:
+    // a growth phase holds every smaller power-of-two buffer of the subtables
+    // in the cache at once).  An allocation that fails flushes the cache and
+    // retries; dyc_trim releases it.
     uint64_t cur = 0;
     for (uint32_t i = 0; i < t->cfg.d; i++) cur += t->nb[i] * t->cfg.bucket_slots * 8;
     t->peak_table_bytes = std::max(t->peak_table_bytes, cur);
-    const uint64_t cap = (256ull << 20) + t->peak_table_bytes;
+    const uint64_t cap = (256ull << 20) + 2 * t->peak_table_bytes;
     while (t->cache_bytes > cap && !t->cache.empty()) {      // oldest first
         cudaEventSynchronize(t->cache.front().ev);
         cudaFree(t->cache.front().p);

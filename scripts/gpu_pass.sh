@@ -16,10 +16,10 @@ for step in "$@"; do
     bench:*) a="${step#bench:}"; n=$(echo "$a" | tr -c 'a-zA-Z0-9' '_'); timeout 1800 python bench.py $a > gpurun_out/bench_${R}_$n.json 2> gpurun_out/bench_${R}_$n.err; tail -2 gpurun_out/bench_${R}_$n.err; head -c 300 gpurun_out/bench_${R}_$n.json; echo ;;
     ref) timeout 900 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/bench_ref_$R.json 2>&1; head -c 300 gpurun_out/bench_ref_$R.json; echo ;;
     launches) timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_$R.csv python bench.py --steps 2 --warmup 1 --profile-only > /dev/null 2>&1; echo "launches rc=$?" ;;
-    ncu) timeout 1500 ncu --set full --clock-control none --import-source on -k regex:"k_upsert|k_find|k_delete|k_place" -c 4 -o gpurun_out/prof_$R python bench.py --steps 1 --warmup 0 --profile-only > gpurun_out/ncu_full_$R.log 2>&1; tail -2 gpurun_out/ncu_full_$R.log ;;
+    ncu) timeout 1500 ncu --set full --clock-control none --import-source on -k regex:"k_upsert|k_find|k_delete|k_place|k_st_" -c 20 -o gpurun_out/prof_$R python bench.py --steps 1 --warmup 0 --profile-only > gpurun_out/ncu_full_$R.log 2>&1; tail -2 gpurun_out/ncu_full_$R.log ;;
     gather) timeout 600 python scripts/gather_wall.py > gpurun_out/gather_$R.log 2>&1; tail -3 gpurun_out/gather_$R.log
             ;;
-    sanitize)
+    sanitize)   # NOTE: compute-sanitizer was closed on the GPU pool during round 2 (r2n); kept for reference
       for tool in memcheck racecheck synccheck; do
         timeout 1500 compute-sanitizer --tool $tool --error-exitcode 9 python scripts/sanitize_streams.py > gpurun_out/${tool}_$R.txt 2>&1; echo "$tool rc=$?"; tail -2 gpurun_out/${tool}_$R.txt
       done ;;

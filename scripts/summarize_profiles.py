@@ -80,6 +80,9 @@ def main(tag):
     # the timed steps are the last 2 groups of probe launches before k_gather
     ours = [(n, ms) for _, n, ms in L if "dyc::" in n and "k_gather" not in n and "k_count" not in n]
     starts = [j for j, (n, _) in enumerate(ours) if "k_upsert" in n]
+    if any("k_st_scatter<1, 1>" in n for n, _ in ours):
+        # a staged insert opens each step: k_st_hist, k_st_scan, k_st_scatter<1, 1>, ...
+        starts = [j - 2 for j, (n, _) in enumerate(ours) if "k_st_scatter<1, 1>" in n]
     last2 = ours[starts[-2]:]                      # the last two timed steps
     per = {}
     for n, ms in last2:
@@ -94,8 +97,8 @@ def main(tag):
           "- `ncu --metrics gpu__time_duration.sum --clock-control none`: the launch list of",
           "  `bench.py --steps 2 --warmup 1 --profile-only`. These launches are cold-cache and serialised, so",
           "  compare shares, not absolutes. The full list of our launches is `" + tag + "_launches.csv`.",
-          "- `ncu --set full --import-source on -k regex:\"k_upsert|k_find|k_delete|k_place\" -c 4`: one capture",
-          "  per probe kernel, on the same C2 2^27 workload.",
+          "- `ncu --set full --import-source on -k regex:\"k_upsert|k_find|k_delete|k_place|k_st_\"`: one capture",
+          "  per kernel launch of one step (staged passes included), on the same C2 2^27 workload.",
           "", "## Kernel shares of one step (ncu launch list, last two timed steps)", "",
           "| kernel | ms per step | share | bench (CUDA events, warm) ms |", "|---|---|---|---|"]
     kms = bench["roofline"]["kernel_ms_per_step"]
@@ -120,6 +123,11 @@ def main(tag):
                                                            1e6 if k["dram__bytes_write.sum"][1] == "Mbyte" else 1)
             if base not in traffic or rd + wr > traffic[base]:
                 traffic[base] = rd + wr
+            if base.startswith("k_st_"):       # the bench's profile kind of a staged pass
+                kind = {"k_st_hist": "st_hist", "k_st_scan": "st_hist", "k_st_scatter": "st_scatter",
+                        "k_st_apply": "st_apply", "k_st_unperm": "st_unperm"}.get(base)
+                if kind:
+                    traffic[kind] = traffic.get(kind, 0.0) + rd + wr
         except (KeyError, ValueError):
             pass
     r = bench["roofline"]
