@@ -1283,6 +1283,8 @@ dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, 
         CU(cudaFuncSetAttribute(k_st_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, kStMaxChunks * 4));
         CU(cudaFuncSetAttribute(k_st_scatter<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 3 * kStTile * 4 + kStTile));
         CU(cudaFuncSetAttribute(k_st_scatter<2, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 3 * kStTile * 4 + kStTile));
+        CU(cudaFuncSetAttribute(k_st_scatter<1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * kStTile * 4 + kStTile));
+        CU(cudaFuncSetAttribute(k_st_scatter<2, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * kStTile * 4 + kStTile));
         attr_set = true;
     }
     t->n_staged++;

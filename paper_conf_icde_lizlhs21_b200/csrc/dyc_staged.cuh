@@ -47,14 +47,26 @@ constexpr int kStLog = 10;                        // buckets per chunk = 1024
 constexpr uint32_t kStChunk = 1u << kStLog;
 constexpr uint32_t kStSlots = kStChunk * 8;       // B = 8: 64 KB of shared memory
 constexpr int kStBins1 = 256;                     // level-1 bins (at most)
-constexpr int kStTile = 4096;                     // ops per partition tile
-constexpr int kStT = 512;                         // threads of the scatter / unperm kernels
-constexpr int kStPer = kStTile / kStT;            // 8 ops per thread
+#ifndef DYC_ST_TILE
+#define DYC_ST_TILE 4096
+#endif
+#ifndef DYC_ST_T
+#define DYC_ST_T 512
+#endif
+#ifndef DYC_ST_SCATTER_MINB
+#define DYC_ST_SCATTER_MINB 3
+#endif
+#ifndef DYC_ST_APPLY_U
+#define DYC_ST_APPLY_U 8
+#endif
+constexpr int kStTile = DYC_ST_TILE;              // ops per partition tile (<= 65536: 16-bit sorted index)
+constexpr int kStT = DYC_ST_T;                    // threads of the scatter / unperm kernels
+constexpr int kStPer = kStTile / kStT;            // ops per thread (8)
 constexpr int kStMaxS1 = 8;                       // 2^s1 chunks per level-1 bin, <= 256
 constexpr uint32_t kStMaxChunks = 32768;          // k_st_hist: one shared counter per chunk
 constexpr int kStHistT = 1024;
 constexpr int kStHistPer = 8;
-constexpr int kStApplyU = 4;                      // ops per lane in flight (apply)
+constexpr int kStApplyU = DYC_ST_APPLY_U;         // ops per lane in flight (apply)
 constexpr int kStNeedBuf = 64;                    // per-warp need-list buffer (apply)
 constexpr int kStRun = 256;                       // bins (level 1) or chunks of a bin (level 2), at most
 
@@ -228,7 +240,7 @@ __device__ __forceinline__ bool st_tile2(const StagedView& s, const uint32_t* ti
 // tile's p-th sorted op went to (what k_st_unperm reads the results back from).
 // Level 2 writes the chunk-local bucket (gb & 1023) as 16 bits instead of gb.
 template <int LEVEL, bool VALS>
-__global__ void __launch_bounds__(kStT, 3) k_st_scatter(StagedView s, const uint32_t* __restrict__ kin,
+__global__ void __launch_bounds__(kStT, DYC_ST_SCATTER_MINB) k_st_scatter(StagedView s, const uint32_t* __restrict__ kin,
                                                      const uint32_t* __restrict__ vin, const uint32_t* __restrict__ gin,
                                                      uint64_t n, const uint32_t* __restrict__ tile_first,
                                                      const uint32_t* __restrict__ tile_bin,
