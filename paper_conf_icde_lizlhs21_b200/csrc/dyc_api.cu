@@ -1315,25 +1315,26 @@ dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, 
     uint32_t* need = b.g;
     {
         ProfScope ps(t, DYC_PROF_ST_APPLY, st);
+        // the need list: positions in g, keys / values in k1 / v1 (free after the level-2 scatter)
         k_st_apply<OP><<<sv.nc, kThreads, kStSlots * 8, st>>>(tv, sv, b.k2, b.v2, b.lb2, b.chunk_off, b.st2, r2, need,
-                                                             b.need_cnt, t->d_ctr);
+                                                             b.k1, b.v1, b.need_cnt, t->d_ctr);
     }
     CU(cudaGetLastError());
-    // the ops their first-choice bucket could not decide (the need list: positions
-    // in the chunk order) run through the direct kernel with the first probe
-    // skipped, reading their keys and writing their results at those positions
+    // the ops their first-choice bucket could not decide (the need list: keys,
+    // values and positions in the chunk order) run through the direct kernel
+    // with the first probe skipped, writing their results at those positions
     const unsigned gneed = (unsigned)t->num_sms * 8;
-    if (OP == 0) TRY(insert_chunk<B>(t, b.k2, b.v2, b.st2, n, true, st, b.need_cnt, gneed, need));
-    else if (OP == 1) TRY(find_impl<B>(t, b.k2, r2, b.st2, n, st, b.need_cnt, gneed, need));
-    else TRY(delete_chunk<B>(t, b.k2, r2, b.st2, n, st, b.need_cnt, gneed, need));
+    if (OP == 0) TRY(insert_chunk<B>(t, b.k1, b.v1, b.st2, n, true, st, b.need_cnt, gneed, need));
+    else if (OP == 1) TRY(find_impl<B>(t, b.k1, r2, b.st2, n, st, b.need_cnt, gneed, need));
+    else TRY(delete_chunk<B>(t, b.k1, r2, b.st2, n, st, b.need_cnt, gneed, need));
     {
         ProfScope ps(t, DYC_PROF_ST_UNPERM, st);
         // back to request order: chunk order -> level-1 order (into st1 / v1) -> caller
         uint32_t* r1 = OP == 0 ? nullptr : b.v1;
-        k_st_unperm<2><<<(unsigned)tiles2, kStT, 0, st>>>(sv, n, b.tile_first, b.tile_bin, b.tile_lo, b.tile_hi,
+        k_st_unperm<2><<<(unsigned)tiles2, kStUT, 0, st>>>(sv, n, b.tile_first, b.tile_bin, b.tile_lo, b.tile_hi,
                                                            b.dmap2, b.spos2, b.st2, r2, b.st1, r1);
         if (out_st || out_r)
-            k_st_unperm<1><<<(unsigned)tiles1, kStT, 0, st>>>(sv, n, b.tile_first, b.tile_bin, b.tile_lo, b.tile_hi,
+            k_st_unperm<1><<<(unsigned)tiles1, kStUT, 0, st>>>(sv, n, b.tile_first, b.tile_bin, b.tile_lo, b.tile_hi,
                                                                b.dmap1, b.spos1, b.st1, r1, out_st, out_r);
     }
     CU(cudaGetLastError());

@@ -180,7 +180,7 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
                                                    uint32_t* __restrict__ vals, uint8_t* __restrict__ found,
                                                    uint64_t n, const unsigned long long* __restrict__ n_dev = nullptr,
                                                    const uint32_t* __restrict__ idx = nullptr) {
-    // S1: op i is keys[idx[i]], its results go to [idx[i]] (a staged batch's need list)
+    // S1: op i (keys[i]) is entry i of a staged batch's need list; its results go to [idx[i]]
     constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
@@ -200,7 +200,7 @@ __global__ void __launch_bounds__(kThreads, DYC_FIND_MINB) k_find(TableView tv, 
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
             const uint64_t i = base + (uint64_t)j * QPW + grp;
-            k[j] = i < n ? __ldg(keys + (S1 ? (uint64_t)__ldg(idx + i) : i)) : kEmptyKey;
+            k[j] = i < n ? __ldg(keys + i) : kEmptyKey;
         }
 #pragma unroll
         for (int j = 0; j < ILP; j++) {
@@ -377,7 +377,7 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
                                                      unsigned long long* __restrict__ defer = nullptr,
                                                      const unsigned long long* __restrict__ n_dev = nullptr,
                                                      const uint32_t* __restrict__ idx = nullptr) {
-    // S1: op i is (keys, vals)[idx[i]], its status goes to status[idx[i]] (a staged batch's need list)
+    // S1: op i ((keys, vals)[i]) is entry i of a staged batch's need list; its status goes to status[idx[i]]
     constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
@@ -410,9 +410,8 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
             for (int u = 0; u < U; u++) {
                 i[u] = base + (uint64_t)u * QPW + grp;
                 const bool valid = i[u] < n;
-                const uint64_t src = (S1 && valid) ? (uint64_t)__ldg(idx + i[u]) : i[u];
-                k[u] = valid ? __ldg(keys + src) : kEmptyKey;
-                kv[u] = make_kv(k[u], valid ? __ldg(vals + src) : 0u);
+                k[u] = valid ? __ldg(keys + i[u]) : kEmptyKey;
+                kv[u] = make_kv(k[u], valid ? __ldg(vals + i[u]) : 0u);
                 const Pair p = pair_of(tv, k[u]);
                 lk1[u] = LK && p.t1 == locked;
                 lk2[u] = LK && p.t2 == locked;
@@ -443,9 +442,8 @@ __global__ void __launch_bounds__(kThreads, DYC_UPSERT_MINB) k_upsert(TableView 
             for (int u = 0; u < U; u++) {
                 i[u] = base + (uint64_t)u * QPW + grp;
                 const bool valid = i[u] < n;
-                const uint64_t src = (S1 && valid) ? (uint64_t)__ldg(idx + i[u]) : i[u];
-                k[u] = valid ? __ldg(keys + src) : kEmptyKey;
-                kv[u] = make_kv(k[u], valid ? __ldg(vals + src) : 0u);
+                k[u] = valid ? __ldg(keys + i[u]) : kEmptyKey;
+                kv[u] = make_kv(k[u], valid ? __ldg(vals + i[u]) : 0u);
                 const Pair p = pair_of(tv, k[u]);
                 lk1[u] = LK && p.t1 == locked;
                 lk2[u] = LK && p.t2 == locked;
@@ -680,7 +678,7 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
                                                      unsigned long long* __restrict__ defer = nullptr,
                                                      const unsigned long long* __restrict__ n_dev = nullptr,
                                                      const uint32_t* __restrict__ idx = nullptr) {
-    // S1: op i is keys[idx[i]], its results go to [idx[i]] (a staged batch's need list)
+    // S1: op i (keys[i]) is entry i of a staged batch's need list; its results go to [idx[i]]
     constexpr int G = B / 4, QPW = 32 / G;
     __shared__ SmemView sv;
     load_view(tv, sv);
@@ -703,7 +701,7 @@ __global__ void __launch_bounds__(kThreads, DYC_DELETE_MINB) k_delete(TableView 
 #pragma unroll
         for (int u = 0; u < U; u++) {
             i[u] = base + (uint64_t)u * QPW + grp;
-            k[u] = i[u] < n ? __ldg(keys + (S1 ? (uint64_t)__ldg(idx + i[u]) : i[u])) : kEmptyKey;
+            k[u] = i[u] < n ? __ldg(keys + i[u]) : kEmptyKey;
             const Pair p = pair_of(tv, k[u]);
             lk1[u] = LK && p.t1 == locked;
             lk2[u] = LK && p.t2 == locked;

@@ -62,6 +62,11 @@ constexpr int kStBins1 = 256;                     // level-1 bins (at most)
 constexpr int kStTile = DYC_ST_TILE;              // ops per partition tile (<= 65536: 16-bit sorted index)
 constexpr int kStT = DYC_ST_T;                    // threads of the scatter / unperm kernels
 constexpr int kStPer = kStTile / kStT;            // ops per thread (8)
+#ifndef DYC_ST_UT
+#define DYC_ST_UT 1024
+#endif
+constexpr int kStUT = DYC_ST_UT;                  // threads of the unperm kernel
+constexpr int kStUPer = kStTile / kStUT;          // positions per thread (unperm)
 constexpr int kStMaxS1 = 8;                       // 2^s1 chunks per level-1 bin, <= 256
 constexpr uint32_t kStMaxChunks = 32768;          // k_st_hist: one shared counter per chunk
 constexpr int kStHistT = 1024;
@@ -343,13 +348,16 @@ __global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView 
                                                        const uint32_t* __restrict__ v2, const uint16_t* __restrict__ lb2,
                                                        const uint32_t* __restrict__ chunk_off,
                                                        uint8_t* __restrict__ st2, uint32_t* __restrict__ r2,
-                                                       uint32_t* __restrict__ need,
+                                                       uint32_t* __restrict__ need, uint32_t* __restrict__ need_k,
+                                                       uint32_t* __restrict__ need_v,
                                                        unsigned long long* __restrict__ need_cnt,
                                                        unsigned long long* __restrict__ ctr) {
     extern __shared__ __align__(128) unsigned long long tab[];
     __shared__ __align__(8) unsigned long long bar;
     __shared__ uint32_t fullw[kStChunk / 32];
-    __shared__ uint32_t nbuf[kThreads / 32][kStNeedBuf];
+    __shared__ uint32_t nbuf[kThreads / 32][kStNeedBuf];     // need list: chunk-order position,
+    __shared__ uint32_t nbufk[kThreads / 32][kStNeedBuf];    // key and (insert) value of each entry
+    __shared__ uint32_t nbufv[OP == 0 ? kThreads / 32 : 1][OP == 0 ? kStNeedBuf : 1];
     __shared__ int changed;
     const uint32_t c = blockIdx.x;
     const uint32_t o0 = chunk_off[c], o1 = chunk_off[c + 1];
@@ -390,7 +398,11 @@ __global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView 
             unsigned long long gb = 0;
             if (lane == 0) gb = atomicAdd(need_cnt, (unsigned long long)ncount);
             gb = __shfl_sync(kFull, gb, 0);
-            for (uint32_t i = lane; i < ncount; i += 32) need[gb + i] = nbuf[w][i];
+            for (uint32_t i = lane; i < ncount; i += 32) {
+                need[gb + i] = nbuf[w][i];
+                need_k[gb + i] = nbufk[w][i];
+                if (OP == 0) need_v[gb + i] = nbufv[w][i];
+            }
             ncount = 0;
         }
         __syncwarp();
@@ -492,7 +504,12 @@ __global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView 
             const unsigned m = __ballot_sync(kFull, to_need);
             if (m) {
                 if (ncount + __popc(m) > (uint32_t)kStNeedBuf) flush();
-                if (to_need) nbuf[w][ncount + __popc(m & lanemask_lt())] = p;
+                if (to_need) {
+                    const uint32_t e = ncount + __popc(m & lanemask_lt());
+                    nbuf[w][e] = p;
+                    nbufk[w][e] = k;
+                    if (OP == 0) nbufv[OP == 0 ? w : 0][OP == 0 ? e : 0] = vv[u];
+                }
                 ncount += __popc(m);
             }
         }
@@ -517,7 +534,7 @@ __global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView 
 // results are gathered through dmap (runs of consecutive positions, so the reads
 // coalesce) into shared memory, then op i of the tile takes entry spos[i].
 template <int LEVEL>
-__global__ void __launch_bounds__(kStT) k_st_unperm(StagedView s, uint64_t n, const uint32_t* __restrict__ tile_first,
+__global__ void __launch_bounds__(kStUT) k_st_unperm(StagedView s, uint64_t n, const uint32_t* __restrict__ tile_first,
                                                     const uint32_t* __restrict__ tile_bin,
                                                     const uint32_t* __restrict__ tile_lo,
                                                     const uint32_t* __restrict__ tile_hi,
@@ -535,12 +552,12 @@ __global__ void __launch_bounds__(kStT) k_st_unperm(StagedView s, uint64_t n, co
         t0 = tile_lo[blockIdx.x];
         tn = tile_hi[blockIdx.x] - t0;
     }
-    uint16_t q[kStPer];
-    uint32_t vr[kStPer];
-    uint8_t vs[kStPer];
+    uint16_t q[kStUPer];
+    uint32_t vr[kStUPer];
+    uint8_t vs[kStUPer];
 #pragma unroll
-    for (int j = 0; j < kStPer; j++) {
-        const uint32_t i = j * kStT + threadIdx.x;
+    for (int j = 0; j < kStUPer; j++) {
+        const uint32_t i = j * kStUT + threadIdx.x;
         const bool ok = i < tn;
         q[j] = ok ? spos[t0 + i] : (uint16_t)0;
         const uint32_t src = ok ? dmap[t0 + i] : 0u;
@@ -548,14 +565,14 @@ __global__ void __launch_bounds__(kStT) k_st_unperm(StagedView s, uint64_t n, co
         vr[j] = (dst_r && ok) ? src_r[src] : 0u;
     }
 #pragma unroll
-    for (int j = 0; j < kStPer; j++) {
-        const uint32_t p = j * kStT + threadIdx.x;
+    for (int j = 0; j < kStUPer; j++) {
+        const uint32_t p = j * kStUT + threadIdx.x;
         if (p < tn) { ss[p] = vs[j]; sr[p] = vr[j]; }
     }
     __syncthreads();
 #pragma unroll
-    for (int j = 0; j < kStPer; j++) {
-        const uint32_t i = j * kStT + threadIdx.x;
+    for (int j = 0; j < kStUPer; j++) {
+        const uint32_t i = j * kStUT + threadIdx.x;
         if (i < tn) {
             if (dst_s) dst_s[t0 + i] = ss[q[j]];
             if (dst_r) dst_r[t0 + i] = sr[q[j]];
