@@ -10,6 +10,7 @@
 //           whose residuals needed a failure upsize ends the loop, Q17b).
 // All comparisons are `(double)m <op> bound*(double)N` on the host (Q29).
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cmath>
 #include <cstdio>
@@ -1275,8 +1276,10 @@ dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, 
     StagedBufs b{};
     TRY(staged_bufs(t, n, sv.nc, tiles1, tiles2, st, b));
     const uint32_t sm_scatter = (VALS ? 3 : 2) * kStTile * 4 + kStTile;
-    static bool attr_set = false;
-    if (!attr_set) {
+    // opt-in shared-memory sizes, once per device (function attributes are per device context)
+    static std::atomic<uint64_t> attr_devices{0};
+    const uint64_t dev_bit = 1ull << (t->device & 63);
+    if (!(attr_devices.load() & dev_bit)) {
         CU(cudaFuncSetAttribute(k_st_apply<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kStSlots * 8));
         CU(cudaFuncSetAttribute(k_st_apply<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, kStSlots * 8));
         CU(cudaFuncSetAttribute(k_st_apply<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, kStSlots * 8));
@@ -1285,7 +1288,7 @@ dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, 
         CU(cudaFuncSetAttribute(k_st_scatter<2, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 3 * kStTile * 4 + kStTile));
         CU(cudaFuncSetAttribute(k_st_scatter<1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * kStTile * 4 + kStTile));
         CU(cudaFuncSetAttribute(k_st_scatter<2, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * kStTile * 4 + kStTile));
-        attr_set = true;
+        attr_devices.fetch_or(dev_bit);
     }
     t->n_staged++;
     const TableView tv = t->view();
