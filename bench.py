@@ -471,6 +471,23 @@ def compute_roofline(args, prof, n_ins, n_find, n_del, s_ins, hit_rate, phi, phi
 
 
 
+def north_star_fracs(n, phase_ms, probes, staged):
+    """north_star's targets (find >= 0.50, insert >= 0.30 of the one-sector-per-probe
+    HBM roofline) at the phase level, with SURVEY §8(d)'s accounting: an insert
+    costs two probed 32-B sectors (the existence check), one written sector and
+    9 B of IO (105 B); a find r_f probed sectors + 9 B, r_f = the direct kernel's
+    measured probes per find.  Phase ops/s x bytes per op over the measured copy peak."""
+    peak, _ = measured_peaks()
+    r_f = 1.0 + probes["find"][1] / max(1, probes["find"][0]) if not staged.get("find") else 1.32
+    ins_bps = n / (phase_ms["insert"] * 1e-3) * 105.0
+    find_bps = n / (phase_ms["find"] * 1e-3) * (r_f * 32.0 + 9.0)
+    return {"insert_frac": ins_bps / (peak * 1e9), "insert_target": 0.30,
+            "find_frac": find_bps / (peak * 1e9), "find_target": 0.50,
+            "bytes_per_op": {"insert": 105.0, "find": r_f * 32.0 + 9.0}, "peak_gbs": peak,
+            "what": "phase ops/s x SURVEY §8(d) bytes per op (32 B per probed sector, 32 B per written sector, "
+                    "streamed IO) / measured copy peak"}
+
+
 # ---------------------------------------------------------------- GPU arm
 def main():
     _redirect_stdout()
@@ -814,6 +831,7 @@ def main():
                 "delete_mops": (n // 2) / phase_ms["delete"] / 1e3},
         "resize": resize,
         "roofline": roofline,
+        "north_star": north_star_fracs(n, phase_ms, probes, staged),
         "cpu_baseline": cpu,
         "e2e": e2e,
         "gpu_launches": launches,
