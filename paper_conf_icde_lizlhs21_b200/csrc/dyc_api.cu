@@ -1234,13 +1234,11 @@ struct StagedBufs {
     unsigned long long* need_cnt;
 };
 
-dyc_status staged_bufs(dyc_table* t, uint64_t n, uint32_t nc, uint64_t tiles1, uint64_t tiles2, cudaStream_t st,
-                       StagedBufs& b) {
+dyc_status staged_bufs(dyc_table* t, uint64_t n, uint32_t nc, uint64_t tiles2, cudaStream_t st, StagedBufs& b) {
     auto al = [](uint64_t x) { return (x + 255) & ~255ull; };
     const uint64_t a4 = al(4 * n), a2 = al(2 * n), a1 = al(n);
     const uint64_t tt = al(4ull * (tiles2 + 1));
     const uint64_t sc = al(4ull * (nc + 1)), sb = al(4ull * (kStBins1 + 1));
-    (void)tiles1;
     const uint64_t bytes = 8 * a4 + 3 * a2 + 2 * a1 + 3 * tt + 3 * sc + 3 * sb + 256;
     if (bytes > t->stg_cap) {
         dev_free(t, t->stg, st);
@@ -1274,7 +1272,7 @@ dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, 
     const uint64_t tiles1 = (n + kStTile - 1) / kStTile;
     const uint64_t tiles2 = tiles1 + sv.nbins;
     StagedBufs b{};
-    TRY(staged_bufs(t, n, sv.nc, tiles1, tiles2, st, b));
+    TRY(staged_bufs(t, n, sv.nc, tiles2, st, b));
     const uint32_t sm_scatter = (VALS ? 3 : 2) * kStTile * 4 + kStTile;
     // opt-in shared-memory sizes, once per device (function attributes are per device context)
     static std::atomic<uint64_t> attr_devices{0};
@@ -1292,7 +1290,6 @@ dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, 
     }
     t->n_staged++;
     const TableView tv = t->view();
-    const unsigned gstream = (unsigned)std::min<uint64_t>(grid_for(n, kThreads), (uint64_t)t->num_sms * 8);
     {
         ProfScope ps(t, DYC_PROF_ST_HIST, st);
         CU(cudaMemsetAsync(b.chunk_cnt, 0, 4ull * (sv.nc + 1), st));
@@ -1319,7 +1316,7 @@ dyc_status staged_run(dyc_table* t, const uint32_t* keys, const uint32_t* vals, 
     {
         ProfScope ps(t, DYC_PROF_ST_APPLY, st);
         // the need list: positions in g, keys / values in k1 / v1 (free after the level-2 scatter)
-        k_st_apply<OP><<<sv.nc, kThreads, kStSlots * 8, st>>>(tv, sv, b.k2, b.v2, b.lb2, b.chunk_off, b.st2, r2, need,
+        k_st_apply<OP><<<sv.nc, kStAT, kStSlots * 8, st>>>(tv, sv, b.k2, b.v2, b.lb2, b.chunk_off, b.st2, r2, need,
                                                              b.k1, b.v1, b.need_cnt, t->d_ctr);
     }
     CU(cudaGetLastError());

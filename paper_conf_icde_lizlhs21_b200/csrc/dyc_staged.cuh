@@ -43,7 +43,14 @@
 
 namespace dyc {
 
-constexpr int kStLog = 10;                        // buckets per chunk = 1024
+#ifndef DYC_ST_LOG
+#define DYC_ST_LOG 10
+#endif
+#ifndef DYC_ST_AT
+#define DYC_ST_AT 256
+#endif
+constexpr int kStLog = DYC_ST_LOG;                // buckets per chunk = 1024
+constexpr int kStAT = DYC_ST_AT;                  // threads of the apply kernel
 constexpr uint32_t kStChunk = 1u << kStLog;
 constexpr uint32_t kStSlots = kStChunk * 8;       // B = 8: 64 KB of shared memory
 constexpr int kStBins1 = 256;                     // level-1 bins (at most)
@@ -68,7 +75,7 @@ constexpr int kStPer = kStTile / kStT;            // ops per thread (8)
 constexpr int kStUT = DYC_ST_UT;                  // threads of the unperm kernel
 constexpr int kStUPer = kStTile / kStUT;          // positions per thread (unperm)
 constexpr int kStMaxS1 = 8;                       // 2^s1 chunks per level-1 bin, <= 256
-constexpr uint32_t kStMaxChunks = 32768;          // k_st_hist: one shared counter per chunk
+constexpr uint32_t kStMaxChunks = kStLog >= 10 ? 32768 : 49152;   // k_st_hist: one shared counter per chunk
 constexpr int kStHistT = 1024;
 constexpr int kStHistPer = 8;
 constexpr int kStApplyU = DYC_ST_APPLY_U;         // ops per lane in flight (apply)
@@ -344,7 +351,7 @@ __global__ void __launch_bounds__(kStT, DYC_ST_SCATTER_MINB) k_st_scatter(Staged
 //       through the direct kernel with the first probe skipped (S1).
 // Insert statuses: 1 INSERTED, 2 UPDATED; delete: 1 DELETED; find: found flag.
 template <int OP>
-__global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView s, const uint32_t* __restrict__ k2,
+__global__ void __launch_bounds__(kStAT) k_st_apply(TableView tv, StagedView s, const uint32_t* __restrict__ k2,
                                                        const uint32_t* __restrict__ v2, const uint16_t* __restrict__ lb2,
                                                        const uint32_t* __restrict__ chunk_off,
                                                        uint8_t* __restrict__ st2, uint32_t* __restrict__ r2,
@@ -355,9 +362,9 @@ __global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView 
     extern __shared__ __align__(128) unsigned long long tab[];
     __shared__ __align__(8) unsigned long long bar;
     __shared__ uint32_t fullw[kStChunk / 32];
-    __shared__ uint32_t nbuf[kThreads / 32][kStNeedBuf];     // need list: chunk-order position,
-    __shared__ uint32_t nbufk[kThreads / 32][kStNeedBuf];    // key and (insert) value of each entry
-    __shared__ uint32_t nbufv[OP == 0 ? kThreads / 32 : 1][OP == 0 ? kStNeedBuf : 1];
+    __shared__ uint32_t nbuf[kStAT / 32][kStNeedBuf];     // need list: chunk-order position,
+    __shared__ uint32_t nbufk[kStAT / 32][kStNeedBuf];    // key and (insert) value of each entry
+    __shared__ uint32_t nbufv[OP == 0 ? kStAT / 32 : 1][OP == 0 ? kStNeedBuf : 1];
     __shared__ int changed;
     const uint32_t c = blockIdx.x;
     const uint32_t o0 = chunk_off[c], o1 = chunk_off[c + 1];
@@ -375,11 +382,11 @@ __global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView 
         changed = 0;
     }
     if (OP == 2)
-        for (uint32_t i = threadIdx.x; i < kStChunk / 32; i += kThreads) fullw[i] = 0;
+        for (uint32_t i = threadIdx.x; i < kStChunk / 32; i += kStAT) fullw[i] = 0;
     __syncthreads();                      // barrier initialized, fullw zeroed
     st_mbar_wait(&bar, 0);
     if (OP == 2) {                        // fullness of every bucket before any erase
-        for (uint32_t q = threadIdx.x; q < nbk; q += kThreads) {
+        for (uint32_t q = threadIdx.x; q < nbk; q += kStAT) {
             bool full = true;
 #pragma unroll
             for (int j = 0; j < 8; j++) full &= tab[q * 8 + ((j + (q >> 1)) & 7u)] != kEmptySlot;   // bank rotation
@@ -408,7 +415,7 @@ __global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView 
         __syncwarp();
     };
     constexpr int U = kStApplyU;
-    for (uint32_t base = o0 + w * 32 * U; base < o1; base += kThreads * U) {
+    for (uint32_t base = o0 + w * 32 * U; base < o1; base += kStAT * U) {
         uint32_t kk[U], vv[U], ll[U];
 #pragma unroll
         for (int u = 0; u < U; u++) {
@@ -516,10 +523,10 @@ __global__ void __launch_bounds__(kThreads) k_st_apply(TableView tv, StagedView 
     }
     flush();
     if (OP == 0) {
-        block_add<kThreads>(ctr + C_INSERTED, n_a);
-        block_add<kThreads>(ctr + C_UPDATED, n_b);
+        block_add<kStAT>(ctr + C_INSERTED, n_a);
+        block_add<kStAT>(ctr + C_UPDATED, n_b);
     } else if (OP == 2) {
-        block_add<kThreads>(ctr + C_REMOVED, n_a);
+        block_add<kStAT>(ctr + C_REMOVED, n_a);
     }
     if (OP != 1) {
         if (mod) changed = 1;

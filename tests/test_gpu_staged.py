@@ -129,3 +129,52 @@ def test_staged_not_used_for_other_bucket_widths(oracle_mod):
     wl = W.random_op_stream(55, n_batches=6, batch=3000, universe=6000, init_capacity=64)
     g, _ = run_staged(oracle_mod, wl, B=4)
     assert g.stats()["n_staged"] == 0
+
+
+def test_staged_with_in_place_subtables(oracle_mod):
+    """Subtables in reserved virtual ranges (DYC_RESIZE_IN_PLACE): the TMA bulk
+    copies address the mapped range like any other device buffer."""
+    wl = W.random_op_stream(4321, n_batches=16, batch=5000, universe=9000, init_capacity=512)
+    g = Table(d=wl.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=8,
+              staged="force", in_place=True)
+    o = oracle_mod.OracleTable(d=wl.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta,
+                               bucket_slots=8)
+    for i, b in enumerate(wl.batches):
+        kd = dev(b.keys)
+        if b.op == "insert":
+            np.testing.assert_array_equal(g.insert(kd, dev(b.values)).cpu().numpy(), o.insert(b.keys, b.values))
+        elif b.op == "find":
+            v, f = g.find(kd)
+            ov, of = o.find(b.keys)
+            np.testing.assert_array_equal(f.cpu().numpy(), of)
+            np.testing.assert_array_equal(host_u32(v), ov)
+        else:
+            v, st = g.delete(kd)
+            ov, os_ = o.delete(b.keys)
+            np.testing.assert_array_equal(st.cpu().numpy(), os_)
+            np.testing.assert_array_equal(host_u32(v), ov)
+        np.testing.assert_array_equal(g.sorted_kv(), o.sorted_kv(), err_msg=f"contents after batch {i}")
+    check_layout(g, o)
+    assert g.stats()["n_staged"] > 0
+
+
+def test_staged_not_used_with_paper_weighted_placement(oracle_mod):
+    """The paper's balancing rule gives up the first-choice-full
+    invariant the chunk pass decides misses with: its batches stay direct."""
+    wl = W.random_op_stream(77, n_batches=8, batch=4000, universe=8000, init_capacity=64)
+    g = Table(d=wl.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=8,
+              staged="force", placement="paper_weighted")
+    o = oracle_mod.OracleTable(d=wl.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta,
+                               bucket_slots=8)
+    for b in wl.batches:
+        if b.op == "insert":
+            np.testing.assert_array_equal(g.insert(dev(b.keys), dev(b.values)).cpu().numpy(),
+                                          o.insert(b.keys, b.values))
+        elif b.op == "find":
+            v, f = g.find(dev(b.keys))
+            np.testing.assert_array_equal(f.cpu().numpy(), o.find(b.keys)[1])
+        else:
+            v, st = g.delete(dev(b.keys))
+            np.testing.assert_array_equal(st.cpu().numpy(), o.delete(b.keys)[1])
+    np.testing.assert_array_equal(g.sorted_kv(), o.sorted_kv())
+    assert g.stats()["n_staged"] == 0
