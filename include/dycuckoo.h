@@ -139,7 +139,7 @@ typedef struct {
  * once; ops the first-choice bucket cannot decide go through the direct kernels.
  * Results are those of the direct path (each op's result depends only on the
  * table before the batch and its own key, P:L464 with distinct keys, Q9); only
- * where new keys land may differ.  Scratch: ~30 bytes per op, kept by the table
+ * where new keys land may differ.  Scratch: ~40 bytes per op, kept by the table
  * until dyc_trim.  Not used with a resize in flight, the paper-weighted
  * placement, a possibly non-empty stash, or the parts / mixed / host-buffer
  * entry points.  DYC_STAGED_OFF disables it; DYC_STAGED_FORCE uses it for every
