@@ -22,22 +22,24 @@
 // as in k_find / k_upsert; a delete takes the fullness of the bucket as it was
 // when its chunk was loaded (deletes of the same batch empty slots).
 //
-// Passes (one CUDA stream, no host wait):
-//   k_st_hist     one hash per op: its global first-choice bucket gb (kept),
-//                 and a per-chunk histogram (shared-memory counters)
-//   k_st_scan     chunk offsets; level-1 bins (2^s1 chunks each) and their tiles
-//   k_st_scatter1 tile-local counting sort by bin in shared memory, coalesced
-//                 runs out; per op its index in the tile's sorted order, per
-//                 tile the (bin -> run) table
-//   k_st_scatter2 the same inside each bin, by chunk
-//   k_st_apply    one CTA per chunk: TMA bulk load, ops in shared memory,
-//                 TMA bulk store; undecided ops -> need list (per-warp
-//                 shared-memory buffers, one global atomic per 64 entries)
-//   (need list)   gathered, run through k_upsert / k_find / k_delete with the
-//                 first probe skipped (S1), scattered back
-//   k_st_unperm   results back to request order, tile by tile: the tile's runs
-//                 are read coalesced into shared memory, then every op takes
-//                 its result from there (level 2, then level 1)
+// Passes (one CUDA stream, no host wait; DESIGN.md §5 "Staged batches"):
+//   k_st_hist       one hash per op: its global first-choice bucket gb (kept),
+//                   and a per-chunk histogram (shared-memory counters)
+//   k_st_scan       chunk offsets; level-1 bins (2^s1 chunks each) and the
+//                   level-2 tile tables
+//   k_st_scatter<1> tile-local counting sort by bin in shared memory, coalesced
+//                   runs out; per op its index in the tile's sorted order, per
+//                   sorted position the global destination (dmap)
+//   k_st_scatter<2> the same inside each bin, by chunk
+//   k_st_apply      one CTA per chunk: TMA bulk load, ops in shared memory,
+//                   TMA bulk store; undecided ops -> need list (per-warp
+//                   shared-memory buffers, one global atomic per 64 entries;
+//                   each entry: key, value, chunk-order position)
+//   (need list)     k_upsert / k_find / k_delete with the first probe skipped
+//                   (S1), results written at the entries' positions
+//   k_st_unperm     results back to request order, tile by tile: the tile's
+//                   sorted results are gathered through dmap into shared memory,
+//                   then every op takes its own (level 2, then level 1)
 #pragma once
 #include "dyc_kernels.cuh"
 
