@@ -960,7 +960,7 @@ def bench_stream(args, local):
                 "grow 16 batches then drain, 2 cycles")
     gen_s = time.time() - t0
     g = Table(d=args.d, init_capacity=wl.init_capacity, alpha=wl.alpha, beta=wl.beta, bucket_slots=args.bucket_slots,
-              placement=args.placement)
+              placement=args.placement, staged=args.staged)
     dev = lambda a: torch.from_numpy(np.ascontiguousarray(a, dtype=np.uint32).view(np.int32)).cuda()  # noqa: E731
     staged = []
     for b in batches:
