@@ -79,7 +79,14 @@ constexpr int kStUPer = kStTile / kStUT;          // positions per thread (unper
 constexpr int kStMaxS1 = 8;                       // 2^s1 chunks per level-1 bin, <= 256
 constexpr uint32_t kStMaxChunks = kStLog >= 10 ? 32768 : 49152;   // k_st_hist: one shared counter per chunk
 constexpr int kStHistT = 1024;
-constexpr int kStHistPer = 8;
+#ifndef DYC_ST_HIST_PER
+#define DYC_ST_HIST_PER 8
+#endif
+constexpr int kStHistPer = DYC_ST_HIST_PER;
+#ifndef DYC_ST_WUNROLL
+#define DYC_ST_WUNROLL 8
+#endif
+constexpr int kStWU = DYC_ST_WUNROLL;             // unroll of the scatter write-out loop
 constexpr int kStApplyU = DYC_ST_APPLY_U;         // ops per lane in flight (apply)
 constexpr int kStNeedBuf = 64;                    // per-warp need-list buffer (apply)
 constexpr int kStRun = 256;                       // bins (level 1) or chunks of a bin (level 2), at most
@@ -329,7 +336,7 @@ __global__ void __launch_bounds__(kStT, DYC_ST_SCATTER_MINB) k_st_scatter(Staged
         }
     }
     __syncthreads();
-#pragma unroll 4
+#pragma unroll kStWU
     for (uint32_t p = threadIdx.x; p < tn; p += kStT) {
         const uint32_t b = sbin[p];
         const uint32_t d = gbase[b] + (p - off[b]);
